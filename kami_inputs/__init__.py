@@ -1,0 +1,122 @@
+"""Seeded synthetic inputs for KAMI batched GEMM -- shared by the oracle side
+(tests, cpu baseline) and the CUDA side (tests, bench).
+
+This module holds NO GEMM arithmetic: it only draws operand values.  Every
+value is a pure function of (seed, operand, global entry index, element
+index) through a counter-based SplitMix64 hash, so
+
+  * entry e is identical whatever the batch chunking or GPU count
+    (multi-GPU shards generate only their own entries);
+  * the same torch code runs on CPU (oracle inputs) and on CUDA (bench inputs,
+    no host->device copy of gigabytes) and yields bit-identical values
+    (checked on the GPU by tests/test_gpu_inputs.py).
+
+Value recipes (the paper never states its value
+distribution, Sec. 5.1 -- reading R17):
+  "unif": uniform in [-1, 1) from 53 random bits, rounded RNE to the dtype;
+  "int" : uniform integer in [-R, R]; R chosen (``int_range``) so that
+          R^2 k <= 2048 (fp16) / 256 (bf16) / 2^40 (fp64): every product and
+          partial sum is an integer exactly representable in FP32 and every
+          result exactly representable in the output dtype, so any summation
+          order gives the same bits (bit-exact parity, north_star).
+"""
+from __future__ import annotations
+
+import torch
+
+MASK64 = (1 << 64) - 1
+_GOLDEN = 0x9E3779B97F4A7C15
+_M1 = 0xBF58476D1CE4E5B9
+_M2 = 0x94D049BB133111EB
+
+OPERAND_A = 0
+OPERAND_B = 1
+
+TORCH_DTYPES = {"f16": torch.float16, "bf16": torch.bfloat16, "f64": torch.float64}
+
+
+def _s64(u: int) -> int:
+    """uint64 constant -> the int64 with the same bits."""
+    u &= MASK64
+    return u - (1 << 64) if u >= (1 << 63) else u
+
+
+def _lshr(x: torch.Tensor, s: int) -> torch.Tensor:
+    """Logical right shift of int64 bit patterns."""
+    return (x >> s) & ((1 << (64 - s)) - 1)
+
+
+def splitmix64(x: torch.Tensor) -> torch.Tensor:
+    """SplitMix64 finaliser of (x + golden) on int64 tensors (two's complement wrap)."""
+    z = x + _s64(_GOLDEN)
+    z = (z ^ _lshr(z, 30)) * _s64(_M1)
+    z = (z ^ _lshr(z, 27)) * _s64(_M2)
+    return z ^ _lshr(z, 31)
+
+
+def splitmix64_py(x: int) -> int:
+    """Pure-Python reference of the same function (used to pin the torch version)."""
+    z = (x + _GOLDEN) & MASK64
+    z = ((z ^ (z >> 30)) * _M1) & MASK64
+    z = ((z ^ (z >> 27)) * _M2) & MASK64
+    return z ^ (z >> 31)
+
+
+def int_range(k: int, dtype: str) -> int:
+    """Largest R with R^2 * k <= limit (fp16 2048, bf16 256, fp64 2^40), R >= 1."""
+    limit = {"f16": 2048, "bf16": 256, "f64": 1 << 40}[dtype]
+    r = 1
+    while (r + 1) * (r + 1) * k <= limit:
+        r += 1
+    return r
+
+
+def counters(seed: int, operand: int, entry0: int, n_entries: int, elems: int,
+             device="cpu") -> torch.Tensor:
+    """int64 counters (seed, operand) * 2^44 + global element index."""
+    assert 0 <= seed < (1 << 17) and operand in (0, 1)
+    base = ((seed * 2 + operand) << 44) + entry0 * elems
+    return torch.arange(n_entries * elems, dtype=torch.int64, device=device) + base
+
+
+def draw(seed: int, operand: int, entry0: int, n_entries: int, rows: int, cols: int,
+         dtype: str, dist: str = "unif", R: int | None = None, device="cpu") -> torch.Tensor:
+    """Operand values for entries [entry0, entry0 + n_entries), packed, as a 1-D
+    tensor of ``dtype`` with n_entries * rows * cols elements.  The element
+    index is the storage index inside the entry, so the values do not depend
+    on the layout flag (the layout only says how they are interpreted)."""
+    elems = rows * cols
+    out = torch.empty(n_entries * elems, dtype=TORCH_DTYPES[dtype], device=device)
+    chunk = 1 << 24
+    total = n_entries * elems
+    base = ((seed * 2 + operand) << 44) + entry0 * elems
+    for s in range(0, total, chunk):
+        e = min(total, s + chunk)
+        z = splitmix64(torch.arange(s, e, dtype=torch.int64, device=device) + base)
+        if dist == "unif":
+            u = _lshr(z, 11).to(torch.float64) * (2.0 ** -52) - 1.0  # [-1, 1), exact
+        elif dist == "int":
+            assert R is not None and R >= 1
+            u = (torch.remainder(_lshr(z, 33), 2 * R + 1) - R).to(torch.float64)
+        else:
+            raise ValueError(dist)
+        out[s:e] = u.to(TORCH_DTYPES[dtype])
+    return out
+
+
+def operands(m: int, n: int, k: int, batch: int, dtype: str, dist: str = "unif",
+             seed: int = 0, entry0: int = 0, device="cpu"):
+    """(A, B) packed operands for entries [entry0, entry0+batch).  A has m*k
+    and B k*n elements per entry (layout-agnostic storage order)."""
+    R = int_range(k, dtype) if dist == "int" else None
+    A = draw(seed, OPERAND_A, entry0, batch, m, k, dtype, dist, R, device)
+    B = draw(seed, OPERAND_B, entry0, batch, k, n, dtype, dist, R, device)
+    return A, B
+
+
+def as_bits(x: torch.Tensor):
+    """numpy view usable by the oracle: uint16 bits for 16-bit dtypes, float64 otherwise."""
+    x = x.detach().cpu().contiguous()
+    if x.dtype in (torch.float16, torch.bfloat16):
+        return x.view(torch.int16).numpy().view("uint16")
+    return x.numpy()

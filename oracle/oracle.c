@@ -1,0 +1,218 @@
+/*
+ * oracle.c -- KAMI batched small-GEMM reference oracle.
+ *
+ * TEST INFRASTRUCTURE ONLY.  Only tests/, __graft_entry__.smoke() and the
+ * cpu_baseline / --impl reference legs of bench.py may load this library.
+ * The product path (paper_conf_sc_wangdltsl25_b200/, include/kami.h) never
+ * links, imports or executes anything under oracle/, and this file includes
+ * nothing from the product tree.
+ *
+ * What it computes (plain definitions, written out, no blocking/fusion):
+ *
+ *   GEMM (Sec. 2.1): C = A * B with A m-by-k, B k-by-n,
+ *   C m-by-n.  Batched GEMM (Sec. 2.1, Fig. 1(e)) applies it to
+ *   every entry b of a batch independently.  KAMI's 1D/2D/3D algorithms
+ *   (Alg. 1-3) only reorder data movement between warps,
+ *   so the exact result they approximate in floating point is
+ *
+ *       C_ref[b,i,j] = sum_{l=0}^{k-1} double(A[b,i,l]) * double(B[b,l,j])
+ *
+ *   accumulated in IEEE binary64 with l ascending.  Inputs are the already
+ *   dtype-rounded fp16 / bf16 / fp64 values, decoded exactly to double.
+ *
+ *   Layout (reading R4; "aligned to cuBLAS"): one
+ *   flag for all three matrices, packed, no leading dimensions.
+ *     row-major: X[b, r, c] at b*R*C + r*C + c
+ *     col-major: X[b, r, c] at b*R*C + c*R + r
+ *
+ *   Error scale (BASELINE.json north_star): S[b,i,j] = sum_l |A[b,i,l]| |B[b,l,j]|.
+ *
+ *   Round-to-nearest-even converters double -> fp16 / bf16 (used to form the
+ *   bit-exact expectation for integer-valued inputs, reading R2),
+ *   written with integer/bit manipulation and C99 rint() under the default
+ *   FE_TONEAREST mode.  No CUDA header is used.
+ *
+ * Pins: tests/test_oracle.py (hand cases, identity/permutation, closed forms,
+ * transpose identity, integer exactness, cross-check vs torch.matmul float64,
+ * RNE converter cases vs the IEEE 754 definition).
+ */
+#include <fenv.h>
+#include <math.h>
+#include <pthread.h>
+#include <stdint.h>
+#include <stdlib.h>
+#include <string.h>
+
+#define ORACLE_F16 0
+#define ORACLE_BF16 1
+#define ORACLE_F64 2
+
+#define ORACLE_ROW 0
+#define ORACLE_COL 1
+
+/* ---------------------------------------------------------------- decoders */
+
+/* IEEE 754 binary16: 1 sign, 5 exponent (bias 15), 10 fraction bits. */
+double oracle_f16_to_f64(uint16_t h) {
+  int s = (h >> 15) & 1;
+  int e = (h >> 10) & 0x1f;
+  int f = h & 0x3ff;
+  double v;
+  if (e == 0) {
+    v = ldexp((double)f, -24); /* subnormal: f * 2^-24 */
+  } else if (e == 31) {
+    v = f ? NAN : INFINITY;
+  } else {
+    v = ldexp((double)(1024 + f), e - 25); /* (1.f) * 2^(e-15) */
+  }
+  return s ? -v : v;
+}
+
+/* bfloat16: the upper 16 bits of an IEEE binary32. */
+double oracle_bf16_to_f64(uint16_t h) {
+  uint32_t u = ((uint32_t)h) << 16;
+  float f;
+  memcpy(&f, &u, sizeof f);
+  return (double)f;
+}
+
+/* ------------------------------------------------------ RNE encoders (f64) */
+
+/* Generic: round |a| (finite, > 0) to a binary format with `mbits` fraction
+ * bits, exponent bias `bias`, max biased exponent `emax_biased` (all-ones
+ * reserved).  Returns the magnitude bits. */
+static uint32_t rne_encode_mag(double a, int mbits, int bias, int emax_biased) {
+  int fe = 0;
+  double fr = frexp(a, &fe);       /* a = fr * 2^fe, fr in [0.5, 1) */
+  int E = fe - 1;                   /* a = (2 fr) * 2^E, 2fr in [1,2) */
+  int emin = 1 - bias;              /* smallest normal exponent */
+  uint32_t one = 1u << mbits;
+  if (E < emin) {
+    /* subnormal range: value = q * 2^(emin - mbits), q integer after RNE */
+    double q = rint(ldexp(a, mbits - emin));
+    /* q == one naturally encodes the smallest normal */
+    return (uint32_t)q;
+  }
+  double q = rint(ldexp(a, mbits - E)); /* in [one, 2*one] */
+  if (q >= (double)(2 * one)) {
+    q = (double)one;
+    E += 1;
+  }
+  int eb = E + bias;
+  if (eb >= emax_biased) return ((uint32_t)emax_biased) << mbits; /* inf */
+  return (((uint32_t)eb) << mbits) | ((uint32_t)q - one);
+}
+
+uint16_t oracle_f64_to_f16_rne(double x) {
+  if (isnan(x)) return 0x7e00;
+  uint16_t s = signbit(x) ? 0x8000 : 0;
+  double a = fabs(x);
+  if (a == 0.0) return s;
+  if (isinf(a)) return s | 0x7c00;
+  return s | (uint16_t)rne_encode_mag(a, 10, 15, 31);
+}
+
+uint16_t oracle_f64_to_bf16_rne(double x) {
+  if (isnan(x)) return 0x7fc0;
+  uint16_t s = signbit(x) ? 0x8000 : 0;
+  double a = fabs(x);
+  if (a == 0.0) return s;
+  if (isinf(a)) return s | 0x7f80;
+  return s | (uint16_t)rne_encode_mag(a, 7, 127, 255);
+}
+
+/* ------------------------------------------------------------ element read */
+
+static double load_elem(const void* base, int dtype, int64_t idx) {
+  switch (dtype) {
+    case ORACLE_F16:
+      return oracle_f16_to_f64(((const uint16_t*)base)[idx]);
+    case ORACLE_BF16:
+      return oracle_bf16_to_f64(((const uint16_t*)base)[idx]);
+    default:
+      return ((const double*)base)[idx];
+  }
+}
+
+/* index of X[b, r, c] for an R-by-C matrix (layout applies to all operands) */
+static int64_t at(int layout, int64_t b, int64_t r, int64_t c, int64_t R, int64_t C) {
+  return layout == ORACLE_ROW ? b * R * C + r * C + c : b * R * C + c * R + r;
+}
+
+/* ------------------------------------------------------------ GEMM oracle */
+
+typedef struct {
+  int m, n, k, dtype, layout;
+  int64_t b0, b1;
+  const void *A, *B;
+  double *C, *S; /* C/S are row-major [batch][m][n] regardless of layout */
+} job_t;
+
+static void* gemm_worker(void* arg) {
+  job_t* j = (job_t*)arg;
+  const int64_t m = j->m, n = j->n, k = j->k;
+  for (int64_t b = j->b0; b < j->b1; ++b) {
+    for (int64_t i = 0; i < m; ++i) {
+      for (int64_t jj = 0; jj < n; ++jj) {
+        double acc = 0.0, sabs = 0.0;
+        for (int64_t l = 0; l < k; ++l) { /* l ascending (R3) */
+          double a = load_elem(j->A, j->dtype, at(j->layout, b, i, l, m, k));
+          double bb = load_elem(j->B, j->dtype, at(j->layout, b, l, jj, k, n));
+          acc += a * bb;
+          sabs += fabs(a) * fabs(bb);
+        }
+        j->C[b * m * n + i * n + jj] = acc;
+        if (j->S) j->S[b * m * n + i * n + jj] = sabs;
+      }
+    }
+  }
+  return NULL;
+}
+
+/*
+ * oracle_gemm: C_ref (and optionally S) for every entry, threads over entries.
+ * C and S are written row-major [batch][m][n] (a host-side convention of the
+ * oracle, independent of the input layout).  Returns 0 on success.
+ */
+int oracle_gemm(int m, int n, int k, int64_t batch, int dtype, int layout,
+                const void* A, const void* B, double* C, double* S, int nthreads) {
+  if (m <= 0 || n <= 0 || k <= 0 || batch < 0) return 1;
+  if (dtype < 0 || dtype > 2 || layout < 0 || layout > 1) return 1;
+  if (batch == 0) return 0;
+  if (fegetround() != FE_TONEAREST) fesetround(FE_TONEAREST);
+  if (nthreads < 1) nthreads = 1;
+  if (nthreads > batch) nthreads = (int)batch;
+  pthread_t* th = (pthread_t*)malloc(sizeof(pthread_t) * nthreads);
+  job_t* jobs = (job_t*)malloc(sizeof(job_t) * nthreads);
+  for (int t = 0; t < nthreads; ++t) {
+    jobs[t].m = m; jobs[t].n = n; jobs[t].k = k;
+    jobs[t].dtype = dtype; jobs[t].layout = layout;
+    jobs[t].b0 = batch * t / nthreads;
+    jobs[t].b1 = batch * (t + 1) / nthreads;
+    jobs[t].A = A; jobs[t].B = B; jobs[t].C = C; jobs[t].S = S;
+  }
+  if (nthreads == 1) {
+    gemm_worker(&jobs[0]);
+  } else {
+    for (int t = 0; t < nthreads; ++t) pthread_create(&th[t], NULL, gemm_worker, &jobs[t]);
+    for (int t = 0; t < nthreads; ++t) pthread_join(th[t], NULL);
+  }
+  free(th);
+  free(jobs);
+  return 0;
+}
+
+/* Round an array of doubles to fp16 / bf16 bits with RNE (expectation for the
+ * bit-exact integer-valued parity cases). */
+void oracle_round_f16(const double* x, uint16_t* out, int64_t n) {
+  for (int64_t i = 0; i < n; ++i) out[i] = oracle_f64_to_f16_rne(x[i]);
+}
+void oracle_round_bf16(const double* x, uint16_t* out, int64_t n) {
+  for (int64_t i = 0; i < n; ++i) out[i] = oracle_f64_to_bf16_rne(x[i]);
+}
+void oracle_decode_f16(const uint16_t* x, double* out, int64_t n) {
+  for (int64_t i = 0; i < n; ++i) out[i] = oracle_f16_to_f64(x[i]);
+}
+void oracle_decode_bf16(const uint16_t* x, double* out, int64_t n) {
+  for (int64_t i = 0; i < n; ++i) out[i] = oracle_bf16_to_f64(x[i]);
+}
