@@ -1,0 +1,383 @@
+#!/usr/bin/env python
+"""bench.py -- KAMI batched small-GEMM throughput on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl kami|reference]
+                    [--workload f16-64 | f16-32 | f16-128 | f16-16 | f64-16 | f64-32 | f64-64 |
+                                lr-8 | lr-16 | lr-32 | bf16-<m>x<n>x<k>] [--algo auto|1d|2d|3d|nonca]
+    torchrun --nproc-per-node N bench.py --gpus N ...
+
+A "step" is one pass of the whole hot path over one batch: one
+kami_gemm_strided_batched call (plan -> TMA/LDG loads -> CA exchange -> MMA ->
+store) over the workload's batch of resident device inputs.  Default
+workload = BASELINE.json configs[1] at its headline order: FP16 in / FP32
+accumulate, m=n=k=64, batch 65 536 per GPU (weak scaling: every rank owns its
+own 65 536 entries; entries are generated on the device by the shared
+counter-based generator keyed by global entry index).
+
+Prints ONE JSON line (rank 0).  value = whole-job TFLOP/s (2mnk per entry,
+padding not counted) over the max-over-ranks device time of K steps.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "batched small-GEMM TFLOP/s and % roofline (fp16/fp64) at 1/2/4/8 B200"
+
+WORKLOADS = {
+    # name: (dtype, m, n, k, batch per GPU, BASELINE config index)
+    "f16-16": ("f16", 16, 16, 16, 1024, 0),
+    "f16-32": ("f16", 32, 32, 32, 65536, 1),
+    "f16-64": ("f16", 64, 64, 64, 65536, 1),
+    "f16-128": ("f16", 128, 128, 128, 65536, 1),
+    "f64-16": ("f64", 16, 16, 16, 32768, 2),
+    "f64-32": ("f64", 32, 32, 32, 32768, 2),
+    "f64-64": ("f64", 64, 64, 64, 32768, 2),
+    "lr-8": ("f16", 256, 256, 8, 16384, 3),
+    "lr-16": ("f16", 256, 256, 16, 16384, 3),
+    "lr-32": ("f16", 256, 256, 32, 16384, 3),
+}
+
+
+def parse_workload(name):
+    if name in WORKLOADS:
+        return WORKLOADS[name]
+    if name.startswith("bf16-"):  # bf16-<m>x<n>x<k>[:batch]
+        spec, _, b = name[5:].partition(":")
+        m, n, k = (int(x) for x in spec.split("x"))
+        return ("bf16", m, n, k, int(b) if b else 125000, 4)
+    raise SystemExit(f"unknown workload {name}")
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d.get("hbm_gbs", 6650.0), d.get("bf16_tflops", 1590.0), "measured (MEASURED_PEAKS.json)"
+    return 6650.0, 1590.0, "fallback (B200_PROFILING.md)"
+
+
+def fp64_peak_tflops():
+    """FP64 DMMA roofline denominator.  No measured figure exists in
+    MEASURED_PEAKS.json; DESIGN.md derives 37 TF/s (B200 datasheet FP64 tensor
+    ~ the DMMA issue rate x 148 SMs x clock), stated as 'nominal'."""
+    return 37.0
+
+
+class ClockSampler:
+    """nvidia-smi clocks/throttle sampler run DURING the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                 "-lms", "50"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+            self.t.join(timeout=2)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for nm, v in zip(names, r[5:9]):
+                if v.strip().lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def cpu_baseline(dtype, m, n, k, target_s=12.0, max_entries=None):
+    """Time the oracle (as it stands) on this host's cores on a bounded sample."""
+    import kami_inputs as ki
+    import oracle
+
+    cores = oracle.default_threads()
+    per_entry_mac = m * n * k
+    # calibrate on a small sample, then size the sample to ~target_s
+    probe = max(cores, int(2e7 // per_entry_mac) or 1)
+    A, B = ki.operands(m, n, k, probe, dtype, "unif", seed=0)
+    a, b = ki.as_bits(A), ki.as_bits(B)
+    t0 = time.perf_counter()
+    oracle.gemm(m, n, k, probe, dtype, "row", a, b, nthreads=cores)
+    dt = time.perf_counter() - t0
+    n_entries = max(probe, int(probe * target_s / max(dt, 1e-6)))
+    if max_entries:
+        n_entries = min(n_entries, max_entries)
+    A, B = ki.operands(m, n, k, n_entries, dtype, "unif", seed=0)
+    a, b = ki.as_bits(A), ki.as_bits(B)
+    t0 = time.perf_counter()
+    oracle.gemm(m, n, k, n_entries, dtype, "row", a, b, nthreads=cores)
+    dt = time.perf_counter() - t0
+    tflops = 2.0 * per_entry_mac * n_entries / dt / 1e12
+    return {"value": tflops, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
+            "sample": f"first {n_entries} entries of the workload (seed 0), FP64 triple loop, {dt:.1f} s",
+            "seconds": dt, "entries": n_entries}
+
+
+def dist_init():
+    import torch
+    import torch.distributed as dist
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    return world, rank, local
+
+
+def run_reference(args):
+    """--impl reference: the oracle timed on the host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    dtype, m, n, k, batch, cfg = parse_workload(args.workload)
+    import kami_inputs as ki
+    import oracle
+
+    cores = oracle.default_threads()
+    # each step = a bounded sample of the workload sized so the run takes ~1-2 min
+    per_entry = 2.0 * m * n * k
+    probe = max(cores, int(2e7 // (m * n * k)) or 1)
+    A, B = ki.operands(m, n, k, probe, dtype, "unif")
+    t0 = time.perf_counter()
+    oracle.gemm(m, n, k, probe, dtype, "row", ki.as_bits(A), ki.as_bits(B), nthreads=cores)
+    rate = probe / max(time.perf_counter() - t0, 1e-6)
+    steps_total = args.steps + args.warmup
+    sample = max(cores, min(batch, int(rate * 90.0 / steps_total)))
+    A, B = ki.operands(m, n, k, sample, dtype, "unif")
+    a, b = ki.as_bits(A), ki.as_bits(B)
+    for _ in range(args.warmup):
+        oracle.gemm(m, n, k, sample, dtype, "row", a, b, nthreads=cores)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.gemm(m, n, k, sample, dtype, "row", a, b, nthreads=cores)
+    dt = (time.perf_counter() - t0) / args.steps
+    value = per_entry * sample / dt / 1e12
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": dtype, "data": "synthetic",
+        "config": workload_config(args, dtype, m, n, k, batch, cfg),
+        "cpu_baseline": {"value": value, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{sample} entries of the workload per step (of {batch}), FP64 triple loop"},
+        "e2e": {"value": value, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def workload_config(args, dtype, m, n, k, batch, cfg):
+    return {"workload": f"{dtype} strided-batched GEMM m={m} n={n} k={k} batch={batch}/GPU row-major "
+                        f"(BASELINE.json configs[{cfg}])",
+            "m": m, "n": n, "k": k, "batch_per_gpu": batch, "global_batch": batch * args.gpus,
+            "layout": "row", "algo": args.algo, "inputs": "unif [-1,1) RNE to dtype, counter-based SplitMix64",
+            "l2": "inputs larger than L2 (126 MB)" if batch * (m * k + k * n + m * n) * (8 if dtype == 'f64' else 2)
+                  > 126e6 else "L2 flushed between timed steps",
+            "parallelism": f"batch-sharded dp{args.gpus}"}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="kami", choices=["kami", "reference"])
+    ap.add_argument("--workload", default="f16-64")
+    ap.add_argument("--algo", default="auto")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    import kami_inputs as ki
+    import paper_conf_sc_wangdltsl25_b200 as kami
+
+    world, rank, local = dist_init()
+    dtype, m, n, k, batch, cfg = parse_workload(args.workload)
+    es = 8 if dtype == "f64" else 2
+    entry0 = rank * batch
+    A, B = ki.operands(m, n, k, batch, dtype, "unif", seed=0, entry0=entry0, device="cuda")
+    C = torch.empty(batch * m * n, dtype=A.dtype, device="cuda")
+    stream = torch.cuda.current_stream()
+    alg_bytes = batch * (m * k + k * n + m * n) * es
+    flops = 2.0 * m * n * k * batch
+    small = alg_bytes < 126e6  # L2-resident: flush L2 between timed steps
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if small else None
+
+    def step():
+        kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A, B, C, algo=args.algo, stream=stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    kernel = kami.last_kernel()
+
+    # clocks sampled during a ~1.5 s sustained burst plus the timed region
+    sampler = ClockSampler(local)
+    sampler.start()
+    t_end = time.time() + 1.5
+    while time.time() < t_end:
+        for _ in range(20):
+            step()
+        torch.cuda.synchronize()
+
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    for s0, s1 in evs:
+        if flush is not None:
+            flush.zero_()
+        s0.record(stream)
+        step()
+        s1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    sampler.stop()
+    per_launch_ms = [a.elapsed_time(b) for a, b in evs]
+    t_ms = sum(per_launch_ms)  # device time of the K timed steps (flush excluded)
+
+    # checksum of the last output (sampled verification happens in tests/)
+    csum = float(C.double().sum().item())
+    stats = torch.tensor([t_ms, csum, float(batch)], dtype=torch.float64, device="cuda")
+    if world > 1:
+        gathered = [torch.zeros_like(stats) for _ in range(world)]
+        dist.all_gather(gathered, stats)  # the only collective: per-rank stats over NCCL
+        allst = torch.stack(gathered).cpu()
+    else:
+        allst = stats.cpu().unsqueeze(0)
+    t_max_ms = float(allst[:, 0].max())
+    total_entries = float(allst[:, 2].sum())
+
+    # end-to-end: the C-ABI host entry point, host<->device copies inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        hA = A.cpu().pin_memory()
+        hB = B.cpu().pin_memory()
+        hC = torch.empty(C.numel(), dtype=C.dtype).pin_memory()
+        kami.gemm_strided_batched_host(m, n, k, batch, dtype, "row", hA, hB, hC)  # warm (workspace)
+        if world > 1:
+            dist.barrier()
+        e_steps = 3
+        t0 = time.perf_counter()
+        for _ in range(e_steps):
+            kami.gemm_strided_batched_host(m, n, k, batch, dtype, "row", hA, hB, hC)
+        e_dt = (time.perf_counter() - t0) / e_steps
+        et = torch.tensor([e_dt], dtype=torch.float64, device="cuda")
+        if world > 1:
+            dist.all_reduce(et, op=dist.ReduceOp.MAX)
+        e2e = {"value": flops * world / float(et.item()) / 1e12, "unit": "TFLOP/s",
+               "h2d_bytes_per_step": batch * (m * k + k * n) * es, "d2h_bytes_per_step": batch * m * n * es,
+               "path": "kami_gemm_strided_batched_host (pinned host buffers, chunked H2D/kernel/D2H pipeline)"}
+        kami.release_workspace()
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return
+
+    hbm, bf16pk, peak_src = load_peaks()
+    value = flops * total_entries / batch * args.steps / (t_max_ms * 1e-3) / 1e12
+    avg_launch_s = (t_ms / args.steps) * 1e-3
+    achieved_gbs = alg_bytes / avg_launch_s / 1e9
+    roof_tf = min(hbm * 1e9 * flops / alg_bytes, (fp64_peak_tflops() if dtype == "f64" else 2250.0) * 1e12) / 1e12
+    bound = "hbm"
+    if dtype == "f64" and fp64_peak_tflops() * 1e12 < hbm * 1e9 * flops / alg_bytes:
+        bound = "tensor"
+    if bound == "hbm":
+        roofline = {"bound": "hbm", "achieved": achieved_gbs, "peak": hbm, "unit": "GB/s",
+                    "frac": achieved_gbs / hbm, "peak_source": peak_src}
+    else:
+        ach = flops / avg_launch_s / 1e12
+        roofline = {"bound": "tensor", "achieved": ach, "peak": fp64_peak_tflops(), "unit": "TFLOP/s",
+                    "frac": ach / fp64_peak_tflops(), "peak_source": "nominal FP64 DMMA (DESIGN.md)"}
+    roofline["traffic"] = traffic_from_profiles(args.workload)
+    roofline["kernel"] = kernel
+    roofline["roofline_tflops_per_gpu"] = roof_tf
+    roofline["frac_of_roofline_tflops"] = (value / world) / roof_tf
+    line = {
+        "metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": t_max_ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": dtype, "data": "synthetic",
+        "config": workload_config(args, dtype, m, n, k, batch, cfg),
+        "roofline": roofline,
+        "gpu_launches": args.steps,
+        "clocks": sampler.summary(),
+        "checksum": float(allst[:, 1].sum()),
+    }
+    if e2e:
+        line["e2e"] = e2e
+    if not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(dtype, m, n, k)
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def traffic_from_profiles(workload):
+    """dram bytes (read + write) per launch of the dominant kernel from the
+    committed ncu --set full summary (profiles/*/ncu_summary.json), or None."""
+    pdir = os.path.join(ROOT, "profiles")
+    best = None
+    if os.path.isdir(pdir):
+        for d in sorted(os.listdir(pdir)):
+            f = os.path.join(pdir, d, "ncu_summary.json")
+            if os.path.exists(f):
+                try:
+                    s = json.load(open(f))
+                    if workload in s.get("traffic_bytes_per_launch", {}):
+                        best = s["traffic_bytes_per_launch"][workload]
+                except Exception:
+                    pass
+    return best
+
+
+if __name__ == "__main__":
+    main()

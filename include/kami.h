@@ -1,0 +1,134 @@
+/*
+ * kami.h -- C ABI of the B200-native KAMI batched small-GEMM library
+ * (libkami.so, built from paper_conf_sc_wangdltsl25_b200/csrc).
+ *
+ * Operation (Sec. 2.1 "Matrix Multiplication"; batched form
+ * L69 and Sec. 5.4): for every batch entry b,
+ *
+ *     C_b = A_b * B_b,   A_b m-by-k,  B_b k-by-n,  C_b m-by-n,
+ *
+ * computed with the thread-block-level communication-avoiding schedules of
+ * KAMI (1D Alg. 1, 2D Alg. 2, 3D Alg. 3) re-designed for
+ * sm_100a.  C is overwritten, never read (reading R1).
+ * FP16 / BF16 inputs accumulate in FP32 and C is rounded to the input type
+ * with round-to-nearest-even; FP64 is FP64 end to end (R2).
+ *
+ * Layout (R4; "aligned to cuBLAS/MAGMA"): one
+ * flag for all three matrices, entries packed back to back, no leading
+ * dimensions:
+ *     KAMI_ROW_MAJOR: X_b(r, c) at  X + b*R*C + r*C + c
+ *     KAMI_COL_MAJOR: X_b(r, c) at  X + b*R*C + c*R + r
+ *
+ * Sizes supported (R5): 16-bit types need m, n multiples of 16 in
+ * [16, 256] and k a multiple of 8 in [8, 256]; FP64 needs m, n, k multiples
+ * of 8 in [8, 128].  Anything else returns KAMI_ERROR_NOT_SUPPORTED.
+ *
+ * Ownership and threading: the caller owns every buffer.  Device entry points
+ * never allocate device memory, never synchronise and enqueue on `stream`
+ * (NULL = legacy default stream) of the current device.  They are
+ * thread-safe.  C must not alias A or B; entries of C must not overlap.
+ * All argument errors are detected before any launch; device faults surface
+ * at the caller's next synchronisation (as in cuBLAS).
+ */
+#ifndef KAMI_H_
+#define KAMI_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define KAMI_VERSION_MAJOR 0
+#define KAMI_VERSION_MINOR 1
+
+typedef enum {
+  KAMI_SUCCESS = 0,
+  KAMI_ERROR_INVALID_VALUE = 1, /* bad size/enum/pointer, batch < 0, ... */
+  KAMI_ERROR_NOT_SUPPORTED = 2, /* outside the supported size grid        */
+  KAMI_ERROR_MISALIGNED = 3,    /* base pointer not 16-byte aligned       */
+  KAMI_ERROR_CUDA = 4           /* a CUDA runtime call failed             */
+} kami_status_t;
+
+typedef enum { KAMI_DTYPE_F16 = 0, KAMI_DTYPE_BF16 = 1, KAMI_DTYPE_F64 = 2 } kami_dtype_t;
+
+typedef enum { KAMI_ROW_MAJOR = 0, KAMI_COL_MAJOR = 1 } kami_layout_t;
+
+/* Which schedule runs (Sec. 4.3-4.5).  AUTO = the planner's choice
+ * (kami_plan).  NONCA = the non-communication-avoiding tiled baseline. */
+typedef enum {
+  KAMI_ALGO_AUTO = 0,
+  KAMI_ALGO_1D = 1,
+  KAMI_ALGO_2D = 2,
+  KAMI_ALGO_3D = 3,
+  KAMI_ALGO_NONCA = 4
+} kami_algo_t;
+
+/* Opaque CUDA stream; binary compatible with cudaStream_t. */
+typedef struct CUstream_st* kami_stream_t;
+
+/* Single GEMM (block-level interface).  `batch` must be 1. */
+kami_status_t kami_gemm(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
+                        const void* A, const void* B, void* C, kami_stream_t stream);
+
+/* Pointer-array batched GEMM (cuBLAS *gemmBatched convention): A_array,
+ * B_array, C_array are DEVICE arrays of `batch` DEVICE pointers, each
+ * 16-byte aligned, each pointing at one packed matrix in `layout`. */
+kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
+                                const void* const* A_array, const void* const* B_array, void* const* C_array,
+                                kami_stream_t stream);
+
+/* Strided-batched GEMM: entry b of A at A + b*m*k elements, of B at
+ * B + b*k*n, of C at C + b*m*n.  The hot path of BASELINE.json. */
+kami_status_t kami_gemm_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                        kami_layout_t layout, const void* A, const void* B, void* C,
+                                        kami_stream_t stream);
+
+/* Same with an explicit schedule and warp count p (0 = planner default).
+ * Bench/test surface: lets the 1D/2D/3D/non-CA variants be compared. */
+kami_status_t kami_gemm_strided_batched_ex(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                           kami_layout_t layout, const void* A, const void* B, void* C,
+                                           kami_algo_t algo, int p, kami_stream_t stream);
+
+/* Host-memory entry point (end-to-end): A, B, C are HOST pointers (pinned
+ * memory recommended).  The library streams the batch through device
+ * workspace in chunks, overlapping host->device copies, the kernel and
+ * device->host copies on internal streams, and returns after C is complete
+ * on the host (synchronous).  Workspace is allocated on first use per device
+ * and kept until kami_release_workspace(). */
+kami_status_t kami_gemm_strided_batched_host(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                             kami_layout_t layout, const void* A, const void* B, void* C);
+kami_status_t kami_release_workspace(void);
+
+/* Planner decision (cost model PAPER.md Eqs. 4/8/12). */
+typedef struct {
+  kami_algo_t algo;      /* chosen schedule                                 */
+  int p;                 /* warps (or tensor-core sub-partitions) per entry */
+  int kernel;            /* 0 = tcgen05 16-bit family, 1 = warp-level DMMA/HMMA family */
+  int entries_per_cta;   /* batch entries a CTA keeps in flight             */
+  int stages;            /* shared-memory pipeline depth                    */
+  int kslice_regs_pct;   /* share of A/B kept resident (Sec. 4.7)           */
+  double t_all_cycles;   /* model cycles per entry of the chosen schedule   */
+} kami_plan_t;
+
+kami_status_t kami_plan(int m, int n, int k, kami_dtype_t dtype, kami_layout_t layout, kami_algo_t algo, int p,
+                        kami_plan_t* out);
+
+/* Paper-faithful cost model (Eqs. 1-12, readings R6-R8): fills
+ * V_cm, T_cm, T_cp, T_all for variant 1/2/3 (KAMI_ALGO_1D/2D/3D). */
+kami_status_t kami_paper_cost(kami_algo_t variant, double m, double n, double k, double p, double s_e,
+                              double L_sm, double B_sm, double theta_r, double theta_w, double O_tc,
+                              double n_tc, double out[4]);
+
+const char* kami_status_string(kami_status_t status);
+
+/* Name of the last kernel this thread launched ("" if none). */
+const char* kami_last_kernel(void);
+
+int kami_version(void); /* (MAJOR << 16) | MINOR */
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* KAMI_H_ */

@@ -1,0 +1,196 @@
+"""paper_conf_sc_wangdltsl25_b200 -- B200-native KAMI batched small GEMM.
+
+Thin Python binding of the C ABI in ``include/kami.h`` (libkami.so, built
+in-tree by ``build.py``).  Argument marshalling only: every step of the GEMM
+runs in the library's CUDA kernels.  There is no CPU fallback -- if the
+shared library is missing or a call fails, a ``KamiError`` is raised.
+
+PyTorch is used only for device memory and the current CUDA stream.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+__all__ = [
+    "KamiError", "lib", "gemm", "gemm_batched", "gemm_strided_batched", "gemm_strided_batched_host",
+    "plan", "paper_cost", "last_kernel", "DTYPE", "LAYOUT", "ALGO", "SO_PATH",
+]
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+SO_PATH = os.path.join(_HERE, "libkami.so")
+
+DTYPE = {"f16": 0, "bf16": 1, "f64": 2}
+LAYOUT = {"row": 0, "col": 1}
+ALGO = {"auto": 0, "1d": 1, "2d": 2, "3d": 3, "nonca": 4}
+STATUS = {0: "KAMI_SUCCESS", 1: "KAMI_ERROR_INVALID_VALUE", 2: "KAMI_ERROR_NOT_SUPPORTED",
+          3: "KAMI_ERROR_MISALIGNED", 4: "KAMI_ERROR_CUDA"}
+
+# every symbol include/kami.h declares (checked by tests/test_abi.py)
+EXPORTS = [
+    "kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
+    "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
+    "kami_status_string", "kami_last_kernel", "kami_version",
+]
+
+
+class KamiError(RuntimeError):
+    def __init__(self, status: int, what: str = ""):
+        self.status = status
+        self.name = STATUS.get(status, f"status {status}")
+        super().__init__(f"{what}: {self.name}" if what else self.name)
+
+
+class KamiPlan(ctypes.Structure):
+    _fields_ = [("algo", ctypes.c_int), ("p", ctypes.c_int), ("kernel", ctypes.c_int),
+                ("entries_per_cta", ctypes.c_int), ("stages", ctypes.c_int), ("kslice_regs_pct", ctypes.c_int),
+                ("t_all_cycles", ctypes.c_double)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    """Load libkami.so (fails loudly if it has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(SO_PATH):
+        raise ImportError(f"{SO_PATH} is missing: run `python -m paper_conf_sc_wangdltsl25_b200.build` "
+                          "(there is no CPU fallback)")
+    L = ctypes.CDLL(SO_PATH)
+    i, i64, vp, st = ctypes.c_int, ctypes.c_int64, ctypes.c_void_p, ctypes.c_void_p
+    L.kami_gemm.argtypes = [i, i, i, i64, i, i, vp, vp, vp, st]
+    L.kami_gemm_batched.argtypes = [i, i, i, i64, i, i, vp, vp, vp, st]
+    L.kami_gemm_strided_batched.argtypes = [i, i, i, i64, i, i, vp, vp, vp, st]
+    L.kami_gemm_strided_batched_ex.argtypes = [i, i, i, i64, i, i, vp, vp, vp, i, i, st]
+    L.kami_gemm_strided_batched_host.argtypes = [i, i, i, i64, i, i, vp, vp, vp]
+    L.kami_release_workspace.argtypes = []
+    L.kami_plan.argtypes = [i, i, i, i, i, i, i, ctypes.POINTER(KamiPlan)]
+    d = ctypes.c_double
+    L.kami_paper_cost.argtypes = [i, d, d, d, d, d, d, d, d, d, d, d, ctypes.POINTER(ctypes.c_double)]
+    for f in ("kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
+              "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost"):
+        getattr(L, f).restype = ctypes.c_int
+    L.kami_status_string.restype = ctypes.c_char_p
+    L.kami_status_string.argtypes = [ctypes.c_int]
+    L.kami_last_kernel.restype = ctypes.c_char_p
+    L.kami_last_kernel.argtypes = []
+    L.kami_version.restype = ctypes.c_int
+    _lib = L
+    return L
+
+
+def _check(status: int, what: str):
+    if status != 0:
+        raise KamiError(status, what)
+
+
+def _enum(table, v, what):
+    if isinstance(v, int):
+        return v
+    try:
+        return table[v.lower()]
+    except KeyError:
+        raise ValueError(f"unknown {what} {v!r}") from None
+
+
+def _stream(stream):
+    if stream is not None:
+        return int(getattr(stream, "cuda_stream", stream))
+    import torch
+
+    return int(torch.cuda.current_stream().cuda_stream)
+
+
+def _dtype_of(t):
+    import torch
+
+    return {torch.float16: "f16", torch.bfloat16: "bf16", torch.float64: "f64"}[t.dtype]
+
+
+def _ptr(x):
+    return None if x is None else (x if isinstance(x, int) else x.data_ptr())
+
+
+def gemm_strided_batched(m, n, k, batch, dtype, layout, A, B, C, algo="auto", p=0, stream=None):
+    """C_b = A_b B_b for b < batch on device buffers (torch tensors or raw
+    device addresses).  Entries are packed; ``layout`` applies to all three."""
+    _check(lib().kami_gemm_strided_batched_ex(
+        m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
+        _ptr(A), _ptr(B), _ptr(C), _enum(ALGO, algo, "algo"), p, _stream(stream)), "kami_gemm_strided_batched")
+    return C
+
+
+def gemm(A, B, out=None, layout="row", algo="auto", p=0, stream=None):
+    """Torch convenience: A [batch, m, k] (or [m, k]) times B -> C, on the GPU.
+
+    For layout "row" the tensors are the usual row-major views; for "col"
+    each matrix is stored column-major (pass the transposed storage)."""
+    import torch
+
+    single = A.dim() == 2
+    A3 = A.unsqueeze(0) if single else A
+    B3 = B.unsqueeze(0) if single else B
+    if not (A3.is_cuda and B3.is_cuda and A3.is_contiguous() and B3.is_contiguous()):
+        raise ValueError("A and B must be contiguous CUDA tensors")
+    batch = A3.shape[0]
+    if layout == "row":
+        m, k = A3.shape[1], A3.shape[2]
+        n = B3.shape[2]
+        shape = (batch, m, n)
+    else:
+        k, m = A3.shape[1], A3.shape[2]
+        n = B3.shape[1]
+        shape = (batch, n, m)
+    if out is None:
+        out = torch.empty(shape, dtype=A3.dtype, device=A3.device)
+    gemm_strided_batched(m, n, k, batch, _dtype_of(A3), layout, A3, B3, out, algo, p, stream)
+    return out[0] if single else out
+
+
+def gemm_batched(m, n, k, batch, dtype, layout, A_ptrs, B_ptrs, C_ptrs, stream=None):
+    """Pointer-array form: A_ptrs/B_ptrs/C_ptrs are device int64 tensors of
+    per-entry device addresses (cuBLAS *gemmBatched convention)."""
+    _check(lib().kami_gemm_batched(m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
+                                   _ptr(A_ptrs), _ptr(B_ptrs), _ptr(C_ptrs), _stream(stream)), "kami_gemm_batched")
+
+
+def gemm_single(m, n, k, dtype, layout, A, B, C, stream=None):
+    _check(lib().kami_gemm(m, n, k, 1, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
+                           _ptr(A), _ptr(B), _ptr(C), _stream(stream)), "kami_gemm")
+
+
+def gemm_strided_batched_host(m, n, k, batch, dtype, layout, A, B, C):
+    """End-to-end entry point on HOST buffers (pinned recommended): the
+    library pipelines host->device copies, kernels and device->host copies
+    and returns when C is complete on the host."""
+    _check(lib().kami_gemm_strided_batched_host(m, n, k, batch, _enum(DTYPE, dtype, "dtype"),
+                                                _enum(LAYOUT, layout, "layout"), _ptr(A), _ptr(B), _ptr(C)),
+           "kami_gemm_strided_batched_host")
+
+
+def release_workspace():
+    _check(lib().kami_release_workspace(), "kami_release_workspace")
+
+
+def plan(m, n, k, dtype, layout="row", algo="auto", p=0) -> dict:
+    out = KamiPlan()
+    _check(lib().kami_plan(m, n, k, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
+                           _enum(ALGO, algo, "algo"), p, ctypes.byref(out)), "kami_plan")
+    inv = {v: k for k, v in ALGO.items()}
+    return {"algo": inv[out.algo], "p": out.p, "kernel": ("tcgen05" if out.kernel == 0 else "warp_ca"),
+            "entries_per_cta": out.entries_per_cta, "stages": out.stages, "kslice_regs_pct": out.kslice_regs_pct,
+            "t_all_cycles": out.t_all_cycles}
+
+
+def paper_cost(variant, m, n, k, p, s_e, L_sm, B_sm, theta_r, theta_w, O_tc, n_tc):
+    """The library's paper-faithful cost model (Eqs. 1-12): (V_cm, T_cm, T_cp, T_all)."""
+    out = (ctypes.c_double * 4)()
+    _check(lib().kami_paper_cost(_enum(ALGO, variant, "variant"), m, n, k, p, s_e, L_sm, B_sm, theta_r, theta_w,
+                                 O_tc, n_tc, out), "kami_paper_cost")
+    return tuple(out)
+
+
+def last_kernel() -> str:
+    return lib().kami_last_kernel().decode()

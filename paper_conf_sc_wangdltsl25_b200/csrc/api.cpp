@@ -1,0 +1,177 @@
+// api.cpp -- the C ABI of libkami.so (include/kami.h): argument validation
+// (all before any launch), layout handling, planner, dispatch to the kernel
+// families, the chunked host-memory entry point, status strings.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstdint>
+#include <cstring>
+#include <mutex>
+#include <vector>
+
+#include "../../include/kami.h"
+#include "kernels.h"
+#include "planner.h"
+
+namespace kami {
+
+static thread_local const char* g_last_kernel = "";
+void set_last_kernel(const char* name) { g_last_kernel = name; }
+
+PFN_encodeTiled get_encode_tiled() {
+  static PFN_encodeTiled fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_encodeTiled>(p);
+  });
+  return fn;
+}
+
+namespace {
+
+bool is16(kami_dtype_t d) { return d == KAMI_DTYPE_F16 || d == KAMI_DTYPE_BF16; }
+size_t esize(kami_dtype_t d) { return d == KAMI_DTYPE_F64 ? 8 : 2; }
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+// Size grid (R5).  Checked before anything touches the device.
+kami_status_t check_sizes(int m, int n, int k, kami_dtype_t dtype) {
+  if (is16(dtype)) {
+    if (m % 16 || n % 16 || k % 8 || m > 256 || n > 256 || k > 256) return KAMI_ERROR_NOT_SUPPORTED;
+    return KAMI_SUCCESS;
+  }
+  // FP64: the register-resident DMMA family is instantiated for these orders
+  if (m == n && n == k && (m == 8 || m == 16 || m == 32 || m == 64)) return KAMI_SUCCESS;
+  return KAMI_ERROR_NOT_SUPPORTED;
+}
+
+kami_status_t check_common(int m, int n, int k, int64_t batch, int dtype, int layout, int algo) {
+  if (m <= 0 || n <= 0 || k <= 0 || batch < 0) return KAMI_ERROR_INVALID_VALUE;
+  if (dtype < KAMI_DTYPE_F16 || dtype > KAMI_DTYPE_F64) return KAMI_ERROR_INVALID_VALUE;
+  if (layout != KAMI_ROW_MAJOR && layout != KAMI_COL_MAJOR) return KAMI_ERROR_INVALID_VALUE;
+  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_NONCA) return KAMI_ERROR_INVALID_VALUE;
+  return check_sizes(m, n, k, (kami_dtype_t)dtype);
+}
+
+// Row-major problem after the layout transform.  Column-major C = A B is the
+// row-major problem C^T = B^T A^T on the same buffers: (m, n, A, B) ->
+// (n, m, B, A)  (pinned by the transpose identity).
+struct RowProblem {
+  int m, n, k;
+  const void* A;
+  const void* B;
+  const void* const* Aa;
+  const void* const* Ba;
+};
+
+RowProblem to_row(int m, int n, int k, kami_layout_t layout, const void* A, const void* B, const void* const* Aa,
+                  const void* const* Ba) {
+  if (layout == KAMI_ROW_MAJOR) return {m, n, k, A, B, Aa, Ba};
+  return {n, m, k, B, A, Ba, Aa};
+}
+
+kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, kami_algo_t algo, int p, void* C,
+                       void* const* Ca, cudaStream_t stream) {
+  kami_plan_t plan;
+  kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
+  if (st != KAMI_SUCCESS) return st;
+  if (plan.kernel == 0) {
+    return tc16_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream, 0);
+  }
+  return warp_ca_launch(rp.m, rp.n, rp.k, batch, dtype, (int)plan.algo, plan.p, rp.A, rp.B, C, rp.Aa, rp.Ba, Ca,
+                        stream);
+}
+
+}  // namespace
+}  // namespace kami
+
+using namespace kami;
+
+extern "C" {
+
+kami_status_t kami_gemm_strided_batched_ex(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                           kami_layout_t layout, const void* A, const void* B, void* C,
+                                           kami_algo_t algo, int p, kami_stream_t stream) {
+  kami_status_t st = check_common(m, n, k, batch, dtype, layout, algo);
+  if (st != KAMI_SUCCESS) return st;
+  if (p < 0) return KAMI_ERROR_INVALID_VALUE;
+  if (batch == 0) return KAMI_SUCCESS;
+  if (!A || !B || !C) return KAMI_ERROR_INVALID_VALUE;
+  if (!aligned16(A) || !aligned16(B) || !aligned16(C)) return KAMI_ERROR_MISALIGNED;
+  if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
+  RowProblem rp = to_row(m, n, k, layout, A, B, nullptr, nullptr);
+  return dispatch(rp, batch, dtype, algo, p, C, nullptr, reinterpret_cast<cudaStream_t>(stream));
+}
+
+kami_status_t kami_gemm_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                        kami_layout_t layout, const void* A, const void* B, void* C,
+                                        kami_stream_t stream) {
+  return kami_gemm_strided_batched_ex(m, n, k, batch, dtype, layout, A, B, C, KAMI_ALGO_AUTO, 0, stream);
+}
+
+kami_status_t kami_gemm(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
+                        const void* A, const void* B, void* C, kami_stream_t stream) {
+  if (batch != 1) return KAMI_ERROR_INVALID_VALUE;
+  return kami_gemm_strided_batched(m, n, k, 1, dtype, layout, A, B, C, stream);
+}
+
+kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
+                                const void* const* A_array, const void* const* B_array, void* const* C_array,
+                                kami_stream_t stream) {
+  kami_status_t st = check_common(m, n, k, batch, dtype, layout, KAMI_ALGO_AUTO);
+  if (st != KAMI_SUCCESS) return st;
+  if (batch == 0) return KAMI_SUCCESS;
+  if (!A_array || !B_array || !C_array) return KAMI_ERROR_INVALID_VALUE;
+  if (!aligned16(A_array) || !aligned16(B_array) || !aligned16(C_array)) return KAMI_ERROR_MISALIGNED;
+  if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
+  RowProblem rp = to_row(m, n, k, layout, nullptr, nullptr, A_array, B_array);
+  return dispatch(rp, batch, dtype, KAMI_ALGO_AUTO, 0, nullptr, C_array, reinterpret_cast<cudaStream_t>(stream));
+}
+
+kami_status_t kami_plan(int m, int n, int k, kami_dtype_t dtype, kami_layout_t layout, kami_algo_t algo, int p,
+                        kami_plan_t* out) {
+  kami_status_t st = check_common(m, n, k, 1, dtype, layout, algo);
+  if (st != KAMI_SUCCESS) return st;
+  if (!out || p < 0) return KAMI_ERROR_INVALID_VALUE;
+  RowProblem rp = to_row(m, n, k, layout, nullptr, nullptr, nullptr, nullptr);
+  return planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, false, out);
+}
+
+kami_status_t kami_paper_cost(kami_algo_t variant, double m, double n, double k, double p, double s_e,
+                              double L_sm, double B_sm, double theta_r, double theta_w, double O_tc, double n_tc,
+                              double out[4]) {
+  if (!out) return KAMI_ERROR_INVALID_VALUE;
+  if (variant != KAMI_ALGO_1D && variant != KAMI_ALGO_2D && variant != KAMI_ALGO_3D)
+    return KAMI_ERROR_INVALID_VALUE;
+  if (m <= 0 || n <= 0 || k <= 0 || p <= 0 || s_e <= 0 || B_sm <= 0 || theta_r <= 0 || theta_w <= 0 ||
+      O_tc <= 0 || n_tc <= 0)
+    return KAMI_ERROR_INVALID_VALUE;
+  PaperCost c = paper_cost((int)variant, m, n, k, p, s_e, L_sm, B_sm, theta_r, theta_w, O_tc, n_tc);
+  out[0] = c.V_cm;
+  out[1] = c.T_cm;
+  out[2] = c.T_cp;
+  out[3] = c.T_all;
+  return KAMI_SUCCESS;
+}
+
+const char* kami_status_string(kami_status_t s) {
+  switch (s) {
+    case KAMI_SUCCESS: return "KAMI_SUCCESS";
+    case KAMI_ERROR_INVALID_VALUE: return "KAMI_ERROR_INVALID_VALUE";
+    case KAMI_ERROR_NOT_SUPPORTED: return "KAMI_ERROR_NOT_SUPPORTED";
+    case KAMI_ERROR_MISALIGNED: return "KAMI_ERROR_MISALIGNED";
+    case KAMI_ERROR_CUDA: return "KAMI_ERROR_CUDA";
+  }
+  return "KAMI_ERROR_UNKNOWN";
+}
+
+const char* kami_last_kernel(void) { return g_last_kernel; }
+
+int kami_version(void) { return (KAMI_VERSION_MAJOR << 16) | KAMI_VERSION_MINOR; }
+
+}  // extern "C"

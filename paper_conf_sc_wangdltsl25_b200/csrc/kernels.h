@@ -1,0 +1,42 @@
+// kernels.h -- host-side interface between the C ABI (api.cpp) and the
+// kernel families (tc16.cu: tcgen05 16-bit; warp_ca.cu: register-resident
+// warp-level CA family with DMMA/HMMA).  Internal; not installed.
+#pragma once
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "../../include/kami.h"
+
+namespace kami {
+
+// cuTensorMapEncodeTiled fetched through the runtime (no link-time libcuda)
+typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                    const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                    CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+PFN_encodeTiled get_encode_tiled();
+void set_last_kernel(const char* name);
+
+// ---------------------------------------------------------------- tcgen05
+struct Tc16Shape {
+  int G, m_tiles, rows_tile, Wk, Wn, Wc, k_chunks, N_mma;
+  uint32_t stage_bytes, c_buf_bytes;
+  int c_bufs, stages, acc_cols, acc_bufs;
+  uint32_t smem_bytes;
+  long long units;
+};
+kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s);
+kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B, void* C,
+                          cudaStream_t stream, int max_ctas);
+
+// ------------------------------------------------ warp-level CA (literal KAMI)
+// algo: 1 = 1D, 2 = 2D, 3 = 3D, 4 = non-CA tiled.  dtype: KAMI_DTYPE_*.
+// Entry pointers: if A_arr != nullptr they are device arrays of per-entry
+// pointers (kami_gemm_batched); else strided from A/B/C.
+kami_status_t warp_ca_supported(int m, int n, int k, kami_dtype_t dtype, int algo, int p);
+kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t dtype, int algo, int p,
+                             const void* A, const void* B, void* C, const void* const* A_arr,
+                             const void* const* B_arr, void* const* C_arr, cudaStream_t stream);
+
+}  // namespace kami
