@@ -84,8 +84,11 @@ kami_status_t kami_gemm_strided_batched(int m, int n, int k, int64_t batch, kami
                                         kami_layout_t layout, const void* A, const void* B, void* C,
                                         kami_stream_t stream);
 
-/* Same with an explicit schedule and warp count p (0 = planner default).
- * Bench/test surface: lets the 1D/2D/3D/non-CA variants be compared. */
+/* Same with an explicit schedule and warp count p.  p = 0 takes the planner
+ * default; for 16-bit KAMI_ALGO_1D with p = 0 that is the tcgen05 kernel
+ * (whose compute units are the 4 sub-partition tensor cores of an SM), while
+ * p > 0 selects the register-resident warp-level kernel with p warps per
+ * entry.  Bench/test surface: lets the 1D/2D/3D/non-CA variants be compared. */
 kami_status_t kami_gemm_strided_batched_ex(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
                                            kami_layout_t layout, const void* A, const void* B, void* C,
                                            kami_algo_t algo, int p, kami_stream_t stream);

@@ -64,8 +64,9 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
   kami_plan_t r{};
   const bool is16 = dtype != KAMI_DTYPE_F64;
   // 16-bit strided: the tcgen05 family implements 1D with p = 4 sub-partition
-  // tensor cores (tc16.cu); it covers the whole 16-bit size grid.
-  if (is16 && !pointer_array && (algo == KAMI_ALGO_AUTO || (algo == KAMI_ALGO_1D && (p == 0 || p == 4)))) {
+  // tensor cores (tc16.cu); it covers the whole 16-bit size grid.  An explicit
+  // p > 0 selects the warp-level family with p warps instead.
+  if (is16 && !pointer_array && (algo == KAMI_ALGO_AUTO || (algo == KAMI_ALGO_1D && p == 0))) {
     Tc16Shape s;
     kami_status_t st = tc16_plan_shape(m, n, k, &s);
     if (st != KAMI_SUCCESS) return st;

@@ -97,23 +97,30 @@ WARP_CASES += [(dt, 64, a) for dt in ("f16", "bf16") for a in ("1d", "2d", "3d",
 WARP_CASES += [("f16", 128, "1d"), ("f16", 128, "2d"), ("f64", 8, "1d")]
 
 
+def warp_p(dtype, s, algo):
+    # 16-bit 1D with p = 0 means the tcgen05 kernel; name the warp count explicitly
+    return {32: 2, 64: 4, 128: 8}[s] if (dtype != "f64" and algo == "1d") else 0
+
+
 @pytest.mark.parametrize("dtype,s,algo", WARP_CASES, ids=lambda x: str(x))
 def test_warp_ca_unif(dtype, s, algo):
-    check(s, s, s, 37, dtype, "row", "unif", algo=algo)
+    check(s, s, s, 37, dtype, "row", "unif", algo=algo, p=warp_p(dtype, s, algo))
     assert "warp" in kami.last_kernel() and (algo in kami.last_kernel() or algo == "nonca")
 
 
 @pytest.mark.parametrize("dtype,s,algo", [c for c in WARP_CASES if c[1] <= 64], ids=lambda x: str(x))
 def test_warp_ca_int_bit_exact_both_layouts(dtype, s, algo):
     for layout in ("row", "col"):
-        check(s, s, s, 19, dtype, layout, "int", algo=algo, seed=2)
+        check(s, s, s, 19, dtype, layout, "int", algo=algo, p=warp_p(dtype, s, algo), seed=2)
 
 
 @pytest.mark.parametrize("dtype,s", [("f64", 64), ("f16", 64), ("bf16", 32)])
 def test_all_variants_agree_bitwise_on_int(dtype, s):
     """All schedules (and the tcgen05 path for 16 bit) produce identical bits on integer data."""
     A, B = ki.operands(s, s, s, 23, dtype, "int", seed=3)
-    outs = [run_gpu(s, s, s, 23, dtype, "row", A, B, algo=a) for a in ("1d", "2d", "nonca")]
+    outs = [run_gpu(s, s, s, 23, dtype, "row", A, B, algo=a, p=warp_p(dtype, s, a)) for a in ("1d", "2d", "nonca")]
+    if dtype != "f64":
+        outs.append(run_gpu(s, s, s, 23, dtype, "row", A, B, algo="1d", p=0))  # tcgen05
     outs.append(run_gpu(s, s, s, 23, dtype, "row", A, B, algo="auto"))
     for o in outs[1:]:
         assert torch.equal(o.view(torch.int16) if o.dtype != torch.float64 else o, outs[0].view(torch.int16)
