@@ -27,9 +27,9 @@
 //   warp 1     MMA issuer (one lane) + TMEM allocator: tcgen05.mma
 //              kind::f16, accumulators double/quad-buffered in TMEM,
 //              tcgen05.commit -> empty[s] (frees the stage) and tfull[a].
-//   warps 2-5  epilogue: tcgen05.ld 32x32b, cvt.rn to fp16/bf16, swizzled
-//              conflict-free st.shared into a C staging tile, one TMA tensor
-//              store per unit (bulk async, double-buffered).
+//   warps 2-9  epilogue, two warpgroups on alternate units: tcgen05.ld
+//              32x32b, cvt.rn to fp16/bf16, swizzled conflict-free st.shared
+//              into a C staging tile, one TMA tensor store per unit.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -42,7 +42,7 @@ namespace kami {
 
 namespace {
 
-constexpr int kThreads = 192;  // 6 warps
+constexpr int kThreads = 320;  // 10 warps: TMA, MMA, 2 x 4 epilogue
 constexpr int kEpiThreads = 128;
 constexpr int kMaxStages = 8;
 constexpr int kMaxAcc = 4;
@@ -161,69 +161,82 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
     }
   } else {
     // ------------------------------------------------------------ epilogue
-    const int sp = warp & 3;  // TMEM sub-partition this warp may access
+    // Two warpgroups (warps 2-5 and 6-9) take alternate units, so one can
+    // drain TMEM / write SMEM while the other's TMA store is in flight.
+    const int wg = (warp - 2) >> 2;
+    const int sp = warp & 3;  // TMEM sub-partition this warp may access (lanes 32sp..)
     const int L = sp * 32 + lane;
-    const bool leader = (warp == 2 && lane == 0);
-    const uint32_t c_smem = smem_base + p.c_off;
-    const int natoms_c = p.n / p.Wc;
-    uint32_t acc_it = 0;
-    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ++acc_it) {
+    const bool leader = ((warp & 3) == 2) && lane == 0;  // warps 2 and 6
+    const uint32_t bar_id = 1 + wg;
+    // ---- per-thread geometry, independent of the unit (no divisions in the loop)
+    int g, r, col_lo, col_hi;
+    bool row_ok;
+    if (p.G > 1) {
+      g = L / p.m;
+      r = L - g * p.m;
+      row_ok = g < p.G;
+      const int glo = (sp * 32) / p.m;
+      int ghi = (sp * 32 + 31) / p.m;
+      if (ghi > p.G - 1) ghi = p.G - 1;
+      col_lo = glo * p.n;
+      col_hi = glo < p.G ? (ghi + 1) * p.n : col_lo;
+    } else {
+      g = 0;
+      r = L;
+      row_ok = L < p.rows_tile;
+      col_lo = 0;
+      col_hi = (sp * 32 < p.rows_tile) ? p.n : 0;
+    }
+    const int my_lo = g * p.n, my_hi = my_lo + p.n;
+    const uint32_t row_bytes = (uint32_t)p.Wc * 2;
+    const uint32_t atom_stride = (uint32_t)p.rows_tile * row_bytes;
+    const uint32_t rowbase = (uint32_t)(g * (p.n / p.Wc) * p.rows_tile + r) * row_bytes;
+    const int wc_shift = p.Wc == 64 ? 6 : p.Wc == 32 ? 5 : 4;
+    const uint32_t c_smem = smem_base + p.c_off + (uint32_t)wg * p.c_bufs * p.c_buf_bytes;
+    uint32_t i = wg, local = 0;
+    for (long long u = blockIdx.x + (long long)wg * gridDim.x; u < p.units;
+         u += 2ll * gridDim.x, i += 2, ++local) {
       const long long grp = u / p.m_tiles;
       const int mt = (int)(u - grp * p.m_tiles);
       const long long e0 = grp * p.G;
-      const uint32_t a = acc_it % p.acc_bufs;
-      const uint32_t aph = (acc_it / p.acc_bufs) & 1;
-      const uint32_t cb = acc_it % p.c_bufs;
+      const uint32_t a = i % p.acc_bufs;
+      const uint32_t aph = (i / p.acc_bufs) & 1;
+      const uint32_t cb = local % p.c_bufs;
+      const bool valid = row_ok && (e0 + g < p.batch) && (p.G > 1 || mt * 128 + L < p.m);
       // the TMA store that last read staging buffer cb must be done reading
       if (leader) {
         if (p.c_bufs == 2) ptx::bulk_wait_read<1>();
         else ptx::bulk_wait_read<0>();
       }
-      ptx::named_bar_sync(1, kEpiThreads);
-
-      // which entry / row this thread's TMEM lane holds
-      int g, r;
-      bool valid;
-      int col_lo, col_hi;
-      if (p.G > 1) {
-        g = L / p.m;
-        r = L - g * p.m;
-        valid = (g < p.G) && (e0 + g < p.batch);
-        const int glo = (sp * 32) / p.m;
-        int ghi = (sp * 32 + 31) / p.m;
-        if (ghi > p.G - 1) ghi = p.G - 1;
-        col_lo = glo * p.n;
-        col_hi = glo < p.G ? (ghi + 1) * p.n : col_lo;
-      } else {
-        g = 0;
-        r = L;
-        valid = (mt * 128 + L < p.m) && (e0 < p.batch);
-        col_lo = 0;
-        col_hi = (sp * 32 < p.rows_tile) ? p.n : 0;
-      }
+      ptx::named_bar_sync(bar_id, kEpiThreads);
       ptx::mbar_wait(&tfull[a], aph);
       ptx::tc_fence_after();
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
       const uint32_t cbase = c_smem + cb * p.c_buf_bytes;
-      const int my_lo = g * p.n, my_hi = g * p.n + p.n;
-      for (int c0 = col_lo; c0 < col_hi; c0 += 32) {
-        uint32_t v[32];
-        if (col_hi - c0 >= 32) {
-          ptx::tmem_ld_32x32b_x32(t_row + c0, v);
-        } else {  // 16 columns left: never read past the accumulator
-          uint32_t (&h)[16] = *reinterpret_cast<uint32_t(*)[16]>(&v[0]);
-          ptx::tmem_ld_32x32b_x16(t_row + c0, h);
+      for (int c0 = col_lo; c0 < col_hi; c0 += 64) {
+        uint32_t v[64];
+        // issue both TMEM loads, then one wait (never read past col_hi)
+        const int left = col_hi - c0;
+        if (left >= 64) {
+          ptx::tmem_ld_32x32b_x32(t_row + c0, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+          ptx::tmem_ld_32x32b_x32(t_row + c0 + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+        } else if (left >= 48) {
+          ptx::tmem_ld_32x32b_x32(t_row + c0, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+          ptx::tmem_ld_32x32b_x16(t_row + c0 + 32, *reinterpret_cast<uint32_t(*)[16]>(&v[32]));
+        } else if (left >= 32) {
+          ptx::tmem_ld_32x32b_x32(t_row + c0, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+        } else {
+          ptx::tmem_ld_32x32b_x16(t_row + c0, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
         }
         ptx::tmem_wait_ld();
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
+        for (int q = 0; q < 8; ++q) {
           const int col = c0 + 8 * q;
           if (valid && col >= my_lo && col < my_hi && col < col_hi) {
-            const int jc = col - my_lo;
-            const int atom = jc / p.Wc;
-            const int ce = jc - atom * p.Wc;
-            uint32_t off = (uint32_t)(((g * natoms_c + atom) * p.rows_tile + r) * (p.Wc * 2) + ce * 2);
-            off = ptx::swz(off, p.c_swz_bits);
+            const uint32_t jc = (uint32_t)(col - my_lo);
+            const uint32_t atom = jc >> wc_shift;
+            const uint32_t ce = jc & (uint32_t)(p.Wc - 1);
+            const uint32_t off = ptx::swz(rowbase + atom * atom_stride + ce * 2, p.c_swz_bits);
             uint32_t w0, w1, w2, w3;
             if (kBF16) {
               w0 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
@@ -246,9 +259,9 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
       if (lane == 0) ptx::mbar_arrive(&tempty[a]);
       // make the generic-proxy smem writes visible to the TMA engine
       ptx::fence_proxy_async_smem();
-      ptx::named_bar_sync(1, kEpiThreads);
+      ptx::named_bar_sync(bar_id, kEpiThreads);
       if (leader) {
-        ptx::tma_store_4d(&p.tmC, smem + p.c_off + cb * p.c_buf_bytes, 0, mt * 128, 0, (int)e0);
+        ptx::tma_store_4d(&p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mt * 128, 0, (int)e0);
         ptx::bulk_commit();
       }
     }
@@ -304,12 +317,13 @@ kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s) {
   const uint32_t b_region = align_up((uint32_t)s->N_mma * s->Wk * 2, 1024);
   s->stage_bytes = a_region + b_region;
   s->c_buf_bytes = align_up((uint32_t)s->G * n * s->rows_tile * 2, 1024);
-  s->c_bufs = (2 * s->c_buf_bytes <= 96 * 1024) ? 2 : 1;
+  // two epilogue warpgroups, each with c_bufs staging tiles
+  s->c_bufs = (4 * s->c_buf_bytes <= 64 * 1024) ? 2 : 1;
   const int budget = kSmemLimit - 1024 /*align slack*/ - 1024 /*barriers*/;
-  int st = (budget - (int)(s->c_bufs * s->c_buf_bytes)) / (int)s->stage_bytes;
+  int st = (budget - (int)(2 * s->c_bufs * s->c_buf_bytes)) / (int)s->stage_bytes;
   if (st > kMaxStages) st = kMaxStages;
   s->stages = st;
-  s->smem_bytes = s->stages * s->stage_bytes + s->c_bufs * s->c_buf_bytes + 1024 + 1024;
+  s->smem_bytes = s->stages * s->stage_bytes + 2 * s->c_bufs * s->c_buf_bytes + 1024 + 1024;
   s->acc_cols = pow2_ceil(s->N_mma);
   s->acc_bufs = 512 / s->acc_cols;
   if (s->acc_bufs > kMaxAcc) s->acc_bufs = kMaxAcc;
@@ -361,7 +375,7 @@ kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const
   p.c_buf_bytes = s.c_buf_bytes;
   p.c_bufs = s.c_bufs;
   p.c_off = s.stages * s.stage_bytes;
-  p.bar_off = p.c_off + s.c_bufs * s.c_buf_bytes;
+  p.bar_off = p.c_off + 2 * s.c_bufs * s.c_buf_bytes;
   const long long groups = (batch + G - 1) / G;
   p.units = groups * s.m_tiles;
 
