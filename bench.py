@@ -210,7 +210,7 @@ def workload_config(args, dtype, m, n, k, batch, cfg):
     return {"workload": f"{dtype} strided-batched GEMM m={m} n={n} k={k} batch={batch}/GPU row-major "
                         f"(BASELINE.json configs[{cfg}])",
             "m": m, "n": n, "k": k, "batch_per_gpu": batch, "global_batch": batch * args.gpus,
-            "layout": "row", "algo": args.algo, "inputs": "unif [-1,1) RNE to dtype, counter-based SplitMix64",
+            "layout": "row", "algo": args.algo, "p": args.p, "inputs": "unif [-1,1) RNE to dtype, counter-based SplitMix64",
             "l2": "inputs larger than L2 (126 MB)" if batch * (m * k + k * n + m * n) * (8 if dtype == 'f64' else 2)
                   > 126e6 else "L2 flushed between timed steps",
             "parallelism": f"batch-sharded dp{args.gpus}"}
@@ -224,6 +224,7 @@ def main():
     ap.add_argument("--impl", default="kami", choices=["kami", "reference"])
     ap.add_argument("--workload", default="f16-64")
     ap.add_argument("--algo", default="auto")
+    ap.add_argument("--p", type=int, default=0, help="warps per entry (0 = planner default)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     args = ap.parse_args()
@@ -251,7 +252,7 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if small else None
 
     def step():
-        kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A, B, C, algo=args.algo, stream=stream)
+        kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A, B, C, algo=args.algo, p=args.p, stream=stream)
 
     for _ in range(args.warmup):
         step()
