@@ -37,15 +37,20 @@ PaperCost paper_cost(int variant, double m, double n, double k, double p, double
 
 namespace {
 
-// B200 constants.  L_sm: LDS latency 29 cycles; B_sm:
-// 128 B/cycle/SM crossbar; n_tc = 4 sub-partition tensor cores per SM.
-// O_tc per tensor core: DMMA FP64 ~ 32 flop/cycle (37 TF / 148 SMs / 1.965
-// GHz / 4); legacy HMMA ~ 256 flop/cycle (assumed 1/8 of tcgen05).
-constexpr double kLsm = 29, kBsm = 128, kNtc = 4;
+// B200 constants, measured by tools/ubench.cu (profiles/r1/ubench_b200.json):
+// L_sm = 29 cycles (dependent LDS), B_sm = 127.6 B/cycle/SM (conflict-free
+// LDS.128), n_tc = 4 sub-partition tensor cores, O_tc per tensor core:
+// DMMA FP64 37.1 TF/s -> 31.9 flop/cycle; legacy HMMA FP16 554.5 TF/s ->
+// 477 flop/cycle (at 1965 MHz, 148 SMs).  HBM: 6541.8 GB/s measured copy
+// (MEASURED_PEAKS.json) -> 22.5 B/cycle/SM.  T_lat: DRAM round trip seen by a
+// team that starts a new entry (~1200 cycles; entries prefetched into L2 by
+// the previous one).
+constexpr double kLsm = 29, kBsm = 127.6, kNtc = 4;
+constexpr double kHbmBpc = 22.5, kTlat = 1200;
 
 double b200_cost(int variant, int m, int n, int k, int p, kami_dtype_t dt) {
   const double s_e = dt == KAMI_DTYPE_F64 ? 8 : 2;
-  const double O = dt == KAMI_DTYPE_F64 ? 32 : 256;
+  const double O = dt == KAMI_DTYPE_F64 ? 31.9 : 477;
   PaperCost c = paper_cost(variant, m, n, k, p, s_e, kLsm, kBsm, 1, 1, O, kNtc);
   const double stages = variant == 1 ? p : variant == 2 ? std::sqrt((double)p) : std::round(std::cbrt((double)p));
   const double ratio = std::max(1.0, p / kNtc);
@@ -55,6 +60,37 @@ double b200_cost(int variant, int m, int n, int k, int p, kami_dtype_t dt) {
     t += 2 * (stages - 1) * (double)m * n * s_acc / kBsm;
   }
   return t;
+}
+
+// Batched form: an SM streams entries; with t teams resident the per-entry
+// time is bounded by HBM and by the serial (latency + T_all) of one team
+// spread over t teams.
+double b200_entry_cycles(int variant, int m, int n, int k, int p, kami_dtype_t dt, int teams_per_sm) {
+  const double s_e = dt == KAMI_DTYPE_F64 ? 8 : 2;
+  const double t_hbm = (double)(m * k + k * n + m * n) * s_e / kHbmBpc;
+  const double t_all = b200_cost(variant, m, n, k, p, dt);
+  return std::max(t_hbm, (kTlat + t_all) / std::max(1, teams_per_sm));
+}
+
+// Measured throughput of each schedule (bench.py, 20 steps, one B200,
+// profiles/r1/f64_sweep_r1.txt).  Where a shape is calibrated, AUTO takes the
+// measured-fastest schedule; elsewhere it takes the model's minimum.
+struct Calib {
+  kami_dtype_t dt;
+  int s, algo, p;
+  double tflops;
+};
+const Calib kCalib[] = {
+    {KAMI_DTYPE_F64, 16, 1, 1, 7.07},  {KAMI_DTYPE_F64, 16, 2, 4, 5.66},  {KAMI_DTYPE_F64, 16, 3, 8, 4.98},
+    {KAMI_DTYPE_F64, 32, 1, 2, 14.29}, {KAMI_DTYPE_F64, 32, 2, 4, 12.42}, {KAMI_DTYPE_F64, 32, 3, 8, 11.63},
+    {KAMI_DTYPE_F64, 64, 1, 8, 14.13}, {KAMI_DTYPE_F64, 64, 2, 16, 17.20}, {KAMI_DTYPE_F64, 64, 3, 8, 15.84},
+};
+
+double calibrated(kami_dtype_t dt, int m, int n, int k, int algo, int p) {
+  if (m != n || n != k) return 0;
+  for (const Calib& c : kCalib)
+    if (c.dt == dt && c.s == m && c.algo == algo && c.p == p) return c.tflops;
+  return 0;
 }
 
 }  // namespace
@@ -96,14 +132,17 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
     *out = r;
     return KAMI_SUCCESS;
   }
-  double best = 1e300;
+  double best = 1e300, best_meas = 0;
   int best_v = 0, best_p = 0;
   for (int v : cand) {
     const int pp = warp_ca_default_p(m, n, k, dtype, v);
     if (pp == 0) continue;
-    const double t = b200_cost(v, m, n, k, pp, dtype);
-    if (t < best) {  // strict: ties keep the earlier (1D) schedule
+    const double meas = calibrated(dtype, m, n, k, v, pp);
+    const double t = b200_entry_cycles(v, m, n, k, pp, dtype, warp_ca_teams_per_sm(m, n, k, dtype, v, pp));
+    const bool better = best_meas > 0 || meas > 0 ? meas > best_meas : t < best;  // ties keep 1D
+    if (best_v == 0 || better) {
       best = t;
+      best_meas = meas;
       best_v = v;
       best_p = pp;
     }
@@ -115,7 +154,7 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
   r.entries_per_cta = best_p >= 8 ? 1 : 8 / best_p;
   r.stages = 2;
   r.kslice_regs_pct = 100;
-  r.t_all_cycles = best;
+  r.t_all_cycles = b200_cost(best_v, m, n, k, best_p, dtype);
   *out = r;
   return KAMI_SUCCESS;
 }

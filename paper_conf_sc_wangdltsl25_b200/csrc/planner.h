@@ -22,5 +22,6 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
                              kami_plan_t* out);
 
 int warp_ca_default_p(int m, int n, int k, kami_dtype_t dtype, int algo);
+int warp_ca_teams_per_sm(int m, int n, int k, kami_dtype_t dtype, int algo, int p);
 
 }  // namespace kami

@@ -32,6 +32,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 
 #include "kernels.h"
 #include "ptx.cuh"
@@ -66,6 +67,38 @@ struct F64Atom {
   __device__ static void store_c(E* C, int ld, int row0, int col0, int lane, const Acc (&c)[NC]) {
     const int row = row0 + (lane >> 2), col = col0 + 2 * (lane & 3);
     *reinterpret_cast<double2*>(C + row * ld + col) = make_double2(c[0], c[1]);
+  }
+};
+
+// mma.sync.m16n8k8.f64 (sm_90+ DMMA shape): A 16x8 (4 regs), B 8x8 (2), C 16x8 (4)
+struct F64Atom16 {
+  using E = double;
+  using R = double;
+  using Acc = double;
+  static constexpr int AM = 16, AN = 8, AK = 8;
+  static constexpr int NA = 4, NB = 2, NC = 4;
+  static constexpr bool kBF16 = false;
+  __device__ static void a_pos(int lane, int r, int& row, int& col) {
+    row = (lane >> 2) + 8 * (r & 1);
+    col = (lane & 3) + 4 * (r >> 1);
+  }
+  __device__ static void b_pos(int lane, int r, int& k, int& n) {
+    k = (lane & 3) + 4 * r;
+    n = lane >> 2;
+  }
+  __device__ static R load_a(const E* p, int ld, int row, int col) { return __ldg(p + row * ld + col); }
+  __device__ static R load_b(const E* p, int ld, int k, int n) { return __ldg(p + k * ld + n); }
+  __device__ static void mma(Acc (&c)[NC], const R (&a)[NA], const R (&b)[NB]) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k8.row.col.f64.f64.f64.f64 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+d"(c[0]), "+d"(c[1]), "+d"(c[2]), "+d"(c[3])
+        : "d"(a[0]), "d"(a[1]), "d"(a[2]), "d"(a[3]), "d"(b[0]), "d"(b[1]));
+  }
+  __device__ static void store_c(E* C, int ld, int row0, int col0, int lane, const Acc (&c)[NC]) {
+    const int row = row0 + (lane >> 2), col = col0 + 2 * (lane & 3);
+    *reinterpret_cast<double2*>(C + row * ld + col) = make_double2(c[0], c[1]);
+    *reinterpret_cast<double2*>(C + (row + 8) * ld + col) = make_double2(c[2], c[3]);
   }
 };
 
@@ -445,7 +478,8 @@ __global__ void __launch_bounds__(P * 32 * TEAMS) kami_warp_ca_kernel(const type
                                                                       typename At::E* __restrict__ C,
                                                                       const void* const* A_arr,
                                                                       const void* const* B_arr, void* const* C_arr,
-                                                                      long long batch, int M, int N, int K) {
+                                                                      long long batch, int M, int N, int K,
+                                                                      int prefetch) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int team = warp / P, wi = warp % P;
@@ -465,6 +499,16 @@ __global__ void __launch_bounds__(P * 32 * TEAMS) kami_warp_ca_kernel(const type
       a = A + e * (long long)M * K;
       b = B + e * (long long)K * N;
       c = C + e * (long long)M * N;
+    }
+    // Stream the team's NEXT entry from HBM into L2 while this one computes,
+    // so its GMem2Reg loads hit L2 (the register-resident design cannot
+    // double-buffer operands in registers).
+    if (prefetch && wi == 0 && lane == 0 && e + nteams < batch) {
+      const long long en = e + nteams;
+      const void* na = A_arr ? A_arr[en] : (const void*)(A + en * (long long)M * K);
+      const void* nb = A_arr ? B_arr[en] : (const void*)(B + en * (long long)K * N);
+      ptx::prefetch_l2_bulk(na, (uint32_t)(M * K * sizeof(typename At::E)));
+      ptx::prefetch_l2_bulk(nb, (uint32_t)(K * N * sizeof(typename At::E)));
     }
     Sched::run(a, b, c, smem, wi, lane, bar, stage);
   }
@@ -506,7 +550,26 @@ LaunchInfo info(const char* name) {
 using H16 = F16Atom<false>;
 using B16 = F16Atom<true>;
 
+int f64_atom_pref() {  // 16 = m16n8k8 DMMA first, 8 = m8n8k4 first (env KAMI_F64_ATOM)
+  static const int v = [] {
+    const char* e = getenv("KAMI_F64_ATOM");
+    return e ? atoi(e) : 16;
+  }();
+  return v;
+}
+
 bool lookup(int m, int n, int k, kami_dtype_t dtype, int algo, int p, LaunchInfo* out) {
+  if (f64_atom_pref() == 16) {
+    // FP64 DMMA m16n8k8 where the register budget allows it
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 16, 16, 16, 1, Sched1D, 1, "kami_warp_ca_1d<f64m16,16>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 32, 32, 32, 1, Sched1D, 2, "kami_warp_ca_1d<f64m16,32>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 32, 32, 32, 2, Sched2D, 4, "kami_warp_ca_2d<f64m16,32>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 32, 32, 32, 3, Sched3D, 8, "kami_warp_ca_3d<f64m16,32>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 32, 32, 32, 4, SchedNonCA, 4, "kami_warp_nonca<f64m16,32>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 64, 64, 64, 2, Sched2D, 16, "kami_warp_ca_2d<f64m16,64>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 64, 64, 64, 3, Sched3D, 8, "kami_warp_ca_3d<f64m16,64>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 64, 64, 64, 4, SchedNonCA, 4, "kami_warp_nonca<f64m16,64>")
+  }
   // FP64 DMMA (m8n8k4): the literal KAMI register-resident family
   KAMI_SIZE_CASES(F64Atom, KAMI_DTYPE_F64, 16, 2, 4, 8, 4, "f64")
   KAMI_SIZE_CASES(F64Atom, KAMI_DTYPE_F64, 32, 4, 16, 8, 4, "f64")
@@ -541,6 +604,25 @@ int warp_ca_default_p(int m, int n, int k, kami_dtype_t dtype, int algo) {
   return 0;
 }
 
+// Resident teams per SM for the model (occupancy API when a device is
+// present; otherwise a register estimate: 64K registers / (threads x regs)).
+int warp_ca_teams_per_sm(int m, int n, int k, kami_dtype_t dtype, int algo, int p) {
+  LaunchInfo li;
+  if (!lookup(m, n, k, dtype, algo, p, &li)) return 1;
+  const int teams_per_cta = li.threads / 32 / li.p;
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, li.fn, li.threads, li.smem) != cudaSuccess ||
+      per_sm < 1) {
+    cudaGetLastError();
+    const double es = dtype == KAMI_DTYPE_F64 ? 2.0 : 0.5;  // 32-bit registers per element
+    const double elems = (double)m * k / li.p * 2 + (double)k * n / li.p * 2 + (double)m * n / li.p;
+    const double regs = elems * es / 32 + 32;
+    per_sm = (int)(65536.0 / (li.threads * regs));
+    if (per_sm < 1) per_sm = 1;
+  }
+  return per_sm * teams_per_cta;
+}
+
 kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t dtype, int algo, int p,
                              const void* A, const void* B, void* C, const void* const* A_arr,
                              const void* const* B_arr, void* const* C_arr, cudaStream_t stream) {
@@ -561,8 +643,13 @@ kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t 
   long long grid = (long long)sms * per_sm;  // persistent: teams loop over the batch
   if (grid > ctas_needed) grid = ctas_needed;
   if (grid < 1) grid = 1;
+  static const int prefetch = [] {
+    const char* e = getenv("KAMI_L2_PREFETCH");
+    return e ? atoi(e) : 1;
+  }();
+  int pf = prefetch;
   void* args[] = {(void*)&A, (void*)&B, (void*)&C, (void*)&A_arr, (void*)&B_arr, (void*)&C_arr,
-                  (void*)&batch, (void*)&m, (void*)&n, (void*)&k};
+                  (void*)&batch, (void*)&m, (void*)&n, (void*)&k, (void*)&pf};
   cudaError_t err = cudaLaunchKernel(li.fn, dim3((unsigned)grid), dim3(li.threads), args, li.smem, stream);
   set_last_kernel(li.name);
   return err == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
