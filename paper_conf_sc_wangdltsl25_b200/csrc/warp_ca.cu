@@ -66,7 +66,7 @@ struct F64Atom {
   // C fragment: lane (g,t) holds (g, 2t) and (g, 2t+1)
   __device__ static void store_c(E* C, int ld, int row0, int col0, int lane, const Acc (&c)[NC]) {
     const int row = row0 + (lane >> 2), col = col0 + 2 * (lane & 3);
-    *reinterpret_cast<double2*>(C + row * ld + col) = make_double2(c[0], c[1]);
+    ptx::st_global_v2_f64(C + row * ld + col, c[0], c[1]);
   }
 };
 
@@ -97,8 +97,8 @@ struct F64Atom16 {
   }
   __device__ static void store_c(E* C, int ld, int row0, int col0, int lane, const Acc (&c)[NC]) {
     const int row = row0 + (lane >> 2), col = col0 + 2 * (lane & 3);
-    *reinterpret_cast<double2*>(C + row * ld + col) = make_double2(c[0], c[1]);
-    *reinterpret_cast<double2*>(C + (row + 8) * ld + col) = make_double2(c[2], c[3]);
+    ptx::st_global_v2_f64(C + row * ld + col, c[0], c[1]);
+    ptx::st_global_v2_f64(C + (row + 8) * ld + col, c[2], c[3]);
   }
 };
 
@@ -146,8 +146,8 @@ struct F16Atom {
     const int row = row0 + (lane >> 2), col = col0 + 2 * (lane & 3);
     const uint32_t lo = BF ? ptx::pack_bf16x2(c[0], c[1]) : ptx::pack_f16x2(c[0], c[1]);
     const uint32_t hi = BF ? ptx::pack_bf16x2(c[2], c[3]) : ptx::pack_f16x2(c[2], c[3]);
-    *reinterpret_cast<uint32_t*>(C + row * ld + col) = lo;
-    *reinterpret_cast<uint32_t*>(C + (row + 8) * ld + col) = hi;
+    ptx::st_global_b32(C + row * ld + col, lo);
+    ptx::st_global_b32(C + (row + 8) * ld + col, hi);
   }
 };
 
@@ -355,7 +355,8 @@ struct Sched3D {
   static constexpr int LWORDS = Cc * TA::WORDS + Cc * TB::WORDS;  // one layer, one stage
   static constexpr int XWORDS = Cc * LWORDS;
   static constexpr int XBYTES = 2 * XWORDS * sizeof(typename At::R);
-  static constexpr int RBYTES = (Cc - 1) * Cc * Cc * TC::WORDS * sizeof(typename At::Acc);
+  // reduce-scatter slots: per cell, per owner layer, per sender layer, one chunk
+  static constexpr int RBYTES = Cc * Cc * Cc * TC::WORDS * sizeof(typename At::Acc);
   static constexpr int SMEM_BYTES = XBYTES + RBYTES;
   static_assert(TM % At::AM == 0 && TK % At::AK == 0 && TN % At::AN == 0, "3D tile shape");
   __device__ static void run(const typename At::E* A, const typename At::E* B, typename At::E* C, uint8_t* smem,
@@ -388,22 +389,61 @@ struct Sched3D {
       if (wr != z) get(br, sb, lane);
       mma_tile(c, ar, br, 0);
     }
-    // K-split reduction across layers (fixed order 0 + 1 + ... )
+    // K-split reduction across layers as a reduce-scatter: the C tile's
+    // fragments are split into Cc chunks, layer l owns chunk l.  Each layer
+    // writes the chunks it does not own, reads the others' partials of its own
+    // chunk, sums them in fixed layer order 0 + 1 + ... (Alg. 3 line 19) and
+    // stores its chunk -- (Cc-1)/Cc of the tile crosses SMEM instead of all of it.
+    constexpr int NF = TC::FM * TC::FN, FW = At::NC * 32;  // fragments, words per fragment
     Acc* red = reinterpret_cast<Acc*>(smem + XBYTES);
     const int cell = wr * Cc + wc;
-    if (l > 0) put(c, red + ((l - 1) * Cc * Cc + cell) * TC::WORDS, lane);
-    ptx::named_bar_sync(bar, P * 32);
-    if (l == 0) {
-#pragma unroll 1
-      for (int ll = 1; ll < Cc; ++ll) {
-        TC t;
-        get(t, red + ((ll - 1) * Cc * Cc + cell) * TC::WORDS, lane);
-        Acc* f = &c.v[0][0][0];
-        const Acc* g = &t.v[0][0][0];
+    if constexpr (NF % Cc == 0) {
+      constexpr int CS = NF / Cc;
+      auto slot = [&](int owner, int sender) { return red + ((cell * Cc + owner) * Cc + sender) * CS * FW; };
 #pragma unroll
-        for (int i = 0; i < (int)(sizeof(c.v) / sizeof(Acc)); ++i) f[i] += g[i];
+      for (int f = 0; f < NF; ++f) {
+        const int o = f / CS;
+        if (o != l) {
+          Acc* dst = slot(o, l) + (f - o * CS) * FW;
+#pragma unroll
+          for (int r = 0; r < At::NC; ++r) dst[r * 32 + lane] = c.v[f / TC::FN][f % TC::FN][r];
+        }
       }
-      store_c(c, C, N, wr * TM, wc * TN, lane);
+      ptx::named_bar_sync(bar, P * 32);
+#pragma unroll
+      for (int f = 0; f < NF; ++f) {
+        if (f / CS == l) {
+          Acc v[At::NC];
+#pragma unroll
+          for (int r = 0; r < At::NC; ++r) {
+            Acc sum = 0;
+#pragma unroll
+            for (int ll = 0; ll < Cc; ++ll) {
+              const Acc x =
+                  (ll == l) ? c.v[f / TC::FN][f % TC::FN][r] : slot(l, ll)[(f - l * CS) * FW + r * 32 + lane];
+              sum = (ll == 0) ? x : sum + x;
+            }
+            v[r] = sum;
+          }
+          At::store_c(C, N, wr * TM + (f / TC::FN) * At::AM, wc * TN + (f % TC::FN) * At::AN, lane, v);
+        }
+      }
+    } else {
+      // a single-fragment tile cannot be split: gather to layer 0
+      if (l > 0) put(c, red + ((l - 1) * Cc * Cc + cell) * TC::WORDS, lane);
+      ptx::named_bar_sync(bar, P * 32);
+      if (l == 0) {
+#pragma unroll 1
+        for (int ll = 1; ll < Cc; ++ll) {
+          TC t;
+          get(t, red + ((ll - 1) * Cc * Cc + cell) * TC::WORDS, lane);
+          Acc* f = &c.v[0][0][0];
+          const Acc* g = &t.v[0][0][0];
+#pragma unroll
+          for (int i = 0; i < (int)(sizeof(c.v) / sizeof(Acc)); ++i) f[i] += g[i];
+        }
+        store_c(c, C, N, wr * TM, wc * TN, lane);
+      }
     }
   }
 };
@@ -413,7 +453,7 @@ struct Sched3D {
 // W_m x W_n warp grid reads its fragments from SMEM for every MMA.
 template <class At, int M, int N, int K, int P>
 struct SchedNonCA {
-  static constexpr int WM = (P == 4) ? 2 : (P == 8 ? 4 : 1), WN = P / WM;
+  static constexpr int WM = (P == 4) ? 2 : (P == 8 || P == 16) ? 4 : 1, WN = P / WM;
   static constexpr int TM = M / WM, TN = N / WN;
   static constexpr int FMT = M / At::AM, FKT = K / At::AK, FNT = N / At::AN;  // whole-matrix fragment grid
   static constexpr int AWORDS = FMT * FKT * At::NA * 32, BWORDS = FKT * FNT * At::NB * 32;
@@ -569,12 +609,18 @@ bool lookup(int m, int n, int k, kami_dtype_t dtype, int algo, int p, LaunchInfo
     KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 64, 64, 64, 2, Sched2D, 16, "kami_warp_ca_2d<f64m16,64>")
     KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 64, 64, 64, 3, Sched3D, 8, "kami_warp_ca_3d<f64m16,64>")
     KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 64, 64, 64, 4, SchedNonCA, 4, "kami_warp_nonca<f64m16,64>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 64, 64, 64, 4, SchedNonCA, 16, "kami_warp_nonca16<f64m16,64>")
+    KAMI_CASE(F64Atom16, KAMI_DTYPE_F64, 64, 64, 64, 4, SchedNonCA, 8, "kami_warp_nonca8<f64m16,64>")
   }
   // FP64 DMMA (m8n8k4): the literal KAMI register-resident family
   KAMI_SIZE_CASES(F64Atom, KAMI_DTYPE_F64, 16, 2, 4, 8, 4, "f64")
   KAMI_SIZE_CASES(F64Atom, KAMI_DTYPE_F64, 32, 4, 16, 8, 4, "f64")
   KAMI_SIZE_CASES(F64Atom, KAMI_DTYPE_F64, 64, 8, 16, 8, 4, "f64")
   KAMI_CASE(F64Atom, KAMI_DTYPE_F64, 8, 8, 8, 1, Sched1D, 1, "kami_warp_ca_1d<f64,8>")
+  KAMI_CASE(F64Atom, KAMI_DTYPE_F64, 32, 32, 32, 4, SchedNonCA, 8, "kami_warp_nonca8<f64,32>")
+  KAMI_CASE(H16, KAMI_DTYPE_F16, 64, 64, 64, 4, SchedNonCA, 8, "kami_warp_nonca8<f16,64>")
+  KAMI_CASE(B16, KAMI_DTYPE_BF16, 64, 64, 64, 4, SchedNonCA, 8, "kami_warp_nonca8<bf16,64>")
+  KAMI_CASE(H16, KAMI_DTYPE_F16, 128, 128, 128, 4, SchedNonCA, 16, "kami_warp_nonca16<f16,128>")
   // FP16 / BF16 HMMA (m16n8k16): CA evidence family
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 1, Sched1D, 2, "kami_warp_ca_1d<f16,32>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 2, Sched2D, 4, "kami_warp_ca_2d<f16,32>")

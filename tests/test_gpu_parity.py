@@ -185,3 +185,12 @@ def test_gpu_generator_matches_cpu():
             assert torch.equal(A.view(torch.int16) if dtype != "f64" else A,
                                Ag.cpu().view(torch.int16) if dtype != "f64" else Ag.cpu())
             assert torch.equal(B.double(), Bg.cpu().double())
+
+
+@pytest.mark.parametrize("dtype,s,algo,p", [("f16", 64, "nonca", 8), ("bf16", 64, "nonca", 8), ("f64", 32, "nonca", 8),
+                                            ("f64", 64, "nonca", 16), ("f64", 64, "nonca", 8),
+                                            ("f16", 128, "nonca", 16), ("f64", 64, "1d", 8), ("f16", 64, "3d", 8)])
+def test_warp_explicit_p(dtype, s, algo, p):
+    """Same-warp-count comparators (non-CA 4x2 / 4x4 grids) and explicit p."""
+    check(s, s, s, 41, dtype, "row", "unif", algo=algo, p=p)
+    check(s, s, s, 13, dtype, "col", "int", algo=algo, p=p, seed=4)
