@@ -56,12 +56,9 @@ def closed_form(dtype, s, algo, p):
         return math.isqrt(p) * (m * k + k * n) * se
     if algo == "3d":
         c = round(p ** (1 / 3))
-        # layer reduction as a reduce-scatter (each layer owns 1/c of the tile)
-        # unless the per-warp tile is a single MMA fragment (then gathered to layer 0)
-        am = 16 if (dtype != "f64" or s >= 32) else 8
-        single = (m // c) * (n // c) <= am * 8
-        red = 2 * (c - 1) * m * n * sacc if single else 2 * (c - 1) * m * n * sacc // c
-        return c * (m * k + k * n) * se + red
+        # layer reduction: gather or reduce-scatter both move (c-1) partial
+        # tiles through SMEM (write + read); reduce-scatter only balances it
+        return c * (m * k + k * n) * se + 2 * (c - 1) * m * n * sacc
     if algo == "nonca":
         wm = {4: 2, 8: 4, 16: 4}[p]
         wn = p // wm
