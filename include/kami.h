@@ -55,13 +55,17 @@ typedef enum { KAMI_DTYPE_F16 = 0, KAMI_DTYPE_BF16 = 1, KAMI_DTYPE_F64 = 2 } kam
 typedef enum { KAMI_ROW_MAJOR = 0, KAMI_COL_MAJOR = 1 } kami_layout_t;
 
 /* Which schedule runs (Sec. 4.3-4.5).  AUTO = the planner's choice
- * (kami_plan).  NONCA = the non-communication-avoiding tiled baseline. */
+ * (kami_plan).  NONCA = the non-communication-avoiding tiled baseline.
+ * 1D_TMA = KAMI-1D whose broadcast operand is written to shared memory by the
+ * TMA engine (16-bit: the tcgen05 kernel; FP64: the DMMA kernel of
+ * dmma_tma.cu, m = n = k in {32, 64}). */
 typedef enum {
   KAMI_ALGO_AUTO = 0,
   KAMI_ALGO_1D = 1,
   KAMI_ALGO_2D = 2,
   KAMI_ALGO_3D = 3,
-  KAMI_ALGO_NONCA = 4
+  KAMI_ALGO_NONCA = 4,
+  KAMI_ALGO_1D_TMA = 5
 } kami_algo_t;
 
 /* Opaque CUDA stream; binary compatible with cudaStream_t. */
@@ -107,7 +111,7 @@ kami_status_t kami_release_workspace(void);
 typedef struct {
   kami_algo_t algo;      /* chosen schedule                                 */
   int p;                 /* warps (or tensor-core sub-partitions) per entry */
-  int kernel;            /* 0 = tcgen05 16-bit family, 1 = warp-level DMMA/HMMA family */
+  int kernel;            /* 0 = tcgen05 16-bit, 1 = warp-level DMMA/HMMA, 2 = FP64 DMMA with TMA broadcast */
   int entries_per_cta;   /* batch entries a CTA keeps in flight             */
   int stages;            /* shared-memory pipeline depth                    */
   int kslice_regs_pct;   /* share of A/B kept resident (Sec. 4.7)           */

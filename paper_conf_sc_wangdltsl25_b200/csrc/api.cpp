@@ -54,7 +54,7 @@ kami_status_t check_common(int m, int n, int k, int64_t batch, int dtype, int la
   if (m <= 0 || n <= 0 || k <= 0 || batch < 0) return KAMI_ERROR_INVALID_VALUE;
   if (dtype < KAMI_DTYPE_F16 || dtype > KAMI_DTYPE_F64) return KAMI_ERROR_INVALID_VALUE;
   if (layout != KAMI_ROW_MAJOR && layout != KAMI_COL_MAJOR) return KAMI_ERROR_INVALID_VALUE;
-  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_NONCA) return KAMI_ERROR_INVALID_VALUE;
+  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_1D_TMA) return KAMI_ERROR_INVALID_VALUE;
   return check_sizes(m, n, k, (kami_dtype_t)dtype);
 }
 
@@ -83,6 +83,7 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
   if (plan.kernel == 0) {
     return tc16_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream, 0);
   }
+  if (plan.kernel == 2) return dmma_tma_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream);
   return warp_ca_launch(rp.m, rp.n, rp.k, batch, dtype, (int)plan.algo, plan.p, rp.A, rp.B, C, rp.Aa, rp.Ba, Ca,
                         stream);
 }

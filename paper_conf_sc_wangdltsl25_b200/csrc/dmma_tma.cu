@@ -1,0 +1,195 @@
+// dmma_tma.cu -- FP64 batched GEMM: KAMI-1D on the DMMA tensor path with the
+// broadcast operand delivered by TMA (the B200 form of the FP64 schedule).
+//
+// KAMI-1D (Alg. 1) partitions one operand among p warps
+// (local, registers) and broadcasts the other through shared memory.  Here we
+// apply it to C^T = B^T A^T, i.e. the warps partition the COLUMNS:
+//   warp w holds B_w = B[:, w n/p:(w+1) n/p] and C_w = C[:, w n/p:(w+1) n/p]
+//   in registers as DMMA fragments (GMem2Reg straight from global);
+//   A (m x k) is the broadcast operand: one TMA tensor copy per entry writes it
+//   into shared memory in the 128-byte-swizzled layout, and every warp reads
+//   its A fragments from there -- bank-conflict free (the 8-row XOR swizzle
+//   spreads the 8 rows of a fragment over distinct 16-byte bank groups).
+// Stage z of Alg. 1 is the z-th k-slice of 4 (one DMMA k-step); all p warps
+// consume the same broadcast slice.  Each team (p warps) double-buffers A:
+// the TMA for its next entry is issued while the current one computes, and
+// the next entry's B is bulk-prefetched into L2, so HBM streaming overlaps the
+// DMMA work.  SMEM traffic per entry: m k s_e written (TMA) + p m k s_e read.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdlib>
+#include <cstring>
+
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace kami {
+namespace {
+
+template <int M, int N, int K, int P, int TEAMS>
+struct DmmaTmaCfg {
+  static constexpr int NP = N / P;        // columns per warp
+  static constexpr int FN = NP / 8;       // 8-wide DMMA n-fragments per warp
+  static constexpr int FM = M / 8;        // 8-tall m-fragments
+  static constexpr int FK = K / 4;        // k-steps
+  static constexpr int A_BYTES = M * K * 8;
+  static constexpr int KCH = K / 16;      // 128-byte (16-double) column chunks of A
+  static constexpr int THREADS = P * 32 * TEAMS;
+  static constexpr int SMEM = TEAMS * 2 * A_BYTES + 1024 /*align*/ + 256 /*barriers*/;
+  static_assert(NP % 8 == 0 && K % 16 == 0 && M % 8 == 0, "shape");
+};
+
+struct DmmaTmaParams {
+  CUtensorMap tmA;  // 4-D (16, m, k/16, batch), box (16, m, k/16, 1), SW128
+  const double* B;
+  double* C;
+  long long batch;
+};
+
+template <int M, int N, int K, int P, int TEAMS>
+__global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(const __grid_constant__ DmmaTmaParams prm) {
+  using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + TEAMS * 2 * Cfg::A_BYTES);  // [TEAMS][2]
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int team = warp / P, w = warp % P;
+  const int g = lane >> 2, t = lane & 3;
+  if (threadIdx.x == 0) {
+    ptx::prefetch_tmap(&prm.tmA);
+    for (int i = 0; i < TEAMS * 2; ++i) ptx::mbar_init(&full[i], 1);
+    ptx::fence_mbar_init();
+    ptx::fence_proxy_async_smem();
+  }
+  __syncthreads();
+  const long long nteams = (long long)gridDim.x * TEAMS;
+  const long long first = (long long)blockIdx.x * TEAMS + team;
+  const bool issuer = (w == 0 && lane == 0);
+  const uint32_t bar = 1 + team;
+  uint8_t* abuf = smem + team * 2 * Cfg::A_BYTES;
+  uint64_t* tfull = full + team * 2;
+  if (issuer && first < prm.batch) {  // prologue: A of the first entry
+    ptx::mbar_arrive_expect_tx(&tfull[0], Cfg::A_BYTES);
+    ptx::tma_load_4d(abuf, &prm.tmA, &tfull[0], 0, 0, 0, (int)first);
+  }
+  uint32_t it = 0;
+  for (long long e = first; e < prm.batch; e += nteams, ++it) {
+    const uint32_t s = it & 1;
+    const long long en = e + nteams;
+    // all warps of the team finished reading buffer s^1 (entry it-1) at the
+    // barrier that ended the previous iteration: refill it with entry it+1
+    if (issuer && en < prm.batch) {
+      ptx::mbar_arrive_expect_tx(&tfull[s ^ 1], Cfg::A_BYTES);
+      ptx::tma_load_4d(abuf + (s ^ 1) * Cfg::A_BYTES, &prm.tmA, &tfull[s ^ 1], 0, 0, 0, (int)en);
+      ptx::prefetch_l2_bulk(prm.B + en * (long long)K * N, (uint32_t)(K * N * 8));
+    }
+    // GMem2Reg: this warp's B_w (k x n/p) as DMMA B fragments (k = t, n = g)
+    const double* Bg = prm.B + e * (long long)K * N + w * Cfg::NP;
+    double b[Cfg::FK][Cfg::FN];
+#pragma unroll
+    for (int kk = 0; kk < Cfg::FK; ++kk)
+#pragma unroll
+      for (int j = 0; j < Cfg::FN; ++j) b[kk][j] = __ldg(Bg + (kk * 4 + t) * N + j * 8 + g);
+    double c[Cfg::FM][Cfg::FN][2];
+#pragma unroll
+    for (int i = 0; i < Cfg::FM; ++i)
+#pragma unroll
+      for (int j = 0; j < Cfg::FN; ++j) c[i][j][0] = c[i][j][1] = 0.0;
+    ptx::mbar_wait(&tfull[s], (it >> 1) & 1);
+    const uint32_t a_s = ptx::smem_u32(abuf + s * Cfg::A_BYTES);
+#pragma unroll
+    for (int kk = 0; kk < Cfg::FK; ++kk) {
+      // A fragment (row g of each 8-row block, column kk*4 + t) from the
+      // swizzled broadcast tile: chunk = col/16, 16-B unit = (col%16)/2 ^ row%8
+      const int col = kk * 4 + t;
+      const uint32_t chunk_off = (uint32_t)(col >> 4) * (M * 128) + ((col & 1) << 3);
+      const uint32_t unit = (uint32_t)((col & 15) >> 1);
+#pragma unroll
+      for (int i = 0; i < Cfg::FM; ++i) {
+        const int row = i * 8 + g;
+        const uint32_t addr = a_s + chunk_off + row * 128 + ((unit ^ (row & 7)) << 4);
+        double a;
+        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(a) : "r"(addr));
+#pragma unroll
+        for (int j = 0; j < Cfg::FN; ++j)
+          asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                       : "+d"(c[i][j][0]), "+d"(c[i][j][1])
+                       : "d"(a), "d"(b[kk][j]));
+      }
+    }
+    // Reg2GMem: C_w, lane holds (row g, cols 2t, 2t+1) of each 8x8 block
+    double* Cg = prm.C + e * (long long)M * N + w * Cfg::NP;
+#pragma unroll
+    for (int i = 0; i < Cfg::FM; ++i)
+#pragma unroll
+      for (int j = 0; j < Cfg::FN; ++j)
+        ptx::st_global_v2_f64(Cg + (i * 8 + g) * N + j * 8 + 2 * t, c[i][j][0], c[i][j][1]);
+    ptx::named_bar_sync(bar, P * 32);  // buffer s free for entry it+2
+  }
+}
+
+template <int M, int N, int K, int P, int TEAMS>
+kami_status_t launch(long long batch, const void* A, const void* B, void* C, cudaStream_t stream, const char* name) {
+  using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
+  PFN_encodeTiled enc = get_encode_tiled();
+  if (!enc) return KAMI_ERROR_CUDA;
+  DmmaTmaParams prm;
+  memset(&prm, 0, sizeof(prm));
+  cuuint64_t dims[4] = {16, (cuuint64_t)M, (cuuint64_t)(K / 16), (cuuint64_t)batch};
+  cuuint64_t strides[3] = {(cuuint64_t)K * 8, 128, (cuuint64_t)M * K * 8};
+  cuuint32_t box[4] = {16, (cuuint32_t)M, (cuuint32_t)(K / 16), 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  if (enc(&prm.tmA, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<void*>(A), dims, strides, box, es,
+          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    return KAMI_ERROR_CUDA;
+  prm.B = static_cast<const double*>(B);
+  prm.C = static_cast<double*>(C);
+  prm.batch = batch;
+  auto fn = kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS>;
+  if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM) != cudaSuccess)
+    return KAMI_ERROR_CUDA;
+  int dev = 0, sms = 148, per_sm = 1;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, Cfg::THREADS, Cfg::SMEM) != cudaSuccess ||
+      per_sm < 1)
+    per_sm = 1;
+  long long grid = (long long)sms * per_sm;
+  const long long need = (batch + TEAMS - 1) / TEAMS;
+  if (grid > need) grid = need;
+  fn<<<(unsigned)grid, Cfg::THREADS, Cfg::SMEM, stream>>>(prm);
+  set_last_kernel(name);
+  return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+}
+
+}  // namespace
+
+bool dmma_tma_supported(int m, int n, int k) { return m == n && n == k && (m == 16 || m == 32 || m == 64); }
+
+// (p, teams) configuration; env KAMI_DMMA_TMA_CFG = 0/1/2 picks an alternative for sweeps
+kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
+                              cudaStream_t stream) {
+  static const int cfg = [] {
+    const char* e = getenv("KAMI_DMMA_TMA_CFG");
+    return e ? atoi(e) : 0;
+  }();
+  if (m == 64 && n == 64 && k == 64) {
+    if (cfg == 1) return launch<64, 64, 64, 8, 2>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,p8>");
+    return launch<64, 64, 64, 4, 3>(batch, A, B, C, stream, "kami_dmma_tma_1d<64>");
+  }
+  if (m == 32 && n == 32 && k == 32) {
+    if (cfg == 1) return launch<32, 32, 32, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,p2>");
+    if (cfg == 2) return launch<32, 32, 32, 4, 6>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,t6>");
+    return launch<32, 32, 32, 4, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32>");
+  }
+  if (m == 16 && n == 16 && k == 16) {
+    if (cfg == 1) return launch<16, 16, 16, 1, 16>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,p1>");
+    return launch<16, 16, 16, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<16>");
+  }
+  return KAMI_ERROR_NOT_SUPPORTED;
+}
+
+}  // namespace kami

@@ -39,4 +39,9 @@ kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t 
                              const void* A, const void* B, void* C, const void* const* A_arr,
                              const void* const* B_arr, void* const* C_arr, cudaStream_t stream);
 
+// ------------------------------------------- FP64 1D with TMA-fed broadcast
+bool dmma_tma_supported(int m, int n, int k);
+kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
+                              cudaStream_t stream);
+
 }  // namespace kami

@@ -93,6 +93,10 @@ double calibrated(kami_dtype_t dt, int m, int n, int k, int algo, int p) {
   return 0;
 }
 
+// measured TFLOP/s of the FP64 TMA-broadcast 1D kernel (0 = not calibrated;
+// bench.py --algo 1d_tma, profiles/r1/dmma_tma_sweep_r1.txt)
+double calibrated_tma(int m) { return m == 16 ? 7.42 : m == 32 ? 15.02 : m == 64 ? 25.45 : 0; }
+
 }  // namespace
 
 kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_t algo, int p, bool pointer_array,
@@ -102,7 +106,8 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
   // 16-bit strided: the tcgen05 family implements 1D with p = 4 sub-partition
   // tensor cores (tc16.cu); it covers the whole 16-bit size grid.  An explicit
   // p > 0 selects the warp-level family with p warps instead.
-  if (is16 && !pointer_array && (algo == KAMI_ALGO_AUTO || (algo == KAMI_ALGO_1D && p == 0))) {
+  if (is16 && !pointer_array &&
+      (algo == KAMI_ALGO_AUTO || algo == KAMI_ALGO_1D_TMA || (algo == KAMI_ALGO_1D && p == 0))) {
     Tc16Shape s;
     kami_status_t st = tc16_plan_shape(m, n, k, &s);
     if (st != KAMI_SUCCESS) return st;
@@ -116,6 +121,30 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
     *out = r;
     return KAMI_SUCCESS;
   }
+  // FP64 1D with the broadcast operand fed by TMA (dmma_tma.cu)
+  const bool tma_ok = !is16 && !pointer_array && dmma_tma_supported(m, n, k);
+  if (algo == KAMI_ALGO_1D_TMA) {
+    if (!tma_ok || (p != 0 && p != 4)) return KAMI_ERROR_NOT_SUPPORTED;
+    r.algo = KAMI_ALGO_1D_TMA;
+    r.p = 4;
+    r.kernel = 2;
+    r.entries_per_cta = m == 64 ? 3 : 8;
+    r.stages = 2;
+    r.kslice_regs_pct = 50;  // B_w resident in registers, A broadcast through SMEM
+    r.t_all_cycles = b200_cost(1, n, m, k, 4, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
+  if (algo == KAMI_ALGO_AUTO && tma_ok) {
+    const double t_tma = calibrated_tma(m);
+    double best_w = 0;
+    for (int v : {1, 2, 3}) {
+      const int pp = warp_ca_default_p(m, n, k, dtype, v);
+      if (pp) best_w = std::max(best_w, calibrated(dtype, m, n, k, v, pp));
+    }
+    if (t_tma > best_w) return planner_choose(m, n, k, dtype, KAMI_ALGO_1D_TMA, 0, pointer_array, out);
+  }
+  if (algo == KAMI_ALGO_1D_TMA) return KAMI_ERROR_NOT_SUPPORTED;
   // warp-level register-resident family
   int cand[3] = {1, 2, 3};
   if (algo != KAMI_ALGO_AUTO) {

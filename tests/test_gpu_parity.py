@@ -194,3 +194,13 @@ def test_warp_explicit_p(dtype, s, algo, p):
     """Same-warp-count comparators (non-CA 4x2 / 4x4 grids) and explicit p."""
     check(s, s, s, 41, dtype, "row", "unif", algo=algo, p=p)
     check(s, s, s, 13, dtype, "col", "int", algo=algo, p=p, seed=4)
+
+
+@pytest.mark.parametrize("s", [16, 32, 64])
+def test_f64_dmma_tma_1d(s):
+    """FP64 1D with the TMA-fed broadcast operand (dmma_tma.cu)."""
+    for batch in (1, 5, 97):
+        check(s, s, s, batch, "f64", "row", "unif", algo="1d_tma")
+    check(s, s, s, 33, "f64", "col", "unif", algo="1d_tma", seed=1)
+    check(s, s, s, 21, "f64", "row", "int", algo="1d_tma", seed=2)
+    assert kami.last_kernel().startswith("kami_dmma_tma_1d")
