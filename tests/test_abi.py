@@ -80,7 +80,10 @@ def test_plan_host_logic():
     # entries in flight per CTA: G = 2 entries per 128-lane MMA tile x stages
     assert p["entries_per_cta"] == 2 * p["stages"]
     p = kami.plan(64, 64, 64, "f64")
-    assert p["kernel"] == "warp_ca" and p["algo"] in ("1d", "2d", "3d")
+    # FP64 AUTO: the measured-fastest schedule (1D with TMA-fed broadcast on DMMA)
+    assert p["kernel"] == "dmma_tma" and p["algo"] == "1d_tma"
+    q = kami.plan(8, 8, 8, "f64")
+    assert q["kernel"] == "warp_ca" and q["algo"] == "1d"
     for algo in ("1d", "2d", "3d", "nonca"):
         q = kami.plan(32, 32, 32, "f64", algo=algo)
         assert q["algo"] == algo and q["kernel"] == "warp_ca"
