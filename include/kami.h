@@ -107,6 +107,21 @@ kami_status_t kami_gemm_strided_batched_host(int m, int n, int k, int64_t batch,
                                              kami_layout_t layout, const void* A, const void* B, void* C);
 kami_status_t kami_release_workspace(void);
 
+/* Block-level (on-chip-resident) mode -- the paper's block-level experiment
+ * (Sec. 5.1, Sec. 5.2, Fig. 8/9): every entry is owned by one
+ * team of p warps that loads A_b and B_b once and runs the CA schedule `reps`
+ * times on chip, accumulating C_b = reps * A_b B_b, stored once; all entries
+ * are launched at once (no persistent loop, no L2 prefetch).  It measures the
+ * schedule without global I/O.  `cycles` (optional, may be NULL) is a DEVICE
+ * int64 array of 2*batch that receives, per entry, the clock64 cycles spent
+ * in communication (SMEM exchange + barrier) and in computation (MMA issue),
+ * summed over the team's warps (Sec. 5.6.2, Fig. 15); it must be zeroed by
+ * the caller.  Register-resident warp-level kernels only: algo 1D/2D/3D/NONCA
+ * (AUTO = 1D) with p = 0 for the default warp count.  reps >= 1. */
+kami_status_t kami_gemm_block_level(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
+                                    kami_algo_t algo, int p, int reps, const void* A, const void* B, void* C,
+                                    int64_t* cycles, kami_stream_t stream);
+
 /* Planner decision (cost model PAPER.md Eqs. 4/8/12). */
 typedef struct {
   kami_algo_t algo;      /* chosen schedule                                 */

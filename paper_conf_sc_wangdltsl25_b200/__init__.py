@@ -30,7 +30,7 @@ STATUS = {0: "KAMI_SUCCESS", 1: "KAMI_ERROR_INVALID_VALUE", 2: "KAMI_ERROR_NOT_S
 EXPORTS = [
     "kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
     "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
-    "kami_status_string", "kami_last_kernel", "kami_version",
+    "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level",
 ]
 
 
@@ -65,11 +65,13 @@ def lib() -> ctypes.CDLL:
     L.kami_gemm_strided_batched.argtypes = [i, i, i, i64, i, i, vp, vp, vp, st]
     L.kami_gemm_strided_batched_ex.argtypes = [i, i, i, i64, i, i, vp, vp, vp, i, i, st]
     L.kami_gemm_strided_batched_host.argtypes = [i, i, i, i64, i, i, vp, vp, vp]
+    L.kami_gemm_block_level.argtypes = [i, i, i, i64, i, i, i, i, i, vp, vp, vp, vp, st]
     L.kami_release_workspace.argtypes = []
     L.kami_plan.argtypes = [i, i, i, i, i, i, i, ctypes.POINTER(KamiPlan)]
     d = ctypes.c_double
     L.kami_paper_cost.argtypes = [i, d, d, d, d, d, d, d, d, d, d, d, ctypes.POINTER(ctypes.c_double)]
     for f in ("kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
+              "kami_gemm_block_level",
               "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost"):
         getattr(L, f).restype = ctypes.c_int
     L.kami_status_string.restype = ctypes.c_char_p
@@ -168,6 +170,17 @@ def gemm_strided_batched_host(m, n, k, batch, dtype, layout, A, B, C):
     _check(lib().kami_gemm_strided_batched_host(m, n, k, batch, _enum(DTYPE, dtype, "dtype"),
                                                 _enum(LAYOUT, layout, "layout"), _ptr(A), _ptr(B), _ptr(C)),
            "kami_gemm_strided_batched_host")
+
+
+def gemm_block_level(m, n, k, batch, dtype, layout, A, B, C, algo="1d", p=0, reps=1000, cycles=None,
+                     stream=None):
+    """Block-level (on-chip-resident) mode: C_b = reps * A_b B_b with the CA
+    schedule repeated ``reps`` times on chip; ``cycles`` (device int64, 2*batch,
+    zeroed) receives per-entry [communication, computation] clock64 sums."""
+    _check(lib().kami_gemm_block_level(m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
+                                       _enum(ALGO, algo, "algo"), p, reps, _ptr(A), _ptr(B), _ptr(C), _ptr(cycles),
+                                       _stream(stream)), "kami_gemm_block_level")
+    return C
 
 
 def release_workspace():

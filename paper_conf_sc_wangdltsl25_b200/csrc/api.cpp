@@ -134,6 +134,24 @@ kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t
   return dispatch(rp, batch, dtype, KAMI_ALGO_AUTO, 0, nullptr, C_array, reinterpret_cast<cudaStream_t>(stream));
 }
 
+kami_status_t kami_gemm_block_level(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
+                                    kami_algo_t algo, int p, int reps, const void* A, const void* B, void* C,
+                                    int64_t* cycles, kami_stream_t stream) {
+  kami_status_t st = check_common(m, n, k, batch, dtype, layout, algo);
+  if (st != KAMI_SUCCESS) return st;
+  if (p < 0 || reps < 1 || algo == KAMI_ALGO_1D_TMA) return KAMI_ERROR_INVALID_VALUE;
+  if (batch == 0) return KAMI_SUCCESS;
+  if (!A || !B || !C) return KAMI_ERROR_INVALID_VALUE;
+  if (!aligned16(A) || !aligned16(B) || !aligned16(C)) return KAMI_ERROR_MISALIGNED;
+  if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
+  RowProblem rp = to_row(m, n, k, layout, A, B, nullptr, nullptr);
+  const int a = algo == KAMI_ALGO_AUTO ? (int)KAMI_ALGO_1D : (int)algo;
+  const int pp = p ? p : warp_ca_default_p(rp.m, rp.n, rp.k, dtype, a);
+  if (pp == 0) return KAMI_ERROR_NOT_SUPPORTED;
+  return warp_ca_launch(rp.m, rp.n, rp.k, batch, dtype, a, pp, rp.A, rp.B, C, nullptr, nullptr, nullptr,
+                        reinterpret_cast<cudaStream_t>(stream), reps, reinterpret_cast<long long*>(cycles));
+}
+
 kami_status_t kami_plan(int m, int n, int k, kami_dtype_t dtype, kami_layout_t layout, kami_algo_t algo, int p,
                         kami_plan_t* out) {
   kami_status_t st = check_common(m, n, k, 1, dtype, layout, algo);

@@ -35,9 +35,13 @@ kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const
 // Entry pointers: if A_arr != nullptr they are device arrays of per-entry
 // pointers (kami_gemm_batched); else strided from A/B/C.
 kami_status_t warp_ca_supported(int m, int n, int k, kami_dtype_t dtype, int algo, int p);
+// reps > 1: block-level mode (operands loaded once, the CA schedule repeated
+// reps times on chip, C = reps * A B stored once).  cycles != nullptr: per-entry
+// [comm, compute] clock64 sums over the team's warps (int64 device array).
 kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t dtype, int algo, int p,
                              const void* A, const void* B, void* C, const void* const* A_arr,
-                             const void* const* B_arr, void* const* C_arr, cudaStream_t stream);
+                             const void* const* B_arr, void* const* C_arr, cudaStream_t stream, int reps = 1,
+                             long long* cycles = nullptr);
 
 // ------------------------------------------- FP64 1D with TMA-fed broadcast
 bool dmma_tma_supported(int m, int n, int k);

@@ -248,6 +248,37 @@ __device__ __forceinline__ void copy_tile(T& dst, const T& src) {
   dst = src;
 }
 
+// Per-phase cycle counters for the block-level mode (Sec. 5.6.2,
+// Fig. 15: clock() around communication and computation phases).  Like the
+// paper's, the compute phase counts issue time of the mma.sync sequence.
+template <bool kTime>
+struct PhaseClock {
+  long long t0 = 0, comm = 0, comp = 0;
+  __device__ __forceinline__ void begin() {
+    if (kTime) t0 = clock64();
+  }
+  __device__ __forceinline__ void comm_done() {
+    if (kTime) {
+      const long long t = clock64();
+      comm += t - t0;
+      t0 = t;
+    }
+  }
+  __device__ __forceinline__ void comp_done() {
+    if (kTime) {
+      const long long t = clock64();
+      comp += t - t0;
+      t0 = t;
+    }
+  }
+  __device__ __forceinline__ void flush(long long* cyc, int lane) {
+    if (kTime && cyc && lane == 0) {
+      atomicAdd(reinterpret_cast<unsigned long long*>(cyc), (unsigned long long)comm);
+      atomicAdd(reinterpret_cast<unsigned long long*>(cyc + 1), (unsigned long long)comp);
+    }
+  }
+};
+
 // ------------------------------------------------------------ schedules
 // Each schedule runs one batch entry on a team of P warps.  wi = warp index
 // in the team, bar = named barrier id of the team, stage = running stage
@@ -266,8 +297,9 @@ struct Sched1D {
   static constexpr int SMEM_WORDS = 2 * XWORDS;     // double buffered
   static constexpr int SMEM_BYTES = SMEM_WORDS * sizeof(typename At::R);
   static_assert(MP % At::AM == 0 && KP % At::AK == 0 && N % At::AN == 0, "1D tile shape");
+  template <bool kTime>
   __device__ static void run(const typename At::E* A, const typename At::E* B, typename At::E* C, uint8_t* smem,
-                             int wi, int lane, int bar, uint32_t& stage) {
+                             int wi, int lane, int bar, uint32_t& stage, int reps, long long* cyc) {
     using W = typename At::R;
     W* xb = reinterpret_cast<W*>(smem);
     TA a;
@@ -276,17 +308,25 @@ struct Sched1D {
     load_a(a, A, K, wi * MP, 0, lane);  // GMem2Reg(A_i)
     load_b(bi, B, N, wi * KP, 0, lane);  // GMem2Reg(B_i)
     zero(c);
+    PhaseClock<kTime> clk;
+#pragma unroll 1
+    for (int rep = 0; rep < reps; ++rep) {  // block-level mode repeats on-chip
 #pragma unroll
-    for (int z = 0; z < P; ++z, ++stage) {
-      W* buf = xb + (stage & 1) * XWORDS;
-      if (wi == z) {
-        put(bi, buf, lane);  // Reg2SMem(SmB <- BSend)
-        copy_tile(br, bi);   // Reg2Reg(BRecv <- BSend)
+      for (int z = 0; z < P; ++z, ++stage) {
+        clk.begin();
+        W* buf = xb + (stage & 1) * XWORDS;
+        if (wi == z) {
+          put(bi, buf, lane);  // Reg2SMem(SmB <- BSend)
+          copy_tile(br, bi);   // Reg2Reg(BRecv <- BSend)
+        }
+        ptx::named_bar_sync(bar, P * 32);
+        if (wi != z) get(br, buf, lane);  // SMem2Reg(BRecv <- SmB)
+        clk.comm_done();
+        mma_tile(c, a, br, z * (KP / At::AK));  // C_i += A_i[:, z k/p:(z+1) k/p] BRecv
+        clk.comp_done();
       }
-      ptx::named_bar_sync(bar, P * 32);
-      if (wi != z) get(br, buf, lane);  // SMem2Reg(BRecv <- SmB)
-      mma_tile(c, a, br, z * (KP / At::AK));  // C_i += A_i[:, z k/p:(z+1) k/p] BRecv
     }
+    clk.flush(cyc, lane);
     store_c(c, C, N, wi * MP, 0, lane);  // Reg2GMem
   }
 };
@@ -307,8 +347,9 @@ struct Sched2D {
   static constexpr int SMEM_WORDS = 2 * XWORDS;
   static constexpr int SMEM_BYTES = SMEM_WORDS * sizeof(typename At::R);
   static_assert(TM % At::AM == 0 && TK % At::AK == 0 && TN % At::AN == 0, "2D tile shape");
+  template <bool kTime>
   __device__ static void run(const typename At::E* A, const typename At::E* B, typename At::E* C, uint8_t* smem,
-                             int wi, int lane, int bar, uint32_t& stage) {
+                             int wi, int lane, int bar, uint32_t& stage, int reps, long long* cyc) {
     using W = typename At::R;
     const int wr = wi / Q, wc = wi % Q;
     TA ai, ar;
@@ -317,24 +358,32 @@ struct Sched2D {
     load_a(ai, A, K, wr * TM, wc * TK, lane);
     load_b(bi, B, N, wr * TK, wc * TN, lane);
     zero(c);
+    PhaseClock<kTime> clk;
+#pragma unroll 1
+    for (int rep = 0; rep < reps; ++rep) {
 #pragma unroll
-    for (int z = 0; z < Q; ++z, ++stage) {
-      W* buf = reinterpret_cast<W*>(smem) + (stage & 1) * XWORDS;
-      W* sa = buf + wr * TA::WORDS;                // SmA of grid row wr
-      W* sb = buf + Q * TA::WORDS + wc * TB::WORDS;  // SmB of grid column wc
-      if (wc == z) {
-        put(ai, sa, lane);
-        copy_tile(ar, ai);
+      for (int z = 0; z < Q; ++z, ++stage) {
+        clk.begin();
+        W* buf = reinterpret_cast<W*>(smem) + (stage & 1) * XWORDS;
+        W* sa = buf + wr * TA::WORDS;                  // SmA of grid row wr
+        W* sb = buf + Q * TA::WORDS + wc * TB::WORDS;  // SmB of grid column wc
+        if (wc == z) {
+          put(ai, sa, lane);
+          copy_tile(ar, ai);
+        }
+        if (wr == z) {
+          put(bi, sb, lane);
+          copy_tile(br, bi);
+        }
+        ptx::named_bar_sync(bar, P * 32);
+        if (wc != z) get(ar, sa, lane);
+        if (wr != z) get(br, sb, lane);
+        clk.comm_done();
+        mma_tile(c, ar, br, 0);
+        clk.comp_done();
       }
-      if (wr == z) {
-        put(bi, sb, lane);
-        copy_tile(br, bi);
-      }
-      ptx::named_bar_sync(bar, P * 32);
-      if (wc != z) get(ar, sa, lane);
-      if (wr != z) get(br, sb, lane);
-      mma_tile(c, ar, br, 0);
     }
+    clk.flush(cyc, lane);
     store_c(c, C, N, wr * TM, wc * TN, lane);
   }
 };
@@ -359,8 +408,9 @@ struct Sched3D {
   static constexpr int RBYTES = Cc * Cc * Cc * TC::WORDS * sizeof(typename At::Acc);
   static constexpr int SMEM_BYTES = XBYTES + RBYTES;
   static_assert(TM % At::AM == 0 && TK % At::AK == 0 && TN % At::AN == 0, "3D tile shape");
+  template <bool kTime>
   __device__ static void run(const typename At::E* A, const typename At::E* B, typename At::E* C, uint8_t* smem,
-                             int wi, int lane, int bar, uint32_t& stage) {
+                             int wi, int lane, int bar, uint32_t& stage, int reps, long long* cyc) {
     using W = typename At::R;
     using Acc = typename At::Acc;
     const int l = wi / (Cc * Cc), wr = (wi / Cc) % Cc, wc = wi % Cc;
@@ -371,24 +421,32 @@ struct Sched3D {
     load_a(ai, A, K, wr * TM, kl + wc * TK, lane);
     load_b(bi, B, N, kl + wr * TK, wc * TN, lane);
     zero(c);
+    PhaseClock<kTime> clk;
+#pragma unroll 1
+    for (int rep = 0; rep < reps; ++rep) {
 #pragma unroll
-    for (int z = 0; z < Cc; ++z, ++stage) {
-      W* buf = reinterpret_cast<W*>(smem) + (stage & 1) * XWORDS + l * LWORDS;
-      W* sa = buf + wr * TA::WORDS;
-      W* sb = buf + Cc * TA::WORDS + wc * TB::WORDS;
-      if (wc == z) {
-        put(ai, sa, lane);
-        copy_tile(ar, ai);
+      for (int z = 0; z < Cc; ++z, ++stage) {
+        clk.begin();
+        W* buf = reinterpret_cast<W*>(smem) + (stage & 1) * XWORDS + l * LWORDS;
+        W* sa = buf + wr * TA::WORDS;
+        W* sb = buf + Cc * TA::WORDS + wc * TB::WORDS;
+        if (wc == z) {
+          put(ai, sa, lane);
+          copy_tile(ar, ai);
+        }
+        if (wr == z) {
+          put(bi, sb, lane);
+          copy_tile(br, bi);
+        }
+        ptx::named_bar_sync(bar, P * 32);
+        if (wc != z) get(ar, sa, lane);
+        if (wr != z) get(br, sb, lane);
+        clk.comm_done();
+        mma_tile(c, ar, br, 0);
+        clk.comp_done();
       }
-      if (wr == z) {
-        put(bi, sb, lane);
-        copy_tile(br, bi);
-      }
-      ptx::named_bar_sync(bar, P * 32);
-      if (wc != z) get(ar, sa, lane);
-      if (wr != z) get(br, sb, lane);
-      mma_tile(c, ar, br, 0);
     }
+    clk.flush(cyc, lane);
     // K-split reduction across layers as a reduce-scatter: the C tile's
     // fragments are split into Cc chunks, layer l owns chunk l.  Each layer
     // writes the chunks it does not own, reads the others' partials of its own
@@ -459,8 +517,9 @@ struct SchedNonCA {
   static constexpr int AWORDS = FMT * FKT * At::NA * 32, BWORDS = FKT * FNT * At::NB * 32;
   static constexpr int SMEM_BYTES = (AWORDS + BWORDS) * sizeof(typename At::R);
   static_assert(TM % At::AM == 0 && TN % At::AN == 0, "non-CA tile shape");
+  template <bool kTime>
   __device__ static void run(const typename At::E* A, const typename At::E* B, typename At::E* C, uint8_t* smem,
-                             int wi, int lane, int bar, uint32_t& stage) {
+                             int wi, int lane, int bar, uint32_t& stage, int reps, long long* cyc) {
     using W = typename At::R;
     W* sA = reinterpret_cast<W*>(smem);
     W* sB = sA + AWORDS;
@@ -489,22 +548,30 @@ struct SchedNonCA {
     const int wm = wi / WN, wn = wi % WN;
     TileC<At, TM, TN> c;
     zero(c);
+    PhaseClock<kTime> clk;
 #pragma unroll 1
-    for (int fk = 0; fk < FKT; ++fk) {
-      TileA<At, TM, At::AK> a;
-      TileB<At, At::AK, TN> b;
+    for (int rep = 0; rep < reps; ++rep) {
+#pragma unroll 1
+      for (int fk = 0; fk < FKT; ++fk) {
+        clk.begin();
+        TileA<At, TM, At::AK> a;
+        TileB<At, At::AK, TN> b;
 #pragma unroll
-      for (int i = 0; i < TileA<At, TM, At::AK>::FM; ++i)
+        for (int i = 0; i < TileA<At, TM, At::AK>::FM; ++i)
 #pragma unroll
-        for (int r = 0; r < At::NA; ++r)
-          a.v[i][0][r] = sA[(((wm * (TM / At::AM) + i) * FKT + fk) * At::NA + r) * 32 + lane];
+          for (int r = 0; r < At::NA; ++r)
+            a.v[i][0][r] = sA[(((wm * (TM / At::AM) + i) * FKT + fk) * At::NA + r) * 32 + lane];
 #pragma unroll
-      for (int j = 0; j < TileB<At, At::AK, TN>::FN; ++j)
+        for (int j = 0; j < TileB<At, At::AK, TN>::FN; ++j)
 #pragma unroll
-        for (int r = 0; r < At::NB; ++r)
-          b.v[0][j][r] = sB[((fk * FNT + wn * (TN / At::AN) + j) * At::NB + r) * 32 + lane];
-      mma_tile(c, a, b, 0);
+          for (int r = 0; r < At::NB; ++r)
+            b.v[0][j][r] = sB[((fk * FNT + wn * (TN / At::AN) + j) * At::NB + r) * 32 + lane];
+        clk.comm_done();
+        mma_tile(c, a, b, 0);
+        clk.comp_done();
+      }
     }
+    clk.flush(cyc, lane);
     store_c(c, C, N, wm * TM, wn * TN, lane);
     ptx::named_bar_sync(bar, P * 32);  // SMEM is reused by the next entry
     ++stage;
@@ -512,14 +579,14 @@ struct SchedNonCA {
 };
 
 // ----------------------------------------------------------- the kernel
-template <class Sched, class At, int P, int TEAMS>
+template <class Sched, class At, int P, int TEAMS, bool kTime>
 __global__ void __launch_bounds__(P * 32 * TEAMS) kami_warp_ca_kernel(const typename At::E* __restrict__ A,
                                                                       const typename At::E* __restrict__ B,
                                                                       typename At::E* __restrict__ C,
                                                                       const void* const* A_arr,
                                                                       const void* const* B_arr, void* const* C_arr,
                                                                       long long batch, int M, int N, int K,
-                                                                      int prefetch) {
+                                                                      int prefetch, int reps, long long* cyc) {
   extern __shared__ __align__(16) uint8_t smem_raw[];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int team = warp / P, wi = warp % P;
@@ -550,13 +617,14 @@ __global__ void __launch_bounds__(P * 32 * TEAMS) kami_warp_ca_kernel(const type
       ptx::prefetch_l2_bulk(na, (uint32_t)(M * K * sizeof(typename At::E)));
       ptx::prefetch_l2_bulk(nb, (uint32_t)(K * N * sizeof(typename At::E)));
     }
-    Sched::run(a, b, c, smem, wi, lane, bar, stage);
+    Sched::template run<kTime>(a, b, c, smem, wi, lane, bar, stage, reps, cyc ? cyc + 2 * e : nullptr);
   }
 }
 
 // ----------------------------------------------------------- host side
 struct LaunchInfo {
   const void* fn;
+  const void* fn_timed;
   int p;
   int threads;
   int smem;
@@ -566,7 +634,8 @@ struct LaunchInfo {
 template <class Sched, class At, int P, int TEAMS>
 LaunchInfo info(const char* name) {
   LaunchInfo li;
-  li.fn = reinterpret_cast<const void*>(&kami_warp_ca_kernel<Sched, At, P, TEAMS>);
+  li.fn = reinterpret_cast<const void*>(&kami_warp_ca_kernel<Sched, At, P, TEAMS, false>);
+  li.fn_timed = reinterpret_cast<const void*>(&kami_warp_ca_kernel<Sched, At, P, TEAMS, true>);
   li.p = P;
   li.threads = P * 32 * TEAMS;
   li.smem = TEAMS * ((Sched::SMEM_BYTES + 127) / 128 * 128);
@@ -671,32 +740,36 @@ int warp_ca_teams_per_sm(int m, int n, int k, kami_dtype_t dtype, int algo, int 
 
 kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t dtype, int algo, int p,
                              const void* A, const void* B, void* C, const void* const* A_arr,
-                             const void* const* B_arr, void* const* C_arr, cudaStream_t stream) {
+                             const void* const* B_arr, void* const* C_arr, cudaStream_t stream, int reps,
+                             long long* cycles) {
   LaunchInfo li;
   if (!lookup(m, n, k, dtype, algo, p, &li)) return KAMI_ERROR_NOT_SUPPORTED;
+  const void* fn = cycles ? li.fn_timed : li.fn;
   if (li.smem > 48 * 1024) {
-    if (cudaFuncSetAttribute(li.fn, cudaFuncAttributeMaxDynamicSharedMemorySize, li.smem) != cudaSuccess)
+    if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, li.smem) != cudaSuccess)
       return KAMI_ERROR_CUDA;
   }
   int dev = 0, sms = 148, per_sm = 1;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, li.fn, li.threads, li.smem) != cudaSuccess ||
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, li.threads, li.smem) != cudaSuccess ||
       per_sm < 1)
     per_sm = 1;
   const long long teams = li.threads / 32 / li.p;
   const long long ctas_needed = (batch + teams - 1) / teams;
-  long long grid = (long long)sms * per_sm;  // persistent: teams loop over the batch
+  // batched: persistent teams loop over the batch; block-level (reps > 1):
+  // one entry per team, every CTA launched at once
+  long long grid = reps > 1 ? ctas_needed : (long long)sms * per_sm;
   if (grid > ctas_needed) grid = ctas_needed;
   if (grid < 1) grid = 1;
   static const int prefetch = [] {
     const char* e = getenv("KAMI_L2_PREFETCH");
     return e ? atoi(e) : 1;
   }();
-  int pf = prefetch;
+  int pf = reps > 1 ? 0 : prefetch;
   void* args[] = {(void*)&A, (void*)&B, (void*)&C, (void*)&A_arr, (void*)&B_arr, (void*)&C_arr,
-                  (void*)&batch, (void*)&m, (void*)&n, (void*)&k, (void*)&pf};
-  cudaError_t err = cudaLaunchKernel(li.fn, dim3((unsigned)grid), dim3(li.threads), args, li.smem, stream);
+                  (void*)&batch, (void*)&m, (void*)&n, (void*)&k, (void*)&pf, (void*)&reps, (void*)&cycles};
+  cudaError_t err = cudaLaunchKernel(fn, dim3((unsigned)grid), dim3(li.threads), args, li.smem, stream);
   set_last_kernel(li.name);
   return err == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
 }
