@@ -82,6 +82,21 @@ kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t
                                 const void* const* A_array, const void* const* B_array, void* const* C_array,
                                 kami_stream_t stream);
 
+/* Variable-size batched GEMM (MAGMA *_vbatched convention; "various matrix
+ * orders in a batch"): entry b is m_array[b] x k_array[b]
+ * times k_array[b] x n_array[b].  m_array, n_array, k_array are DEVICE int
+ * arrays; A_array, B_array, C_array are DEVICE arrays of DEVICE pointers (each
+ * 16-byte aligned, packed matrices in `layout`).  max_m/max_n/max_k are host
+ * upper bounds used for planning and validated against the size grid; every
+ * entry must itself be on the grid (16-bit: m, n multiples of 16 <= 256, k a
+ * multiple of 8 <= 256) -- entries off the grid are undefined behaviour (the
+ * sizes live on the device and are not read by the host).  16-bit types only
+ * (FP64 returns KAMI_ERROR_NOT_SUPPORTED). */
+kami_status_t kami_gemm_vbatched(int64_t batch, const int* m_array, const int* n_array, const int* k_array,
+                                 int max_m, int max_n, int max_k, kami_dtype_t dtype, kami_layout_t layout,
+                                 const void* const* A_array, const void* const* B_array, void* const* C_array,
+                                 kami_stream_t stream);
+
 /* Strided-batched GEMM: entry b of A at A + b*m*k elements, of B at
  * B + b*k*n, of C at C + b*m*n.  The hot path of BASELINE.json. */
 kami_status_t kami_gemm_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,

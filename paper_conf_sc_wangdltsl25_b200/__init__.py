@@ -30,7 +30,7 @@ STATUS = {0: "KAMI_SUCCESS", 1: "KAMI_ERROR_INVALID_VALUE", 2: "KAMI_ERROR_NOT_S
 EXPORTS = [
     "kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
     "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
-    "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level",
+    "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level", "kami_gemm_vbatched",
 ]
 
 
@@ -66,12 +66,13 @@ def lib() -> ctypes.CDLL:
     L.kami_gemm_strided_batched_ex.argtypes = [i, i, i, i64, i, i, vp, vp, vp, i, i, st]
     L.kami_gemm_strided_batched_host.argtypes = [i, i, i, i64, i, i, vp, vp, vp]
     L.kami_gemm_block_level.argtypes = [i, i, i, i64, i, i, i, i, i, vp, vp, vp, vp, st]
+    L.kami_gemm_vbatched.argtypes = [i64, vp, vp, vp, i, i, i, i, i, vp, vp, vp, st]
     L.kami_release_workspace.argtypes = []
     L.kami_plan.argtypes = [i, i, i, i, i, i, i, ctypes.POINTER(KamiPlan)]
     d = ctypes.c_double
     L.kami_paper_cost.argtypes = [i, d, d, d, d, d, d, d, d, d, d, d, ctypes.POINTER(ctypes.c_double)]
     for f in ("kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
-              "kami_gemm_block_level",
+              "kami_gemm_block_level", "kami_gemm_vbatched",
               "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost"):
         getattr(L, f).restype = ctypes.c_int
     L.kami_status_string.restype = ctypes.c_char_p
@@ -156,6 +157,15 @@ def gemm_batched(m, n, k, batch, dtype, layout, A_ptrs, B_ptrs, C_ptrs, stream=N
     per-entry device addresses (cuBLAS *gemmBatched convention)."""
     _check(lib().kami_gemm_batched(m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
                                    _ptr(A_ptrs), _ptr(B_ptrs), _ptr(C_ptrs), _stream(stream)), "kami_gemm_batched")
+
+
+def gemm_vbatched(batch, m_arr, n_arr, k_arr, max_m, max_n, max_k, dtype, layout, A_ptrs, B_ptrs, C_ptrs,
+                  stream=None):
+    """Variable-size batched GEMM: per-entry sizes and pointers in device int32 /
+    int64 tensors (MAGMA vbatched convention)."""
+    _check(lib().kami_gemm_vbatched(batch, _ptr(m_arr), _ptr(n_arr), _ptr(k_arr), max_m, max_n, max_k,
+                                    _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"), _ptr(A_ptrs),
+                                    _ptr(B_ptrs), _ptr(C_ptrs), _stream(stream)), "kami_gemm_vbatched")
 
 
 def gemm_single(m, n, k, dtype, layout, A, B, C, stream=None):

@@ -77,6 +77,10 @@ RowProblem to_row(int m, int n, int k, kami_layout_t layout, const void* A, cons
 
 kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, kami_algo_t algo, int p, void* C,
                        void* const* Ca, cudaStream_t stream) {
+  // 16-bit pointer arrays: the LDG-fed tcgen05 kernel covers the whole size grid
+  if (Ca && is16(dtype) && algo == KAMI_ALGO_AUTO)
+    return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, rp.m, rp.n, rp.k, nullptr, nullptr, nullptr, rp.m, rp.Aa,
+                          rp.Ba, Ca, stream);
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
@@ -132,6 +136,24 @@ kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t
   if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
   RowProblem rp = to_row(m, n, k, layout, nullptr, nullptr, A_array, B_array);
   return dispatch(rp, batch, dtype, KAMI_ALGO_AUTO, 0, nullptr, C_array, reinterpret_cast<cudaStream_t>(stream));
+}
+
+kami_status_t kami_gemm_vbatched(int64_t batch, const int* m_array, const int* n_array, const int* k_array,
+                                 int max_m, int max_n, int max_k, kami_dtype_t dtype, kami_layout_t layout,
+                                 const void* const* A_array, const void* const* B_array, void* const* C_array,
+                                 kami_stream_t stream) {
+  kami_status_t st = check_common(max_m, max_n, max_k, batch, dtype, layout, KAMI_ALGO_AUTO);
+  if (st != KAMI_SUCCESS) return st;
+  if (!is16(dtype)) return KAMI_ERROR_NOT_SUPPORTED;
+  if (batch == 0) return KAMI_SUCCESS;
+  if (!m_array || !n_array || !k_array || !A_array || !B_array || !C_array) return KAMI_ERROR_INVALID_VALUE;
+  if (!aligned16(A_array) || !aligned16(B_array) || !aligned16(C_array)) return KAMI_ERROR_MISALIGNED;
+  if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
+  // column-major: C^T = B^T A^T per entry -> swap m<->n and A<->B
+  const bool col = layout == KAMI_COL_MAJOR;
+  return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, 0, 0, 0, col ? n_array : m_array, col ? m_array : n_array,
+                        k_array, col ? max_n : max_m, col ? B_array : A_array, col ? A_array : B_array, C_array,
+                        reinterpret_cast<cudaStream_t>(stream));
 }
 
 kami_status_t kami_gemm_block_level(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,

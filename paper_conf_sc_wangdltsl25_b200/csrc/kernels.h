@@ -48,4 +48,10 @@ bool dmma_tma_supported(int m, int n, int k);
 kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
                               cudaStream_t stream);
 
+// ------------------------- 16-bit pointer-array / variable-size (tc16_vb.cu)
+// dm/dn/dk: device arrays of per-entry sizes, or nullptr for uniform m, n, k.
+kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, const int* dm, const int* dn,
+                             const int* dk, int max_m, const void* const* A, const void* const* B, void* const* C,
+                             cudaStream_t stream);
+
 }  // namespace kami
