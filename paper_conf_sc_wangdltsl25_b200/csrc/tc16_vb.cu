@@ -6,10 +6,11 @@
 // B broadcast through shared memory), but the operands cannot be described by
 // one TMA tensor map (every entry has its own pointer and possibly its own
 // m, n, k), so a producer warpgroup performs the paper's GMem2Reg + Reg2SMem
-// itself: coalesced 16-byte LDGs of A and B rows into registers, then
-// swizzled STS into the UMMA canonical layouts (128-byte swizzle, K-major A,
-// N-major B), zero-filling k beyond the entry's order; a generic->async proxy
-// fence and an mbarrier arrive hand the stage to the MMA warp.
+// itself: coalesced 16-byte cp.async (LDGSTS) copies of A and B rows straight
+// into the UMMA canonical layouts (128-byte swizzle, K-major A, N-major B),
+// zero-filling k beyond the entry's order; once a stage's copy group has
+// landed, a generic->async proxy fence and an mbarrier arrive hand it to the
+// MMA warp.
 //
 // Warps: 0-3 producer, 4 MMA issuer + TMEM allocator, 5-12 epilogue (two
 // warpgroups on alternate units; tcgen05.ld -> cvt.rn -> 16-byte st.global).
@@ -88,8 +89,24 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
 
   if (warp < 4) {
     // ------------------------------------------------ producer warpgroup
+    // cp.async (LDGSTS) straight into the swizzled stage buffers, zero-filled
+    // outside the entry; a stage is handed to the MMA warp (fence.proxy.async
+    // + mbarrier arrive) once its copy group has landed, kLag stages later, so
+    // several stages stream concurrently without register staging.
+    constexpr int kLag = kVbStages - 1;
     const int tid = threadIdx.x;  // 0..127
-    uint32_t it = 0;
+    uint32_t it = 0, handed = 0;
+    auto hand_over = [&](int pending) {
+      // copies of stage `handed` are complete when at most `pending` groups remain
+      static_assert(kLag <= 3, "wait_group depth");
+      if (pending >= 3) ptx::cp_async_wait<3>();
+      else if (pending == 2) ptx::cp_async_wait<2>();
+      else if (pending == 1) ptx::cp_async_wait<1>();
+      else ptx::cp_async_wait<0>();
+      ptx::fence_proxy_async_smem();
+      ptx::mbar_arrive(&full[handed % kVbStages]);
+      ++handed;
+    };
     for (long long u = blockIdx.x; u < units; u += gridDim.x) {
       const long long e = u / p.mtiles;
       const int mt = (int)(u - e * p.mtiles);
@@ -105,27 +122,27 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         ptx::mbar_wait(&empty[s], ((it / kVbStages) & 1) ^ 1);
         const uint32_t sa = smem_base + s * kStage, sb = sa + kAReg;
         // A: 128 rows x 8 chunks; a warp covers 4 whole 128-byte row segments
-#pragma unroll 2
+#pragma unroll 4
         for (int i = tid; i < 128 * 8; i += 128) {
           const int r = i >> 3, j = i & 7;
           const int gr = mt * 128 + r, gc = kc * 64 + j * 8;
-          uint4 v = make_uint4(0, 0, 0, 0);
-          if (gr < m && gc < k) v = __ldg(reinterpret_cast<const uint4*>(A + (long long)gr * k + gc));
-          ptx::st_shared_v4(sa + r * 128 + ((j ^ (r & 7)) << 4), v.x, v.y, v.z, v.w);
+          const bool ok = gr < m && gc < k;
+          const uint16_t* src = ok ? A + (long long)gr * k + gc : A;
+          ptx::cp_async_16(sa + r * 128 + ((j ^ (r & 7)) << 4), src, ok ? 16 : 0);
         }
         // B: 64 k-rows x n/8 chunks into N-atoms of 64 columns
         for (int i = tid; i < 64 * nc8; i += 128) {
           const int kr = i / nc8, j = i - kr * nc8;
           const int gk = kc * 64 + kr;
-          uint4 v = make_uint4(0, 0, 0, 0);
-          if (gk < k) v = __ldg(reinterpret_cast<const uint4*>(B + (long long)gk * n + j * 8));
-          const int atom = j >> 3, jj = j & 7;
-          ptx::st_shared_v4(sb + atom * 8192 + kr * 128 + ((jj ^ (kr & 7)) << 4), v.x, v.y, v.z, v.w);
+          const bool ok = gk < k;
+          const uint16_t* src = ok ? B + (long long)gk * n + j * 8 : B;
+          ptx::cp_async_16(sb + (j >> 3) * 8192 + kr * 128 + (((j & 7) ^ (kr & 7)) << 4), src, ok ? 16 : 0);
         }
-        ptx::fence_proxy_async_smem();  // generic-proxy writes -> visible to the tensor core
-        ptx::mbar_arrive(&full[s]);
+        ptx::cp_async_commit();
+        if (it + 1 - handed > (uint32_t)kLag) hand_over(kLag);
       }
     }
+    while (handed < it) hand_over((int)(it - handed - 1));
   } else if (warp == 4) {
     // ------------------------------------------------------------- MMA
     uint32_t it = 0, acc_it = 0;
