@@ -120,3 +120,64 @@ def as_bits(x: torch.Tensor):
     if x.dtype in (torch.float16, torch.bfloat16):
         return x.view(torch.int16).numpy().view("uint16")
     return x.numpy()
+
+
+# ------------------------------------------------- block-sparse A (SpMM, f3)
+BLK = 16  # dense block order (Sec. 4.6: user-configurable, default 16 x 16)
+
+
+def _key(seed: int, op: int, idx: torch.Tensor) -> torch.Tensor:
+    # a counter space disjoint from draw(): bit 62 set
+    assert 0 <= seed < (1 << 13) and 0 <= op < 16
+    return splitmix64(idx + ((1 << 62) + (seed << 48) + (op << 44)))
+
+
+def bsr_operands(m: int, n: int, k: int, batch: int, dtype: str, density: float = 0.5, dist: str = "unif",
+                 seed: int = 0, entry0: int = 0, device="cpu"):
+    """Batched block-sparse A (BSR, 16 x 16 dense blocks, block-row order --
+    the 1D storage of PAPER.md Fig. 7(a)) and dense B.
+
+    Block (i, j) of entry e is present iff a counter-based draw keyed by
+    (seed, e, i, j) falls below ``density`` (the paper's "50 % random
+    sparsity", Sec. 5.1); its values are keyed by (seed, e, i, j, element) so
+    they do not depend on the sparsity of other blocks.  Layout, per entry
+    (max_nnzb = (m/16) (k/16), unused tail slots zero / -1):
+      row_ptr [batch, m/16 + 1] int32, col_blk [batch, max_nnzb] int32 (sorted
+      within a block row), vals [batch, max_nnzb, 16, 16] (row-major blocks),
+      B [batch * k * n] packed row-major."""
+    assert m % BLK == 0 and k % BLK == 0
+    mb, kb = m // BLK, k // BLK
+    nb = mb * kb
+    ids = torch.arange(batch * nb, dtype=torch.int64, device=device) + entry0 * nb
+    z = _key(seed, 0, ids)
+    u = _lshr(z, 11).to(torch.float64) * (2.0 ** -53)
+    present = (u < density).view(batch, mb, kb)
+    counts = present.sum(2, dtype=torch.int32)                       # [batch, mb]
+    row_ptr = torch.zeros(batch, mb + 1, dtype=torch.int32, device=device)
+    row_ptr[:, 1:] = torch.cumsum(counts, 1)
+    # col_blk: present columns of each row, in order, packed per entry
+    cols = torch.arange(kb, dtype=torch.int32, device=device).expand(batch, mb, kb)
+    order = torch.argsort((~present).to(torch.int8), dim=2, stable=True)  # present first, ascending col
+    sorted_cols = torch.gather(cols, 2, order)
+    col_blk = torch.full((batch, nb), -1, dtype=torch.int32, device=device)
+    vals = torch.zeros(batch, nb, BLK, BLK, dtype=TORCH_DTYPES[dtype], device=device)
+    R = int_range(k, dtype) if dist == "int" else None
+    # vectorised scatter: slot of block (e, i, j-th present) = row_ptr[e, i] + j
+    jpos = torch.arange(kb, device=device).expand(batch, mb, kb)
+    valid = jpos < counts.unsqueeze(2)
+    slot = (row_ptr[:, :mb].unsqueeze(2) + jpos).masked_select(valid)
+    eidx = torch.arange(batch, device=device).view(batch, 1, 1).expand(batch, mb, kb).masked_select(valid)
+    bi = torch.arange(mb, device=device).view(1, mb, 1).expand(batch, mb, kb).masked_select(valid)
+    bj = sorted_cols.masked_select(valid).to(torch.int64)
+    col_blk[eidx, slot.to(torch.int64)] = bj.to(torch.int32)
+    # block values keyed by (entry, block row, block col, element)
+    bid = ((eidx + entry0) * nb + bi * kb + bj)                       # [nnz_total]
+    el = torch.arange(BLK * BLK, dtype=torch.int64, device=device)
+    zz = _key(seed, 1, bid.unsqueeze(1) * (BLK * BLK) + el.unsqueeze(0))
+    if dist == "unif":
+        v = _lshr(zz, 11).to(torch.float64) * (2.0 ** -52) - 1.0
+    else:
+        v = (torch.remainder(_lshr(zz, 33), 2 * R + 1) - R).to(torch.float64)
+    vals[eidx, slot.to(torch.int64)] = v.view(-1, BLK, BLK).to(TORCH_DTYPES[dtype])
+    _, B = operands(m, n, k, batch, dtype, dist, seed=seed, entry0=entry0, device=device)
+    return row_ptr, col_blk, vals, B

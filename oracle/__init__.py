@@ -151,3 +151,27 @@ def normalised_error(c_gpu: np.ndarray, c_ref: np.ndarray, s: np.ndarray) -> flo
     with np.errstate(divide="ignore", invalid="ignore"):
         e = np.where(zero, 0.0, diff / np.where(zero, 1.0, s))
     return float(e.max()) if e.size else 0.0
+
+
+def spmm_bsr(m: int, n: int, k: int, batch: int, dtype: str, row_ptr, col_blk, vals, B, blk: int = 16,
+             with_scale: bool = False):
+    """C_ref = A B for block-sparse A (BSR, Sec. 4.6): A densified
+    (absent blocks = 0), then the plain GEMM definition.  Returns [batch, m, n]."""
+    L = lib()
+    if not hasattr(L, "_spmm_set"):
+        L.oracle_spmm_bsr.restype = ctypes.c_int
+        L.oracle_spmm_bsr.argtypes = [ctypes.c_int] * 4 + [ctypes.c_int64, ctypes.c_int] + [ctypes.c_void_p] * 3 + \
+            [ctypes.c_int] + [ctypes.c_void_p] * 3 + [ctypes.c_int]
+        L._spmm_set = True
+    rp = np.ascontiguousarray(np.asarray(row_ptr), dtype=np.int32).reshape(-1)
+    cb = np.ascontiguousarray(np.asarray(col_blk), dtype=np.int32).reshape(batch, -1)
+    max_nnzb = cb.shape[1]
+    v = _raw(np.asarray(vals).reshape(-1), dtype)
+    b = _raw(np.asarray(B).reshape(-1), dtype)
+    C = np.empty((batch, m, n), dtype=np.float64)
+    S = np.empty((batch, m, n), dtype=np.float64) if with_scale else None
+    rc = L.oracle_spmm_bsr(m, n, k, blk, batch, DTYPES[dtype], rp.ctypes.data, cb.ctypes.data, v.ctypes.data,
+                           max_nnzb, b.ctypes.data, C.ctypes.data, S.ctypes.data if S is not None else None, 1)
+    if rc != 0:
+        raise ValueError(f"oracle_spmm_bsr rejected its arguments ({rc})")
+    return (C, S) if with_scale else C

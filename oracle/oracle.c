@@ -216,3 +216,43 @@ void oracle_decode_f16(const uint16_t* x, double* out, int64_t n) {
 void oracle_decode_bf16(const uint16_t* x, double* out, int64_t n) {
   for (int64_t i = 0; i < n; ++i) out[i] = oracle_bf16_to_f64(x[i]);
 }
+
+/* ---------------------------------------------------------- SpMM oracle
+ * PAPER.md Sec. 4.6 (L407-418): SpMM multiplies a sparse A, stored as dense
+ * blk x blk blocks in block-row order (Fig. 7(a), the 1D storage: row_ptr /
+ * col_blk / vals), by a dense B into a dense C.  The plain definition: expand
+ * A to its dense m x k matrix (absent blocks are zero) and run the GEMM
+ * definition above.  Per entry b: row_ptr[b*(m/blk+1) + i] .. row_ptr[...+i+1]
+ * index the blocks of block row i in col_blk[b*max_nnzb + j] and
+ * vals[(b*max_nnzb + j)*blk*blk + r*blk + c].  B and C row-major. */
+int oracle_spmm_bsr(int m, int n, int k, int blk, int64_t batch, int dtype, const int* row_ptr,
+                    const int* col_blk, const void* vals, int max_nnzb, const void* B, double* C, double* S,
+                    int nthreads) {
+  if (m <= 0 || n <= 0 || k <= 0 || blk <= 0 || batch < 0 || m % blk || k % blk) return 1;
+  const int mb = m / blk;
+  double* Ad = (double*)malloc(sizeof(double) * (size_t)m * k);
+  double* Bd = (double*)malloc(sizeof(double) * (size_t)k * n);
+  if (!Ad || !Bd) return 2;
+  int rc = 0;
+  for (int64_t b = 0; b < batch && rc == 0; ++b) {
+    memset(Ad, 0, sizeof(double) * (size_t)m * k);
+    const int* rp = row_ptr + b * (mb + 1);
+    for (int i = 0; i < mb; ++i) {
+      for (int j = rp[i]; j < rp[i + 1]; ++j) {
+        const int bc = col_blk[b * max_nnzb + j];
+        if (bc < 0 || (bc + 1) * blk > k) { rc = 3; break; }
+        for (int r = 0; r < blk; ++r)
+          for (int c = 0; c < blk; ++c)
+            Ad[(size_t)(i * blk + r) * k + bc * blk + c] =
+                load_elem(vals, dtype, (b * max_nnzb + j) * (int64_t)blk * blk + r * blk + c);
+      }
+    }
+    for (int64_t t = 0; t < (int64_t)k * n; ++t) Bd[t] = load_elem(B, dtype, b * (int64_t)k * n + t);
+    rc = rc ? rc : oracle_gemm(m, n, k, 1, ORACLE_F64, ORACLE_ROW, Ad, Bd, C + b * (int64_t)m * n,
+                               S ? S + b * (int64_t)m * n : NULL, 1);
+  }
+  (void)nthreads;
+  free(Ad);
+  free(Bd);
+  return rc;
+}
