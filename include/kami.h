@@ -122,6 +122,20 @@ kami_status_t kami_gemm_strided_batched_host(int m, int n, int k, int64_t batch,
                                              kami_layout_t layout, const void* A, const void* B, void* C);
 kami_status_t kami_release_workspace(void);
 
+/* SpMM: C_b = A_b * B_b with block-sparse A_b (Sec. 4.6):
+ * A is stored as 16 x 16 dense blocks in block-row order (the 1D storage of
+ * Fig. 7(a), i.e. BSR): for entry b, block row i owns blocks
+ * row_ptr[b*(m/16+1) + i] .. row_ptr[b*(m/16+1) + i + 1] - 1 (indices local to
+ * the entry), block j has block column col_blk[b*max_nnzb + j] and values
+ * vals[(b*max_nnzb + j)*256 + r*16 + c] (row-major block).  B (k x n) and C
+ * (m x n) are dense, row-major, packed strided batches.  All arrays are
+ * DEVICE memory.  m, n, k multiples of 16 in [16, 256]; 16-bit types only.
+ * Absent blocks are zero; the kernel densifies A on load (HBM traffic is the
+ * nonzero blocks only) and runs the dense tcgen05 1D schedule. */
+kami_status_t kami_spmm_bsr_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                            const int* row_ptr, const int* col_blk, const void* vals,
+                                            int max_nnzb, const void* B, void* C, kami_stream_t stream);
+
 /* Block-level (on-chip-resident) mode -- the paper's block-level experiment
  * (Sec. 5.1, Sec. 5.2, Fig. 8/9): every entry is owned by one
  * team of p warps that loads A_b and B_b once and runs the CA schedule `reps`

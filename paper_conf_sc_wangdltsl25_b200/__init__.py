@@ -31,6 +31,7 @@ EXPORTS = [
     "kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
     "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
     "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level", "kami_gemm_vbatched",
+    "kami_spmm_bsr_strided_batched",
 ]
 
 
@@ -67,12 +68,13 @@ def lib() -> ctypes.CDLL:
     L.kami_gemm_strided_batched_host.argtypes = [i, i, i, i64, i, i, vp, vp, vp]
     L.kami_gemm_block_level.argtypes = [i, i, i, i64, i, i, i, i, i, vp, vp, vp, vp, st]
     L.kami_gemm_vbatched.argtypes = [i64, vp, vp, vp, i, i, i, i, i, vp, vp, vp, st]
+    L.kami_spmm_bsr_strided_batched.argtypes = [i, i, i, i64, i, vp, vp, vp, i, vp, vp, st]
     L.kami_release_workspace.argtypes = []
     L.kami_plan.argtypes = [i, i, i, i, i, i, i, ctypes.POINTER(KamiPlan)]
     d = ctypes.c_double
     L.kami_paper_cost.argtypes = [i, d, d, d, d, d, d, d, d, d, d, d, ctypes.POINTER(ctypes.c_double)]
     for f in ("kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
-              "kami_gemm_block_level", "kami_gemm_vbatched",
+              "kami_gemm_block_level", "kami_gemm_vbatched", "kami_spmm_bsr_strided_batched",
               "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost"):
         getattr(L, f).restype = ctypes.c_int
     L.kami_status_string.restype = ctypes.c_char_p
@@ -166,6 +168,17 @@ def gemm_vbatched(batch, m_arr, n_arr, k_arr, max_m, max_n, max_k, dtype, layout
     _check(lib().kami_gemm_vbatched(batch, _ptr(m_arr), _ptr(n_arr), _ptr(k_arr), max_m, max_n, max_k,
                                     _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"), _ptr(A_ptrs),
                                     _ptr(B_ptrs), _ptr(C_ptrs), _stream(stream)), "kami_gemm_vbatched")
+
+
+def spmm_bsr_strided_batched(m, n, k, batch, dtype, row_ptr, col_blk, vals, B, C, stream=None):
+    """Block-sparse A (BSR, 16x16 blocks; Sec. 4.6) times dense B.
+    row_ptr [batch, m/16+1] and col_blk [batch, max_nnzb] int32, vals
+    [batch, max_nnzb, 16, 16], B/C packed row-major -- all device tensors."""
+    max_nnzb = col_blk.shape[-1]
+    _check(lib().kami_spmm_bsr_strided_batched(m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _ptr(row_ptr),
+                                               _ptr(col_blk), _ptr(vals), max_nnzb, _ptr(B), _ptr(C),
+                                               _stream(stream)), "kami_spmm_bsr_strided_batched")
+    return C
 
 
 def gemm_single(m, n, k, dtype, layout, A, B, C, stream=None):

@@ -32,7 +32,7 @@ constexpr int kVbStages = 4;
 constexpr uint32_t kAReg = 128 * 128;       // 128 rows x 64 k (128 B)
 constexpr uint32_t kBReg = 4 * 64 * 128;    // 4 N-atoms x 64 k-rows x 128 B
 constexpr uint32_t kStage = kAReg + kBReg;  // 48 KB
-constexpr uint32_t kVbSmem = kVbStages * kStage + 1024 + 256;
+constexpr uint32_t kVbSmem = kVbStages * kStage + 1024 + 1024;
 
 struct VbParams {
   const void* const* A;
@@ -44,7 +44,22 @@ struct VbParams {
   int m, n, k;
   int mtiles;  // m-tiles per entry slot (1 or 2)
   long long batch;
+  // SpMM (Sec. 4.6): A block-sparse in BSR with 16 x 16 dense blocks
+  // (block-row order, the 1D storage of Fig. 7(a)); B, C dense and strided.
+  int bsr, max_nnzb;
+  const int* rowptr;
+  const int* colblk;
+  const uint16_t* vals;
+  const uint16_t* Bs;
+  uint16_t* Cs;
 };
+
+__device__ __forceinline__ const uint16_t* entry_B(const VbParams& p, long long e, int k, int n) {
+  return p.bsr ? p.Bs + e * (long long)k * n : reinterpret_cast<const uint16_t*>(p.B[e]);
+}
+__device__ __forceinline__ uint16_t* entry_C(const VbParams& p, long long e, int m, int n) {
+  return p.bsr ? p.Cs + e * (long long)m * n : reinterpret_cast<uint16_t*>(p.C[e]);
+}
 
 __device__ __forceinline__ void entry_dims(const VbParams& p, long long e, int& m, int& n, int& k) {
   if (p.dm) {
@@ -67,6 +82,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   uint64_t* tfull = empty + kVbStages;
   uint64_t* tempty = tfull + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  int* blk_tab = reinterpret_cast<int*>(tmem_slot + 4);  // SpMM: [8 block rows][16 block cols] -> block index
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < kVbStages; ++s) {
@@ -113,9 +129,25 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       int m, n, k;
       entry_dims(p, e, m, n, k);
       if (mt * 128 >= m) continue;
-      const uint16_t* A = reinterpret_cast<const uint16_t*>(p.A[e]);
-      const uint16_t* B = reinterpret_cast<const uint16_t*>(p.B[e]);
+      const uint16_t* A = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[e]);
+      const uint16_t* B = entry_B(p, e, k, n);
       const int kchunks = (k + 63) / 64;
+      if (p.bsr) {
+        // this m-tile's block lookup table: -1 = absent block (zero-filled)
+        ptx::named_bar_sync(3, 128);  // previous unit's copies issued: table reusable
+        blk_tab[tid] = -1;
+        ptx::named_bar_sync(3, 128);
+        const int mb = m / 16;
+        const int br0 = mt * 8, br1 = min(br0 + 8, mb);
+        const int* rp = p.rowptr + e * (mb + 1);
+        const int j0 = __ldg(rp + br0), j1 = __ldg(rp + br1);
+        for (int j = j0 + tid; j < j1; j += 128) {
+          int br = br0;
+          while (__ldg(rp + br + 1) <= j) ++br;
+          blk_tab[(br - br0) * 16 + __ldg(p.colblk + e * (long long)p.max_nnzb + j)] = j;
+        }
+        ptx::named_bar_sync(3, 128);
+      }
       const int nc8 = n / 8;  // 16-byte chunks per B row
       for (int kc = 0; kc < kchunks; ++kc, ++it) {
         const uint32_t s = it % kVbStages;
@@ -126,8 +158,15 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         for (int i = tid; i < 128 * 8; i += 128) {
           const int r = i >> 3, j = i & 7;
           const int gr = mt * 128 + r, gc = kc * 64 + j * 8;
-          const bool ok = gr < m && gc < k;
-          const uint16_t* src = ok ? A + (long long)gr * k + gc : A;
+          bool ok = gr < m && gc < k;
+          const uint16_t* src;
+          if (p.bsr) {  // densify on load: block (r/16, gc/16) or zeros
+            const int idx = ok ? blk_tab[(r >> 4) * 16 + (gc >> 4)] : -1;
+            ok = idx >= 0;
+            src = ok ? p.vals + ((e * (long long)p.max_nnzb + idx) * 256 + (r & 15) * 16 + (gc & 15)) : p.vals;
+          } else {
+            src = ok ? A + (long long)gr * k + gc : A;
+          }
           ptx::cp_async_16(sa + r * 128 + ((j ^ (r & 7)) << 4), src, ok ? 16 : 0);
         }
         // B: 64 k-rows x n/8 chunks into N-atoms of 64 columns
@@ -199,7 +238,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       ptx::tc_fence_after();
       const int row = mt * 128 + L;
       const bool warp_live = mt * 128 + sp * 32 < m;
-      uint16_t* Crow = reinterpret_cast<uint16_t*>(p.C[e]) + (long long)row * n;
+      uint16_t* Crow = entry_C(p, e, m, n) + (long long)row * n;
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * 256;
       if (warp_live) {
         for (int c0 = 0; c0 < n; c0 += 32) {
@@ -242,6 +281,30 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
 
 }  // namespace
 
+namespace {
+kami_status_t vb_launch(const VbParams& p, bool bf16, cudaStream_t stream);
+}
+
+kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf16, const int* row_ptr,
+                                   const int* col_blk, const void* vals, int max_nnzb, const void* B, void* C,
+                                   cudaStream_t stream) {
+  VbParams p;
+  memset(&p, 0, sizeof(p));
+  p.m = m;
+  p.n = n;
+  p.k = k;
+  p.mtiles = (m + 127) / 128;
+  p.batch = batch;
+  p.bsr = 1;
+  p.max_nnzb = max_nnzb;
+  p.rowptr = row_ptr;
+  p.colblk = col_blk;
+  p.vals = static_cast<const uint16_t*>(vals);
+  p.Bs = static_cast<const uint16_t*>(B);
+  p.Cs = static_cast<uint16_t*>(C);
+  return vb_launch(p, bf16, stream);
+}
+
 kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, const int* dm, const int* dn,
                              const int* dk, int max_m, const void* const* A, const void* const* B, void* const* C,
                              cudaStream_t stream) {
@@ -258,6 +321,12 @@ kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, co
   p.k = k;
   p.mtiles = (max_m + 127) / 128;
   p.batch = batch;
+  return vb_launch(p, bf16, stream);
+}
+
+namespace {
+kami_status_t vb_launch(const VbParams& p, bool bf16, cudaStream_t stream) {
+  const long long batch = p.batch;
   auto fn = bf16 ? kami_tc16_vb_kernel<true> : kami_tc16_vb_kernel<false>;
   if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kVbSmem) != cudaSuccess)
     return KAMI_ERROR_CUDA;
@@ -267,8 +336,10 @@ kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, co
   const long long units = batch * p.mtiles;
   const long long grid = units < sms ? units : sms;
   fn<<<(unsigned)grid, kVbThreads, kVbSmem, stream>>>(p);
-  set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>");
+  set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
+                        : (bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>"));
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
 }
+}  // namespace
 
 }  // namespace kami
