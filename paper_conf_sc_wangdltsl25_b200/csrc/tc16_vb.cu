@@ -13,7 +13,8 @@
 // MMA warp.
 //
 // Warps: 0-3 producer, 4 MMA issuer + TMEM allocator, 5-12 epilogue (two
-// warpgroups on alternate units; tcgen05.ld -> cvt.rn -> 16-byte st.global).
+// warpgroups on alternate units; tcgen05.ld -> cvt.rn -> padded SMEM staging
+// -> coalesced 16-byte st.global).
 // A unit is one (entry, 128-row m-tile); N = the entry's n (<= 256).
 #include <cuda.h>
 #include <cuda_runtime.h>
@@ -28,11 +29,15 @@ namespace kami {
 namespace {
 
 constexpr int kVbThreads = 416;  // 13 warps
-constexpr int kVbStages = 4;
+constexpr int kVbStages = 3;
 constexpr uint32_t kAReg = 128 * 128;       // 128 rows x 64 k (128 B)
 constexpr uint32_t kBReg = 4 * 64 * 128;    // 4 N-atoms x 64 k-rows x 128 B
 constexpr uint32_t kStage = kAReg + kBReg;  // 48 KB
-constexpr uint32_t kVbSmem = kVbStages * kStage + 1024 + 1024;
+constexpr uint32_t kCRow = 128 * 2 + 16;               // padded staging row (128 columns)
+constexpr uint32_t kCBuf = 128 * kCRow;                 // one warpgroup's C staging (34 KB)
+constexpr uint32_t kCStage = kVbStages * kStage;        // offset of the C staging buffers
+constexpr uint32_t kBarOff = kCStage + 2 * kCBuf;       // barriers + tables
+constexpr uint32_t kVbSmem = kBarOff + 1024 + 1024;
 
 struct VbParams {
   const void* const* A;
@@ -77,7 +82,7 @@ template <bool kBF16>
 __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __grid_constant__ VbParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kVbStages * kStage);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kBarOff);
   uint64_t* empty = full + kVbStages;
   uint64_t* tfull = empty + kVbStages;
   uint64_t* tempty = tfull + 2;
@@ -236,37 +241,52 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       if (!mine) continue;
       ptx::mbar_wait(&tfull[a], ((acc_it - 1) >> 1) & 1);
       ptx::tc_fence_after();
-      const int row = mt * 128 + L;
-      const bool warp_live = mt * 128 + sp * 32 < m;
-      uint16_t* Crow = entry_C(p, e, m, n) + (long long)row * n;
+      // Stage the tile through padded shared memory (row stride 272 B: rows
+      // land on different banks, conflict-free) in 128-column halves, then
+      // copy out with coalesced 16-byte stores (a warp writes whole rows).
+      const int rows = min(128, m - mt * 128);
+      const bool warp_live = sp * 32 < rows;
+      uint16_t* Cbase = entry_C(p, e, m, n) + (long long)mt * 128 * n;
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * 256;
-      if (warp_live) {
-        for (int c0 = 0; c0 < n; c0 += 32) {
-          uint32_t v[32];
-          if (n - c0 >= 32) ptx::tmem_ld_32x32b_x32(t_row + c0, v);
-          else ptx::tmem_ld_32x32b_x16(t_row + c0, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
-          ptx::tmem_wait_ld();
-          if (row < m) {
+      const uint32_t cst = smem_base + kCStage + wg * kCBuf;
+      for (int h0 = 0; h0 < n; h0 += 128) {
+        const int hw = min(128, n - h0);
+        if (warp_live) {
+          for (int c0 = 0; c0 < hw; c0 += 32) {
+            uint32_t v[32];
+            if (hw - c0 >= 32) ptx::tmem_ld_32x32b_x32(t_row + h0 + c0, v);
+            else ptx::tmem_ld_32x32b_x16(t_row + h0 + c0, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
+            ptx::tmem_wait_ld();
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
-              if (c0 + 8 * q < n) {
-                uint4 w;
+              if (c0 + 8 * q < hw) {
+                uint32_t w0, w1, w2, w3;
                 if (kBF16) {
-                  w.x = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
-                  w.y = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
-                  w.z = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
-                  w.w = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
+                  w0 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
+                  w1 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
+                  w2 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
+                  w3 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
                 } else {
-                  w.x = ptx::pack_f16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
-                  w.y = ptx::pack_f16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
-                  w.z = ptx::pack_f16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
-                  w.w = ptx::pack_f16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
+                  w0 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
+                  w1 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
+                  w2 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
+                  w3 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
                 }
-                ptx::st_global_v4(Crow + c0 + 8 * q, w);
+                ptx::st_shared_v4(cst + L * kCRow + (c0 + 8 * q) * 2, w0, w1, w2, w3);
               }
             }
           }
         }
+        ptx::named_bar_sync(1 + wg, 128);
+        // copy-out: chunk index i -> (row i / cpr, 16-byte chunk i % cpr)
+        const int cpr = hw / 8;
+        for (int i = L; i < rows * cpr; i += 128) {
+          const int r = i / cpr, c = i - r * cpr;
+          uint32_t x0, x1, x2, x3;
+          ptx::ld_shared_v4(cst + r * kCRow + c * 16, x0, x1, x2, x3);
+          ptx::st_global_v4(Cbase + (long long)r * n + h0 + c * 8, make_uint4(x0, x1, x2, x3));
+        }
+        ptx::named_bar_sync(1 + wg, 128);  // staging buffer reusable
       }
       ptx::tc_fence_before();
       __syncwarp();

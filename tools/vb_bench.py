@@ -25,10 +25,19 @@ ap.add_argument("--dtype", default="f16")
 ap.add_argument("--shape", default="64x64x64")
 ap.add_argument("--batch", type=int, default=65536)
 ap.add_argument("--reps", type=int, default=10)
+ap.add_argument("--density", type=float, default=0.5)
 a = ap.parse_args()
 hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
     os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
-if a.mode == "ptr":
+if a.mode == "spmm":
+    m, n, k = (int(x) for x in a.shape.split("x"))
+    rp, cb, v, B = ki.bsr_operands(m, n, k, a.batch, a.dtype, density=a.density, device="cuda")
+    C = torch.empty(a.batch * m * n, dtype=B.dtype, device="cuda")
+    run = lambda: kami.spmm_bsr_strided_batched(m, n, k, a.batch, a.dtype, rp, cb, v, B, C)  # noqa: E731
+    nnzb = float(rp[:, -1].sum())
+    flops = 2.0 * nnzb * 256 * n  # useful (sparse) flops
+    byts = nnzb * (512 + 4) + a.batch * ((m // 16 + 1) * 4 + (k * n + m * n) * 2)
+elif a.mode == "ptr":
     m, n, k = (int(x) for x in a.shape.split("x"))
     A, B = ki.operands(m, n, k, a.batch, a.dtype, "unif", device="cuda")
     C = torch.empty(a.batch * m * n, dtype=A.dtype, device="cuda")
