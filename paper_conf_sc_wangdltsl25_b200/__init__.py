@@ -18,7 +18,8 @@ __all__ = [
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-SO_PATH = os.path.join(_HERE, "libkami.so")
+# KAMI_LIB may point at another build of the same library (A/B experiments)
+SO_PATH = os.environ.get("KAMI_LIB") or os.path.join(_HERE, "libkami.so")
 
 DTYPE = {"f16": 0, "bf16": 1, "f64": 2}
 LAYOUT = {"row": 0, "col": 1}

@@ -79,8 +79,8 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
                        void* const* Ca, cudaStream_t stream) {
   // 16-bit pointer arrays: the LDG-fed tcgen05 kernel covers the whole size grid
   if (Ca && is16(dtype) && algo == KAMI_ALGO_AUTO)
-    return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, rp.m, rp.n, rp.k, nullptr, nullptr, nullptr, rp.m, rp.Aa,
-                          rp.Ba, Ca, stream);
+    return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, rp.m, rp.n, rp.k, nullptr, nullptr, nullptr, rp.m, rp.n,
+                          rp.Aa, rp.Ba, Ca, stream);
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
@@ -152,8 +152,8 @@ kami_status_t kami_gemm_vbatched(int64_t batch, const int* m_array, const int* n
   // column-major: C^T = B^T A^T per entry -> swap m<->n and A<->B
   const bool col = layout == KAMI_COL_MAJOR;
   return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, 0, 0, 0, col ? n_array : m_array, col ? m_array : n_array,
-                        k_array, col ? max_n : max_m, col ? B_array : A_array, col ? A_array : B_array, C_array,
-                        reinterpret_cast<cudaStream_t>(stream));
+                        k_array, col ? max_n : max_m, col ? max_m : max_n, col ? B_array : A_array,
+                        col ? A_array : B_array, C_array, reinterpret_cast<cudaStream_t>(stream));
 }
 
 kami_status_t kami_spmm_bsr_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,

@@ -51,8 +51,8 @@ kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* 
 // ------------------------- 16-bit pointer-array / variable-size (tc16_vb.cu)
 // dm/dn/dk: device arrays of per-entry sizes, or nullptr for uniform m, n, k.
 kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, const int* dm, const int* dn,
-                             const int* dk, int max_m, const void* const* A, const void* const* B, void* const* C,
-                             cudaStream_t stream);
+                             const int* dk, int max_m, int max_n, const void* const* A, const void* const* B,
+                             void* const* C, cudaStream_t stream);
 
 // SpMM: block-sparse A (BSR, 16x16 blocks) x dense B on tcgen05 (densify on load)
 kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf16, const int* row_ptr,

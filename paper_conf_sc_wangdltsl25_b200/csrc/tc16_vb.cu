@@ -1,21 +1,22 @@
 // tc16_vb.cu -- FP16/BF16 batched GEMM on tcgen05 for POINTER-ARRAY and
 // VARIABLE-SIZE batches ("supports various matrix orders in
-// a batch").
+// a batch") and for SpMM with block-sparse A (f3, Sec. 4.6).
 //
 // Same KAMI-1D mapping as tc16.cu (4 sub-partition tensor cores, C_i in TMEM,
-// B broadcast through shared memory), but the operands cannot be described by
-// one TMA tensor map (every entry has its own pointer and possibly its own
-// m, n, k), so a producer warpgroup performs the paper's GMem2Reg + Reg2SMem
-// itself: coalesced 16-byte cp.async (LDGSTS) copies of A and B rows straight
-// into the UMMA canonical layouts (128-byte swizzle, K-major A, N-major B),
-// zero-filling k beyond the entry's order; once a stage's copy group has
-// landed, a generic->async proxy fence and an mbarrier arrive hand it to the
-// MMA warp.
+// B broadcast through shared memory, G = min(128/m, 256/n) same-size entries
+// packed block-diagonally per 128-lane MMA tile), but the operands cannot be
+// described by one TMA tensor map (every entry has its own pointer, possibly
+// its own m, n, k, or a sparse A), so a producer warpgroup performs the
+// paper's GMem2Reg + Reg2SMem itself: coalesced 16-byte cp.async (LDGSTS)
+// copies of A and B rows straight into the UMMA canonical layouts (128-byte
+// swizzle, K-major A, N-major B), zero-filling k beyond the entry's order
+// (SpMM: absent 16x16 blocks of A are zero-filled -- A is densified on load,
+// only its nonzero blocks cross HBM).  Once a stage's copy group has landed, a
+// generic->async proxy fence and an mbarrier arrive hand it to the MMA warp.
 //
 // Warps: 0-3 producer, 4 MMA issuer + TMEM allocator, 5-12 epilogue (two
 // warpgroups on alternate units; tcgen05.ld -> cvt.rn -> padded SMEM staging
-// -> coalesced 16-byte st.global).
-// A unit is one (entry, 128-row m-tile); N = the entry's n (<= 256).
+// -> coalesced 16-byte st.global).  A unit is G entries x one 128-row m-tile.
 #include <cuda.h>
 #include <cuda_runtime.h>
 
@@ -29,15 +30,12 @@ namespace kami {
 namespace {
 
 constexpr int kVbThreads = 416;  // 13 warps
-constexpr int kVbStages = 3;
-constexpr uint32_t kAReg = 128 * 128;       // 128 rows x 64 k (128 B)
-constexpr uint32_t kBReg = 4 * 64 * 128;    // 4 N-atoms x 64 k-rows x 128 B
-constexpr uint32_t kStage = kAReg + kBReg;  // 48 KB
-constexpr uint32_t kCRow = 128 * 2 + 16;               // padded staging row (128 columns)
-constexpr uint32_t kCBuf = 128 * kCRow;                 // one warpgroup's C staging (34 KB)
-constexpr uint32_t kCStage = kVbStages * kStage;        // offset of the C staging buffers
-constexpr uint32_t kBarOff = kCStage + 2 * kCBuf;       // barriers + tables
-constexpr uint32_t kVbSmem = kBarOff + 1024 + 1024;
+constexpr int kMaxStages = 8;
+constexpr int kMaxAcc = 4;
+constexpr uint32_t kAReg = 128 * 128;                 // 128 rows x 64 k (128 B)
+constexpr uint32_t kCRow = 128 * 2 + 16;              // padded staging row (128 columns)
+constexpr uint32_t kCBuf = 128 * kCRow;               // one warpgroup's C staging (34 KB)
+constexpr int kSmemLimit = 232448;
 
 struct VbParams {
   const void* const* A;
@@ -47,8 +45,12 @@ struct VbParams {
   const int* dn;
   const int* dk;
   int m, n, k;
-  int mtiles;  // m-tiles per entry slot (1 or 2)
-  long long batch;
+  int G;       // entries per unit (block-diagonal packing; 1 for mixed sizes)
+  int mtiles;  // m-tiles per unit slot
+  long long batch, units;
+  int stages;
+  uint32_t stage_bytes, c_off, bar_off;
+  int acc_cols, acc_bufs;
   // SpMM (Sec. 4.6): A block-sparse in BSR with 16 x 16 dense blocks
   // (block-row order, the 1D storage of Fig. 7(a)); B, C dense and strided.
   int bsr, max_nnzb;
@@ -65,7 +67,6 @@ __device__ __forceinline__ const uint16_t* entry_B(const VbParams& p, long long 
 __device__ __forceinline__ uint16_t* entry_C(const VbParams& p, long long e, int m, int n) {
   return p.bsr ? p.Cs + e * (long long)m * n : reinterpret_cast<uint16_t*>(p.C[e]);
 }
-
 __device__ __forceinline__ void entry_dims(const VbParams& p, long long e, int& m, int& n, int& k) {
   if (p.dm) {
     m = __ldg(p.dm + e);
@@ -77,138 +78,182 @@ __device__ __forceinline__ void entry_dims(const VbParams& p, long long e, int& 
     k = p.k;
   }
 }
+// unit -> first entry, m-tile, live entries, sizes
+struct Unit {
+  long long e0;
+  int mt, ng, m, n, k;
+};
+__device__ __forceinline__ bool unit_of(const VbParams& p, long long u, Unit& U) {
+  const long long grp = u / p.mtiles;
+  U.mt = (int)(u - grp * p.mtiles);
+  U.e0 = grp * p.G;
+  const long long left = p.batch - U.e0;
+  U.ng = left < p.G ? (int)left : p.G;
+  entry_dims(p, U.e0, U.m, U.n, U.k);
+  return U.mt * 128 < U.m;  // mixed sizes: an entry may have fewer m-tiles
+}
+
+__device__ __forceinline__ void cp_async_wait_n(int n) {
+  switch (n) {
+    case 0: ptx::cp_async_wait<0>(); break;
+    case 1: ptx::cp_async_wait<1>(); break;
+    case 2: ptx::cp_async_wait<2>(); break;
+    case 3: ptx::cp_async_wait<3>(); break;
+    case 4: ptx::cp_async_wait<4>(); break;
+    case 5: ptx::cp_async_wait<5>(); break;
+    default: ptx::cp_async_wait<6>(); break;
+  }
+}
 
 template <bool kBF16>
 __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __grid_constant__ VbParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kBarOff);
-  uint64_t* empty = full + kVbStages;
-  uint64_t* tfull = empty + kVbStages;
-  uint64_t* tempty = tfull + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
-  int* blk_tab = reinterpret_cast<int*>(tmem_slot + 4);  // SpMM: [8 block rows][16 block cols] -> block index
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + p.bar_off);
+  uint64_t* empty = full + kMaxStages;
+  uint64_t* tfull = empty + kMaxStages;
+  uint64_t* tempty = tfull + kMaxAcc;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + kMaxAcc);
+  int* blk_tab = reinterpret_cast<int*>(tmem_slot + 4);  // SpMM: [8 tile block rows][16 block cols]
+  // per-unit entry pointer tables (loaded once per unit, not once per copy)
+  const uint16_t** a_tab = reinterpret_cast<const uint16_t**>(blk_tab + 128);
+  const uint16_t** b_tab = a_tab + 8;
+  uint16_t** c_tab = reinterpret_cast<uint16_t**>(b_tab + 8);  // [2 warpgroups][8]
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
-    for (int s = 0; s < kVbStages; ++s) {
+    for (int s = 0; s < p.stages; ++s) {
       ptx::mbar_init(&full[s], 128);
       ptx::mbar_init(&empty[s], 1);
     }
-    for (int a = 0; a < 2; ++a) {
+    for (int a = 0; a < p.acc_bufs; ++a) {
       ptx::mbar_init(&tfull[a], 1);
       ptx::mbar_init(&tempty[a], 4);
     }
     ptx::fence_mbar_init();
   }
-  if (warp == 4) ptx::tmem_alloc(tmem_slot, 512);
+  if (warp == 4) ptx::tmem_alloc(tmem_slot, p.acc_cols * p.acc_bufs);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   const uint32_t smem_base = ptx::smem_u32(smem);
-  const long long units = p.batch * p.mtiles;
 
   if (warp < 4) {
     // ------------------------------------------------ producer warpgroup
-    // cp.async (LDGSTS) straight into the swizzled stage buffers, zero-filled
-    // outside the entry; a stage is handed to the MMA warp (fence.proxy.async
-    // + mbarrier arrive) once its copy group has landed, kLag stages later, so
+    // cp.async straight into the swizzled stage buffers; a stage is handed to
+    // the MMA warp once its copy group has landed, `lag` stages later, so
     // several stages stream concurrently without register staging.
-    constexpr int kLag = kVbStages - 1;
+    const int lag = p.stages - 1 < 6 ? p.stages - 1 : 6;
     const int tid = threadIdx.x;  // 0..127
     uint32_t it = 0, handed = 0;
     auto hand_over = [&](int pending) {
-      // copies of stage `handed` are complete when at most `pending` groups remain
-      static_assert(kLag <= 3, "wait_group depth");
-      if (pending >= 3) ptx::cp_async_wait<3>();
-      else if (pending == 2) ptx::cp_async_wait<2>();
-      else if (pending == 1) ptx::cp_async_wait<1>();
-      else ptx::cp_async_wait<0>();
+      cp_async_wait_n(pending);  // the oldest un-handed group has landed
       ptx::fence_proxy_async_smem();
-      ptx::mbar_arrive(&full[handed % kVbStages]);
+      ptx::mbar_arrive(&full[handed % p.stages]);
       ++handed;
     };
-    for (long long u = blockIdx.x; u < units; u += gridDim.x) {
-      const long long e = u / p.mtiles;
-      const int mt = (int)(u - e * p.mtiles);
-      int m, n, k;
-      entry_dims(p, e, m, n, k);
-      if (mt * 128 >= m) continue;
-      const uint16_t* A = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[e]);
-      const uint16_t* B = entry_B(p, e, k, n);
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
+      Unit U;
+      if (!unit_of(p, u, U)) continue;
+      const int m = U.m, n = U.n, k = U.k, G = p.G;
       const int kchunks = (k + 63) / 64;
+      const int rows = G > 1 ? U.ng * m : min(128, m - U.mt * 128);  // live tile rows
+      ptx::named_bar_sync(3, 128);  // previous unit's items issued: tables reusable
+      if (tid < U.ng) {
+        a_tab[tid] = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[U.e0 + tid]);
+        b_tab[tid] = entry_B(p, U.e0 + tid, k, n);
+      }
+      if (p.bsr) blk_tab[tid] = -1;
+      ptx::named_bar_sync(3, 128);
       if (p.bsr) {
-        // this m-tile's block lookup table: -1 = absent block (zero-filled)
-        ptx::named_bar_sync(3, 128);  // previous unit's copies issued: table reusable
-        blk_tab[tid] = -1;
-        ptx::named_bar_sync(3, 128);
+        // block lookup table of this tile: tile block row -> global block slot
         const int mb = m / 16;
-        const int br0 = mt * 8, br1 = min(br0 + 8, mb);
-        const int* rp = p.rowptr + e * (mb + 1);
-        const int j0 = __ldg(rp + br0), j1 = __ldg(rp + br1);
-        for (int j = j0 + tid; j < j1; j += 128) {
-          int br = br0;
-          while (__ldg(rp + br + 1) <= j) ++br;
-          blk_tab[(br - br0) * 16 + __ldg(p.colblk + e * (long long)p.max_nnzb + j)] = j;
+        for (int g = 0; g < U.ng; ++g) {
+          const long long e = U.e0 + g;
+          const int br0 = U.mt * 8, br1 = min(br0 + 8, mb);
+          const int tb0 = g * (m / 16) - br0;  // tile block row of the entry's block row 0
+          const int* rp = p.rowptr + e * (mb + 1);
+          const int j0 = __ldg(rp + br0), j1 = __ldg(rp + br1);
+          for (int j = j0 + tid; j < j1; j += 128) {
+            int br = br0;
+            while (__ldg(rp + br + 1) <= j) ++br;
+            blk_tab[(tb0 + br) * 16 + __ldg(p.colblk + e * (long long)p.max_nnzb + j)] =
+                (int)(e * p.max_nnzb + j);
+          }
         }
         ptx::named_bar_sync(3, 128);
       }
-      const int nc8 = n / 8;  // 16-byte chunks per B row
+      const int nc8 = n / 8;  // 16-byte chunks per B row of one entry
+      const int nc8_shift = (nc8 & (nc8 - 1)) == 0 ? __ffs(nc8) - 1 : -1;  // power-of-two fast path
       for (int kc = 0; kc < kchunks; ++kc, ++it) {
-        const uint32_t s = it % kVbStages;
-        ptx::mbar_wait(&empty[s], ((it / kVbStages) & 1) ^ 1);
-        const uint32_t sa = smem_base + s * kStage, sb = sa + kAReg;
-        // A: 128 rows x 8 chunks; a warp covers 4 whole 128-byte row segments
-#pragma unroll 4
-        for (int i = tid; i < 128 * 8; i += 128) {
+        const uint32_t s = it % p.stages;
+        ptx::mbar_wait(&empty[s], ((it / p.stages) & 1) ^ 1);
+        const uint32_t sa = smem_base + s * p.stage_bytes, sb = sa + kAReg;
+        // A: live rows x 8 chunks of 16 B; a warp covers 4 whole row segments
+        for (int i = tid; i < rows * 8; i += 128) {
           const int r = i >> 3, j = i & 7;
-          const int gr = mt * 128 + r, gc = kc * 64 + j * 8;
-          bool ok = gr < m && gc < k;
+          const int g = G > 1 ? r / m : 0;
+          const int er = G > 1 ? r - g * m : U.mt * 128 + r;  // row inside the entry
+          const int gc = kc * 64 + j * 8;
+          bool ok = gc < k;
           const uint16_t* src;
           if (p.bsr) {  // densify on load: block (r/16, gc/16) or zeros
-            const int idx = ok ? blk_tab[(r >> 4) * 16 + (gc >> 4)] : -1;
-            ok = idx >= 0;
-            src = ok ? p.vals + ((e * (long long)p.max_nnzb + idx) * 256 + (r & 15) * 16 + (gc & 15)) : p.vals;
+            const int slot = ok ? blk_tab[(r >> 4) * 16 + (gc >> 4)] : -1;
+            ok = slot >= 0;
+            src = ok ? p.vals + ((long long)slot * 256 + (er & 15) * 16 + (gc & 15)) : p.vals;
           } else {
-            src = ok ? A + (long long)gr * k + gc : A;
+            const uint16_t* A = a_tab[g];
+            src = ok ? A + (long long)er * k + gc : A;
           }
           ptx::cp_async_16(sa + r * 128 + ((j ^ (r & 7)) << 4), src, ok ? 16 : 0);
         }
-        // B: 64 k-rows x n/8 chunks into N-atoms of 64 columns
-        for (int i = tid; i < 64 * nc8; i += 128) {
-          const int kr = i / nc8, j = i - kr * nc8;
+        // B: per entry 64 k-rows x n/8 chunks at columns [g n, g n + n) of the
+        // N-major tile (atoms of 64 columns x 64 k-rows)
+        const int per = 64 * nc8;
+        for (int i = tid; i < U.ng * per; i += 128) {
+          int g, kr, j;
+          if (nc8_shift >= 0) {
+            const int row = i >> nc8_shift;  // = g * 64 + kr
+            g = row >> 6;
+            kr = row & 63;
+            j = i & (nc8 - 1);
+          } else {
+            g = i / per;
+            const int rem = i - g * per;
+            kr = rem / nc8;
+            j = rem - kr * nc8;
+          }
           const int gk = kc * 64 + kr;
           const bool ok = gk < k;
+          const uint16_t* B = b_tab[g];
           const uint16_t* src = ok ? B + (long long)gk * n + j * 8 : B;
-          ptx::cp_async_16(sb + (j >> 3) * 8192 + kr * 128 + (((j & 7) ^ (kr & 7)) << 4), src, ok ? 16 : 0);
+          const int cc = g * nc8 + j;  // 16-byte chunk column in the tile
+          ptx::cp_async_16(sb + (cc >> 3) * 8192 + kr * 128 + (((cc & 7) ^ (kr & 7)) << 4), src, ok ? 16 : 0);
         }
         ptx::cp_async_commit();
-        if (it + 1 - handed > (uint32_t)kLag) hand_over(kLag);
+        if ((int)(it + 1 - handed) > lag) hand_over(lag);
       }
     }
     while (handed < it) hand_over((int)(it - handed - 1));
   } else if (warp == 4) {
     // ------------------------------------------------------------- MMA
     uint32_t it = 0, acc_it = 0;
-    for (long long u = blockIdx.x; u < units; u += gridDim.x) {
-      const long long e = u / p.mtiles;
-      const int mt = (int)(u - e * p.mtiles);
-      int m, n, k;
-      entry_dims(p, e, m, n, k);
-      if (mt * 128 >= m) continue;
-      const uint32_t a = acc_it & 1;
-      ptx::mbar_wait(&tempty[a], ((acc_it >> 1) & 1) ^ 1);
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
+      Unit U;
+      if (!unit_of(p, u, U)) continue;
+      const uint32_t a = acc_it % p.acc_bufs;
+      ptx::mbar_wait(&tempty[a], ((acc_it / p.acc_bufs) & 1) ^ 1);
       ptx::tc_fence_after();
-      const uint32_t d_tmem = tmem_base + a * 256;
-      const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, n, 0, 1);
-      const int kpad = (k + 15) / 16 * 16;
-      const int kchunks = (k + 63) / 64;
+      const uint32_t d_tmem = tmem_base + a * p.acc_cols;
+      const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, p.G * U.n, 0, 1);
+      const int kpad = (U.k + 15) / 16 * 16;
+      const int kchunks = (U.k + 63) / 64;
       for (int kc = 0; kc < kchunks; ++kc, ++it) {
-        const uint32_t s = it % kVbStages;
-        ptx::mbar_wait(&full[s], (it / kVbStages) & 1);
+        const uint32_t s = it % p.stages;
+        ptx::mbar_wait(&full[s], (it / p.stages) & 1);
         ptx::tc_fence_after();
         if (lane == 0) {
-          const uint32_t sa = smem_base + s * kStage, sb = sa + kAReg;
+          const uint32_t sa = smem_base + s * p.stage_bytes, sb = sa + kAReg;
           const int nsteps = (kpad - kc * 64) >= 64 ? 4 : (kpad - kc * 64) / 16;
           for (int ks = 0; ks < nsteps; ++ks) {
             const uint64_t adesc = ptx::make_smem_desc(sa + ks * 32, 16, 1024, 2);
@@ -228,63 +273,71 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     const int wg = (warp - 5) >> 2;
     const int sp = warp & 3;
     const int L = sp * 32 + lane;
+    const uint32_t cst = smem_base + p.c_off + wg * kCBuf;
     uint32_t acc_it = 0;
-    for (long long u = blockIdx.x; u < units; u += gridDim.x) {
-      const long long e = u / p.mtiles;
-      const int mt = (int)(u - e * p.mtiles);
-      int m, n, k;
-      entry_dims(p, e, m, n, k);
-      if (mt * 128 >= m) continue;
-      const uint32_t a = acc_it & 1;
-      const bool mine = (int)(acc_it & 1) == wg;  // accumulator a is drained by warpgroup a
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
+      Unit U;
+      if (!unit_of(p, u, U)) continue;
+      const uint32_t a = acc_it % p.acc_bufs;
+      const uint32_t aph = (acc_it / p.acc_bufs) & 1;
+      const bool mine = (int)(acc_it & 1) == wg;  // warpgroups take alternate units
       ++acc_it;
       if (!mine) continue;
-      ptx::mbar_wait(&tfull[a], ((acc_it - 1) >> 1) & 1);
-      ptx::tc_fence_after();
-      // Stage the tile through padded shared memory (row stride 272 B: rows
-      // land on different banks, conflict-free) in 128-column halves, then
-      // copy out with coalesced 16-byte stores (a warp writes whole rows).
-      const int rows = min(128, m - mt * 128);
+      const int m = U.m, n = U.n, G = p.G;
+      const int rows = G > 1 ? U.ng * m : min(128, m - U.mt * 128);
+      // lanes -> (entry g, row); the warp's lanes may span several entries
+      const int g = G > 1 ? L / m : 0;
+      const bool row_ok = L < rows;
+      const int glo = G > 1 ? (sp * 32) / m : 0;
+      const int ghi = G > 1 ? min(U.ng - 1, (sp * 32 + 31) / m) : 0;
       const bool warp_live = sp * 32 < rows;
-      uint16_t* Cbase = entry_C(p, e, m, n) + (long long)mt * 128 * n;
-      const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * 256;
-      const uint32_t cst = smem_base + kCStage + wg * kCBuf;
+      if (L < U.ng) c_tab[wg * 8 + L] = entry_C(p, U.e0 + L, m, n);  // read after the staging barrier
+      ptx::mbar_wait(&tfull[a], aph);
+      ptx::tc_fence_after();
+      const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
       for (int h0 = 0; h0 < n; h0 += 128) {
         const int hw = min(128, n - h0);
         if (warp_live) {
-          for (int c0 = 0; c0 < hw; c0 += 32) {
-            uint32_t v[32];
-            if (hw - c0 >= 32) ptx::tmem_ld_32x32b_x32(t_row + h0 + c0, v);
-            else ptx::tmem_ld_32x32b_x16(t_row + h0 + c0, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
-            ptx::tmem_wait_ld();
+          for (int gg = glo; gg <= ghi; ++gg) {  // warp-uniform
+            for (int c0 = 0; c0 < hw; c0 += 32) {
+              uint32_t v[32];
+              const uint32_t col = (uint32_t)(gg * n + h0 + c0);
+              if (hw - c0 >= 32) ptx::tmem_ld_32x32b_x32(t_row + col, v);
+              else ptx::tmem_ld_32x32b_x16(t_row + col, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
+              ptx::tmem_wait_ld();
+              if (row_ok && g == gg) {
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              if (c0 + 8 * q < hw) {
-                uint32_t w0, w1, w2, w3;
-                if (kBF16) {
-                  w0 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
-                  w1 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
-                  w2 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
-                  w3 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
-                } else {
-                  w0 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
-                  w1 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
-                  w2 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
-                  w3 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
+                for (int q = 0; q < 4; ++q) {
+                  if (c0 + 8 * q < hw) {
+                    uint32_t w0, w1, w2, w3;
+                    if (kBF16) {
+                      w0 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
+                      w1 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
+                      w2 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
+                      w3 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
+                    } else {
+                      w0 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
+                      w1 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
+                      w2 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
+                      w3 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
+                    }
+                    ptx::st_shared_v4(cst + L * kCRow + (c0 + 8 * q) * 2, w0, w1, w2, w3);
+                  }
                 }
-                ptx::st_shared_v4(cst + L * kCRow + (c0 + 8 * q) * 2, w0, w1, w2, w3);
               }
             }
           }
         }
         ptx::named_bar_sync(1 + wg, 128);
-        // copy-out: chunk index i -> (row i / cpr, 16-byte chunk i % cpr)
+        // copy-out: chunk index i -> (tile row i / cpr, 16-byte chunk i % cpr)
         const int cpr = hw / 8;
         for (int i = L; i < rows * cpr; i += 128) {
           const int r = i / cpr, c = i - r * cpr;
+          const int ge = G > 1 ? r / m : 0;
+          const int er = G > 1 ? r - ge * m : U.mt * 128 + r;
           uint32_t x0, x1, x2, x3;
           ptx::ld_shared_v4(cst + r * kCRow + c * 16, x0, x1, x2, x3);
-          ptx::st_global_v4(Cbase + (long long)r * n + h0 + c * 8, make_uint4(x0, x1, x2, x3));
+          ptx::st_global_v4(c_tab[wg * 8 + ge] + (long long)er * n + h0 + c * 8, make_uint4(x0, x1, x2, x3));
         }
         ptx::named_bar_sync(1 + wg, 128);  // staging buffer reusable
       }
@@ -296,14 +349,53 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
-  if (warp == 4) ptx::tmem_dealloc(tmem_base, 512);
+  if (warp == 4) ptx::tmem_dealloc(tmem_base, p.acc_cols * p.acc_bufs);
+}
+
+int pow2_ceil(int x) {
+  int q = 32;
+  while (q < x) q <<= 1;
+  return q;
+}
+
+// n_max: widest B tile (columns) a unit can need; G entries per unit
+kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream_t stream) {
+  const int N = p.G * n_max;
+  const uint32_t b_region = (uint32_t)((N + 63) / 64) * 8192;
+  p.stage_bytes = kAReg + b_region;
+  p.acc_cols = pow2_ceil(N);
+  p.acc_bufs = 512 / p.acc_cols < kMaxAcc ? 512 / p.acc_cols : kMaxAcc;
+  const int budget = kSmemLimit - 1024 /*align*/ - 2048 /*barriers, tables*/ - 2 * (int)kCBuf;
+  int st = budget / (int)p.stage_bytes;
+  if (st > kMaxStages) st = kMaxStages;
+  if (st < 2) return KAMI_ERROR_NOT_SUPPORTED;
+  p.stages = st;
+  p.c_off = st * p.stage_bytes;
+  p.bar_off = p.c_off + 2 * kCBuf;
+  p.mtiles = p.G > 1 ? 1 : (max_m + 127) / 128;
+  p.units = ((p.batch + p.G - 1) / p.G) * p.mtiles;
+  const uint32_t smem = p.bar_off + 2048 + 1024;
+  auto fn = bf16 ? kami_tc16_vb_kernel<true> : kami_tc16_vb_kernel<false>;
+  if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
+    return KAMI_ERROR_CUDA;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long grid = p.units < sms ? p.units : sms;
+  fn<<<(unsigned)grid, kVbThreads, smem, stream>>>(p);
+  set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
+                        : (bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>"));
+  return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+}
+
+int packing(int m, int n) {  // entries per 128-lane tile (same rule as tc16.cu)
+  if (m > 128) return 1;
+  const int g1 = 128 / m, g2 = 256 / n;
+  const int g = g1 < g2 ? g1 : g2;
+  return g < 1 ? 1 : g;
 }
 
 }  // namespace
-
-namespace {
-kami_status_t vb_launch(const VbParams& p, bool bf16, cudaStream_t stream);
-}
 
 kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf16, const int* row_ptr,
                                    const int* col_blk, const void* vals, int max_nnzb, const void* B, void* C,
@@ -313,8 +405,8 @@ kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf
   p.m = m;
   p.n = n;
   p.k = k;
-  p.mtiles = (m + 127) / 128;
   p.batch = batch;
+  p.G = packing(m, n);
   p.bsr = 1;
   p.max_nnzb = max_nnzb;
   p.rowptr = row_ptr;
@@ -322,12 +414,12 @@ kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf
   p.vals = static_cast<const uint16_t*>(vals);
   p.Bs = static_cast<const uint16_t*>(B);
   p.Cs = static_cast<uint16_t*>(C);
-  return vb_launch(p, bf16, stream);
+  return vb_launch(p, bf16, n, m, stream);
 }
 
 kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, const int* dm, const int* dn,
-                             const int* dk, int max_m, const void* const* A, const void* const* B, void* const* C,
-                             cudaStream_t stream) {
+                             const int* dk, int max_m, int max_n, const void* const* A, const void* const* B,
+                             void* const* C, cudaStream_t stream) {
   VbParams p;
   memset(&p, 0, sizeof(p));
   p.A = A;
@@ -339,27 +431,9 @@ kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, co
   p.m = m;
   p.n = n;
   p.k = k;
-  p.mtiles = (max_m + 127) / 128;
   p.batch = batch;
-  return vb_launch(p, bf16, stream);
+  p.G = dm ? 1 : packing(m, n);  // mixed sizes cannot share a tile
+  return vb_launch(p, bf16, dm ? max_n : n, dm ? max_m : m, stream);
 }
-
-namespace {
-kami_status_t vb_launch(const VbParams& p, bool bf16, cudaStream_t stream) {
-  const long long batch = p.batch;
-  auto fn = bf16 ? kami_tc16_vb_kernel<true> : kami_tc16_vb_kernel<false>;
-  if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kVbSmem) != cudaSuccess)
-    return KAMI_ERROR_CUDA;
-  int dev = 0, sms = 148;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const long long units = batch * p.mtiles;
-  const long long grid = units < sms ? units : sms;
-  fn<<<(unsigned)grid, kVbThreads, kVbSmem, stream>>>(p);
-  set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
-                        : (bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>"));
-  return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
-}
-}  // namespace
 
 }  // namespace kami
