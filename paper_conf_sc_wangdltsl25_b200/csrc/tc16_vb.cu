@@ -189,46 +189,63 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         const uint32_t s = it % p.stages;
         ptx::mbar_wait(&empty[s], ((it / p.stages) & 1) ^ 1);
         const uint32_t sa = smem_base + s * p.stage_bytes, sb = sa + kAReg;
-        // A: live rows x 8 chunks of 16 B; a warp covers 4 whole row segments
-        for (int i = tid; i < rows * 8; i += 128) {
-          const int r = i >> 3, j = i & 7;
-          const int g = G > 1 ? r / m : 0;
-          const int er = G > 1 ? r - g * m : U.mt * 128 + r;  // row inside the entry
+        // A: thread = (16-byte chunk j, row r0 + 16 q): a warp covers 4 whole
+        // 128-byte row segments, the swizzle phase (r & 7) is fixed per thread
+        // and the addresses advance by constant strides.
+        {
+          const int j = tid & 7, r0 = tid >> 3;
           const int gc = kc * 64 + j * 8;
-          bool ok = gc < k;
-          const uint16_t* src;
-          if (p.bsr) {  // densify on load: block (r/16, gc/16) or zeros
-            const int slot = ok ? blk_tab[(r >> 4) * 16 + (gc >> 4)] : -1;
-            ok = slot >= 0;
-            src = ok ? p.vals + ((long long)slot * 256 + (er & 15) * 16 + (gc & 15)) : p.vals;
-          } else {
-            const uint16_t* A = a_tab[g];
-            src = ok ? A + (long long)er * k + gc : A;
+          const bool col_ok = gc < k;
+          const uint32_t dst0 = sa + r0 * 128 + ((j ^ (r0 & 7)) << 4);
+          for (int g = 0; g < U.ng; ++g) {
+            const int tbase = G > 1 ? g * m : 0;                 // first tile row of the entry
+            const int ebase = G > 1 ? 0 : U.mt * 128;            // first entry row in the tile
+            const int cnt = G > 1 ? m : rows;                    // entry rows in the tile
+            if (p.bsr) {
+              for (int q = r0; q < cnt; q += 16) {
+                const int r = tbase + q;
+                const int slot = col_ok ? blk_tab[(r >> 4) * 16 + (gc >> 4)] : -1;
+                const bool ok = slot >= 0;
+                const uint16_t* src =
+                    ok ? p.vals + ((long long)slot * 256 + ((ebase + q) & 15) * 16 + (gc & 15)) : p.vals;
+                ptx::cp_async_16(dst0 + (tbase + q - r0) * 128, src, ok ? 16 : 0);
+              }
+            } else {
+              const uint16_t* A = a_tab[g];
+              const uint16_t* src = A + (long long)(ebase + r0) * k + gc;
+              const long long step = 16ll * k;
+              for (int q = r0; q < cnt; q += 16, src += step)
+                ptx::cp_async_16(dst0 + (tbase + q - r0) * 128, col_ok ? src : A, col_ok ? 16 : 0);
+            }
           }
-          ptx::cp_async_16(sa + r * 128 + ((j ^ (r & 7)) << 4), src, ok ? 16 : 0);
         }
         // B: per entry 64 k-rows x n/8 chunks at columns [g n, g n + n) of the
         // N-major tile (atoms of 64 columns x 64 k-rows)
-        const int per = 64 * nc8;
-        for (int i = tid; i < U.ng * per; i += 128) {
-          int g, kr, j;
-          if (nc8_shift >= 0) {
-            const int row = i >> nc8_shift;  // = g * 64 + kr
-            g = row >> 6;
-            kr = row & 63;
-            j = i & (nc8 - 1);
-          } else {
-            g = i / per;
-            const int rem = i - g * per;
-            kr = rem / nc8;
-            j = rem - kr * nc8;
+        if (nc8_shift >= 0 && nc8 <= 128) {
+          const int j = tid & (nc8 - 1), kr0 = tid >> nc8_shift, kstep = 128 >> nc8_shift;
+          for (int g = 0; g < U.ng; ++g) {
+            const uint16_t* B = b_tab[g];
+            const int cc = g * nc8 + j;  // 16-byte chunk column in the tile
+            const uint32_t dcol = sb + (cc >> 3) * 8192;
+            const uint16_t* src = B + (long long)(kc * 64 + kr0) * n + j * 8;
+            const long long step = (long long)kstep * n;
+            for (int kr = kr0; kr < 64; kr += kstep, src += step) {
+              const bool ok = kc * 64 + kr < k;
+              ptx::cp_async_16(dcol + kr * 128 + (((cc & 7) ^ (kr & 7)) << 4), ok ? src : B, ok ? 16 : 0);
+            }
           }
-          const int gk = kc * 64 + kr;
-          const bool ok = gk < k;
-          const uint16_t* B = b_tab[g];
-          const uint16_t* src = ok ? B + (long long)gk * n + j * 8 : B;
-          const int cc = g * nc8 + j;  // 16-byte chunk column in the tile
-          ptx::cp_async_16(sb + (cc >> 3) * 8192 + kr * 128 + (((cc & 7) ^ (kr & 7)) << 4), src, ok ? 16 : 0);
+        } else {
+          const int per = 64 * nc8;
+          for (int i = tid; i < U.ng * per; i += 128) {
+            const int g = i / per, rem = i - g * per;
+            const int kr = rem / nc8, j = rem - kr * nc8;
+            const int gk = kc * 64 + kr;
+            const bool ok = gk < k;
+            const uint16_t* B = b_tab[g];
+            const uint16_t* src = ok ? B + (long long)gk * n + j * 8 : B;
+            const int cc = g * nc8 + j;
+            ptx::cp_async_16(sb + (cc >> 3) * 8192 + kr * 128 + (((cc & 7) ^ (kr & 7)) << 4), src, ok ? 16 : 0);
+          }
         }
         ptx::cp_async_commit();
         if ((int)(it + 1 - handed) > lag) hand_over(lag);

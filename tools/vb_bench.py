@@ -26,6 +26,7 @@ ap.add_argument("--shape", default="64x64x64")
 ap.add_argument("--batch", type=int, default=65536)
 ap.add_argument("--reps", type=int, default=10)
 ap.add_argument("--density", type=float, default=0.5)
+ap.add_argument("--noperm", action="store_true", help="ptr mode: pointers in entry order (no scatter)")
 a = ap.parse_args()
 hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
     os.path.join(ROOT, "MEASURED_PEAKS.json")) else 6650.0
@@ -41,7 +42,7 @@ elif a.mode == "ptr":
     m, n, k = (int(x) for x in a.shape.split("x"))
     A, B = ki.operands(m, n, k, a.batch, a.dtype, "unif", device="cuda")
     C = torch.empty(a.batch * m * n, dtype=A.dtype, device="cuda")
-    perm = torch.randperm(a.batch, device="cuda")
+    perm = torch.arange(a.batch, device="cuda") if a.noperm else torch.randperm(a.batch, device="cuda")
     es = A.element_size()
     pa = (A.data_ptr() + perm * (m * k * es)).to(torch.int64)
     pb = (B.data_ptr() + perm * (k * n * es)).to(torch.int64)
