@@ -21,6 +21,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 
 #include "kernels.h"
@@ -59,6 +60,7 @@ struct VbParams {
   const uint16_t* vals;
   const uint16_t* Bs;
   uint16_t* Cs;
+  int dbg;  // experiments only (env KAMI_VB_DEBUG): 1 = skip C stores, 2 = skip A/B copies
 };
 
 __device__ __forceinline__ const uint16_t* entry_B(const VbParams& p, long long e, int k, int n) {
@@ -105,6 +107,12 @@ __device__ __forceinline__ void cp_async_wait_n(int n) {
   }
 }
 
+// debug trace (KAMI_VB_DEBUG bit 4): clock64 of role events of CTA 0
+__device__ long long g_vb_trace[8][1024];
+__device__ __forceinline__ void trace(int ev, uint32_t i) {
+  if (blockIdx.x == 0 && (threadIdx.x & 31) == 0 && i < 1024) g_vb_trace[ev][i] = clock64();
+}
+
 template <bool kBF16>
 __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __grid_constant__ VbParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -118,7 +126,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   // per-unit entry pointer tables (loaded once per unit, not once per copy)
   const uint16_t** a_tab = reinterpret_cast<const uint16_t**>(blk_tab + 128);
   const uint16_t** b_tab = a_tab + 8;
-  uint16_t** c_tab = reinterpret_cast<uint16_t**>(b_tab + 8);  // [2 warpgroups][8]
+  uint16_t** c_tab = reinterpret_cast<uint16_t**>(const_cast<uint16_t**>(b_tab + 8));  // [2 warpgroups][8]
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < p.stages; ++s) {
@@ -143,15 +151,8 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     // cp.async straight into the swizzled stage buffers; a stage is handed to
     // the MMA warp once its copy group has landed, `lag` stages later, so
     // several stages stream concurrently without register staging.
-    const int lag = p.stages - 1 < 6 ? p.stages - 1 : 6;
     const int tid = threadIdx.x;  // 0..127
-    uint32_t it = 0, handed = 0;
-    auto hand_over = [&](int pending) {
-      cp_async_wait_n(pending);  // the oldest un-handed group has landed
-      ptx::fence_proxy_async_smem();
-      ptx::mbar_arrive(&full[handed % p.stages]);
-      ++handed;
-    };
+    uint32_t it = 0;
     for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
       Unit U;
       if (!unit_of(p, u, U)) continue;
@@ -188,7 +189,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       for (int kc = 0; kc < kchunks; ++kc, ++it) {
         const uint32_t s = it % p.stages;
         ptx::mbar_wait(&empty[s], ((it / p.stages) & 1) ^ 1);
+        if (p.dbg & 4) trace(0, it);
         const uint32_t sa = smem_base + s * p.stage_bytes, sb = sa + kAReg;
+        if (!(p.dbg & 2)) {
         // A: thread = (16-byte chunk j, row r0 + 16 q): a warp covers 4 whole
         // 128-byte row segments, the swizzle phase (r & 7) is fixed per thread
         // and the addresses advance by constant strides.
@@ -247,11 +250,14 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
             ptx::cp_async_16(sb + (cc >> 3) * 8192 + kr * 128 + (((cc & 7) ^ (kr & 7)) << 4), src, ok ? 16 : 0);
           }
         }
-        ptx::cp_async_commit();
-        if ((int)(it + 1 - handed) > lag) hand_over(lag);
+        }  // dbg & 2
+        // full[s] completes when all 128 threads' copies of this stage landed;
+        // the MMA warp fences generic->async proxy before reading the stage
+        ptx::cp_async_mbar_arrive_noinc(&full[s]);
+        if (p.dbg & 4) trace(1, it);
       }
     }
-    while (handed < it) hand_over((int)(it - handed - 1));
+    ptx::cp_async_wait<0>();  // nothing may be in flight when the CTA exits
   } else if (warp == 4) {
     // ------------------------------------------------------------- MMA
     uint32_t it = 0, acc_it = 0;
@@ -260,6 +266,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       if (!unit_of(p, u, U)) continue;
       const uint32_t a = acc_it % p.acc_bufs;
       ptx::mbar_wait(&tempty[a], ((acc_it / p.acc_bufs) & 1) ^ 1);
+      if (p.dbg & 4) trace(6, acc_it);
       ptx::tc_fence_after();
       const uint32_t d_tmem = tmem_base + a * p.acc_cols;
       const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, p.G * U.n, 0, 1);
@@ -268,6 +275,8 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       for (int kc = 0; kc < kchunks; ++kc, ++it) {
         const uint32_t s = it % p.stages;
         ptx::mbar_wait(&full[s], (it / p.stages) & 1);
+        if (p.dbg & 4) trace(2, it);
+        ptx::fence_proxy_async_smem();  // cp.async (generic proxy) writes -> tensor-core reads
         ptx::tc_fence_after();
         if (lane == 0) {
           const uint32_t sa = smem_base + s * p.stage_bytes, sb = sa + kAReg;
@@ -282,6 +291,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         __syncwarp();
       }
       if (lane == 0) ptx::umma_commit(&tfull[a]);
+      if (p.dbg & 4) trace(3, acc_it);
       __syncwarp();
       ++acc_it;
     }
@@ -310,6 +320,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       const bool warp_live = sp * 32 < rows;
       if (L < U.ng) c_tab[wg * 8 + L] = entry_C(p, U.e0 + L, m, n);  // read after the staging barrier
       ptx::mbar_wait(&tfull[a], aph);
+      if (p.dbg & 4) trace(4, acc_it);
       ptx::tc_fence_after();
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
       for (int h0 = 0; h0 < n; h0 += 128) {
@@ -348,10 +359,12 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         ptx::named_bar_sync(1 + wg, 128);
         // copy-out: chunk index i -> (tile row i / cpr, 16-byte chunk i % cpr)
         const int cpr = hw / 8;
+        const int cpr_shift = (cpr & (cpr - 1)) == 0 ? __ffs(cpr) - 1 : -1;
         for (int i = L; i < rows * cpr; i += 128) {
-          const int r = i / cpr, c = i - r * cpr;
+          const int r = cpr_shift >= 0 ? i >> cpr_shift : i / cpr, c = i - r * cpr;
           const int ge = G > 1 ? r / m : 0;
           const int er = G > 1 ? r - ge * m : U.mt * 128 + r;
+          if (p.dbg & 1) continue;
           uint32_t x0, x1, x2, x3;
           ptx::ld_shared_v4(cst + r * kCRow + c * 16, x0, x1, x2, x3);
           ptx::st_global_v4(c_tab[wg * 8 + ge] + (long long)er * n + h0 + c * 8, make_uint4(x0, x1, x2, x3));
@@ -361,6 +374,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[a]);
+      if (p.dbg & 4) trace(5, acc_it);
     }
   }
   ptx::tc_fence_before();
@@ -391,6 +405,10 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   p.bar_off = p.c_off + 2 * kCBuf;
   p.mtiles = p.G > 1 ? 1 : (max_m + 127) / 128;
   p.units = ((p.batch + p.G - 1) / p.G) * p.mtiles;
+  {
+    const char* d = getenv("KAMI_VB_DEBUG");
+    p.dbg = d ? atoi(d) : 0;
+  }
   const uint32_t smem = p.bar_off + 2048 + 1024;
   auto fn = bf16 ? kami_tc16_vb_kernel<true> : kami_tc16_vb_kernel<false>;
   if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
@@ -413,6 +431,10 @@ int packing(int m, int n) {  // entries per 128-lane tile (same rule as tc16.cu)
 }
 
 }  // namespace
+
+extern "C" int kami_debug_vb_trace(long long* out) {
+  return cudaMemcpyFromSymbol(out, g_vb_trace, sizeof(long long) * 8 * 1024) == cudaSuccess ? 0 : 1;
+}
 
 kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf16, const int* row_ptr,
                                    const int* col_blk, const void* vals, int max_nnzb, const void* B, void* C,
