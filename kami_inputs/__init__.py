@@ -32,7 +32,18 @@ _M2 = 0x94D049BB133111EB
 OPERAND_A = 0
 OPERAND_B = 1
 
-TORCH_DTYPES = {"f16": torch.float16, "bf16": torch.bfloat16, "f64": torch.float64}
+TORCH_DTYPES = {"f16": torch.float16, "bf16": torch.bfloat16, "f64": torch.float64, "f32": torch.float32,
+                "tf32": torch.float32, "e4m3": torch.float8_e4m3fn, "e5m2": torch.float8_e5m2}
+# output (C) storage type of each input type (DESIGN.md f4)
+OUT_DTYPE = {"f16": "f16", "bf16": "bf16", "f64": "f64", "tf32": "f32", "e4m3": "f16", "e5m2": "f16"}
+
+
+def _to_tf32(x: torch.Tensor) -> torch.Tensor:
+    """RNE of float64 values to TF32 precision (8-bit exponent, 10-bit
+    fraction), stored as float32 -- the values a kind::tf32 MMA reads exactly."""
+    u = x.to(torch.float32).view(torch.int32)
+    u = (u + 0xFFF + ((u >> 13) & 1)) & ~0x1FFF
+    return u.view(torch.float32)
 
 
 def _s64(u: int) -> int:
@@ -63,10 +74,13 @@ def splitmix64_py(x: int) -> int:
 
 
 def int_range(k: int, dtype: str) -> int:
-    """Largest R with R^2 * k <= limit (fp16 2048, bf16 256, fp64 2^40), R >= 1."""
-    limit = {"f16": 2048, "bf16": 256, "f64": 1 << 40}[dtype]
+    """Largest R with R^2 * k <= limit (fp16/fp8->fp16 2048, bf16 256, fp64 2^40,
+    tf32->fp32 2^24) and R exactly representable in the input type, R >= 1."""
+    limit = {"f16": 2048, "bf16": 256, "f64": 1 << 40, "tf32": 1 << 24, "f32": 1 << 24, "e4m3": 2048,
+             "e5m2": 2048}[dtype]
+    rmax = {"e4m3": 16, "e5m2": 8, "tf32": 2048, "f32": 2048}.get(dtype, 1 << 20)
     r = 1
-    while (r + 1) * (r + 1) * k <= limit:
+    while (r + 1) * (r + 1) * k <= limit and r + 1 <= rmax:
         r += 1
     return r
 
@@ -100,7 +114,7 @@ def draw(seed: int, operand: int, entry0: int, n_entries: int, rows: int, cols: 
             u = (torch.remainder(_lshr(z, 33), 2 * R + 1) - R).to(torch.float64)
         else:
             raise ValueError(dist)
-        out[s:e] = u.to(TORCH_DTYPES[dtype])
+        out[s:e] = _to_tf32(u) if dtype == "tf32" else u.to(TORCH_DTYPES[dtype])
     return out
 
 
@@ -115,10 +129,13 @@ def operands(m: int, n: int, k: int, batch: int, dtype: str, dist: str = "unif",
 
 
 def as_bits(x: torch.Tensor):
-    """numpy view usable by the oracle: uint16 bits for 16-bit dtypes, float64 otherwise."""
+    """numpy view usable by the oracle: uint16 bits for 16-bit dtypes, uint8
+    bits for fp8, float32 / float64 otherwise."""
     x = x.detach().cpu().contiguous()
     if x.dtype in (torch.float16, torch.bfloat16):
         return x.view(torch.int16).numpy().view("uint16")
+    if x.dtype in (torch.float8_e4m3fn, torch.float8_e5m2):
+        return x.view(torch.uint8).numpy()
     return x.numpy()
 
 

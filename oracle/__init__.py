@@ -30,7 +30,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 _SO = os.path.join(_HERE, "liboracle.so")
 _SRC = os.path.join(_HERE, "oracle.c")
 
-DTYPES = {"f16": 0, "bf16": 1, "f64": 2}
+DTYPES = {"f16": 0, "bf16": 1, "f64": 2, "f32": 3, "tf32": 3, "e4m3": 4, "e5m2": 5}
 LAYOUTS = {"row": 0, "col": 1}
 
 
@@ -72,9 +72,15 @@ def lib() -> ctypes.CDLL:
 
 
 def _raw(x: np.ndarray, dtype: str) -> np.ndarray:
-    """Contiguous raw storage: uint16 bit patterns for 16-bit types, float64 for f64."""
+    """Contiguous raw storage: uint16 bit patterns for 16-bit types, float64 for
+    f64, float32 for f32/tf32, uint8 bit patterns for fp8."""
     if dtype == "f64":
         return np.ascontiguousarray(x, dtype=np.float64)
+    if dtype in ("f32", "tf32"):
+        return np.ascontiguousarray(x, dtype=np.float32)
+    if dtype in ("e4m3", "e5m2"):
+        return np.ascontiguousarray(np.asarray(x).view(np.uint8) if np.asarray(x).dtype != np.uint8 else x,
+                                    dtype=np.uint8)
     if x.dtype == np.float16:
         x = x.view(np.uint16)
     return np.ascontiguousarray(x, dtype=np.uint16)
@@ -115,6 +121,8 @@ def round_to(x: np.ndarray, dtype: str) -> np.ndarray:
     x = np.ascontiguousarray(x, dtype=np.float64).reshape(-1)
     if dtype == "f64":
         return x.copy()
+    if dtype in ("f32", "tf32"):  # binary32 output (f4): IEEE cast, RNE
+        return x.astype(np.float32)
     out = np.empty(x.size, dtype=np.uint16)
     fn = lib().oracle_round_f16 if dtype == "f16" else lib().oracle_round_bf16
     fn(x.ctypes.data, out.ctypes.data, x.size)
@@ -122,9 +130,20 @@ def round_to(x: np.ndarray, dtype: str) -> np.ndarray:
 
 
 def decode(bits: np.ndarray, dtype: str) -> np.ndarray:
-    """Exact decode of uint16 fp16/bf16 bit patterns (or float64) to float64."""
+    """Exact decode of uint16 fp16/bf16 bit patterns, uint8 fp8 bit patterns,
+    float32 or float64 to float64."""
     if dtype == "f64":
         return np.asarray(bits, dtype=np.float64).reshape(-1)
+    if dtype in ("f32", "tf32"):
+        return np.asarray(bits, dtype=np.float32).astype(np.float64).reshape(-1)
+    if dtype in ("e4m3", "e5m2"):
+        b = np.ascontiguousarray(np.asarray(bits).reshape(-1), dtype=np.uint8)
+        out = np.empty(b.size, dtype=np.float64)
+        L = lib()
+        L.oracle_decode_fp8.restype = None
+        L.oracle_decode_fp8.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_int64, ctypes.c_int]
+        L.oracle_decode_fp8(b.ctypes.data, out.ctypes.data, b.size, 1 if dtype == "e5m2" else 0)
+        return out
     b = _raw(np.asarray(bits).reshape(-1), dtype)
     out = np.empty(b.size, dtype=np.float64)
     fn = lib().oracle_decode_f16 if dtype == "f16" else lib().oracle_decode_bf16
@@ -175,3 +194,14 @@ def spmm_bsr(m: int, n: int, k: int, batch: int, dtype: str, row_ptr, col_blk, v
     if rc != 0:
         raise ValueError(f"oracle_spmm_bsr rejected its arguments ({rc})")
     return (C, S) if with_scale else C
+
+
+def axpby(C_ref: np.ndarray, C_in: np.ndarray, alpha: float, beta: float) -> np.ndarray:
+    """alpha * C_ref + beta * C_in in binary64 (the C-update form, DESIGN.md f4)."""
+    out = np.ascontiguousarray(C_ref, dtype=np.float64).copy()
+    cin = np.ascontiguousarray(C_in, dtype=np.float64).reshape(out.shape)
+    L = lib()
+    L.oracle_axpby.restype = None
+    L.oracle_axpby.argtypes = [ctypes.c_void_p, ctypes.c_void_p, ctypes.c_double, ctypes.c_double, ctypes.c_int64]
+    L.oracle_axpby(out.ctypes.data, cin.ctypes.data, alpha, beta, out.size)
+    return out

@@ -46,6 +46,9 @@
 #define ORACLE_F16 0
 #define ORACLE_BF16 1
 #define ORACLE_F64 2
+#define ORACLE_F32 3  /* IEEE binary32 storage (TF32 inputs are FP32 values with a 10-bit mantissa) */
+#define ORACLE_E4M3 4 /* OCP FP8 E4M3 ("fn": no infinities, 0x7f/0xff NaN) */
+#define ORACLE_E5M2 5 /* OCP FP8 E5M2 (IEEE-like) */
 
 #define ORACLE_ROW 0
 #define ORACLE_COL 1
@@ -74,6 +77,26 @@ double oracle_bf16_to_f64(uint16_t h) {
   float f;
   memcpy(&f, &u, sizeof f);
   return (double)f;
+}
+
+/* FP8 E4M3 (bias 7, 3 fraction bits, max 448, S.1111.111 = NaN). */
+double oracle_e4m3_to_f64(uint8_t h) {
+  int s = (h >> 7) & 1, e = (h >> 3) & 0xf, f = h & 7;
+  double v;
+  if (e == 15 && f == 7) v = NAN;
+  else if (e == 0) v = ldexp((double)f, -9); /* f * 2^-3 * 2^-6 */
+  else v = ldexp((double)(8 + f), e - 10);   /* (1.f) * 2^(e-7) */
+  return s ? -v : v;
+}
+
+/* FP8 E5M2 (bias 15, 2 fraction bits, IEEE specials). */
+double oracle_e5m2_to_f64(uint8_t h) {
+  int s = (h >> 7) & 1, e = (h >> 2) & 0x1f, f = h & 3;
+  double v;
+  if (e == 31) v = f ? NAN : INFINITY;
+  else if (e == 0) v = ldexp((double)f, -16); /* f * 2^-2 * 2^-14 */
+  else v = ldexp((double)(4 + f), e - 17);    /* (1.f) * 2^(e-15) */
+  return s ? -v : v;
 }
 
 /* ------------------------------------------------------ RNE encoders (f64) */
@@ -129,6 +152,12 @@ static double load_elem(const void* base, int dtype, int64_t idx) {
       return oracle_f16_to_f64(((const uint16_t*)base)[idx]);
     case ORACLE_BF16:
       return oracle_bf16_to_f64(((const uint16_t*)base)[idx]);
+    case ORACLE_F32:
+      return (double)((const float*)base)[idx];
+    case ORACLE_E4M3:
+      return oracle_e4m3_to_f64(((const uint8_t*)base)[idx]);
+    case ORACLE_E5M2:
+      return oracle_e5m2_to_f64(((const uint8_t*)base)[idx]);
     default:
       return ((const double*)base)[idx];
   }
@@ -177,7 +206,7 @@ static void* gemm_worker(void* arg) {
 int oracle_gemm(int m, int n, int k, int64_t batch, int dtype, int layout,
                 const void* A, const void* B, double* C, double* S, int nthreads) {
   if (m <= 0 || n <= 0 || k <= 0 || batch < 0) return 1;
-  if (dtype < 0 || dtype > 2 || layout < 0 || layout > 1) return 1;
+  if (dtype < 0 || dtype > 5 || layout < 0 || layout > 1) return 1;
   if (batch == 0) return 0;
   if (fegetround() != FE_TONEAREST) fesetround(FE_TONEAREST);
   if (nthreads < 1) nthreads = 1;
@@ -255,4 +284,16 @@ int oracle_spmm_bsr(int m, int n, int k, int blk, int64_t batch, int dtype, cons
   free(Ad);
   free(Bd);
   return rc;
+}
+
+/* ------------------------------------------------- alpha A B + beta C_in
+ * The GEMM-update form the algorithms' GMem2Reg(C_i <- C) implies (Alg. 1-3
+ * load C, R1/f4):  C_ref = alpha * (A B)_ref + beta * C_in, both
+ * terms in binary64; C_in given as doubles (already decoded, row-major
+ * [batch][m][n]).  Writes the result in place over C (which holds (A B)_ref). */
+void oracle_axpby(double* C, const double* Cin, double alpha, double beta, int64_t count) {
+  for (int64_t i = 0; i < count; ++i) C[i] = alpha * C[i] + beta * Cin[i];
+}
+void oracle_decode_fp8(const uint8_t* x, double* out, int64_t n, int e5m2) {
+  for (int64_t i = 0; i < n; ++i) out[i] = e5m2 ? oracle_e5m2_to_f64(x[i]) : oracle_e4m3_to_f64(x[i]);
 }
