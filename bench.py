@@ -45,7 +45,20 @@ WORKLOADS = {
     "lr-8": ("f16", 256, 256, 8, 16384, 3),
     "lr-16": ("f16", 256, 256, 16, 16384, 3),
     "lr-32": ("f16", 256, 256, 32, 16384, 3),
+    # SURVEY f4 variants (not BASELINE configs; same shape as configs[1] 64^3)
+    "tf32-64": ("tf32", 64, 64, 64, 65536, 1),
+    "e4m3-64": ("e4m3", 64, 64, 64, 65536, 1),
+    "e5m2-64": ("e5m2", 64, 64, 64, 65536, 1),
+    "f16upd-64": ("f16", 64, 64, 64, 65536, 1),   # C = A B + C (beta = 1: C read and written)
 }
+ES_IN = {"f64": 8, "tf32": 4, "e4m3": 1, "e5m2": 1}
+ES_OUT = {"f64": 8, "tf32": 4}
+
+
+def op_bytes(dtype, m, n, k, update=False):
+    """Algorithmic bytes of one entry: A, B read once, C written once (and
+    read once more when beta != 0)."""
+    return (m * k + k * n) * ES_IN.get(dtype, 2) + m * n * ES_OUT.get(dtype, 2) * (2 if update else 1)
 
 
 def parse_workload(name):
@@ -211,8 +224,8 @@ def workload_config(args, dtype, m, n, k, batch, cfg):
                         f"(BASELINE.json configs[{cfg}])",
             "m": m, "n": n, "k": k, "batch_per_gpu": batch, "global_batch": batch * args.gpus,
             "layout": "row", "algo": args.algo, "p": args.p, "inputs": "unif [-1,1) RNE to dtype, counter-based SplitMix64",
-            "l2": "inputs larger than L2 (126 MB)" if batch * (m * k + k * n + m * n) * (8 if dtype == 'f64' else 2)
-                  > 126e6 else "L2 flushed between timed steps",
+            "l2": "inputs larger than L2 (126 MB)" if batch * op_bytes(dtype, m, n, k) > 126e6
+                  else "L2 flushed between timed steps",
             "parallelism": f"batch-sharded dp{args.gpus}"}
 
 
@@ -241,18 +254,23 @@ def main():
 
     world, rank, local = dist_init()
     dtype, m, n, k, batch, cfg = parse_workload(args.workload)
-    es = 8 if dtype == "f64" else 2
+    update = "upd" in args.workload
+    esi, eso = ES_IN.get(dtype, 2), ES_OUT.get(dtype, 2)
     entry0 = rank * batch
     A, B = ki.operands(m, n, k, batch, dtype, "unif", seed=0, entry0=entry0, device="cuda")
-    C = torch.empty(batch * m * n, dtype=A.dtype, device="cuda")
+    C = torch.zeros(batch * m * n, dtype=ki.TORCH_DTYPES[ki.OUT_DTYPE[dtype]], device="cuda")
     stream = torch.cuda.current_stream()
-    alg_bytes = batch * (m * k + k * n + m * n) * es
+    alg_bytes = batch * op_bytes(dtype, m, n, k, update)
     flops = 2.0 * m * n * k * batch
     small = alg_bytes < 126e6  # L2-resident: flush L2 between timed steps
     flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if small else None
 
     def step():
-        kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A, B, C, algo=args.algo, p=args.p, stream=stream)
+        if update:  # C <- A B + C
+            kami.gemm_strided_batched_axpby(m, n, k, batch, dtype, "row", 1.0, A, B, 1.0, C, stream=stream)
+        else:
+            kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A, B, C, algo=args.algo, p=args.p,
+                                      stream=stream)
 
     for _ in range(args.warmup):
         step()
@@ -299,7 +317,7 @@ def main():
 
     # end-to-end: the C-ABI host entry point, host<->device copies inside the timed region
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and not update:
         hA = A.cpu().pin_memory()
         hB = B.cpu().pin_memory()
         hC = torch.empty(C.numel(), dtype=C.dtype).pin_memory()
@@ -315,7 +333,7 @@ def main():
         if world > 1:
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
         e2e = {"value": flops * world / float(et.item()) / 1e12, "unit": "TFLOP/s",
-               "h2d_bytes_per_step": batch * (m * k + k * n) * es, "d2h_bytes_per_step": batch * m * n * es,
+               "h2d_bytes_per_step": batch * (m * k + k * n) * esi, "d2h_bytes_per_step": batch * m * n * eso,
                "path": "kami_gemm_strided_batched_host (pinned host buffers, chunked H2D/kernel/D2H pipeline)"}
         kami.release_workspace()
 
@@ -328,7 +346,8 @@ def main():
     value = flops * total_entries / batch * args.steps / (t_max_ms * 1e-3) / 1e12
     avg_launch_s = (t_ms / args.steps) * 1e-3
     achieved_gbs = alg_bytes / avg_launch_s / 1e9
-    roof_tf = min(hbm * 1e9 * flops / alg_bytes, (fp64_peak_tflops() if dtype == "f64" else 2250.0) * 1e12) / 1e12
+    tensor_peak = {"f64": fp64_peak_tflops(), "tf32": 1125.0, "e4m3": 4500.0, "e5m2": 4500.0}.get(dtype, 2250.0)
+    roof_tf = min(hbm * 1e9 * flops / alg_bytes, tensor_peak * 1e12) / 1e12
     bound = "hbm"
     if dtype == "f64" and fp64_peak_tflops() * 1e12 < hbm * 1e9 * flops / alg_bytes:
         bound = "tensor"

@@ -20,8 +20,10 @@
  *     KAMI_COL_MAJOR: X_b(r, c) at  X + b*R*C + c*R + r
  *
  * Sizes supported (R5): 16-bit types need m, n multiples of 16 in
- * [16, 256] and k a multiple of 8 in [8, 256]; FP64 needs m, n, k multiples
- * of 8 in [8, 128].  Anything else returns KAMI_ERROR_NOT_SUPPORTED.
+ * [16, 256] and k a multiple of 8 in [8, 256]; TF32 the same with k a
+ * multiple of 4; FP8 m, n multiples of 32 and k of 16 (all <= 256); FP64
+ * m = n = k in {8, 16, 32, 64}.  Anything else returns
+ * KAMI_ERROR_NOT_SUPPORTED.
  *
  * Ownership and threading: the caller owns every buffer.  Device entry points
  * never allocate device memory, never synchronise and enqueue on `stream`
@@ -50,7 +52,19 @@ typedef enum {
   KAMI_ERROR_CUDA = 4           /* a CUDA runtime call failed             */
 } kami_status_t;
 
-typedef enum { KAMI_DTYPE_F16 = 0, KAMI_DTYPE_BF16 = 1, KAMI_DTYPE_F64 = 2 } kami_dtype_t;
+/* Element types.  F16/BF16: A, B, C in that type, FP32 accumulation, C
+ * rounded RNE.  F64: FP64 end to end.  TF32: A, B, C are FP32
+ * arrays, the tensor core reads A and B at TF32 precision (10-bit fraction),
+ * FP32 accumulation, C FP32.  E4M3 / E5M2 (f4): A, B are OCP FP8 bytes, FP32
+ * accumulation, C FP16 (RNE). */
+typedef enum {
+  KAMI_DTYPE_F16 = 0,
+  KAMI_DTYPE_BF16 = 1,
+  KAMI_DTYPE_F64 = 2,
+  KAMI_DTYPE_TF32 = 3,
+  KAMI_DTYPE_E4M3 = 4,
+  KAMI_DTYPE_E5M2 = 5
+} kami_dtype_t;
 
 typedef enum { KAMI_ROW_MAJOR = 0, KAMI_COL_MAJOR = 1 } kami_layout_t;
 
@@ -102,6 +116,15 @@ kami_status_t kami_gemm_vbatched(int64_t batch, const int* m_array, const int* n
 kami_status_t kami_gemm_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
                                         kami_layout_t layout, const void* A, const void* B, void* C,
                                         kami_stream_t stream);
+
+/* C <- alpha * A B + beta * C (the C-update form of Alg. 1-3, whose
+ * GMem2Reg loads C).  C is read iff beta != 0.  alpha and beta are
+ * applied in FP32 for the tensor-core types (FP64 for F64).  Strided batches,
+ * planner-chosen kernel; NOT_SUPPORTED where that kernel has no update form
+ * (FP64 order 8). */
+kami_status_t kami_gemm_strided_batched_axpby(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                              kami_layout_t layout, double alpha, const void* A, const void* B,
+                                              double beta, void* C, kami_stream_t stream);
 
 /* Same with an explicit schedule and warp count p.  p = 0 takes the planner
  * default; for 16-bit KAMI_ALGO_1D with p = 0 that is the tcgen05 kernel

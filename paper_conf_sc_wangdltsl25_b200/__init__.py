@@ -21,7 +21,7 @@ _HERE = os.path.dirname(os.path.abspath(__file__))
 # KAMI_LIB may point at another build of the same library (A/B experiments)
 SO_PATH = os.environ.get("KAMI_LIB") or os.path.join(_HERE, "libkami.so")
 
-DTYPE = {"f16": 0, "bf16": 1, "f64": 2}
+DTYPE = {"f16": 0, "bf16": 1, "f64": 2, "tf32": 3, "e4m3": 4, "e5m2": 5}
 LAYOUT = {"row": 0, "col": 1}
 ALGO = {"auto": 0, "1d": 1, "2d": 2, "3d": 3, "nonca": 4, "1d_tma": 5}
 STATUS = {0: "KAMI_SUCCESS", 1: "KAMI_ERROR_INVALID_VALUE", 2: "KAMI_ERROR_NOT_SUPPORTED",
@@ -32,7 +32,7 @@ EXPORTS = [
     "kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
     "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
     "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level", "kami_gemm_vbatched",
-    "kami_spmm_bsr_strided_batched",
+    "kami_spmm_bsr_strided_batched", "kami_gemm_strided_batched_axpby",
 ]
 
 
@@ -70,12 +70,15 @@ def lib() -> ctypes.CDLL:
     L.kami_gemm_block_level.argtypes = [i, i, i, i64, i, i, i, i, i, vp, vp, vp, vp, st]
     L.kami_gemm_vbatched.argtypes = [i64, vp, vp, vp, i, i, i, i, i, vp, vp, vp, st]
     L.kami_spmm_bsr_strided_batched.argtypes = [i, i, i, i64, i, vp, vp, vp, i, vp, vp, st]
+    L.kami_gemm_strided_batched_axpby.argtypes = [i, i, i, i64, i, i, ctypes.c_double, vp, vp, ctypes.c_double, vp,
+                                                  st]
     L.kami_release_workspace.argtypes = []
     L.kami_plan.argtypes = [i, i, i, i, i, i, i, ctypes.POINTER(KamiPlan)]
     d = ctypes.c_double
     L.kami_paper_cost.argtypes = [i, d, d, d, d, d, d, d, d, d, d, d, ctypes.POINTER(ctypes.c_double)]
     for f in ("kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
               "kami_gemm_block_level", "kami_gemm_vbatched", "kami_spmm_bsr_strided_batched",
+              "kami_gemm_strided_batched_axpby",
               "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost"):
         getattr(L, f).restype = ctypes.c_int
     L.kami_status_string.restype = ctypes.c_char_p
@@ -112,7 +115,8 @@ def _stream(stream):
 def _dtype_of(t):
     import torch
 
-    return {torch.float16: "f16", torch.bfloat16: "bf16", torch.float64: "f64"}[t.dtype]
+    return {torch.float16: "f16", torch.bfloat16: "bf16", torch.float64: "f64", torch.float32: "tf32",
+            torch.float8_e4m3fn: "e4m3", torch.float8_e5m2: "e5m2"}[t.dtype]
 
 
 def _ptr(x):
@@ -125,6 +129,14 @@ def gemm_strided_batched(m, n, k, batch, dtype, layout, A, B, C, algo="auto", p=
     _check(lib().kami_gemm_strided_batched_ex(
         m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
         _ptr(A), _ptr(B), _ptr(C), _enum(ALGO, algo, "algo"), p, _stream(stream)), "kami_gemm_strided_batched")
+    return C
+
+
+def gemm_strided_batched_axpby(m, n, k, batch, dtype, layout, alpha, A, B, beta, C, stream=None):
+    """C <- alpha A B + beta C per entry (C read iff beta != 0)."""
+    _check(lib().kami_gemm_strided_batched_axpby(
+        m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"), float(alpha), _ptr(A),
+        _ptr(B), float(beta), _ptr(C), _stream(stream)), "kami_gemm_strided_batched_axpby")
     return C
 
 

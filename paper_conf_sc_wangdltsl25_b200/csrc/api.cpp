@@ -36,15 +36,20 @@ PFN_encodeTiled get_encode_tiled() {
 namespace {
 
 bool is16(kami_dtype_t d) { return d == KAMI_DTYPE_F16 || d == KAMI_DTYPE_BF16; }
-size_t esize(kami_dtype_t d) { return d == KAMI_DTYPE_F64 ? 8 : 2; }
+bool is_tc(kami_dtype_t d) { return d != KAMI_DTYPE_F64; }  // tcgen05 types
+int in_kind(kami_dtype_t d) {  // tc16.cu input kinds
+  return d == KAMI_DTYPE_F16 ? 0 : d == KAMI_DTYPE_BF16 ? 1 : d == KAMI_DTYPE_TF32 ? 2 : d == KAMI_DTYPE_E4M3 ? 3 : 4;
+}
+int out_kind(kami_dtype_t d) { return d == KAMI_DTYPE_BF16 ? 1 : d == KAMI_DTYPE_TF32 ? 2 : 0; }
 bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
 
 // Size grid (R5).  Checked before anything touches the device.
 kami_status_t check_sizes(int m, int n, int k, kami_dtype_t dtype) {
-  if (is16(dtype)) {
-    if (m % 16 || n % 16 || k % 8 || m > 256 || n > 256 || k > 256) return KAMI_ERROR_NOT_SUPPORTED;
-    return KAMI_SUCCESS;
-  }
+  if (m > 256 || n > 256 || k > 256) return KAMI_ERROR_NOT_SUPPORTED;
+  if (is16(dtype)) return (m % 16 || n % 16 || k % 8) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
+  if (dtype == KAMI_DTYPE_TF32) return (m % 16 || n % 16 || k % 4) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
+  if (dtype == KAMI_DTYPE_E4M3 || dtype == KAMI_DTYPE_E5M2)
+    return (m % 32 || n % 32 || k % 16) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
   // FP64: the register-resident DMMA family is instantiated for these orders
   if (m == n && n == k && (m == 8 || m == 16 || m == 32 || m == 64)) return KAMI_SUCCESS;
   return KAMI_ERROR_NOT_SUPPORTED;
@@ -52,7 +57,7 @@ kami_status_t check_sizes(int m, int n, int k, kami_dtype_t dtype) {
 
 kami_status_t check_common(int m, int n, int k, int64_t batch, int dtype, int layout, int algo) {
   if (m <= 0 || n <= 0 || k <= 0 || batch < 0) return KAMI_ERROR_INVALID_VALUE;
-  if (dtype < KAMI_DTYPE_F16 || dtype > KAMI_DTYPE_F64) return KAMI_ERROR_INVALID_VALUE;
+  if (dtype < KAMI_DTYPE_F16 || dtype > KAMI_DTYPE_E5M2) return KAMI_ERROR_INVALID_VALUE;
   if (layout != KAMI_ROW_MAJOR && layout != KAMI_COL_MAJOR) return KAMI_ERROR_INVALID_VALUE;
   if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_1D_TMA) return KAMI_ERROR_INVALID_VALUE;
   return check_sizes(m, n, k, (kami_dtype_t)dtype);
@@ -76,7 +81,14 @@ RowProblem to_row(int m, int n, int k, kami_layout_t layout, const void* A, cons
 }
 
 kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, kami_algo_t algo, int p, void* C,
-                       void* const* Ca, cudaStream_t stream) {
+                       void* const* Ca, cudaStream_t stream, double alpha = 1.0, double beta = 0.0) {
+  const bool update = alpha != 1.0 || beta != 0.0;
+  if (!is16(dtype) && dtype != KAMI_DTYPE_F64) {  // TF32 / FP8: tcgen05 1D only, strided only
+    if (Ca || (algo != KAMI_ALGO_AUTO && algo != KAMI_ALGO_1D && algo != KAMI_ALGO_1D_TMA) || p)
+      return KAMI_ERROR_NOT_SUPPORTED;
+    return tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), rp.A, rp.B, C, (float)alpha,
+                            (float)beta, stream, 0);
+  }
   // 16-bit pointer arrays: the LDG-fed tcgen05 kernel covers the whole size grid
   if (Ca && is16(dtype) && algo == KAMI_ALGO_AUTO)
     return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, rp.m, rp.n, rp.k, nullptr, nullptr, nullptr, rp.m, rp.n,
@@ -85,9 +97,11 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
   if (plan.kernel == 0) {
-    return tc16_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream, 0);
+    return tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), rp.A, rp.B, C, (float)alpha,
+                            (float)beta, stream, 0);
   }
-  if (plan.kernel == 2) return dmma_tma_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream);
+  if (plan.kernel == 2) return dmma_tma_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream, alpha, beta);
+  if (update) return KAMI_ERROR_NOT_SUPPORTED;  // the warp-level family has no update form
   return warp_ca_launch(rp.m, rp.n, rp.k, batch, dtype, (int)plan.algo, plan.p, rp.A, rp.B, C, rp.Aa, rp.Ba, Ca,
                         stream);
 }
@@ -111,6 +125,21 @@ kami_status_t kami_gemm_strided_batched_ex(int m, int n, int k, int64_t batch, k
   if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
   RowProblem rp = to_row(m, n, k, layout, A, B, nullptr, nullptr);
   return dispatch(rp, batch, dtype, algo, p, C, nullptr, reinterpret_cast<cudaStream_t>(stream));
+}
+
+kami_status_t kami_gemm_strided_batched_axpby(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                              kami_layout_t layout, double alpha, const void* A, const void* B,
+                                              double beta, void* C, kami_stream_t stream) {
+  kami_status_t st = check_common(m, n, k, batch, dtype, layout, KAMI_ALGO_AUTO);
+  if (st != KAMI_SUCCESS) return st;
+  if (batch == 0) return KAMI_SUCCESS;
+  if (!A || !B || !C) return KAMI_ERROR_INVALID_VALUE;
+  if (!aligned16(A) || !aligned16(B) || !aligned16(C)) return KAMI_ERROR_MISALIGNED;
+  if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
+  // column-major: C^T = alpha B^T A^T + beta C^T on the same buffers
+  RowProblem rp = to_row(m, n, k, layout, A, B, nullptr, nullptr);
+  return dispatch(rp, batch, dtype, KAMI_ALGO_AUTO, 0, C, nullptr, reinterpret_cast<cudaStream_t>(stream), alpha,
+                  beta);
 }
 
 kami_status_t kami_gemm_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,

@@ -46,6 +46,7 @@ struct DmmaTmaParams {
   const double* B;
   double* C;
   long long batch;
+  double alpha, beta;  // C = alpha A B + beta C (C read iff beta != 0)
 };
 
 template <int M, int N, int K, int P, int TEAMS>
@@ -125,13 +126,26 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
     for (int i = 0; i < Cfg::FM; ++i)
 #pragma unroll
       for (int j = 0; j < Cfg::FN; ++j)
-        ptx::st_global_v2_f64(Cg + (i * 8 + g) * N + j * 8 + 2 * t, c[i][j][0], c[i][j][1]);
+      {
+        double* dst = Cg + (i * 8 + g) * N + j * 8 + 2 * t;
+        double r0 = c[i][j][0], r1 = c[i][j][1];
+        if (prm.beta != 0.0) {
+          const double2 o = *reinterpret_cast<const double2*>(dst);
+          r0 = fma(prm.beta, o.x, prm.alpha * r0);
+          r1 = fma(prm.beta, o.y, prm.alpha * r1);
+        } else if (prm.alpha != 1.0) {
+          r0 *= prm.alpha;
+          r1 *= prm.alpha;
+        }
+        ptx::st_global_v2_f64(dst, r0, r1);
+      }
     ptx::named_bar_sync(bar, P * 32);  // buffer s free for entry it+2
   }
 }
 
 template <int M, int N, int K, int P, int TEAMS>
-kami_status_t launch(long long batch, const void* A, const void* B, void* C, cudaStream_t stream, const char* name) {
+kami_status_t launch(long long batch, const void* A, const void* B, void* C, cudaStream_t stream, const char* name,
+                     double alpha, double beta) {
   using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
   PFN_encodeTiled enc = get_encode_tiled();
   if (!enc) return KAMI_ERROR_CUDA;
@@ -148,6 +162,8 @@ kami_status_t launch(long long batch, const void* A, const void* B, void* C, cud
   prm.B = static_cast<const double*>(B);
   prm.C = static_cast<double*>(C);
   prm.batch = batch;
+  prm.alpha = alpha;
+  prm.beta = beta;
   auto fn = kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS>;
   if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM) != cudaSuccess)
     return KAMI_ERROR_CUDA;
@@ -171,23 +187,23 @@ bool dmma_tma_supported(int m, int n, int k) { return m == n && n == k && (m == 
 
 // (p, teams) configuration; env KAMI_DMMA_TMA_CFG = 0/1/2 picks an alternative for sweeps
 kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
-                              cudaStream_t stream) {
+                              cudaStream_t stream, double alpha, double beta) {
   static const int cfg = [] {
     const char* e = getenv("KAMI_DMMA_TMA_CFG");
     return e ? atoi(e) : 0;
   }();
   if (m == 64 && n == 64 && k == 64) {
-    if (cfg == 1) return launch<64, 64, 64, 8, 2>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,p8>");
-    return launch<64, 64, 64, 4, 3>(batch, A, B, C, stream, "kami_dmma_tma_1d<64>");
+    if (cfg == 1) return launch<64, 64, 64, 8, 2>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,p8>", alpha, beta);
+    return launch<64, 64, 64, 4, 3>(batch, A, B, C, stream, "kami_dmma_tma_1d<64>", alpha, beta);
   }
   if (m == 32 && n == 32 && k == 32) {
-    if (cfg == 1) return launch<32, 32, 32, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,p2>");
-    if (cfg == 2) return launch<32, 32, 32, 4, 6>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,t6>");
-    return launch<32, 32, 32, 4, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32>");
+    if (cfg == 1) return launch<32, 32, 32, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,p2>", alpha, beta);
+    if (cfg == 2) return launch<32, 32, 32, 4, 6>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,t6>", alpha, beta);
+    return launch<32, 32, 32, 4, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32>", alpha, beta);
   }
   if (m == 16 && n == 16 && k == 16) {
-    if (cfg == 1) return launch<16, 16, 16, 1, 16>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,p1>");
-    return launch<16, 16, 16, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<16>");
+    if (cfg == 1) return launch<16, 16, 16, 1, 16>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,p1>", alpha, beta);
+    return launch<16, 16, 16, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<16>", alpha, beta);
   }
   return KAMI_ERROR_NOT_SUPPORTED;
 }

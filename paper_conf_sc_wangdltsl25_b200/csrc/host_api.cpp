@@ -59,8 +59,10 @@ extern "C" kami_status_t kami_gemm_strided_batched_host(int m, int n, int k, int
   if (st != KAMI_SUCCESS) return st;
   if (batch == 0) return KAMI_SUCCESS;
   if (!A || !B || !C) return KAMI_ERROR_INVALID_VALUE;
-  const size_t es = dtype == KAMI_DTYPE_F64 ? 8 : 2;
-  const size_t ea = (size_t)m * k * es, eb = (size_t)k * n * es, ec = (size_t)m * n * es;
+  const size_t esi = dtype == KAMI_DTYPE_F64 ? 8 : dtype == KAMI_DTYPE_TF32 ? 4
+                    : (dtype == KAMI_DTYPE_E4M3 || dtype == KAMI_DTYPE_E5M2) ? 1 : 2;
+  const size_t eso = dtype == KAMI_DTYPE_F64 ? 8 : dtype == KAMI_DTYPE_TF32 ? 4 : 2;
+  const size_t ea = (size_t)m * k * esi, eb = (size_t)k * n * esi, ec = (size_t)m * n * eso;
   const size_t per_entry = ea + eb + ec;
   // ~64 MiB per chunk: large enough to amortise launches, small enough to pipeline
   int64_t chunk = (int64_t)((64ull << 20) / per_entry);

@@ -29,6 +29,11 @@ struct Tc16Shape {
 kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s);
 kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B, void* C,
                           cudaStream_t stream, int max_ctas);
+// in_kind: 0 f16, 1 bf16, 2 tf32, 3 e4m3, 4 e5m2; out_kind: 0 f16, 1 bf16, 2 f32.
+// C = alpha A B + beta C (C is read iff beta != 0).
+kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kind, Tc16Shape* s);
+kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind, int out_kind, const void* A,
+                               const void* B, void* C, float alpha, float beta, cudaStream_t stream, int max_ctas);
 
 // ------------------------------------------------ warp-level CA (literal KAMI)
 // algo: 1 = 1D, 2 = 2D, 3 = 3D, 4 = non-CA tiled.  dtype: KAMI_DTYPE_*.
@@ -46,7 +51,7 @@ kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t 
 // ------------------------------------------- FP64 1D with TMA-fed broadcast
 bool dmma_tma_supported(int m, int n, int k);
 kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
-                              cudaStream_t stream);
+                              cudaStream_t stream, double alpha = 1.0, double beta = 0.0);
 
 // ------------------------- 16-bit pointer-array / variable-size (tc16_vb.cu)
 // dm/dn/dk: device arrays of per-entry sizes, or nullptr for uniform m, n, k.

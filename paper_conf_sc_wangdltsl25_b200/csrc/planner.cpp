@@ -102,14 +102,17 @@ double calibrated_tma(int m) { return m == 16 ? 7.42 : m == 32 ? 15.02 : m == 64
 kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_t algo, int p, bool pointer_array,
                              kami_plan_t* out) {
   kami_plan_t r{};
-  const bool is16 = dtype != KAMI_DTYPE_F64;
+  const bool is16 = dtype != KAMI_DTYPE_F64;  // all tcgen05 types (f16, bf16, tf32, fp8)
   // 16-bit strided: the tcgen05 family implements 1D with p = 4 sub-partition
   // tensor cores (tc16.cu); it covers the whole 16-bit size grid.  An explicit
   // p > 0 selects the warp-level family with p warps instead.
   if (is16 && !pointer_array &&
       (algo == KAMI_ALGO_AUTO || algo == KAMI_ALGO_1D_TMA || (algo == KAMI_ALGO_1D && p == 0))) {
     Tc16Shape s;
-    kami_status_t st = tc16_plan_shape(m, n, k, &s);
+    const int ik = dtype == KAMI_DTYPE_F16 ? 0 : dtype == KAMI_DTYPE_BF16 ? 1 : dtype == KAMI_DTYPE_TF32 ? 2
+                 : dtype == KAMI_DTYPE_E4M3 ? 3 : 4;
+    const int ok = dtype == KAMI_DTYPE_BF16 ? 1 : dtype == KAMI_DTYPE_TF32 ? 2 : 0;
+    kami_status_t st = tc16_plan_shape_kind(m, n, k, ik, ok, &s);
     if (st != KAMI_SUCCESS) return st;
     r.algo = KAMI_ALGO_1D;
     r.p = 4;

@@ -230,6 +230,21 @@ __host__ __device__ __forceinline__ uint32_t make_idesc_f16(int is_bf16, int M, 
   return d;
 }
 
+// Instruction descriptor with explicit operand formats: kind::tf32 (fmt 2 =
+// TF32) and kind::f8f6f4 (fmt 0 = E4M3, 1 = E5M2), fp32 accumulation.
+__host__ __device__ __forceinline__ uint32_t make_idesc_fmt(int a_fmt, int b_fmt, int M, int N, int a_mn_major,
+                                                             int b_mn_major) {
+  uint32_t d = 0;
+  d |= 1u << 4;
+  d |= (uint32_t)(a_fmt & 7) << 7;
+  d |= (uint32_t)(b_fmt & 7) << 10;
+  d |= (uint32_t)(a_mn_major & 1) << 15;
+  d |= (uint32_t)(b_mn_major & 1) << 16;
+  d |= (uint32_t)((N >> 3) & 0x3F) << 17;
+  d |= (uint32_t)((M >> 4) & 0x1F) << 24;
+  return d;
+}
+
 // Swizzle<B,4,3> on a byte offset inside a 1024-B aligned region: XOR the
 // 16-byte chunk index (bits [4,4+B)) with bits [7,7+B).  B = log2(sw/16).
 __device__ __forceinline__ uint32_t swz(uint32_t off, uint32_t bbits) {
@@ -263,6 +278,11 @@ __device__ __forceinline__ void st_global_b32(void* p, uint32_t v) {
 
 __device__ __forceinline__ void ld_shared_v4(uint32_t addr, uint32_t& a, uint32_t& b, uint32_t& c, uint32_t& d) {
   asm volatile("ld.shared.v4.b32 {%0, %1, %2, %3}, [%4];" : "=r"(a), "=r"(b), "=r"(c), "=r"(d) : "r"(addr) : "memory");
+}
+__device__ __forceinline__ uint32_t ld_shared_u32(uint32_t addr) {
+  uint32_t v;
+  asm volatile("ld.shared.b32 %0, [%1];" : "=r"(v) : "r"(addr) : "memory");
+  return v;
 }
 __device__ __forceinline__ void st_shared_v4(uint32_t addr, uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
   asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c), "r"(d)

@@ -1,6 +1,7 @@
-// tc16.cu -- FP16/BF16 batched small GEMM on 5th-generation tensor cores
-// (tcgen05 + TMEM + TMA), sm_100a.  Hot path of BASELINE.json configs 0, 1,
-// 3 and 4.
+// tc16.cu -- batched small GEMM on 5th-generation tensor cores (tcgen05 +
+// TMEM + TMA), sm_100a.  Hot path of BASELINE.json configs 0, 1, 3 and 4
+// (FP16 / BF16 in, FP32 accumulate) and of the f4 extensions (TF32 in / FP32
+// out, FP8 E4M3 / E5M2 in / FP16 out, C = alpha A B + beta C).
 //
 // KAMI mapping (Table 1):
 //   compute unit  = one SM sub-partition tensor core (n_tc = 4 per SM).  A
@@ -11,7 +12,7 @@
 //   communication = shared memory: the B tile is written once (TMA) and
 //                   broadcast to all four units by every MMA -- KAMI-1D
 //                   (Alg. 1) with p = 4, where stage z of Alg. 1 is
-//                   the z-th K=16 slice (k-slicing, Sec. 4.7).
+//                   the z-th 32-byte K slice (k-slicing, Sec. 4.7).
 //   batching      = G = min(128/m, 256/n) entries packed block-diagonally
 //                   into one 128 x (G n) MMA tile: entry g's A rows occupy
 //                   TMEM lanes [g m, g m + m) and its B columns [g n, g n + n),
@@ -24,13 +25,24 @@
 //   warp 0     TMA producer: per (unit, k-chunk) one 3-D box of A (K-major,
 //              swizzled) and one 4-D box of B (N-major, swizzled) into an
 //              S-stage shared-memory ring guarded by full/empty mbarriers.
-//   warp 1     MMA issuer (one lane) + TMEM allocator: tcgen05.mma
-//              kind::f16, accumulators double/quad-buffered in TMEM,
-//              tcgen05.commit -> empty[s] (frees the stage) and tfull[a].
+//   warp 1     MMA issuer (one lane) + TMEM allocator: tcgen05.mma,
+//              accumulators double/quad-buffered in TMEM, tcgen05.commit ->
+//              empty[s] (frees the stage) and tfull[a].
 //   warps 2-9  epilogue, two warpgroups on alternate units: tcgen05.ld
-//              32x32b, cvt.rn to fp16/bf16, swizzled conflict-free st.shared
-//              into a C staging tile, one TMA tensor store per unit.
+//              32x32b, (beta != 0: TMA-load the old C tile into the staging
+//              buffer first), alpha/beta, cvt.rn, swizzled conflict-free
+//              st.shared into the C staging tile, one TMA tensor store.
+//              FP32 output (TF32 inputs): alpha/beta and 32-byte full-sector
+//              st.global straight from registers (a 128 x 256 FP32 staging
+//              tile per warpgroup would not fit next to the ring).
+//   warps 10-13 (TF32 only) B transposer.  kind::tf32 reads both operands
+//              K-major only (an MN-major B descriptor yields zeros on sm_100a,
+//              DESIGN.md R25), and TMA cannot transpose 4-byte elements, so
+//              B lands N-major in a raw slot of the stage and these warps
+//              rewrite it K-major (SW-swizzled, same canonical layout as A)
+//              before arriving on bready[s], which the MMA issuer waits on.
 #include <cuda.h>
+#include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
 #include <cstring>
@@ -43,9 +55,23 @@ namespace kami {
 namespace {
 
 constexpr int kThreads = 320;  // 10 warps: TMA, MMA, 2 x 4 epilogue
+constexpr int kXposeThreads = 128;  // TF32: 4 more warps transpose B
 constexpr int kEpiThreads = 128;
 constexpr int kMaxStages = 8;
 constexpr int kMaxAcc = 4;
+
+// input kinds (A, B) and output kinds (C)
+enum { IN_F16 = 0, IN_BF16 = 1, IN_TF32 = 2, IN_E4M3 = 3, IN_E5M2 = 4 };
+enum { OUT_F16 = 0, OUT_BF16 = 1, OUT_F32 = 2 };
+template <int kIn>
+struct InTraits {
+  static constexpr int ES = kIn == IN_TF32 ? 4 : (kIn >= IN_E4M3 ? 1 : 2);
+};
+constexpr int threads_for(int in) { return kThreads + (in == IN_TF32 ? kXposeThreads : 0); }
+template <int kOut>
+struct OutTraits {
+  static constexpr int ES = kOut == OUT_F32 ? 4 : 2;
+};
 
 struct alignas(64) Tc16Params {
   CUtensorMap tmA;  // 3-D (k, m, batch), box (Wk, rowsA, G)
@@ -55,23 +81,134 @@ struct alignas(64) Tc16Params {
   long long units;
   int m, n, k;
   int G, m_tiles, rows_tile;
-  int k_chunks, Wk, Wn, Wc;
+  int k_chunks, Wk, Wn, Wc;  // atom widths in ELEMENTS of their operand
   int ksteps_full, ksteps_last;
   int N_mma;
   uint32_t idesc;
   uint32_t a_layout, b_layout, c_swz_bits;
-  uint32_t a_sbo, b_lbo, b_sbo;
-  uint32_t a_region, stage_bytes, tx_bytes;
+  uint32_t a_sbo, b_lbo, b_sbo, b_kstep;  // bytes
+  uint32_t a_region, stage_bytes, tx_bytes, c_tx_bytes;
   int stages;
   int acc_cols, acc_bufs, tmem_cols;
   uint32_t c_buf_bytes;
   int c_bufs;
   uint32_t c_off;    // byte offset of C staging
   uint32_t bar_off;  // byte offset of barriers
+  float alpha, beta;
+  uint32_t b_raw_off;       // TF32: byte offset in the stage of the N-major raw B slot
+  uint32_t raw_swz_bits, k_swz_bits;
+  int wn_b, wk_b;           // atom widths in bytes
+  void* Cg;                 // FP32 output: direct stores
+  int scale;  // 0: C = AB, 1: C = alpha AB, 2: C = alpha AB + beta C (C read)
 };
 
-template <bool kBF16>
-__global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_constant__ Tc16Params p) {
+template <int kIn>
+__device__ __forceinline__ void umma(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
+  if constexpr (kIn == IN_TF32) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc)
+        : "memory");
+  } else if constexpr (kIn >= IN_E4M3) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::f8f6f4 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
+        "l"(a), "l"(b), "r"(idesc), "r"(acc)
+        : "memory");
+  } else {
+    ptx::umma_f16_ss(d, a, b, idesc, acc);
+  }
+}
+
+// 8 fp32 accumulators -> the output type, written as 16-byte chunks of the
+// swizzled staging tile.  `off` is the unswizzled byte offset of the first
+// element; old values (beta != 0) are read from the same locations.
+template <int kOut>
+__device__ __forceinline__ void emit8(uint32_t cbase, uint32_t off, uint32_t swz_bits, const uint32_t* v,
+                                      const Tc16Params& p) {
+  float x[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) x[i] = __uint_as_float(v[i]);
+  if (p.scale) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) x[i] *= p.alpha;
+  }
+  if constexpr (kOut == OUT_F32) {
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      const uint32_t a = cbase + ptx::swz(off + 16 * h, swz_bits);
+      if (p.scale == 2) {
+        uint32_t o0, o1, o2, o3;
+        ptx::ld_shared_v4(a, o0, o1, o2, o3);
+        x[4 * h + 0] = fmaf(p.beta, __uint_as_float(o0), x[4 * h + 0]);
+        x[4 * h + 1] = fmaf(p.beta, __uint_as_float(o1), x[4 * h + 1]);
+        x[4 * h + 2] = fmaf(p.beta, __uint_as_float(o2), x[4 * h + 2]);
+        x[4 * h + 3] = fmaf(p.beta, __uint_as_float(o3), x[4 * h + 3]);
+      }
+      ptx::st_shared_v4(a, __float_as_uint(x[4 * h + 0]), __float_as_uint(x[4 * h + 1]),
+                        __float_as_uint(x[4 * h + 2]), __float_as_uint(x[4 * h + 3]));
+    }
+  } else {
+    const uint32_t a = cbase + ptx::swz(off, swz_bits);
+    if (p.scale == 2) {
+      uint32_t o[4];
+      ptx::ld_shared_v4(a, o[0], o[1], o[2], o[3]);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        float lo, hi;
+        if (kOut == OUT_BF16) {
+          lo = __uint_as_float(o[i] << 16);
+          hi = __uint_as_float(o[i] & 0xffff0000u);
+        } else {
+          const __half2 h2 = *reinterpret_cast<const __half2*>(&o[i]);
+          lo = __low2float(h2);
+          hi = __high2float(h2);
+        }
+        x[2 * i] = fmaf(p.beta, lo, x[2 * i]);
+        x[2 * i + 1] = fmaf(p.beta, hi, x[2 * i + 1]);
+      }
+    }
+    uint32_t w[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+      w[i] = kOut == OUT_BF16 ? ptx::pack_bf16x2(x[2 * i], x[2 * i + 1]) : ptx::pack_f16x2(x[2 * i], x[2 * i + 1]);
+    ptx::st_shared_v4(a, w[0], w[1], w[2], w[3]);
+  }
+}
+
+// FP32 output: 8 accumulators -> 32 contiguous bytes of C (one full sector).
+__device__ __forceinline__ void emit8_f32_global(float* dst, const uint32_t* v, const Tc16Params& p) {
+  float x[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) x[i] = __uint_as_float(v[i]);
+  if (p.scale) {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) x[i] *= p.alpha;
+  }
+  if (p.scale == 2) {
+    const float4 o0 = *reinterpret_cast<const float4*>(dst);
+    const float4 o1 = *reinterpret_cast<const float4*>(dst + 4);
+    x[0] = fmaf(p.beta, o0.x, x[0]);
+    x[1] = fmaf(p.beta, o0.y, x[1]);
+    x[2] = fmaf(p.beta, o0.z, x[2]);
+    x[3] = fmaf(p.beta, o0.w, x[3]);
+    x[4] = fmaf(p.beta, o1.x, x[4]);
+    x[5] = fmaf(p.beta, o1.y, x[5]);
+    x[6] = fmaf(p.beta, o1.z, x[6]);
+    x[7] = fmaf(p.beta, o1.w, x[7]);
+  }
+  ptx::st_global_v4(dst, make_uint4(__float_as_uint(x[0]), __float_as_uint(x[1]), __float_as_uint(x[2]),
+                                    __float_as_uint(x[3])));
+  ptx::st_global_v4(dst + 4, make_uint4(__float_as_uint(x[4]), __float_as_uint(x[5]), __float_as_uint(x[6]),
+                                        __float_as_uint(x[7])));
+}
+
+template <int kIn, int kOut>
+__global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const __grid_constant__ Tc16Params p) {
+  constexpr bool kXpose = kIn == IN_TF32;
+  constexpr bool kDirect = kOut == OUT_F32;
+  constexpr int ESO = OutTraits<kOut>::ES;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-byte alignment for the 128B swizzle atoms
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -79,7 +216,9 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
   uint64_t* empty = full + kMaxStages;
   uint64_t* tfull = empty + kMaxStages;
   uint64_t* tempty = tfull + kMaxAcc;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + kMaxAcc);
+  uint64_t* cfull = tempty + kMaxAcc;  // [2 warpgroups][2 staging buffers]: old C landed
+  uint64_t* bready = cfull + 4;  // TF32: K-major B of stage s written
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bready + kMaxStages);
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -91,11 +230,13 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
     for (int s = 0; s < p.stages; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
+      ptx::mbar_init(&bready[s], kXposeThreads);
     }
     for (int a = 0; a < p.acc_bufs; ++a) {
       ptx::mbar_init(&tfull[a], 1);
       ptx::mbar_init(&tempty[a], kEpiThreads / 32);
     }
+    for (int c = 0; c < 4; ++c) ptx::mbar_init(&cfull[c], 1);
     ptx::fence_mbar_init();
     ptx::fence_proxy_async_smem();
   }
@@ -123,7 +264,7 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
           uint8_t* sa = smem + s * p.stage_bytes;
           uint8_t* sb = sa + p.a_region;
           ptx::tma_load_3d(sa, &p.tmA, &full[s], kc * p.Wk, mt * 128, e0);
-          ptx::tma_load_4d(sb, &p.tmB, &full[s], 0, kc * p.Wk, 0, e0);
+          ptx::tma_load_4d(kXpose ? sa + p.b_raw_off : sb, &p.tmB, &full[s], 0, kc * p.Wk, 0, e0);
         }
       }
     }
@@ -139,18 +280,19 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
       for (int kc = 0; kc < p.k_chunks; ++kc, ++it) {
         const uint32_t s = it % p.stages;
         const uint32_t ph = (it / p.stages) & 1;
-        ptx::mbar_wait(&full[s], ph);
+        ptx::mbar_wait(kXpose ? &bready[s] : &full[s], ph);
         ptx::tc_fence_after();
         if (lane == 0) {
           const uint32_t sa = smem_base + s * p.stage_bytes;
           const uint32_t sb = sa + p.a_region;
           const int nsteps = (kc == p.k_chunks - 1) ? p.ksteps_last : p.ksteps_full;
           for (int ks = 0; ks < nsteps; ++ks) {
-            // A: K-major, 16 elements = 32 bytes further along the swizzled row
+            // A: K-major, one K step = 32 bytes further along the swizzled row
             const uint64_t adesc = ptx::make_smem_desc(sa + ks * 32, 16, p.a_sbo, p.a_layout);
-            // B: N-major, 16 K-rows further = 2 core-row groups
-            const uint64_t bdesc = ptx::make_smem_desc(sb + ks * 2 * p.b_sbo, p.b_lbo, p.b_sbo, p.b_layout);
-            ptx::umma_f16_ss(d_tmem, adesc, bdesc, p.idesc, (kc | ks) != 0);
+            // B: N-major, one K step = 32 bytes of K = 32/es rows further
+            // (TF32: K-major like A, one K step = 32 bytes along the row)
+            const uint64_t bdesc = ptx::make_smem_desc(sb + ks * p.b_kstep, p.b_lbo, p.b_sbo, p.b_layout);
+            umma<kIn>(d_tmem, adesc, bdesc, p.idesc, (kc | ks) != 0);
           }
           ptx::umma_commit(&empty[s]);  // stage s may be refilled once these MMAs retire
         }
@@ -158,6 +300,38 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
       }
       if (lane == 0) ptx::umma_commit(&tfull[a]);  // accumulator a complete
       __syncwarp();
+    }
+  } else if (kXpose && warp >= kThreads / 32) {
+    // ------------------------------------------------- TF32 B transposer
+    // raw (N-major) element (kk, c) of the stage: atom c / Wn, row kk:
+    //   ((c / Wn) Wk + kk) wn_b + (c % Wn) 4    [swizzled with raw_swz_bits]
+    // K-major element (c, kk): c wk_b + 4 kk  [swizzled with k_swz_bits]
+    // Thread t takes columns c = t, t + 128, ... (conflict-free 4-byte reads
+    // along a raw row) and 4 consecutive kk (one 16-byte K-major chunk).
+    const int t = threadIdx.x - kThreads;
+    const int wn_shift = 31 - __clz(p.Wn);
+    const int kq = p.Wk >> 2;
+    uint32_t it = 0;
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
+      for (int kc = 0; kc < p.k_chunks; ++kc, ++it) {
+        const uint32_t s = it % p.stages;
+        const uint32_t ph = (it / p.stages) & 1;
+        ptx::mbar_wait(&full[s], ph);
+        const uint32_t raw = smem_base + s * p.stage_bytes + p.b_raw_off;
+        const uint32_t dst = smem_base + s * p.stage_bytes + p.a_region;
+        for (int c = t; c < p.N_mma; c += kXposeThreads) {
+          const uint32_t cbase = (uint32_t)((c >> wn_shift) * p.Wk) * p.wn_b + (uint32_t)(c & (p.Wn - 1)) * 4;
+          for (int q = 0; q < kq; ++q) {
+            uint32_t w[4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) w[j] = ptx::ld_shared_u32(raw + ptx::swz(cbase + (4 * q + j) * p.wn_b,
+                                                                                  p.raw_swz_bits));
+            ptx::st_shared_v4(dst + ptx::swz((uint32_t)c * p.wk_b + 16 * q, p.k_swz_bits), w[0], w[1], w[2], w[3]);
+          }
+        }
+        ptx::fence_proxy_async_smem();  // generic writes -> the MMA's async-proxy reads
+        ptx::mbar_arrive(&bready[s]);
+      }
     }
   } else {
     // ------------------------------------------------------------ epilogue
@@ -188,10 +362,10 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
       col_hi = (sp * 32 < p.rows_tile) ? p.n : 0;
     }
     const int my_lo = g * p.n, my_hi = my_lo + p.n;
-    const uint32_t row_bytes = (uint32_t)p.Wc * 2;
+    const uint32_t row_bytes = (uint32_t)p.Wc * ESO;
     const uint32_t atom_stride = (uint32_t)p.rows_tile * row_bytes;
     const uint32_t rowbase = (uint32_t)(g * (p.n / p.Wc) * p.rows_tile + r) * row_bytes;
-    const int wc_shift = p.Wc == 64 ? 6 : p.Wc == 32 ? 5 : 4;
+    const int wc_shift = 31 - __clz(p.Wc);
     const uint32_t c_smem = smem_base + p.c_off + (uint32_t)wg * p.c_bufs * p.c_buf_bytes;
     uint32_t i = wg, local = 0;
     for (long long u = blockIdx.x + (long long)wg * gridDim.x; u < p.units;
@@ -204,13 +378,22 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
       const uint32_t cb = local % p.c_bufs;
       const bool valid = row_ok && (e0 + g < p.batch) && (p.G > 1 || mt * 128 + L < p.m);
       // the TMA store that last read staging buffer cb must be done reading
-      if (leader) {
+      if (!kDirect && leader) {
         if (p.c_bufs == 2) ptx::bulk_wait_read<1>();
         else ptx::bulk_wait_read<0>();
+        if (p.scale == 2) {  // C update: bring the old C tile into the staging buffer
+          uint64_t* cf = &cfull[wg * 2 + cb];
+          ptx::mbar_arrive_expect_tx(cf, p.c_tx_bytes);
+          ptx::tma_load_4d(smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, &p.tmC, cf, 0, mt * 128, 0,
+                           (int)e0);
+        }
       }
       ptx::named_bar_sync(bar_id, kEpiThreads);
       ptx::mbar_wait(&tfull[a], aph);
       ptx::tc_fence_after();
+      if (!kDirect && p.scale == 2) ptx::mbar_wait(&cfull[wg * 2 + cb], (local / p.c_bufs) & 1);
+      float* crow = nullptr;
+      if constexpr (kDirect) crow = reinterpret_cast<float*>(p.Cg) + ((e0 + g) * p.m + mt * 128 + r) * (long long)p.n;
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
       const uint32_t cbase = c_smem + cb * p.c_buf_bytes;
       for (int c0 = col_lo; c0 < col_hi; c0 += 64) {
@@ -234,22 +417,13 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
           const int col = c0 + 8 * q;
           if (valid && col >= my_lo && col < my_hi && col < col_hi) {
             const uint32_t jc = (uint32_t)(col - my_lo);
-            const uint32_t atom = jc >> wc_shift;
-            const uint32_t ce = jc & (uint32_t)(p.Wc - 1);
-            const uint32_t off = ptx::swz(rowbase + atom * atom_stride + ce * 2, p.c_swz_bits);
-            uint32_t w0, w1, w2, w3;
-            if (kBF16) {
-              w0 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
-              w1 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
-              w2 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
-              w3 = ptx::pack_bf16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
+            if constexpr (kDirect) {
+              emit8_f32_global(crow + jc, &v[8 * q], p);
             } else {
-              w0 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 0]), __uint_as_float(v[8 * q + 1]));
-              w1 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 2]), __uint_as_float(v[8 * q + 3]));
-              w2 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 4]), __uint_as_float(v[8 * q + 5]));
-              w3 = ptx::pack_f16x2(__uint_as_float(v[8 * q + 6]), __uint_as_float(v[8 * q + 7]));
+              const uint32_t atom = jc >> wc_shift;
+              const uint32_t ce = jc & (uint32_t)(p.Wc - 1);
+              emit8<kOut>(cbase, rowbase + atom * atom_stride + ce * ESO, p.c_swz_bits, &v[8 * q], p);
             }
-            ptx::st_shared_v4(cbase + off, w0, w1, w2, w3);
           }
         }
       }
@@ -257,6 +431,7 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[a]);
+      if constexpr (kDirect) continue;
       // make the generic-proxy smem writes visible to the TMA engine
       ptx::fence_proxy_async_smem();
       ptx::named_bar_sync(bar_id, kEpiThreads);
@@ -265,7 +440,7 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
         ptx::bulk_commit();
       }
     }
-    if (leader) ptx::bulk_wait<0>();
+    if (!kDirect && leader) ptx::bulk_wait<0>();
   }
 
   ptx::tc_fence_before();
@@ -276,15 +451,16 @@ __global__ void __launch_bounds__(kThreads, 1) kami_tc16_1d_kernel(const __grid_
 
 // ------------------------------------------------------------------- host
 
-int pick_atom(int elems) {  // largest swizzle atom width (elements) dividing elems
-  if (elems % 64 == 0) return 64;
-  if (elems % 32 == 0) return 32;
-  return 16;
+int pick_atom_bytes(int bytes) {  // largest swizzle atom (bytes) dividing the row bytes
+  if (bytes % 128 == 0) return 128;
+  if (bytes % 64 == 0) return 64;
+  if (bytes % 32 == 0) return 32;
+  return 0;
 }
-int swz_bits_for(int atom_elems) { return atom_elems == 64 ? 3 : atom_elems == 32 ? 2 : 1; }
-CUtensorMapSwizzle swz_mode_for(int atom_elems) {
-  return atom_elems == 64 ? CU_TENSOR_MAP_SWIZZLE_128B
-         : atom_elems == 32 ? CU_TENSOR_MAP_SWIZZLE_64B
+int swz_bits_for(int atom_bytes) { return atom_bytes == 128 ? 3 : atom_bytes == 64 ? 2 : 1; }
+CUtensorMapSwizzle swz_mode_for(int atom_bytes) {
+  return atom_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+         : atom_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
                             : CU_TENSOR_MAP_SWIZZLE_32B;
 }
 uint32_t align_up(uint32_t x, uint32_t a) { return (x + a - 1) / a * a; }
@@ -293,12 +469,22 @@ int pow2_ceil(int x) {
   while (p < x) p <<= 1;
   return p;
 }
+int in_es(int in) { return in == IN_TF32 ? 4 : (in >= IN_E4M3 ? 1 : 2); }
+int out_es(int out) { return out == OUT_F32 ? 4 : 2; }
 
 constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 
+template <int kIn, int kOut>
+void launch_kernel(const Tc16Params& p, unsigned grid, size_t smem, cudaStream_t stream, const char* name) {
+  cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  kami_tc16_1d_kernel<kIn, kOut><<<grid, threads_for(kIn), smem, stream>>>(p);
+  set_last_kernel(name);
+}
+
 }  // namespace
 
-kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s) {
+kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kind, Tc16Shape* s) {
+  const int esi = in_es(in_kind), eso = out_es(out_kind);
   s->G = 1;
   if (m <= 128) {
     int g1 = 128 / m, g2 = 256 / n;
@@ -307,16 +493,21 @@ kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s) {
   }
   s->m_tiles = (s->G > 1 || m <= 128) ? 1 : (m + 127) / 128;
   s->rows_tile = m < 128 ? m : 128;
-  const int kpad = (k + 15) / 16 * 16;
-  s->Wk = pick_atom(kpad);
-  s->Wn = pick_atom(n);
-  s->Wc = s->Wn;
+  const int kgran = 32 / esi;  // elements per 32-byte MMA K step
+  const int kpad = (k + kgran - 1) / kgran * kgran;
+  const int wk_b = pick_atom_bytes(kpad * esi), wn_b = pick_atom_bytes(n * esi), wc_b = pick_atom_bytes(n * eso);
+  if (!wk_b || !wn_b || !wc_b) return KAMI_ERROR_NOT_SUPPORTED;
+  s->Wk = wk_b / esi;
+  s->Wn = wn_b / esi;
+  s->Wc = wc_b / eso;
   s->k_chunks = (kpad + s->Wk - 1) / s->Wk;
   s->N_mma = s->G > 1 ? s->G * n : n;
-  const uint32_t a_region = align_up(128u * s->Wk * 2, 1024);
-  const uint32_t b_region = align_up((uint32_t)s->N_mma * s->Wk * 2, 1024);
-  s->stage_bytes = a_region + b_region;
-  s->c_buf_bytes = align_up((uint32_t)s->G * n * s->rows_tile * 2, 1024);
+  const uint32_t a_region = align_up(128u * wk_b, 1024);
+  const uint32_t b_region = align_up((uint32_t)s->N_mma * wk_b, 1024);
+  // TF32: + the raw N-major B slot the transposer reads
+  s->stage_bytes = a_region + b_region * (in_kind == IN_TF32 ? 2 : 1);
+  // FP32 output is stored straight from registers (no staging)
+  s->c_buf_bytes = out_kind == OUT_F32 ? 0 : align_up((uint32_t)s->G * n * s->rows_tile * eso, 1024);
   // two epilogue warpgroups, each with c_bufs staging tiles
   s->c_bufs = (4 * s->c_buf_bytes <= 64 * 1024) ? 2 : 1;
   const int budget = kSmemLimit - 1024 /*align slack*/ - 1024 /*barriers*/;
@@ -331,13 +522,18 @@ kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s) {
   return st >= 2 ? KAMI_SUCCESS : KAMI_ERROR_NOT_SUPPORTED;
 }
 
-kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B, void* C,
-                          cudaStream_t stream, int max_ctas) {
+kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s) {
+  return tc16_plan_shape_kind(m, n, k, IN_F16, OUT_F16, s);
+}
+
+kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind, int out_kind, const void* A,
+                               const void* B, void* C, float alpha, float beta, cudaStream_t stream, int max_ctas) {
   Tc16Shape s;
-  kami_status_t st = tc16_plan_shape(m, n, k, &s);
+  kami_status_t st = tc16_plan_shape_kind(m, n, k, in_kind, out_kind, &s);
   if (st != KAMI_SUCCESS) return st;
   PFN_encodeTiled enc = get_encode_tiled();
   if (!enc) return KAMI_ERROR_CUDA;
+  const int esi = in_es(in_kind), eso = out_es(out_kind);
 
   Tc16Params p;
   memset(&p, 0, sizeof(p));
@@ -352,22 +548,46 @@ kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const
   p.Wk = s.Wk;
   p.Wn = s.Wn;
   p.Wc = s.Wc;
-  const int kpad = (k + 15) / 16 * 16;
-  p.ksteps_full = s.Wk / 16;
-  p.ksteps_last = (kpad - (s.k_chunks - 1) * s.Wk) / 16;
+  const int wk_b = s.Wk * esi, wn_b = s.Wn * esi, wc_b = s.Wc * eso;
+  const int kgran = 32 / esi;
+  const int kpad = (k + kgran - 1) / kgran * kgran;
+  p.ksteps_full = wk_b / 32;
+  p.ksteps_last = (kpad - (s.k_chunks - 1) * s.Wk) / kgran;
   p.N_mma = s.N_mma;
-  p.idesc = ptx::make_idesc_f16(bf16 ? 1 : 0, 128, s.N_mma, /*a MN-major*/ 0, /*b MN-major*/ 1);
-  p.a_layout = ptx::umma_layout_code(s.Wk * 2);
-  p.b_layout = ptx::umma_layout_code(s.Wn * 2);
-  p.c_swz_bits = swz_bits_for(s.Wc);
-  p.a_sbo = 8 * s.Wk * 2;          // 8 rows of the K-major A tile
-  p.b_sbo = 8 * s.Wn * 2;          // 8 K-rows of one N-atom
-  p.b_lbo = s.Wk * s.Wn * 2;       // next N-atom (next 64/32/16 columns)
-  p.a_region = align_up(128u * s.Wk * 2, 1024);
+  if (in_kind == IN_TF32) {
+    p.idesc = ptx::make_idesc_fmt(2, 2, 128, s.N_mma, 0, 0);  // both K-major (R25)
+  } else if (in_kind >= IN_E4M3) {
+    const int f = in_kind == IN_E5M2 ? 1 : 0;
+    p.idesc = ptx::make_idesc_fmt(f, f, 128, s.N_mma, 0, 1);
+  } else {
+    p.idesc = ptx::make_idesc_f16(in_kind == IN_BF16 ? 1 : 0, 128, s.N_mma, /*a MN-major*/ 0, /*b MN-major*/ 1);
+  }
+  if (const char* e = getenv("KAMI_TC_IDESC_XOR")) p.idesc ^= (uint32_t)strtoul(e, nullptr, 0);  // debug
+  p.a_layout = ptx::umma_layout_code(wk_b);
+  p.b_layout = ptx::umma_layout_code(wn_b);
+  p.c_swz_bits = swz_bits_for(wc_b);
+  p.a_sbo = 8 * wk_b;                      // 8 rows of the K-major A tile
+  p.b_sbo = 8 * wn_b;                      // 8 K-rows of one N-atom
+  p.b_lbo = s.Wk * wn_b;                   // next N-atom
+  p.b_kstep = (uint32_t)(kgran / 8) * p.b_sbo;  // one 32-byte K step of B rows
+  p.a_region = align_up(128u * wk_b, 1024);
+  p.wn_b = wn_b;
+  p.wk_b = wk_b;
+  p.raw_swz_bits = swz_bits_for(wn_b);
+  p.k_swz_bits = swz_bits_for(wk_b);
+  p.Cg = C;
+  if (in_kind == IN_TF32) {  // B is transposed in shared memory to K-major (same geometry as A)
+    p.b_raw_off = p.a_region + align_up((uint32_t)s.N_mma * wk_b, 1024);
+    p.b_layout = p.a_layout;
+    p.b_sbo = p.a_sbo;
+    p.b_lbo = 16;
+    p.b_kstep = 32;
+  }
   p.stage_bytes = s.stage_bytes;
   const int G = s.G;
   const int rowsA = s.rows_tile;
-  p.tx_bytes = (uint32_t)(s.Wk * rowsA * G * 2) + (uint32_t)(s.Wn * s.Wk * (n / s.Wn) * G * 2);
+  p.tx_bytes = (uint32_t)(wk_b * rowsA * G) + (uint32_t)(wk_b * n * G);
+  p.c_tx_bytes = (uint32_t)(G * n * s.rows_tile * eso);
   p.stages = s.stages;
   p.acc_cols = s.acc_cols;
   p.acc_bufs = s.acc_bufs;
@@ -376,34 +596,43 @@ kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const
   p.c_bufs = s.c_bufs;
   p.c_off = s.stages * s.stage_bytes;
   p.bar_off = p.c_off + 2 * s.c_bufs * s.c_buf_bytes;
+  p.alpha = alpha;
+  p.beta = beta;
+  p.scale = beta != 0.0f ? 2 : (alpha != 1.0f ? 1 : 0);
   const long long groups = (batch + G - 1) / G;
   p.units = groups * s.m_tiles;
 
-  const CUtensorMapDataType dt = bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+  const CUtensorMapDataType dti = in_kind == IN_BF16   ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                  : in_kind == IN_F16  ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                                  : in_kind == IN_TF32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                                       : CU_TENSOR_MAP_DATA_TYPE_UINT8;
+  const CUtensorMapDataType dto = out_kind == OUT_BF16  ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
+                                  : out_kind == OUT_F16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                                                        : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
   {  // A: (k, m, batch)
     cuuint64_t dims[3] = {(cuuint64_t)k, (cuuint64_t)m, (cuuint64_t)batch};
-    cuuint64_t strides[2] = {(cuuint64_t)k * 2, (cuuint64_t)m * k * 2};
+    cuuint64_t strides[2] = {(cuuint64_t)k * esi, (cuuint64_t)m * k * esi};
     cuuint32_t box[3] = {(cuuint32_t)s.Wk, (cuuint32_t)rowsA, (cuuint32_t)G};
     cuuint32_t es[3] = {1, 1, 1};
-    if (enc(&p.tmA, dt, 3, const_cast<void*>(A), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-            swz_mode_for(s.Wk), CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    if (enc(&p.tmA, dti, 3, const_cast<void*>(A), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            swz_mode_for(wk_b), CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
   {  // B: (Wn, k, n/Wn, batch)
     cuuint64_t dims[4] = {(cuuint64_t)s.Wn, (cuuint64_t)k, (cuuint64_t)(n / s.Wn), (cuuint64_t)batch};
-    cuuint64_t strides[3] = {(cuuint64_t)n * 2, (cuuint64_t)s.Wn * 2, (cuuint64_t)k * n * 2};
+    cuuint64_t strides[3] = {(cuuint64_t)n * esi, (cuuint64_t)wn_b, (cuuint64_t)k * n * esi};
     cuuint32_t box[4] = {(cuuint32_t)s.Wn, (cuuint32_t)s.Wk, (cuuint32_t)(n / s.Wn), (cuuint32_t)G};
     cuuint32_t es[4] = {1, 1, 1, 1};
-    if (enc(&p.tmB, dt, 4, const_cast<void*>(B), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-            swz_mode_for(s.Wn), CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    if (enc(&p.tmB, dti, 4, const_cast<void*>(B), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            swz_mode_for(wn_b), CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
   {  // C: (Wc, m, n/Wc, batch)
     cuuint64_t dims[4] = {(cuuint64_t)s.Wc, (cuuint64_t)m, (cuuint64_t)(n / s.Wc), (cuuint64_t)batch};
-    cuuint64_t strides[3] = {(cuuint64_t)n * 2, (cuuint64_t)s.Wc * 2, (cuuint64_t)m * n * 2};
+    cuuint64_t strides[3] = {(cuuint64_t)n * eso, (cuuint64_t)wc_b, (cuuint64_t)m * n * eso};
     cuuint32_t box[4] = {(cuuint32_t)s.Wc, (cuuint32_t)s.rows_tile, (cuuint32_t)(n / s.Wc), (cuuint32_t)G};
     cuuint32_t es[4] = {1, 1, 1, 1};
-    if (enc(&p.tmC, dt, 4, C, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz_mode_for(s.Wc),
+    if (enc(&p.tmC, dto, 4, C, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz_mode_for(wc_b),
             CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
@@ -414,16 +643,21 @@ kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const
   long long grid = p.units < sms ? p.units : sms;
   if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
   const size_t smem = s.smem_bytes;
-  if (bf16) {
-    cudaFuncSetAttribute(kami_tc16_1d_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    kami_tc16_1d_kernel<true><<<(unsigned)grid, kThreads, smem, stream>>>(p);
-    set_last_kernel("kami_tc16_1d_kernel<bf16>");
-  } else {
-    cudaFuncSetAttribute(kami_tc16_1d_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    kami_tc16_1d_kernel<false><<<(unsigned)grid, kThreads, smem, stream>>>(p);
-    set_last_kernel("kami_tc16_1d_kernel<f16>");
+  const unsigned g = (unsigned)grid;
+  switch (in_kind) {
+    case IN_F16: launch_kernel<IN_F16, OUT_F16>(p, g, smem, stream, "kami_tc16_1d_kernel<f16>"); break;
+    case IN_BF16: launch_kernel<IN_BF16, OUT_BF16>(p, g, smem, stream, "kami_tc16_1d_kernel<bf16>"); break;
+    case IN_TF32: launch_kernel<IN_TF32, OUT_F32>(p, g, smem, stream, "kami_tc16_1d_kernel<tf32,f32>"); break;
+    case IN_E4M3: launch_kernel<IN_E4M3, OUT_F16>(p, g, smem, stream, "kami_tc16_1d_kernel<e4m3,f16>"); break;
+    default: launch_kernel<IN_E5M2, OUT_F16>(p, g, smem, stream, "kami_tc16_1d_kernel<e5m2,f16>"); break;
   }
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+}
+
+kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B, void* C,
+                          cudaStream_t stream, int max_ctas) {
+  return tc16_launch_kind(m, n, k, batch, bf16 ? IN_BF16 : IN_F16, bf16 ? OUT_BF16 : OUT_F16, A, B, C, 1.0f, 0.0f,
+                          stream, max_ctas);
 }
 
 }  // namespace kami
