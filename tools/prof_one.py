@@ -24,8 +24,11 @@ dtype, m, n, k, batch, _ = parse_workload(a.workload)
 if a.batch:
     batch = a.batch
 A, B = ki.operands(m, n, k, batch, dtype, "unif", device="cuda")
-C = torch.empty(batch * m * n, dtype=A.dtype, device="cuda")
+C = torch.zeros(batch * m * n, dtype=ki.TORCH_DTYPES[ki.OUT_DTYPE[dtype]], device="cuda")
 for _ in range(a.iters):
-    kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A, B, C, algo=a.algo, p=a.p)
+    if "upd" in a.workload:
+        kami.gemm_strided_batched_axpby(m, n, k, batch, dtype, "row", 1.0, A, B, 1.0, C)
+    else:
+        kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A, B, C, algo=a.algo, p=a.p)
 torch.cuda.synchronize()
 print(kami.last_kernel())
