@@ -91,7 +91,8 @@ class ClockSampler:
 
     Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
          "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap,clocks.mem,"
+         "temperature.gpu,temperature.memory")
 
     def __init__(self, index):
         self.index = index
@@ -132,8 +133,12 @@ class ClockSampler:
             for nm, v in zip(names, r[5:9]):
                 if v.strip().lower() == "active":
                     reasons.add(nm)
+        def med(i):
+            v = [float(r[i]) for r in self.rows if len(r) > i and r[i].replace(".", "").isdigit()]
+            return statistics.median(v) if v else None
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(self.rows)}
+                "reasons": sorted(reasons), "samples": len(self.rows), "mem_mhz": med(9), "power_w": med(3),
+                "gpu_temp_c": med(10), "mem_temp_c": med(11)}
 
 
 def cpu_baseline(dtype, m, n, k, target_s=12.0, max_entries=None):

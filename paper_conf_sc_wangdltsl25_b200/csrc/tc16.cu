@@ -45,6 +45,8 @@
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 
 #include "kernels.h"
@@ -124,13 +126,13 @@ __device__ __forceinline__ void umma(uint32_t d, uint64_t a, uint64_t b, uint32_
 // 8 fp32 accumulators -> the output type, written as 16-byte chunks of the
 // swizzled staging tile.  `off` is the unswizzled byte offset of the first
 // element; old values (beta != 0) are read from the same locations.
-template <int kOut>
+template <int kOut, bool kUpd>
 __device__ __forceinline__ void emit8(uint32_t cbase, uint32_t off, uint32_t swz_bits, const uint32_t* v,
                                       const Tc16Params& p) {
   float x[8];
 #pragma unroll
   for (int i = 0; i < 8; ++i) x[i] = __uint_as_float(v[i]);
-  if (p.scale) {
+  if (kUpd && p.scale) {
 #pragma unroll
     for (int i = 0; i < 8; ++i) x[i] *= p.alpha;
   }
@@ -138,7 +140,7 @@ __device__ __forceinline__ void emit8(uint32_t cbase, uint32_t off, uint32_t swz
 #pragma unroll
     for (int h = 0; h < 2; ++h) {
       const uint32_t a = cbase + ptx::swz(off + 16 * h, swz_bits);
-      if (p.scale == 2) {
+      if (kUpd && p.scale == 2) {
         uint32_t o0, o1, o2, o3;
         ptx::ld_shared_v4(a, o0, o1, o2, o3);
         x[4 * h + 0] = fmaf(p.beta, __uint_as_float(o0), x[4 * h + 0]);
@@ -151,7 +153,7 @@ __device__ __forceinline__ void emit8(uint32_t cbase, uint32_t off, uint32_t swz
     }
   } else {
     const uint32_t a = cbase + ptx::swz(off, swz_bits);
-    if (p.scale == 2) {
+    if (kUpd && p.scale == 2) {
       uint32_t o[4];
       ptx::ld_shared_v4(a, o[0], o[1], o[2], o[3]);
 #pragma unroll
@@ -178,15 +180,16 @@ __device__ __forceinline__ void emit8(uint32_t cbase, uint32_t off, uint32_t swz
 }
 
 // FP32 output: 8 accumulators -> 32 contiguous bytes of C (one full sector).
+template <bool kUpd>
 __device__ __forceinline__ void emit8_f32_global(float* dst, const uint32_t* v, const Tc16Params& p) {
   float x[8];
 #pragma unroll
   for (int i = 0; i < 8; ++i) x[i] = __uint_as_float(v[i]);
-  if (p.scale) {
+  if (kUpd && p.scale) {
 #pragma unroll
     for (int i = 0; i < 8; ++i) x[i] *= p.alpha;
   }
-  if (p.scale == 2) {
+  if (kUpd && p.scale == 2) {
     const float4 o0 = *reinterpret_cast<const float4*>(dst);
     const float4 o1 = *reinterpret_cast<const float4*>(dst + 4);
     x[0] = fmaf(p.beta, o0.x, x[0]);
@@ -204,7 +207,9 @@ __device__ __forceinline__ void emit8_f32_global(float* dst, const uint32_t* v, 
                                         __float_as_uint(x[7])));
 }
 
-template <int kIn, int kOut>
+// kUpd: the C-update epilogue (alpha != 1 or beta != 0); the plain C = AB
+// instantiation carries none of its code.
+template <int kIn, int kOut, bool kUpd>
 __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const __grid_constant__ Tc16Params p) {
   constexpr bool kXpose = kIn == IN_TF32;
   constexpr bool kDirect = kOut == OUT_F32;
@@ -381,7 +386,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       if (!kDirect && leader) {
         if (p.c_bufs == 2) ptx::bulk_wait_read<1>();
         else ptx::bulk_wait_read<0>();
-        if (p.scale == 2) {  // C update: bring the old C tile into the staging buffer
+        if (kUpd && p.scale == 2) {  // C update: bring the old C tile into the staging buffer
           uint64_t* cf = &cfull[wg * 2 + cb];
           ptx::mbar_arrive_expect_tx(cf, p.c_tx_bytes);
           ptx::tma_load_4d(smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, &p.tmC, cf, 0, mt * 128, 0,
@@ -391,7 +396,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       ptx::named_bar_sync(bar_id, kEpiThreads);
       ptx::mbar_wait(&tfull[a], aph);
       ptx::tc_fence_after();
-      if (!kDirect && p.scale == 2) ptx::mbar_wait(&cfull[wg * 2 + cb], (local / p.c_bufs) & 1);
+      if (kUpd && !kDirect && p.scale == 2) ptx::mbar_wait(&cfull[wg * 2 + cb], (local / p.c_bufs) & 1);
       float* crow = nullptr;
       if constexpr (kDirect) crow = reinterpret_cast<float*>(p.Cg) + ((e0 + g) * p.m + mt * 128 + r) * (long long)p.n;
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
@@ -418,11 +423,11 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
           if (valid && col >= my_lo && col < my_hi && col < col_hi) {
             const uint32_t jc = (uint32_t)(col - my_lo);
             if constexpr (kDirect) {
-              emit8_f32_global(crow + jc, &v[8 * q], p);
+              emit8_f32_global<kUpd>(crow + jc, &v[8 * q], p);
             } else {
               const uint32_t atom = jc >> wc_shift;
               const uint32_t ce = jc & (uint32_t)(p.Wc - 1);
-              emit8<kOut>(cbase, rowbase + atom * atom_stride + ce * ESO, p.c_swz_bits, &v[8 * q], p);
+              emit8<kOut, kUpd>(cbase, rowbase + atom * atom_stride + ce * ESO, p.c_swz_bits, &v[8 * q], p);
             }
           }
         }
@@ -474,10 +479,32 @@ int out_es(int out) { return out == OUT_F32 ? 4 : 2; }
 
 constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 
+// Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo"
+// (0 / -1 = planner default; promo = TMA L2 promotion 0 none, 1 64B, 2 128B, 3 256B),
+// KAMI_TC_IDESC_XOR (debug of the instruction descriptor).
+struct TcTune {
+  int stages = 0, cbufs = 0, grid = 0, promo = -1;
+  uint32_t idesc_xor = 0;
+};
+const TcTune& tc_tune() {
+  static const TcTune t = [] {
+    TcTune r;
+    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo);
+    if (const char* e = getenv("KAMI_TC_IDESC_XOR")) r.idesc_xor = (uint32_t)strtoul(e, nullptr, 0);
+    return r;
+  }();
+  return t;
+}
+
 template <int kIn, int kOut>
 void launch_kernel(const Tc16Params& p, unsigned grid, size_t smem, cudaStream_t stream, const char* name) {
-  cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  kami_tc16_1d_kernel<kIn, kOut><<<grid, threads_for(kIn), smem, stream>>>(p);
+  if (p.scale) {
+    cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    kami_tc16_1d_kernel<kIn, kOut, true><<<grid, threads_for(kIn), smem, stream>>>(p);
+  } else {
+    cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    kami_tc16_1d_kernel<kIn, kOut, false><<<grid, threads_for(kIn), smem, stream>>>(p);
+  }
   set_last_kernel(name);
 }
 
@@ -510,9 +537,20 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   s->c_buf_bytes = out_kind == OUT_F32 ? 0 : align_up((uint32_t)s->G * n * s->rows_tile * eso, 1024);
   // two epilogue warpgroups, each with c_bufs staging tiles
   s->c_bufs = (4 * s->c_buf_bytes <= 64 * 1024) ? 2 : 1;
+  if (tc_tune().cbufs) s->c_bufs = tc_tune().cbufs;
   const int budget = kSmemLimit - 1024 /*align slack*/ - 1024 /*barriers*/;
   int st = (budget - (int)(2 * s->c_bufs * s->c_buf_bytes)) / (int)s->stage_bytes;
   if (st > kMaxStages) st = kMaxStages;
+  // Bytes in flight per SM: beyond ~96 KB of outstanding TMA loads per SM the
+  // sustained HBM throughput DROPS (measured, profiles/r1/stage_sweep_r1.txt:
+  // f16 64^3 119 -> 137 TFLOP/s, f16 128^3 245 -> 283 going from 5 / 4 stages
+  // of 32 KB to 3); shapes with smaller stages are insensitive.
+  const int cap = (96 * 1024) / (int)s->stage_bytes;
+  if (tc_tune().stages > 0) {
+    if (st > tc_tune().stages) st = tc_tune().stages;
+  } else if (st > cap) {
+    st = cap < 2 ? 2 : cap;
+  }
   s->stages = st;
   s->smem_bytes = s->stages * s->stage_bytes + 2 * s->c_bufs * s->c_buf_bytes + 1024 + 1024;
   s->acc_cols = pow2_ceil(s->N_mma);
@@ -562,7 +600,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   } else {
     p.idesc = ptx::make_idesc_f16(in_kind == IN_BF16 ? 1 : 0, 128, s.N_mma, /*a MN-major*/ 0, /*b MN-major*/ 1);
   }
-  if (const char* e = getenv("KAMI_TC_IDESC_XOR")) p.idesc ^= (uint32_t)strtoul(e, nullptr, 0);  // debug
+  p.idesc ^= tc_tune().idesc_xor;
   p.a_layout = ptx::umma_layout_code(wk_b);
   p.b_layout = ptx::umma_layout_code(wn_b);
   p.c_swz_bits = swz_bits_for(wc_b);
@@ -609,13 +647,15 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   const CUtensorMapDataType dto = out_kind == OUT_BF16  ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
                                   : out_kind == OUT_F16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
                                                         : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
+  const CUtensorMapL2promotion promo =
+      tc_tune().promo < 0 ? CU_TENSOR_MAP_L2_PROMOTION_L2_256B : (CUtensorMapL2promotion)tc_tune().promo;
   {  // A: (k, m, batch)
     cuuint64_t dims[3] = {(cuuint64_t)k, (cuuint64_t)m, (cuuint64_t)batch};
     cuuint64_t strides[2] = {(cuuint64_t)k * esi, (cuuint64_t)m * k * esi};
     cuuint32_t box[3] = {(cuuint32_t)s.Wk, (cuuint32_t)rowsA, (cuuint32_t)G};
     cuuint32_t es[3] = {1, 1, 1};
     if (enc(&p.tmA, dti, 3, const_cast<void*>(A), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-            swz_mode_for(wk_b), CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            swz_mode_for(wk_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
   {  // B: (Wn, k, n/Wn, batch)
@@ -624,7 +664,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
     cuuint32_t box[4] = {(cuuint32_t)s.Wn, (cuuint32_t)s.Wk, (cuuint32_t)(n / s.Wn), (cuuint32_t)G};
     cuuint32_t es[4] = {1, 1, 1, 1};
     if (enc(&p.tmB, dti, 4, const_cast<void*>(B), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-            swz_mode_for(wn_b), CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+            swz_mode_for(wn_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
   {  // C: (Wc, m, n/Wc, batch)
@@ -641,6 +681,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   long long grid = p.units < sms ? p.units : sms;
+  if (tc_tune().grid > 0 && tc_tune().grid < grid) grid = tc_tune().grid;
   if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
   const size_t smem = s.smem_bytes;
   const unsigned g = (unsigned)grid;
