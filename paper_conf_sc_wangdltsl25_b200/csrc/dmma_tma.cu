@@ -49,7 +49,8 @@ struct DmmaTmaParams {
   double alpha, beta;  // C = alpha A B + beta C (C read iff beta != 0)
 };
 
-template <int M, int N, int K, int P, int TEAMS>
+// kUpd: C = alpha A B + beta C epilogue; the plain instantiation has none of it.
+template <int M, int N, int K, int P, int TEAMS, bool kUpd>
 __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(const __grid_constant__ DmmaTmaParams prm) {
   using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -129,11 +130,11 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
       {
         double* dst = Cg + (i * 8 + g) * N + j * 8 + 2 * t;
         double r0 = c[i][j][0], r1 = c[i][j][1];
-        if (prm.beta != 0.0) {
+        if (kUpd && prm.beta != 0.0) {
           const double2 o = *reinterpret_cast<const double2*>(dst);
           r0 = fma(prm.beta, o.x, prm.alpha * r0);
           r1 = fma(prm.beta, o.y, prm.alpha * r1);
-        } else if (prm.alpha != 1.0) {
+        } else if (kUpd && prm.alpha != 1.0) {
           r0 *= prm.alpha;
           r1 *= prm.alpha;
         }
@@ -164,7 +165,8 @@ kami_status_t launch(long long batch, const void* A, const void* B, void* C, cud
   prm.batch = batch;
   prm.alpha = alpha;
   prm.beta = beta;
-  auto fn = kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS>;
+  auto fn = (alpha != 1.0 || beta != 0.0) ? kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, true>
+                                          : kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, false>;
   if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM) != cudaSuccess)
     return KAMI_ERROR_CUDA;
   int dev = 0, sms = 148, per_sm = 1;
