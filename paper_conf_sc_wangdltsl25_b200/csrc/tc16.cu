@@ -179,6 +179,40 @@ __device__ __forceinline__ void emit8(uint32_t cbase, uint32_t off, uint32_t swz
   }
 }
 
+// Incremental (unit -> entry group, m-tile) and ring (slot, phase) counters:
+// the single-thread producer / MMA roles run one iteration per unit, and with
+// small units their serial instruction latency bounds the kernel (ncu: ~190
+// instructions per unit in the MMA lane with 64-bit divisions), so no
+// divisions or modulos inside the loops.
+struct UnitIter {
+  long long grp;
+  int mt, gstep, mstep, m_tiles;
+  __device__ __forceinline__ UnitIter(long long u0, long long step, int mtiles) {
+    m_tiles = mtiles;
+    grp = u0 / mtiles;
+    mt = (int)(u0 - grp * mtiles);
+    gstep = (int)(step / mtiles);
+    mstep = (int)(step - (long long)gstep * mtiles);
+  }
+  __device__ __forceinline__ void next() {
+    grp += gstep;
+    mt += mstep;
+    if (mt >= m_tiles) {
+      mt -= m_tiles;
+      ++grp;
+    }
+  }
+};
+struct RingPos {
+  uint32_t s = 0, ph = 0;
+  __device__ __forceinline__ void next(uint32_t n) {
+    if (++s == n) {
+      s = 0;
+      ph ^= 1;
+    }
+  }
+};
+
 // FP32 output: 8 accumulators -> 32 contiguous bytes of C (one full sector).
 template <bool kUpd>
 __device__ __forceinline__ void emit8_f32_global(float* dst, const uint32_t* v, const Tc16Params& p) {
@@ -256,54 +290,48 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
   if (warp == 0) {
     // ------------------------------------------------------------ producer
     if (lane == 0) {
-      uint32_t it = 0;
-      for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
-        const long long grp = u / p.m_tiles;
-        const int mt = (int)(u - grp * p.m_tiles);
-        const int e0 = (int)(grp * p.G);
-        for (int kc = 0; kc < p.k_chunks; ++kc, ++it) {
-          const uint32_t s = it % p.stages;
-          const uint32_t ph = (it / p.stages) & 1;
-          ptx::mbar_wait(&empty[s], ph ^ 1);
-          ptx::mbar_arrive_expect_tx(&full[s], p.tx_bytes);
-          uint8_t* sa = smem + s * p.stage_bytes;
+      RingPos r;
+      UnitIter ui(blockIdx.x, gridDim.x, p.m_tiles);
+      for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ui.next()) {
+        const int e0 = (int)(ui.grp * p.G);
+        for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
+          ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
+          ptx::mbar_arrive_expect_tx(&full[r.s], p.tx_bytes);
+          uint8_t* sa = smem + r.s * p.stage_bytes;
           uint8_t* sb = sa + p.a_region;
-          ptx::tma_load_3d(sa, &p.tmA, &full[s], kc * p.Wk, mt * 128, e0);
-          ptx::tma_load_4d(kXpose ? sa + p.b_raw_off : sb, &p.tmB, &full[s], 0, kc * p.Wk, 0, e0);
+          ptx::tma_load_3d(sa, &p.tmA, &full[r.s], kc * p.Wk, ui.mt * 128, e0);
+          ptx::tma_load_4d(kXpose ? sa + p.b_raw_off : sb, &p.tmB, &full[r.s], 0, kc * p.Wk, 0, e0);
         }
       }
     }
   } else if (warp == 1) {
     // ---------------------------------------------------------- MMA issuer
-    uint32_t it = 0, acc_it = 0;
-    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ++acc_it) {
-      const uint32_t a = acc_it % p.acc_bufs;
-      const uint32_t aph = (acc_it / p.acc_bufs) & 1;
-      ptx::mbar_wait(&tempty[a], aph ^ 1);
+    RingPos r, ra;
+    // descriptors of stage 0; a stage / K step only moves the 14-bit start
+    // address field (addresses are < 256 KB, so the field never carries)
+    const uint64_t adesc0 = ptx::make_smem_desc(smem_base, 16, p.a_sbo, p.a_layout);
+    const uint64_t bdesc0 = ptx::make_smem_desc(smem_base + p.a_region, p.b_lbo, p.b_sbo, p.b_layout);
+    const uint32_t stage16 = p.stage_bytes >> 4, bstep16 = p.b_kstep >> 4;
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ra.next(p.acc_bufs)) {
+      ptx::mbar_wait(&tempty[ra.s], ra.ph ^ 1);
       ptx::tc_fence_after();
-      const uint32_t d_tmem = tmem_base + a * p.acc_cols;
-      for (int kc = 0; kc < p.k_chunks; ++kc, ++it) {
-        const uint32_t s = it % p.stages;
-        const uint32_t ph = (it / p.stages) & 1;
-        ptx::mbar_wait(kXpose ? &bready[s] : &full[s], ph);
+      const uint32_t d_tmem = tmem_base + ra.s * p.acc_cols;
+      for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
+        ptx::mbar_wait(kXpose ? &bready[r.s] : &full[r.s], r.ph);
         ptx::tc_fence_after();
         if (lane == 0) {
-          const uint32_t sa = smem_base + s * p.stage_bytes;
-          const uint32_t sb = sa + p.a_region;
+          const uint64_t ad = adesc0 + r.s * stage16, bd = bdesc0 + r.s * stage16;
           const int nsteps = (kc == p.k_chunks - 1) ? p.ksteps_last : p.ksteps_full;
           for (int ks = 0; ks < nsteps; ++ks) {
-            // A: K-major, one K step = 32 bytes further along the swizzled row
-            const uint64_t adesc = ptx::make_smem_desc(sa + ks * 32, 16, p.a_sbo, p.a_layout);
-            // B: N-major, one K step = 32 bytes of K = 32/es rows further
-            // (TF32: K-major like A, one K step = 32 bytes along the row)
-            const uint64_t bdesc = ptx::make_smem_desc(sb + ks * p.b_kstep, p.b_lbo, p.b_sbo, p.b_layout);
-            umma<kIn>(d_tmem, adesc, bdesc, p.idesc, (kc | ks) != 0);
+            // A: K-major, one K step = 32 bytes further along the swizzled row;
+            // B: N-major, one K step = 32/es K rows further (TF32: K-major, 32 bytes)
+            umma<kIn>(d_tmem, ad + 2 * ks, bd + bstep16 * ks, p.idesc, (kc | ks) != 0);
           }
-          ptx::umma_commit(&empty[s]);  // stage s may be refilled once these MMAs retire
+          ptx::umma_commit(&empty[r.s]);  // stage s may be refilled once these MMAs retire
         }
         __syncwarp();
       }
-      if (lane == 0) ptx::umma_commit(&tfull[a]);  // accumulator a complete
+      if (lane == 0) ptx::umma_commit(&tfull[ra.s]);  // accumulator complete
       __syncwarp();
     }
   } else if (kXpose && warp >= kThreads / 32) {
@@ -316,12 +344,11 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     const int t = threadIdx.x - kThreads;
     const int wn_shift = 31 - __clz(p.Wn);
     const int kq = p.Wk >> 2;
-    uint32_t it = 0;
+    RingPos r;
     for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
-      for (int kc = 0; kc < p.k_chunks; ++kc, ++it) {
-        const uint32_t s = it % p.stages;
-        const uint32_t ph = (it / p.stages) & 1;
-        ptx::mbar_wait(&full[s], ph);
+      for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
+        const uint32_t s = r.s;
+        ptx::mbar_wait(&full[s], r.ph);
         const uint32_t raw = smem_base + s * p.stage_bytes + p.b_raw_off;
         const uint32_t dst = smem_base + s * p.stage_bytes + p.a_region;
         for (int c = t; c < p.N_mma; c += kXposeThreads) {
@@ -372,15 +399,20 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     const uint32_t rowbase = (uint32_t)(g * (p.n / p.Wc) * p.rows_tile + r) * row_bytes;
     const int wc_shift = 31 - __clz(p.Wc);
     const uint32_t c_smem = smem_base + p.c_off + (uint32_t)wg * p.c_bufs * p.c_buf_bytes;
-    uint32_t i = wg, local = 0;
-    for (long long u = blockIdx.x + (long long)wg * gridDim.x; u < p.units;
-         u += 2ll * gridDim.x, i += 2, ++local) {
-      const long long grp = u / p.m_tiles;
-      const int mt = (int)(u - grp * p.m_tiles);
-      const long long e0 = grp * p.G;
-      const uint32_t a = i % p.acc_bufs;
-      const uint32_t aph = (i / p.acc_bufs) & 1;
-      const uint32_t cb = local % p.c_bufs;
+    // this warpgroup's units: u0 + 2j gridDim; accumulators wg, wg + 2, ... (mod acc_bufs);
+    // staging buffers 0, 1, 0, ... (mod c_bufs) -- all advanced incrementally
+    const long long u0 = blockIdx.x + (long long)wg * gridDim.x;
+    UnitIter ui(u0, 2ll * gridDim.x, p.m_tiles);
+    uint32_t a = wg, aph = 0;
+    if (a >= (uint32_t)p.acc_bufs) {  // acc_bufs >= 2 always (N_mma <= 256); kept general
+      a -= p.acc_bufs;
+      aph = 1;
+    }
+    RingPos cpos;
+    for (long long u = u0; u < p.units; u += 2ll * gridDim.x, ui.next()) {
+      const int mt = ui.mt;
+      const long long e0 = ui.grp * p.G;
+      const uint32_t cb = cpos.s;
       const bool valid = row_ok && (e0 + g < p.batch) && (p.G > 1 || mt * 128 + L < p.m);
       // the TMA store that last read staging buffer cb must be done reading
       if (!kDirect && leader) {
@@ -396,7 +428,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       ptx::named_bar_sync(bar_id, kEpiThreads);
       ptx::mbar_wait(&tfull[a], aph);
       ptx::tc_fence_after();
-      if (kUpd && !kDirect && p.scale == 2) ptx::mbar_wait(&cfull[wg * 2 + cb], (local / p.c_bufs) & 1);
+      if (kUpd && !kDirect && p.scale == 2) ptx::mbar_wait(&cfull[wg * 2 + cb], cpos.ph);
       float* crow = nullptr;
       if constexpr (kDirect) crow = reinterpret_cast<float*>(p.Cg) + ((e0 + g) * p.m + mt * 128 + r) * (long long)p.n;
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
@@ -436,6 +468,12 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[a]);
+      a += 2;
+      if (a >= (uint32_t)p.acc_bufs) {
+        a -= p.acc_bufs;
+        aph ^= 1;
+      }
+      cpos.next(p.c_bufs);
       if constexpr (kDirect) continue;
       // make the generic-proxy smem writes visible to the TMA engine
       ptx::fence_proxy_async_smem();
