@@ -86,6 +86,8 @@ struct alignas(64) Tc16Params {
   int k_chunks, Wk, Wn, Wc;  // atom widths in ELEMENTS of their operand
   int ksteps_full, ksteps_last;
   int N_mma;
+  int U, GU;               // sub-tiles (MMA tiles) per unit; entries per unit = G * U
+  uint32_t a_sub, b_sub;   // byte offsets between sub-tiles' A and B operands
   uint32_t idesc;
   uint32_t a_layout, b_layout, c_swz_bits;
   uint32_t a_sbo, b_lbo, b_sbo, b_kstep;  // bytes
@@ -293,7 +295,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       RingPos r;
       UnitIter ui(blockIdx.x, gridDim.x, p.m_tiles);
       for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ui.next()) {
-        const int e0 = (int)(ui.grp * p.G);
+        const int e0 = (int)(ui.grp * p.GU);
         for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
           ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
           ptx::mbar_arrive_expect_tx(&full[r.s], p.tx_bytes);
@@ -322,10 +324,13 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
         if (lane == 0) {
           const uint64_t ad = adesc0 + r.s * stage16, bd = bdesc0 + r.s * stage16;
           const int nsteps = (kc == p.k_chunks - 1) ? p.ksteps_last : p.ksteps_full;
-          for (int ks = 0; ks < nsteps; ++ks) {
-            // A: K-major, one K step = 32 bytes further along the swizzled row;
-            // B: N-major, one K step = 32/es K rows further (TF32: K-major, 32 bytes)
-            umma<kIn>(d_tmem, ad + 2 * ks, bd + bstep16 * ks, p.idesc, (kc | ks) != 0);
+          for (int j = 0; j < p.U; ++j) {  // sub-tile j: entries [jG, jG + G) of the unit
+            const uint64_t adj = ad + j * (p.a_sub >> 4), bdj = bd + j * (p.b_sub >> 4);
+            for (int ks = 0; ks < nsteps; ++ks) {
+              // A: K-major, one K step = 32 bytes further along the swizzled row;
+              // B: N-major, one K step = 32/es K rows further (TF32: K-major, 32 bytes)
+              umma<kIn>(d_tmem + j * p.N_mma, adj + 2 * ks, bdj + bstep16 * ks, p.idesc, (kc | ks) != 0);
+            }
           }
           ptx::umma_commit(&empty[r.s]);  // stage s may be refilled once these MMAs retire
         }
@@ -351,7 +356,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
         ptx::mbar_wait(&full[s], r.ph);
         const uint32_t raw = smem_base + s * p.stage_bytes + p.b_raw_off;
         const uint32_t dst = smem_base + s * p.stage_bytes + p.a_region;
-        for (int c = t; c < p.N_mma; c += kXposeThreads) {
+        for (int c = t; c < p.U * p.N_mma; c += kXposeThreads) {
           const uint32_t cbase = (uint32_t)((c >> wn_shift) * p.Wk) * p.wn_b + (uint32_t)(c & (p.Wn - 1)) * 4;
           for (int q = 0; q < kq; ++q) {
             uint32_t w[4];
@@ -411,9 +416,9 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     RingPos cpos;
     for (long long u = u0; u < p.units; u += 2ll * gridDim.x, ui.next()) {
       const int mt = ui.mt;
-      const long long e0 = ui.grp * p.G;
+      const long long e0 = ui.grp * p.GU;
       const uint32_t cb = cpos.s;
-      const bool valid = row_ok && (e0 + g < p.batch) && (p.G > 1 || mt * 128 + L < p.m);
+      const bool valid0 = row_ok && (p.G > 1 || mt * 128 + L < p.m);
       // the TMA store that last read staging buffer cb must be done reading
       if (!kDirect && leader) {
         if (p.c_bufs == 2) ptx::bulk_wait_read<1>();
@@ -429,10 +434,14 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       ptx::mbar_wait(&tfull[a], aph);
       ptx::tc_fence_after();
       if (kUpd && !kDirect && p.scale == 2) ptx::mbar_wait(&cfull[wg * 2 + cb], cpos.ph);
-      float* crow = nullptr;
-      if constexpr (kDirect) crow = reinterpret_cast<float*>(p.Cg) + ((e0 + g) * p.m + mt * 128 + r) * (long long)p.n;
-      const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
       const uint32_t cbase = c_smem + cb * p.c_buf_bytes;
+      for (int j = 0; j < p.U; ++j) {
+      const bool valid = valid0 && (e0 + j * p.G + g < p.batch);
+      float* crow = nullptr;
+      if constexpr (kDirect)
+        crow = reinterpret_cast<float*>(p.Cg) + ((e0 + j * p.G + g) * p.m + mt * 128 + r) * (long long)p.n;
+      const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols + j * p.N_mma;
+      const uint32_t rowbase_j = rowbase + (uint32_t)(j * p.G * (p.n / p.Wc)) * atom_stride;
       for (int c0 = col_lo; c0 < col_hi; c0 += 64) {
         uint32_t v[64];
         // issue both TMEM loads, then one wait (never read past col_hi)
@@ -459,11 +468,12 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
             } else {
               const uint32_t atom = jc >> wc_shift;
               const uint32_t ce = jc & (uint32_t)(p.Wc - 1);
-              emit8<kOut, kUpd>(cbase, rowbase + atom * atom_stride + ce * ESO, p.c_swz_bits, &v[8 * q], p);
+              emit8<kOut, kUpd>(cbase, rowbase_j + atom * atom_stride + ce * ESO, p.c_swz_bits, &v[8 * q], p);
             }
           }
         }
       }
+      }  // sub-tiles
       // accumulator a may be overwritten by the next MMA chain
       ptx::tc_fence_before();
       __syncwarp();
@@ -517,17 +527,17 @@ int out_es(int out) { return out == OUT_F32 ? 4 : 2; }
 
 constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 
-// Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo"
+// Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo,U"
 // (0 / -1 = planner default; promo = TMA L2 promotion 0 none, 1 64B, 2 128B, 3 256B),
 // KAMI_TC_IDESC_XOR (debug of the instruction descriptor).
 struct TcTune {
-  int stages = 0, cbufs = 0, grid = 0, promo = -1;
+  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0;
   uint32_t idesc_xor = 0;
 };
 const TcTune& tc_tune() {
   static const TcTune t = [] {
     TcTune r;
-    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo);
+    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U);
     if (const char* e = getenv("KAMI_TC_IDESC_XOR")) r.idesc_xor = (uint32_t)strtoul(e, nullptr, 0);
     return r;
   }();
@@ -567,35 +577,53 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   s->Wc = wc_b / eso;
   s->k_chunks = (kpad + s->Wk - 1) / s->Wk;
   s->N_mma = s->G > 1 ? s->G * n : n;
-  const uint32_t a_region = align_up(128u * wk_b, 1024);
-  const uint32_t b_region = align_up((uint32_t)s->N_mma * wk_b, 1024);
-  // TF32: + the raw N-major B slot the transposer reads
-  s->stage_bytes = a_region + b_region * (in_kind == IN_TF32 ? 2 : 1);
-  // FP32 output is stored straight from registers (no staging)
-  s->c_buf_bytes = out_kind == OUT_F32 ? 0 : align_up((uint32_t)s->G * n * s->rows_tile * eso, 1024);
-  // two epilogue warpgroups, each with c_bufs staging tiles
-  s->c_bufs = (4 * s->c_buf_bytes <= 64 * 1024) ? 2 : 1;
-  if (tc_tune().cbufs) s->c_bufs = tc_tune().cbufs;
-  const int budget = kSmemLimit - 1024 /*align slack*/ - 1024 /*barriers*/;
-  int st = (budget - (int)(2 * s->c_bufs * s->c_buf_bytes)) / (int)s->stage_bytes;
-  if (st > kMaxStages) st = kMaxStages;
-  // Bytes in flight per SM: beyond ~96 KB of outstanding TMA loads per SM the
-  // sustained HBM throughput DROPS (measured, profiles/r1/stage_sweep_r1.txt:
-  // f16 64^3 119 -> 137 TFLOP/s, f16 128^3 245 -> 283 going from 5 / 4 stages
-  // of 32 KB to 3); shapes with smaller stages are insensitive.
-  const int cap = (96 * 1024) / (int)s->stage_bytes;
-  if (tc_tune().stages > 0) {
-    if (st > tc_tune().stages) st = tc_tune().stages;
-  } else if (st > cap) {
-    st = cap < 2 ? 2 : cap;
+  // Sub-tiles per unit: small tiles are bound by the per-unit fixed cost of
+  // the single-thread producer / MMA roles and the epilogue barriers, so
+  // U MMA tiles (G U entries) share one unit until a unit moves >= 32 KB
+  // (f16 32^3: 48.6 -> 61.4 TFLOP/s, bf16 48^3: 45 -> 68; fp8 64^3 at 32 KB
+  // per tile is faster unsplit: U = 2 would halve its C double-buffering).
+  s->U = 1;
+  if (s->m_tiles == 1) {
+    const long long tile_bytes =
+        (long long)s->G * ((long long)m * k * esi + (long long)k * n * esi + (long long)m * n * eso);
+    while (s->U < 4 && tile_bytes * s->U < 32 * 1024 && 2 * s->U * s->N_mma <= 256 && s->G * 2 * s->U <= 256)
+      s->U *= 2;
   }
-  s->stages = st;
-  s->smem_bytes = s->stages * s->stage_bytes + 2 * s->c_bufs * s->c_buf_bytes + 1024 + 1024;
-  s->acc_cols = pow2_ceil(s->N_mma);
-  s->acc_bufs = 512 / s->acc_cols;
-  if (s->acc_bufs > kMaxAcc) s->acc_bufs = kMaxAcc;
+  if (tc_tune().U > 0) s->U = tc_tune().U;
+  for (;; s->U /= 2) {  // fall back to fewer sub-tiles if the ring does not fit
+    const int rowsA = s->G > 1 ? m : s->rows_tile;
+    const uint32_t a_region = align_up((uint32_t)((s->U - 1) * s->G * rowsA + 128) * wk_b, 1024);
+    const uint32_t b_region = align_up((uint32_t)(s->U * s->N_mma) * wk_b, 1024);
+    // TF32: + the raw N-major B slot the transposer reads
+    s->stage_bytes = a_region + b_region * (in_kind == IN_TF32 ? 2 : 1);
+    // FP32 output is stored straight from registers (no staging)
+    s->c_buf_bytes = out_kind == OUT_F32 ? 0 : align_up((uint32_t)(s->U * s->G) * n * s->rows_tile * eso, 1024);
+    // two epilogue warpgroups, each with c_bufs staging tiles
+    s->c_bufs = (4 * s->c_buf_bytes <= 64 * 1024) ? 2 : 1;
+    if (tc_tune().cbufs) s->c_bufs = tc_tune().cbufs;
+    const int budget = kSmemLimit - 1024 /*align slack*/ - 1024 /*barriers*/;
+    int st = (budget - (int)(2 * s->c_bufs * s->c_buf_bytes)) / (int)s->stage_bytes;
+    if (st > kMaxStages) st = kMaxStages;
+    // Bytes in flight per SM: beyond ~96 KB of outstanding TMA loads per SM the
+    // sustained HBM throughput DROPS (measured, profiles/r1/stage_sweep_r1.txt:
+    // f16 64^3 119 -> 137 TFLOP/s, f16 128^3 245 -> 283 going from 5 / 4 stages
+    // of 32 KB to 3); shapes with smaller stages are insensitive.
+    const int cap = (96 * 1024) / (int)s->stage_bytes;
+    if (tc_tune().stages > 0) {
+      if (st > tc_tune().stages) st = tc_tune().stages;
+    } else if (st > cap) {
+      st = cap < 2 ? 2 : cap;
+    }
+    s->stages = st;
+    s->smem_bytes = s->stages * s->stage_bytes + 2 * s->c_bufs * s->c_buf_bytes + 1024 + 1024;
+    s->acc_cols = pow2_ceil(s->U * s->N_mma);
+    if (s->acc_cols > 256) return KAMI_ERROR_NOT_SUPPORTED;
+    s->acc_bufs = 512 / s->acc_cols;
+    if (s->acc_bufs > kMaxAcc) s->acc_bufs = kMaxAcc;
+    if (st >= 2 || s->U == 1) break;
+  }
   s->units = 0;
-  return st >= 2 ? KAMI_SUCCESS : KAMI_ERROR_NOT_SUPPORTED;
+  return s->stages >= 2 ? KAMI_SUCCESS : KAMI_ERROR_NOT_SUPPORTED;
 }
 
 kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s) {
@@ -646,24 +674,28 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   p.b_sbo = 8 * wn_b;                      // 8 K-rows of one N-atom
   p.b_lbo = s.Wk * wn_b;                   // next N-atom
   p.b_kstep = (uint32_t)(kgran / 8) * p.b_sbo;  // one 32-byte K step of B rows
-  p.a_region = align_up(128u * wk_b, 1024);
+  const int U = s.U, G = s.G, rowsA = s.rows_tile;
+  p.U = U;
+  p.GU = G * U;
+  p.a_region = align_up((uint32_t)((U - 1) * G * rowsA + 128) * wk_b, 1024);
+  p.a_sub = (uint32_t)(G * rowsA * wk_b);      // sub-tile j's A rows start j G m rows further
+  p.b_sub = (uint32_t)(G * (n / s.Wn)) * p.b_lbo;  // and its B columns j G n columns further
   p.wn_b = wn_b;
   p.wk_b = wk_b;
   p.raw_swz_bits = swz_bits_for(wn_b);
   p.k_swz_bits = swz_bits_for(wk_b);
   p.Cg = C;
   if (in_kind == IN_TF32) {  // B is transposed in shared memory to K-major (same geometry as A)
-    p.b_raw_off = p.a_region + align_up((uint32_t)s.N_mma * wk_b, 1024);
+    p.b_raw_off = p.a_region + align_up((uint32_t)(U * s.N_mma) * wk_b, 1024);
+    p.b_sub = (uint32_t)(G * n * wk_b);  // K-major: one row per column
     p.b_layout = p.a_layout;
     p.b_sbo = p.a_sbo;
     p.b_lbo = 16;
     p.b_kstep = 32;
   }
   p.stage_bytes = s.stage_bytes;
-  const int G = s.G;
-  const int rowsA = s.rows_tile;
-  p.tx_bytes = (uint32_t)(wk_b * rowsA * G) + (uint32_t)(wk_b * n * G);
-  p.c_tx_bytes = (uint32_t)(G * n * s.rows_tile * eso);
+  p.tx_bytes = (uint32_t)(wk_b * rowsA * G * U) + (uint32_t)(wk_b * n * G * U);
+  p.c_tx_bytes = (uint32_t)(G * U * n * s.rows_tile * eso);
   p.stages = s.stages;
   p.acc_cols = s.acc_cols;
   p.acc_bufs = s.acc_bufs;
@@ -675,7 +707,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   p.alpha = alpha;
   p.beta = beta;
   p.scale = beta != 0.0f ? 2 : (alpha != 1.0f ? 1 : 0);
-  const long long groups = (batch + G - 1) / G;
+  const long long groups = (batch + G * U - 1) / (G * U);
   p.units = groups * s.m_tiles;
 
   const CUtensorMapDataType dti = in_kind == IN_BF16   ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
@@ -690,7 +722,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   {  // A: (k, m, batch)
     cuuint64_t dims[3] = {(cuuint64_t)k, (cuuint64_t)m, (cuuint64_t)batch};
     cuuint64_t strides[2] = {(cuuint64_t)k * esi, (cuuint64_t)m * k * esi};
-    cuuint32_t box[3] = {(cuuint32_t)s.Wk, (cuuint32_t)rowsA, (cuuint32_t)G};
+    cuuint32_t box[3] = {(cuuint32_t)s.Wk, (cuuint32_t)rowsA, (cuuint32_t)(G * U)};
     cuuint32_t es[3] = {1, 1, 1};
     if (enc(&p.tmA, dti, 3, const_cast<void*>(A), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
             swz_mode_for(wk_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
@@ -699,7 +731,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   {  // B: (Wn, k, n/Wn, batch)
     cuuint64_t dims[4] = {(cuuint64_t)s.Wn, (cuuint64_t)k, (cuuint64_t)(n / s.Wn), (cuuint64_t)batch};
     cuuint64_t strides[3] = {(cuuint64_t)n * esi, (cuuint64_t)wn_b, (cuuint64_t)k * n * esi};
-    cuuint32_t box[4] = {(cuuint32_t)s.Wn, (cuuint32_t)s.Wk, (cuuint32_t)(n / s.Wn), (cuuint32_t)G};
+    cuuint32_t box[4] = {(cuuint32_t)s.Wn, (cuuint32_t)s.Wk, (cuuint32_t)(n / s.Wn), (cuuint32_t)(G * U)};
     cuuint32_t es[4] = {1, 1, 1, 1};
     if (enc(&p.tmB, dti, 4, const_cast<void*>(B), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
             swz_mode_for(wn_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
@@ -708,7 +740,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   {  // C: (Wc, m, n/Wc, batch)
     cuuint64_t dims[4] = {(cuuint64_t)s.Wc, (cuuint64_t)m, (cuuint64_t)(n / s.Wc), (cuuint64_t)batch};
     cuuint64_t strides[3] = {(cuuint64_t)n * eso, (cuuint64_t)wc_b, (cuuint64_t)m * n * eso};
-    cuuint32_t box[4] = {(cuuint32_t)s.Wc, (cuuint32_t)s.rows_tile, (cuuint32_t)(n / s.Wc), (cuuint32_t)G};
+    cuuint32_t box[4] = {(cuuint32_t)s.Wc, (cuuint32_t)s.rows_tile, (cuuint32_t)(n / s.Wc), (cuuint32_t)(G * U)};
     cuuint32_t es[4] = {1, 1, 1, 1};
     if (enc(&p.tmC, dto, 4, C, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz_mode_for(wc_b),
             CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
