@@ -583,9 +583,10 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   // (f16 32^3: 48.6 -> 61.4 TFLOP/s, bf16 48^3: 45 -> 68; fp8 64^3 at 32 KB
   // per tile is faster unsplit: U = 2 would halve its C double-buffering).
   s->U = 1;
-  if (s->m_tiles == 1) {
+  {  // (m > 128: the U sub-tiles are U entries at the same m-tile)
+    const long long rt = s->rows_tile;
     const long long tile_bytes =
-        (long long)s->G * ((long long)m * k * esi + (long long)k * n * esi + (long long)m * n * eso);
+        (long long)s->G * (rt * k * esi + (long long)k * n * esi + rt * n * eso);
     while (s->U < 4 && tile_bytes * s->U < 32 * 1024 && 2 * s->U * s->N_mma <= 256 && s->G * 2 * s->U <= 256)
       s->U *= 2;
   }
