@@ -528,17 +528,15 @@ int out_es(int out) { return out == OUT_F32 ? 4 : 2; }
 constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 
 // Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo,U"
-// (0 / -1 = planner default; promo = TMA L2 promotion 0 none, 1 64B, 2 128B, 3 256B),
-// KAMI_TC_IDESC_XOR (debug of the instruction descriptor).
+// (0 / -1 = planner default; promo = TMA L2 promotion 0 none, 1 64B, 2 128B, 3 256B;
+// U = sub-tiles per unit).  Unset in production.
 struct TcTune {
   int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0;
-  uint32_t idesc_xor = 0;
 };
 const TcTune& tc_tune() {
   static const TcTune t = [] {
     TcTune r;
     if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U);
-    if (const char* e = getenv("KAMI_TC_IDESC_XOR")) r.idesc_xor = (uint32_t)strtoul(e, nullptr, 0);
     return r;
   }();
   return t;
@@ -667,7 +665,6 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   } else {
     p.idesc = ptx::make_idesc_f16(in_kind == IN_BF16 ? 1 : 0, 128, s.N_mma, /*a MN-major*/ 0, /*b MN-major*/ 1);
   }
-  p.idesc ^= tc_tune().idesc_xor;
   p.a_layout = ptx::umma_layout_code(wk_b);
   p.b_layout = ptx::umma_layout_code(wn_b);
   p.c_swz_bits = swz_bits_for(wc_b);
