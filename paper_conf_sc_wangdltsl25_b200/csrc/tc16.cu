@@ -51,6 +51,7 @@
 
 #include "kernels.h"
 #include "ptx.cuh"
+#include "sched.cuh"
 
 namespace kami {
 
@@ -180,40 +181,6 @@ __device__ __forceinline__ void emit8(uint32_t cbase, uint32_t off, uint32_t swz
     ptx::st_shared_v4(a, w[0], w[1], w[2], w[3]);
   }
 }
-
-// Incremental (unit -> entry group, m-tile) and ring (slot, phase) counters:
-// the single-thread producer / MMA roles run one iteration per unit, and with
-// small units their serial instruction latency bounds the kernel (ncu: ~190
-// instructions per unit in the MMA lane with 64-bit divisions), so no
-// divisions or modulos inside the loops.
-struct UnitIter {
-  long long grp;
-  int mt, gstep, mstep, m_tiles;
-  __device__ __forceinline__ UnitIter(long long u0, long long step, int mtiles) {
-    m_tiles = mtiles;
-    grp = u0 / mtiles;
-    mt = (int)(u0 - grp * mtiles);
-    gstep = (int)(step / mtiles);
-    mstep = (int)(step - (long long)gstep * mtiles);
-  }
-  __device__ __forceinline__ void next() {
-    grp += gstep;
-    mt += mstep;
-    if (mt >= m_tiles) {
-      mt -= m_tiles;
-      ++grp;
-    }
-  }
-};
-struct RingPos {
-  uint32_t s = 0, ph = 0;
-  __device__ __forceinline__ void next(uint32_t n) {
-    if (++s == n) {
-      s = 0;
-      ph ^= 1;
-    }
-  }
-};
 
 // FP32 output: 8 accumulators -> 32 contiguous bytes of C (one full sector).
 template <bool kUpd>

@@ -26,6 +26,7 @@
 
 #include "kernels.h"
 #include "ptx.cuh"
+#include "sched.cuh"
 
 namespace kami {
 namespace {
@@ -85,14 +86,16 @@ struct Unit {
   long long e0;
   int mt, ng, m, n, k;
 };
-__device__ __forceinline__ bool unit_of(const VbParams& p, long long u, Unit& U) {
-  const long long grp = u / p.mtiles;
-  U.mt = (int)(u - grp * p.mtiles);
+// Fills U for (entry group grp, m-tile mt).  The size loads (variable-size
+// batches) are consumed one unit later by the callers, so their latency hides
+// behind the current unit's work.  A unit is live iff mt * 128 < m (mixed
+// sizes: an entry may have fewer m-tiles than the widest one).
+__device__ __forceinline__ void unit_fill(const VbParams& p, long long grp, int mt, Unit& U) {
+  U.mt = mt;
   U.e0 = grp * p.G;
   const long long left = p.batch - U.e0;
   U.ng = left < p.G ? (int)left : p.G;
   entry_dims(p, U.e0, U.m, U.n, U.k);
-  return U.mt * 128 < U.m;  // mixed sizes: an entry may have fewer m-tiles
 }
 
 __device__ __forceinline__ void cp_async_wait_n(int n) {
@@ -152,17 +155,35 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     // the MMA warp once its copy group has landed, `lag` stages later, so
     // several stages stream concurrently without register staging.
     const int tid = threadIdx.x;  // 0..127
-    uint32_t it = 0;
+    RingPos rs;
+    uint32_t it = 0;  // stages issued (trace index)
+    UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
+    // the next unit's sizes and entry pointers are fetched one unit ahead:
+    // their global-load latency (the pointer arrays live in HBM) hides behind
+    // this unit's copy issue instead of stalling the table hand-over
+    Unit Un;
+    const uint16_t *pa_n = nullptr, *pb_n = nullptr;
+    auto fetch = [&]() {
+      unit_fill(p, ui.grp, ui.mt, Un);
+      if (tid < Un.ng) {
+        pa_n = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[Un.e0 + tid]);
+        pb_n = p.bsr ? p.Bs + (Un.e0 + tid) * (long long)p.k * p.n : reinterpret_cast<const uint16_t*>(p.B[Un.e0 + tid]);
+      }
+    };
+    if ((long long)blockIdx.x < p.units) fetch();
     for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
-      Unit U;
-      if (!unit_of(p, u, U)) continue;
+      const Unit U = Un;
+      const uint16_t *pa = pa_n, *pb = pb_n;
+      ui.next();
+      if (u + gridDim.x < p.units) fetch();
+      if (U.mt * 128 >= U.m) continue;
       const int m = U.m, n = U.n, k = U.k, G = p.G;
       const int kchunks = (k + 63) / 64;
       const int rows = G > 1 ? U.ng * m : min(128, m - U.mt * 128);  // live tile rows
       ptx::named_bar_sync(3, 128);  // previous unit's items issued: tables reusable
       if (tid < U.ng) {
-        a_tab[tid] = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[U.e0 + tid]);
-        b_tab[tid] = entry_B(p, U.e0 + tid, k, n);
+        a_tab[tid] = pa;
+        b_tab[tid] = pb;
       }
       if (p.bsr) blk_tab[tid] = -1;
       ptx::named_bar_sync(3, 128);
@@ -186,9 +207,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       }
       const int nc8 = n / 8;  // 16-byte chunks per B row of one entry
       const int nc8_shift = (nc8 & (nc8 - 1)) == 0 ? __ffs(nc8) - 1 : -1;  // power-of-two fast path
-      for (int kc = 0; kc < kchunks; ++kc, ++it) {
-        const uint32_t s = it % p.stages;
-        ptx::mbar_wait(&empty[s], ((it / p.stages) & 1) ^ 1);
+      for (int kc = 0; kc < kchunks; ++kc, rs.next(p.stages), ++it) {
+        const uint32_t s = rs.s;
+        ptx::mbar_wait(&empty[s], rs.ph ^ 1);
         if (p.dbg & 4) trace(0, it);
         const uint32_t sa = smem_base + s * p.stage_bytes, sb = sa + kAReg;
         if (!(p.dbg & 2)) {
@@ -260,21 +281,27 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     ptx::cp_async_wait<0>();  // nothing may be in flight when the CTA exits
   } else if (warp == 4) {
     // ------------------------------------------------------------- MMA
-    uint32_t it = 0, acc_it = 0;
+    RingPos rs, ra;
+    uint32_t it = 0, acc_it = 0;  // trace indices
+    UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
+    Unit Un;
+    if ((long long)blockIdx.x < p.units) unit_fill(p, ui.grp, ui.mt, Un);
     for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
-      Unit U;
-      if (!unit_of(p, u, U)) continue;
-      const uint32_t a = acc_it % p.acc_bufs;
-      ptx::mbar_wait(&tempty[a], ((acc_it / p.acc_bufs) & 1) ^ 1);
+      const Unit U = Un;
+      ui.next();
+      if (u + gridDim.x < p.units) unit_fill(p, ui.grp, ui.mt, Un);
+      if (U.mt * 128 >= U.m) continue;
+      const uint32_t a = ra.s;
+      ptx::mbar_wait(&tempty[a], ra.ph ^ 1);
       if (p.dbg & 4) trace(6, acc_it);
       ptx::tc_fence_after();
       const uint32_t d_tmem = tmem_base + a * p.acc_cols;
       const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, p.G * U.n, 0, 1);
       const int kpad = (U.k + 15) / 16 * 16;
       const int kchunks = (U.k + 63) / 64;
-      for (int kc = 0; kc < kchunks; ++kc, ++it) {
-        const uint32_t s = it % p.stages;
-        ptx::mbar_wait(&full[s], (it / p.stages) & 1);
+      for (int kc = 0; kc < kchunks; ++kc, rs.next(p.stages), ++it) {
+        const uint32_t s = rs.s;
+        ptx::mbar_wait(&full[s], rs.ph);
         if (p.dbg & 4) trace(2, it);
         ptx::fence_proxy_async_smem();  // cp.async (generic proxy) writes -> tensor-core reads
         ptx::tc_fence_after();
@@ -293,6 +320,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       if (lane == 0) ptx::umma_commit(&tfull[a]);
       if (p.dbg & 4) trace(3, acc_it);
       __syncwarp();
+      ra.next(p.acc_bufs);
       ++acc_it;
     }
   } else {
@@ -301,14 +329,27 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     const int sp = warp & 3;
     const int L = sp * 32 + lane;
     const uint32_t cst = smem_base + p.c_off + wg * kCBuf;
-    uint32_t acc_it = 0;
+    RingPos ra;
+    uint32_t live = 0;  // live units seen (the warpgroups take alternate live units)
+    UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
+    Unit Un;
+    uint16_t* pc_n = nullptr;
+    auto fetch = [&]() {
+      unit_fill(p, ui.grp, ui.mt, Un);
+      if (L < Un.ng) pc_n = entry_C(p, Un.e0 + L, Un.m, Un.n);
+    };
+    if ((long long)blockIdx.x < p.units) fetch();
     for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
-      Unit U;
-      if (!unit_of(p, u, U)) continue;
-      const uint32_t a = acc_it % p.acc_bufs;
-      const uint32_t aph = (acc_it / p.acc_bufs) & 1;
-      const bool mine = (int)(acc_it & 1) == wg;  // warpgroups take alternate units
-      ++acc_it;
+      const Unit U = Un;
+      uint16_t* const pc = pc_n;
+      ui.next();
+      if (u + gridDim.x < p.units) fetch();
+      if (U.mt * 128 >= U.m) continue;
+      const uint32_t a = ra.s;
+      const uint32_t aph = ra.ph;
+      ra.next(p.acc_bufs);
+      const bool mine = (int)(live & 1) == wg;
+      ++live;
       if (!mine) continue;
       const int m = U.m, n = U.n, G = p.G;
       const int rows = G > 1 ? U.ng * m : min(128, m - U.mt * 128);
@@ -318,9 +359,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       const int glo = G > 1 ? (sp * 32) / m : 0;
       const int ghi = G > 1 ? min(U.ng - 1, (sp * 32 + 31) / m) : 0;
       const bool warp_live = sp * 32 < rows;
-      if (L < U.ng) c_tab[wg * 8 + L] = entry_C(p, U.e0 + L, m, n);  // read after the staging barrier
+      if (L < U.ng) c_tab[wg * 8 + L] = pc;  // read after the staging barrier
       ptx::mbar_wait(&tfull[a], aph);
-      if (p.dbg & 4) trace(4, acc_it);
+      if (p.dbg & 4) trace(4, live);
       ptx::tc_fence_after();
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
       for (int h0 = 0; h0 < n; h0 += 128) {
@@ -374,7 +415,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) ptx::mbar_arrive(&tempty[a]);
-      if (p.dbg & 4) trace(5, acc_it);
+      if (p.dbg & 4) trace(5, live);
     }
   }
   ptx::tc_fence_before();
