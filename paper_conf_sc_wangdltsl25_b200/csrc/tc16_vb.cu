@@ -130,6 +130,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   const uint16_t** a_tab = reinterpret_cast<const uint16_t**>(blk_tab + 128);
   const uint16_t** b_tab = a_tab + 8;
   uint16_t** c_tab = reinterpret_cast<uint16_t**>(const_cast<uint16_t**>(b_tab + 8));  // [2 warpgroups][8]
+  int* rp_tab = reinterpret_cast<int*>(c_tab + 16);  // SpMM: the unit's row_ptr values [G][mb + 1] (<= 32)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < p.stages; ++s) {
@@ -163,17 +164,31 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     // this unit's copy issue instead of stalling the table hand-over
     Unit Un;
     const uint16_t *pa_n = nullptr, *pb_n = nullptr;
+    // SpMM: the next unit's block structure is fetched ahead too, without the
+    // row_ptr -> col_blk dependency: every col_blk slot of the unit's entries
+    // (<= 2 per thread: G mb kb <= 256) and every row_ptr value (<= 17)
+    const int mbk = p.bsr ? p.m / 16 : 0, rpn = mbk + 1;
+    int cb_n[2] = {-1, -1}, rp_n = 0;
     auto fetch = [&]() {
       unit_fill(p, ui.grp, ui.mt, Un);
       if (tid < Un.ng) {
         pa_n = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[Un.e0 + tid]);
         pb_n = p.bsr ? p.Bs + (Un.e0 + tid) * (long long)p.k * p.n : reinterpret_cast<const uint16_t*>(p.B[Un.e0 + tid]);
       }
+      if (p.bsr) {
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          const int idx = tid + 128 * q;
+          cb_n[q] = idx < Un.ng * p.max_nnzb ? __ldg(p.colblk + Un.e0 * (long long)p.max_nnzb + idx) : -1;
+        }
+        if (tid < Un.ng * rpn) rp_n = __ldg(p.rowptr + Un.e0 * (long long)rpn + tid);
+      }
     };
     if ((long long)blockIdx.x < p.units) fetch();
     for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
       const Unit U = Un;
       const uint16_t *pa = pa_n, *pb = pb_n;
+      const int cb0 = cb_n[0], cb1 = cb_n[1], rpv = rp_n;
       ui.next();
       if (u + gridDim.x < p.units) fetch();
       if (U.mt * 128 >= U.m) continue;
@@ -185,23 +200,28 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         a_tab[tid] = pa;
         b_tab[tid] = pb;
       }
-      if (p.bsr) blk_tab[tid] = -1;
+      if (p.bsr) {
+        blk_tab[tid] = -1;
+        if (tid < U.ng * rpn) rp_tab[tid] = rpv;
+      }
       ptx::named_bar_sync(3, 128);
       if (p.bsr) {
-        // block lookup table of this tile: tile block row -> global block slot
-        const int mb = m / 16;
-        for (int g = 0; g < U.ng; ++g) {
-          const long long e = U.e0 + g;
-          const int br0 = U.mt * 8, br1 = min(br0 + 8, mb);
-          const int tb0 = g * (m / 16) - br0;  // tile block row of the entry's block row 0
-          const int* rp = p.rowptr + e * (mb + 1);
-          const int j0 = __ldg(rp + br0), j1 = __ldg(rp + br1);
-          for (int j = j0 + tid; j < j1; j += 128) {
-            int br = br0;
-            while (__ldg(rp + br + 1) <= j) ++br;
-            blk_tab[(tb0 + br) * 16 + __ldg(p.colblk + e * (long long)p.max_nnzb + j)] =
-                (int)(e * p.max_nnzb + j);
-          }
+        // block lookup table of this tile: tile block row -> global block slot.
+        // Slot idx = g max_nnzb + j of entry g lies in block row br with
+        // rp[br] <= j < rp[br + 1]; only rows [br0, br1) belong to this m-tile.
+        const int br0 = U.mt * 8, br1 = min(br0 + 8, mbk);
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          const int idx = tid + 128 * q;
+          const int col = q ? cb1 : cb0;
+          if (col < 0) continue;
+          const int g = idx / p.max_nnzb, j = idx - g * p.max_nnzb;
+          const int* rpg = rp_tab + g * rpn;
+          if (j >= rpg[mbk]) continue;  // unused tail slot
+          int br = 0;
+          while (rpg[br + 1] <= j) ++br;
+          if (br < br0 || br >= br1) continue;
+          blk_tab[(g * mbk + br - br0) * 16 + col] = (int)((U.e0 + g) * p.max_nnzb + j);
         }
         ptx::named_bar_sync(3, 128);
       }
