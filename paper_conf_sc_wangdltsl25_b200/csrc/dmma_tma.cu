@@ -54,7 +54,9 @@ template <int M, int N, int K, int P, int TEAMS, bool kUpd>
 __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(const __grid_constant__ DmmaTmaParams prm) {
   using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-byte aligned base; pointer arithmetic on the __shared__ array keeps
+  // the address space, so table reads compile to LDS rather than generic loads
+  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + TEAMS * 2 * Cfg::A_BYTES);  // [TEAMS][2]
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int team = warp / P, w = warp % P;

@@ -119,7 +119,9 @@ __device__ __forceinline__ void trace(int ev, uint32_t i) {
 template <bool kBF16>
 __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __grid_constant__ VbParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
-  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  // 1024-byte aligned base; pointer arithmetic on the __shared__ array keeps
+  // the address space, so table reads compile to LDS rather than generic loads
+  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + p.bar_off);
   uint64_t* empty = full + kMaxStages;
   uint64_t* tfull = empty + kMaxStages;
@@ -233,20 +235,27 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         if (p.dbg & 4) trace(0, it);
         const uint32_t sa = smem_base + s * p.stage_bytes, sb = sa + kAReg;
         if (!(p.dbg & 2)) {
-        // A: thread = (16-byte chunk j, row r0 + 16 q): a warp covers 4 whole
-        // 128-byte row segments, the swizzle phase (r & 7) is fixed per thread
-        // and the addresses advance by constant strides.
+        // Only the K columns the MMA reads in this chunk are written (kpad_c,
+        // a multiple of 16; zero-filled past k): for k < 64 the copy issue --
+        // the producer's bottleneck (tools/trace_vb.py) -- shrinks with k.
+        const int kpad_c = min(64, ((k + 15) & ~15) - kc * 64);
+        // A: thread = (16-byte chunk j, row r0 + rstep q): the chunks of a row
+        // are spread over 2^cshift threads, the swizzle phase (r & 7) is fixed
+        // per thread (rstep is a multiple of 8) and addresses advance by
+        // constant strides.
         {
-          const int j = tid & 7, r0 = tid >> 3;
+          const int cpa = kpad_c >> 3;  // live chunks per row: 2, 4, 6 or 8
+          const int cshift = cpa <= 2 ? 1 : cpa <= 4 ? 2 : 3;
+          const int j = tid & ((1 << cshift) - 1), r0 = tid >> cshift, rstep = 128 >> cshift;
           const int gc = kc * 64 + j * 8;
           const bool col_ok = gc < k;
           const uint32_t dst0 = sa + r0 * 128 + ((j ^ (r0 & 7)) << 4);
-          for (int g = 0; g < U.ng; ++g) {
+          for (int g = 0; g < U.ng && j < cpa; ++g) {
             const int tbase = G > 1 ? g * m : 0;                 // first tile row of the entry
             const int ebase = G > 1 ? 0 : U.mt * 128;            // first entry row in the tile
             const int cnt = G > 1 ? m : rows;                    // entry rows in the tile
             if (p.bsr) {
-              for (int q = r0; q < cnt; q += 16) {
+              for (int q = r0; q < cnt; q += rstep) {
                 const int r = tbase + q;
                 const int slot = col_ok ? blk_tab[(r >> 4) * 16 + (gc >> 4)] : -1;
                 const bool ok = slot >= 0;
@@ -257,8 +266,8 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
             } else {
               const uint16_t* A = a_tab[g];
               const uint16_t* src = A + (long long)(ebase + r0) * k + gc;
-              const long long step = 16ll * k;
-              for (int q = r0; q < cnt; q += 16, src += step)
+              const long long step = (long long)rstep * k;
+              for (int q = r0; q < cnt; q += rstep, src += step)
                 ptx::cp_async_16(dst0 + (tbase + q - r0) * 128, col_ok ? src : A, col_ok ? 16 : 0);
             }
           }
@@ -273,13 +282,13 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
             const uint32_t dcol = sb + (cc >> 3) * 8192;
             const uint16_t* src = B + (long long)(kc * 64 + kr0) * n + j * 8;
             const long long step = (long long)kstep * n;
-            for (int kr = kr0; kr < 64; kr += kstep, src += step) {
+            for (int kr = kr0; kr < kpad_c; kr += kstep, src += step) {
               const bool ok = kc * 64 + kr < k;
               ptx::cp_async_16(dcol + kr * 128 + (((cc & 7) ^ (kr & 7)) << 4), ok ? src : B, ok ? 16 : 0);
             }
           }
         } else {
-          const int per = 64 * nc8;
+          const int per = kpad_c * nc8;
           for (int i = tid; i < U.ng * per; i += 128) {
             const int g = i / per, rem = i - g * per;
             const int kr = rem / nc8, j = rem - kr * nc8;
@@ -421,9 +430,10 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         // copy-out: chunk index i -> (tile row i / cpr, 16-byte chunk i % cpr)
         const int cpr = hw / 8;
         const int cpr_shift = (cpr & (cpr - 1)) == 0 ? __ffs(cpr) - 1 : -1;
+        const uint32_t inv_m = (65536u + m - 1) / m;  // r / m == (r inv_m) >> 16 for r < 256
         for (int i = L; i < rows * cpr; i += 128) {
           const int r = cpr_shift >= 0 ? i >> cpr_shift : i / cpr, c = i - r * cpr;
-          const int ge = G > 1 ? r / m : 0;
+          const int ge = G > 1 ? (int)(((uint32_t)r * inv_m) >> 16) : 0;
           const int er = G > 1 ? r - ge * m : U.mt * 128 + r;
           if (p.dbg & 1) continue;
           uint32_t x0, x1, x2, x3;
