@@ -49,8 +49,44 @@ struct DmmaTmaParams {
   double alpha, beta;  // C = alpha A B + beta C (C read iff beta != 0)
 };
 
+// B_w fragments of k-steps [K0, K1) of one entry (k = t, n = g of each 8x8 block).
+// volatile asm keeps the loads where the schedule puts them relative to the MMAs.
+template <int N, int FN, int K0, int K1, int FK>
+__device__ __forceinline__ void load_b_steps(double (&b)[FK][FN], const double* Bg, int t, int g) {
+#pragma unroll
+  for (int kk = K0; kk < K1; ++kk)
+#pragma unroll
+    for (int j = 0; j < FN; ++j)
+      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(b[kk][j]) : "l"(Bg + (kk * 4 + t) * N + j * 8 + g));
+}
+
+// One k-step range of the entry: A fragments from the swizzled broadcast tile
+// (chunk = col/16, 16-B unit = (col%16)/2 ^ row%8), B_w and C_w in registers.
+template <int M, int FM, int FN, int K0, int K1, int FK>
+__device__ __forceinline__ void mma_steps(double (&c)[FM][FN][2], const double (&b)[FK][FN], uint32_t a_s, int t,
+                                          int g) {
+#pragma unroll
+  for (int kk = K0; kk < K1; ++kk) {
+    const int col = kk * 4 + t;
+    const uint32_t chunk_off = (uint32_t)(col >> 4) * (M * 128) + ((col & 1) << 3);
+    const uint32_t unit = (uint32_t)((col & 15) >> 1);
+#pragma unroll
+    for (int i = 0; i < FM; ++i) {
+      const int row = i * 8 + g;
+      const uint32_t addr = a_s + chunk_off + row * 128 + ((unit ^ (row & 7)) << 4);
+      double a;
+      asm volatile("ld.shared.f64 %0, [%1];" : "=d"(a) : "r"(addr));
+#pragma unroll
+      for (int j = 0; j < FN; ++j)
+        asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                     : "+d"(c[i][j][0]), "+d"(c[i][j][1])
+                     : "d"(a), "d"(b[kk][j]));
+    }
+  }
+}
+
 // kUpd: C = alpha A B + beta C epilogue; the plain instantiation has none of it.
-template <int M, int N, int K, int P, int TEAMS, bool kUpd>
+template <int M, int N, int K, int P, int TEAMS, bool kUpd, bool kRot>
 __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(const __grid_constant__ DmmaTmaParams prm) {
   using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -78,6 +114,14 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
     ptx::mbar_arrive_expect_tx(&tfull[0], Cfg::A_BYTES);
     ptx::tma_load_4d(abuf, &prm.tmA, &tfull[0], 0, 0, 0, (int)first);
   }
+  constexpr int H = Cfg::FK / 2;
+  double b[Cfg::FK][Cfg::FN];
+  // kRot: B_w rotates through the registers half an entry ahead -- the first
+  // k-half of entry e+1 is loaded into the slots of entry e's first k-half as
+  // soon as those MMAs have issued, so the next entry starts without an L2
+  // round trip and no extra registers are needed.
+  if (kRot && first < prm.batch)
+    load_b_steps<N, Cfg::FN, 0, H>(b, prm.B + first * (long long)K * N + w * Cfg::NP, t, g);
   uint32_t it = 0;
   for (long long e = first; e < prm.batch; e += nteams, ++it) {
     const uint32_t s = it & 1;
@@ -91,11 +135,14 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
     }
     // GMem2Reg: this warp's B_w (k x n/p) as DMMA B fragments (k = t, n = g)
     const double* Bg = prm.B + e * (long long)K * N + w * Cfg::NP;
-    double b[Cfg::FK][Cfg::FN];
+    if (kRot) {
+      load_b_steps<N, Cfg::FN, H, Cfg::FK>(b, Bg, t, g);
+    } else {
 #pragma unroll
-    for (int kk = 0; kk < Cfg::FK; ++kk)
+      for (int kk = 0; kk < Cfg::FK; ++kk)
 #pragma unroll
-      for (int j = 0; j < Cfg::FN; ++j) b[kk][j] = __ldg(Bg + (kk * 4 + t) * N + j * 8 + g);
+        for (int j = 0; j < Cfg::FN; ++j) b[kk][j] = __ldg(Bg + (kk * 4 + t) * N + j * 8 + g);
+    }
     double c[Cfg::FM][Cfg::FN][2];
 #pragma unroll
     for (int i = 0; i < Cfg::FM; ++i)
@@ -103,26 +150,10 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
       for (int j = 0; j < Cfg::FN; ++j) c[i][j][0] = c[i][j][1] = 0.0;
     ptx::mbar_wait(&tfull[s], (it >> 1) & 1);
     const uint32_t a_s = ptx::smem_u32(abuf + s * Cfg::A_BYTES);
-#pragma unroll
-    for (int kk = 0; kk < Cfg::FK; ++kk) {
-      // A fragment (row g of each 8-row block, column kk*4 + t) from the
-      // swizzled broadcast tile: chunk = col/16, 16-B unit = (col%16)/2 ^ row%8
-      const int col = kk * 4 + t;
-      const uint32_t chunk_off = (uint32_t)(col >> 4) * (M * 128) + ((col & 1) << 3);
-      const uint32_t unit = (uint32_t)((col & 15) >> 1);
-#pragma unroll
-      for (int i = 0; i < Cfg::FM; ++i) {
-        const int row = i * 8 + g;
-        const uint32_t addr = a_s + chunk_off + row * 128 + ((unit ^ (row & 7)) << 4);
-        double a;
-        asm volatile("ld.shared.f64 %0, [%1];" : "=d"(a) : "r"(addr));
-#pragma unroll
-        for (int j = 0; j < Cfg::FN; ++j)
-          asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
-                       : "+d"(c[i][j][0]), "+d"(c[i][j][1])
-                       : "d"(a), "d"(b[kk][j]));
-      }
-    }
+    mma_steps<M, Cfg::FM, Cfg::FN, 0, H>(c, b, a_s, t, g);
+    if (kRot && en < prm.batch)
+      load_b_steps<N, Cfg::FN, 0, H>(b, prm.B + en * (long long)K * N + w * Cfg::NP, t, g);
+    mma_steps<M, Cfg::FM, Cfg::FN, H, Cfg::FK>(c, b, a_s, t, g);
     // Reg2GMem: C_w, lane holds (row g, cols 2t, 2t+1) of each 8x8 block
     double* Cg = prm.C + e * (long long)M * N + w * Cfg::NP;
 #pragma unroll
@@ -146,7 +177,7 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
   }
 }
 
-template <int M, int N, int K, int P, int TEAMS>
+template <int M, int N, int K, int P, int TEAMS, bool kRot = false>
 kami_status_t launch(long long batch, const void* A, const void* B, void* C, cudaStream_t stream, const char* name,
                      double alpha, double beta) {
   using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
@@ -167,8 +198,8 @@ kami_status_t launch(long long batch, const void* A, const void* B, void* C, cud
   prm.batch = batch;
   prm.alpha = alpha;
   prm.beta = beta;
-  auto fn = (alpha != 1.0 || beta != 0.0) ? kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, true>
-                                          : kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, false>;
+  auto fn = (alpha != 1.0 || beta != 0.0) ? kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, true, kRot>
+                                          : kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, false, kRot>;
   if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM) != cudaSuccess)
     return KAMI_ERROR_CUDA;
   int dev = 0, sms = 148, per_sm = 1;
@@ -189,7 +220,9 @@ kami_status_t launch(long long batch, const void* A, const void* B, void* C, cud
 
 bool dmma_tma_supported(int m, int n, int k) { return m == n && n == k && (m == 16 || m == 32 || m == 64); }
 
-// (p, teams) configuration; env KAMI_DMMA_TMA_CFG = 0/1/2 picks an alternative for sweeps
+// (p, teams) configuration; env KAMI_DMMA_TMA_CFG = 1/2/3/4 picks an alternative for sweeps
+// (64^3 default rotates B half an entry ahead: 25.3 -> 26.1 TF/s, profiles/r1/dmma_tma_sweep_r1.txt;
+// at 16^3 / 32^3 it made no difference and the plain form stays)
 kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
                               cudaStream_t stream, double alpha, double beta) {
   static const int cfg = [] {
@@ -198,14 +231,17 @@ kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* 
   }();
   if (m == 64 && n == 64 && k == 64) {
     if (cfg == 1) return launch<64, 64, 64, 8, 2>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,p8>", alpha, beta);
-    return launch<64, 64, 64, 4, 3>(batch, A, B, C, stream, "kami_dmma_tma_1d<64>", alpha, beta);
+    if (cfg == 4) return launch<64, 64, 64, 4, 3>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,norot>", alpha, beta);
+    return launch<64, 64, 64, 4, 3, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<64>", alpha, beta);
   }
   if (m == 32 && n == 32 && k == 32) {
+    if (cfg == 3) return launch<32, 32, 32, 4, 8, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,rot>", alpha, beta);
     if (cfg == 1) return launch<32, 32, 32, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,p2>", alpha, beta);
     if (cfg == 2) return launch<32, 32, 32, 4, 6>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,t6>", alpha, beta);
     return launch<32, 32, 32, 4, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32>", alpha, beta);
   }
   if (m == 16 && n == 16 && k == 16) {
+    if (cfg == 3) return launch<16, 16, 16, 2, 8, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,rot>", alpha, beta);
     if (cfg == 1) return launch<16, 16, 16, 1, 16>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,p1>", alpha, beta);
     return launch<16, 16, 16, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<16>", alpha, beta);
   }
