@@ -216,7 +216,7 @@ def run_reference(args):
         "impl": "reference", "metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": dtype, "data": "synthetic",
-        "config": workload_config(args, dtype, m, n, k, batch, cfg),
+        "config": dict(workload_config(args, dtype, m, n, k, batch, cfg), timing="host wall clock"),
         "cpu_baseline": {"value": value, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
                          "sample": f"{sample} entries of the workload per step (of {batch}), FP64 triple loop"},
         "e2e": {"value": value, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -229,8 +229,13 @@ def workload_config(args, dtype, m, n, k, batch, cfg):
                         f"(BASELINE.json configs[{cfg}])",
             "m": m, "n": n, "k": k, "batch_per_gpu": batch, "global_batch": batch * args.gpus,
             "layout": "row", "algo": args.algo, "p": args.p, "inputs": "unif [-1,1) RNE to dtype, counter-based SplitMix64",
-            "l2": "inputs larger than L2 (126 MB)" if batch * op_bytes(dtype, m, n, k) > 126e6
-                  else "L2 flushed between timed steps",
+            "l2": "inputs larger than L2 (126 MB)" if batch * op_bytes(dtype, m, n, k) >= 126e6
+                  else f"inputs rotated over {int(-(-3 * 126e6 // (batch * op_bytes(dtype, m, n, k))))} distinct "
+                       "sets (> 3x the 126 MB L2), no flush",
+            "timing": {"graph": "K steps captured in one CUDA graph, replayed between two CUDA events on the "
+                                "launch stream",
+                       "b2b": "K steps launched back to back between two CUDA events on the launch stream",
+                       "events": "one CUDA event pair per step on the launch stream, summed"}[args.timing],
             "parallelism": f"batch-sharded dp{args.gpus}"}
 
 
@@ -245,6 +250,9 @@ def main():
     ap.add_argument("--p", type=int, default=0, help="warps per entry (0 = planner default)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--timing", default="graph", choices=["graph", "b2b", "events"],
+                    help="graph: K steps in one CUDA graph between two events; b2b: K launches back to back "
+                         "between two events; events: one event pair per launch, summed")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
 
@@ -261,24 +269,32 @@ def main():
     dtype, m, n, k, batch, cfg = parse_workload(args.workload)
     update = "upd" in args.workload
     esi, eso = ES_IN.get(dtype, 2), ES_OUT.get(dtype, 2)
-    entry0 = rank * batch
-    A, B = ki.operands(m, n, k, batch, dtype, "unif", seed=0, entry0=entry0, device="cuda")
-    C = torch.zeros(batch * m * n, dtype=ki.TORCH_DTYPES[ki.OUT_DTYPE[dtype]], device="cuda")
-    stream = torch.cuda.current_stream()
     alg_bytes = batch * op_bytes(dtype, m, n, k, update)
     flops = 2.0 * m * n * k * batch
-    small = alg_bytes < 126e6  # L2-resident: flush L2 between timed steps
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda") if small else None
+    # L2-resident workloads (configs[0]: 1.5 MB) rotate over R distinct input /
+    # output sets whose total exceeds 3x the 126 MB L2, so every timed step
+    # reads cold inputs without an L2 flush inside the timed region
+    R = 1 if alg_bytes >= 126e6 else int(-(-3 * 126e6 // alg_bytes))
+    sets = []
+    for r_ in range(R):
+        entry0 = (rank * R + r_) * batch
+        A, B = ki.operands(m, n, k, batch, dtype, "unif", seed=0, entry0=entry0, device="cuda")
+        C = torch.zeros(batch * m * n, dtype=ki.TORCH_DTYPES[ki.OUT_DTYPE[dtype]], device="cuda")
+        sets.append((A, B, C))
+    A, B, C = sets[0]
+    stream = torch.cuda.current_stream()
 
-    def step():
+    def step(i=0):
+        A_, B_, C_ = sets[i % R]
+        st = torch.cuda.current_stream()  # the capture stream while a graph is being recorded
         if update:  # C <- A B + C
-            kami.gemm_strided_batched_axpby(m, n, k, batch, dtype, "row", 1.0, A, B, 1.0, C, stream=stream)
+            kami.gemm_strided_batched_axpby(m, n, k, batch, dtype, "row", 1.0, A_, B_, 1.0, C_, stream=st)
         else:
-            kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A, B, C, algo=args.algo, p=args.p,
-                                      stream=stream)
+            kami.gemm_strided_batched(m, n, k, batch, dtype, "row", A_, B_, C_, algo=args.algo, p=args.p,
+                                      stream=st)
 
-    for _ in range(args.warmup):
-        step()
+    for i in range(args.warmup):
+        step(i)
     torch.cuda.synchronize()
     kernel = kami.last_kernel()
 
@@ -287,26 +303,50 @@ def main():
     sampler.start()
     t_end = time.time() + 1.5
     while time.time() < t_end:
-        for _ in range(20):
-            step()
+        for i in range(20):
+            step(i)
         torch.cuda.synchronize()
 
+    # The K steps are captured once into a CUDA graph (the launch-bound small
+    # configs would otherwise time the host's per-call cost, ~10 us, instead of
+    # the kernels) and replayed between one pair of events on the launch
+    # stream; the per-step average is the kernel's launch duration, gaps
+    # between launches included.  --timing b2b / events for comparison.
+    graph = None
+    if args.timing == "graph":
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            for i in range(args.steps):
+                step(i)
+        graph.replay()  # untimed
+        torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    for s0, s1 in evs:
-        if flush is not None:
-            flush.zero_()
-        s0.record(stream)
-        step()
-        s1.record(stream)
+    if args.timing == "events":
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(args.steps)]
+        for i, (e0, e1) in enumerate(evs):
+            e0.record(stream)
+            step(i)
+            e1.record(stream)
+    else:
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(stream)
+        if graph is not None:
+            graph.replay()
+        else:
+            for i in range(args.steps):
+                step(i)
+        ev1.record(stream)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     sampler.stop()
-    per_launch_ms = [a.elapsed_time(b) for a, b in evs]
-    t_ms = sum(per_launch_ms)  # device time of the K timed steps (flush excluded)
+    if args.timing == "events":
+        t_ms = sum(a.elapsed_time(b) for a, b in evs)
+    else:
+        t_ms = ev0.elapsed_time(ev1)  # device time of the K timed steps
 
     # checksum of the last output (sampled verification happens in tests/)
     csum = float(C.double().sum().item())

@@ -19,12 +19,16 @@ from concurrent.futures import ThreadPoolExecutor
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-OUT = os.path.join(HERE, "libkami.so")
-BUILD = os.path.join(HERE, "_build")
+# KAMI_BUILD_TAG builds an experiment variant (libkami_<tag>.so, objects in
+# _build_<tag>/) with KAMI_EXTRA_FLAGS added, for A/B runs via KAMI_LIB; unset
+# in production.
+_TAG = os.environ.get("KAMI_BUILD_TAG", "")
+OUT = os.path.join(HERE, f"libkami_{_TAG}.so" if _TAG else "libkami.so")
+BUILD = os.path.join(HERE, f"_build_{_TAG}" if _TAG else "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", "--expt-relaxed-constexpr",
-         "-Xptxas", "-v,-warn-spills"]
+         "-Xptxas", "-v,-warn-spills"] + os.environ.get("KAMI_EXTRA_FLAGS", "").split()
 
 
 def _sources():

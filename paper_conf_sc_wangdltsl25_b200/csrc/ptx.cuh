@@ -44,6 +44,9 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
+#ifndef KAMI_MBAR_HINT_NS
+#define KAMI_MBAR_HINT_NS 0x989680
+#endif
 // Waits with a suspend-time hint so a waiting warp is parked by the hardware
 // instead of re-issuing try_wait (spinning warps steal issue slots from the
 // producer / epilogue warps that share their SM sub-partition).
@@ -54,7 +57,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       "WAIT_%=:\n\t"
       "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1, %2;\n\t"
       "@!P1 bra WAIT_%=;\n\t}" ::"r"(addr),
-      "r"(parity), "r"(0x989680)
+      "r"(parity), "r"(KAMI_MBAR_HINT_NS)
       : "memory");
 }
 

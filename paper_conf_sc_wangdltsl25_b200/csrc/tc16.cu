@@ -57,6 +57,14 @@ namespace kami {
 
 namespace {
 
+// Diagnostic builds only (-DKAMI_PHASE_TIMING, tools/latency.py): CTA 0 records
+// clock64 at the pipeline's phase boundaries and prints them at exit.
+#ifdef KAMI_PHASE_TIMING
+#define KAMI_TS(i) (kami_ts[i] = clock64())
+#else
+#define KAMI_TS(i) ((void)0)
+#endif
+
 constexpr int kThreads = 320;  // 10 warps: TMA, MMA, 2 x 4 epilogue
 constexpr int kXposeThreads = 128;  // TF32: 4 more warps transpose B
 constexpr int kEpiThreads = 128;
@@ -232,6 +240,10 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
+#ifdef KAMI_PHASE_TIMING
+  __shared__ long long kami_ts[12];
+  if (threadIdx.x == 0) KAMI_TS(0);
+#endif
 
   if (threadIdx.x == 0) {
     ptx::prefetch_tmap(&p.tmA);
@@ -255,6 +267,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (threadIdx.x == 0 && blockIdx.x == 0) KAMI_TS(1);
 
   const uint32_t smem_base = ptx::smem_u32(smem);
 
@@ -272,6 +285,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
           uint8_t* sb = sa + p.a_region;
           ptx::tma_load_3d(sa, &p.tmA, &full[r.s], kc * p.Wk, ui.mt * 128, e0);
           ptx::tma_load_4d(kXpose ? sa + p.b_raw_off : sb, &p.tmB, &full[r.s], 0, kc * p.Wk, 0, e0);
+          if (u == blockIdx.x && kc == 0) KAMI_TS(2);
         }
       }
     }
@@ -290,6 +304,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
         ptx::mbar_wait(kXpose ? &bready[r.s] : &full[r.s], r.ph);
         ptx::tc_fence_after();
+        if (lane == 0 && u == blockIdx.x && kc == 0) KAMI_TS(3);
         if (lane == 0) {
           const uint64_t ad = adesc0 + r.s * stage16, bd = bdesc0 + r.s * stage16;
           const int nsteps = (kc == p.k_chunks - 1) ? p.ksteps_last : p.ksteps_full;
@@ -306,6 +321,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
         __syncwarp();
       }
       if (lane == 0) ptx::umma_commit(&tfull[ra.s]);  // accumulator complete
+      if (lane == 0) KAMI_TS(4);
       __syncwarp();
     }
   } else if (kXpose && warp >= kThreads / 32) {
@@ -402,6 +418,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       ptx::named_bar_sync(bar_id, kEpiThreads);
       ptx::mbar_wait(&tfull[a], aph);
       ptx::tc_fence_after();
+      if (leader && wg == 0 && u == u0) KAMI_TS(5);
       if (kUpd && !kDirect && p.scale == 2) ptx::mbar_wait(&cfull[wg * 2 + cb], cpos.ph);
       const uint32_t cbase = c_smem + cb * p.c_buf_bytes;
       for (int j = 0; j < p.U; ++j) {
@@ -460,15 +477,26 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       if (leader) {
         ptx::tma_store_4d(&p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mt * 128, 0, (int)e0);
         ptx::bulk_commit();
+        if (wg == 0) KAMI_TS(6);
       }
     }
     if (!kDirect && leader) ptx::bulk_wait<0>();
+    if (leader && wg == 0) KAMI_TS(7);
   }
 
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
   if (warp == 1) ptx::tmem_dealloc(tmem_base, p.tmem_cols);
+#ifdef KAMI_PHASE_TIMING
+  if (threadIdx.x == 0 && blockIdx.x == 0) {
+    KAMI_TS(8);
+    printf("KAMI_TS setup %lld firstTMA %lld dataLanded %lld lastCommit %lld accReady %lld storeIssued %lld "
+           "storeDone %lld exit %lld\n",
+           kami_ts[1] - kami_ts[0], kami_ts[2] - kami_ts[0], kami_ts[3] - kami_ts[0], kami_ts[4] - kami_ts[0],
+           kami_ts[5] - kami_ts[0], kami_ts[6] - kami_ts[0], kami_ts[7] - kami_ts[0], kami_ts[8] - kami_ts[0]);
+  }
+#endif
 }
 
 // ------------------------------------------------------------------- host
