@@ -89,13 +89,23 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
     return tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), rp.A, rp.B, C, (float)alpha,
                             (float)beta, stream, 0);
   }
-  // 16-bit pointer arrays: the LDG-fed tcgen05 kernel covers the whole size grid
+  // 16-bit pointer arrays: the LDG-fed tcgen05 kernel covers the whole size
+  // grid; square orders 16 and 32 go to the warp-level HMMA 1D instead, which
+  // is faster there (f16 x 65 536: 16^3 4.4 -> 22.0, 32^3 26.5 -> 47.9 TFLOP/s;
+  // tcgen05 wins from 64^3 on, profiles/r1/ptr_ab_r1.txt)
+  const bool ptr_warp = Ca && is16(dtype) && algo == KAMI_ALGO_AUTO && rp.m == rp.n && rp.n == rp.k &&
+                        rp.m <= 32 && warp_ca_default_p(rp.m, rp.n, rp.k, dtype, 1) != 0;
+  if (ptr_warp && !update)
+    return warp_ca_launch(rp.m, rp.n, rp.k, batch, dtype, 1, warp_ca_default_p(rp.m, rp.n, rp.k, dtype, 1), rp.A,
+                          rp.B, C, rp.Aa, rp.Ba, Ca, stream);
   if (Ca && is16(dtype) && algo == KAMI_ALGO_AUTO)
     return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, rp.m, rp.n, rp.k, nullptr, nullptr, nullptr, rp.m, rp.n,
                           rp.Aa, rp.Ba, Ca, stream);
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
+  if (plan.kernel == 1 && update && is16(dtype) && algo == KAMI_ALGO_AUTO && !Ca)
+    plan.kernel = 0;  // the update form (C read) exists on tcgen05 only
   if (plan.kernel == 0) {
     return tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), rp.A, rp.B, C, (float)alpha,
                             (float)beta, stream, 0);

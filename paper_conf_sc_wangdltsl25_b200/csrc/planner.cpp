@@ -106,6 +106,13 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
   // 16-bit strided: the tcgen05 family implements 1D with p = 4 sub-partition
   // tensor cores (tc16.cu); it covers the whole 16-bit size grid.  An explicit
   // p > 0 selects the warp-level family with p warps instead.
+  // 16^3 FP16 / BF16 AUTO: the warp-level HMMA 1D (p = 1, LDG-fed, register
+  // resident) beats the tcgen05 kernel at every batch measured -- 32-byte TMA
+  // rows and a per-unit fixed cost bound tcgen05 there (configs[0] 4.8 ->
+  // 2.2 us per launch; 65 536 entries 19 -> 27 TFLOP/s, profiles/r1/small16_r1.txt)
+  if (algo == KAMI_ALGO_AUTO && !pointer_array && m == 16 && n == 16 && k == 16 &&
+      (dtype == KAMI_DTYPE_F16 || dtype == KAMI_DTYPE_BF16))
+    return planner_choose(m, n, k, dtype, KAMI_ALGO_1D, 1, pointer_array, out);
   if (is16 && !pointer_array &&
       (algo == KAMI_ALGO_AUTO || algo == KAMI_ALGO_1D_TMA || (algo == KAMI_ALGO_1D && p == 0))) {
     Tc16Shape s;

@@ -691,6 +691,8 @@ bool lookup(int m, int n, int k, kami_dtype_t dtype, int algo, int p, LaunchInfo
   KAMI_CASE(B16, KAMI_DTYPE_BF16, 64, 64, 64, 4, SchedNonCA, 8, "kami_warp_nonca8<bf16,64>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 128, 128, 128, 4, SchedNonCA, 16, "kami_warp_nonca16<f16,128>")
   // FP16 / BF16 HMMA (m16n8k16): CA evidence family
+  KAMI_CASE(H16, KAMI_DTYPE_F16, 16, 16, 16, 1, Sched1D, 1, "kami_warp_ca_1d<f16,16>")
+  KAMI_CASE(B16, KAMI_DTYPE_BF16, 16, 16, 16, 1, Sched1D, 1, "kami_warp_ca_1d<bf16,16>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 1, Sched1D, 2, "kami_warp_ca_1d<f16,32>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 2, Sched2D, 4, "kami_warp_ca_2d<f16,32>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 4, SchedNonCA, 4, "kami_warp_nonca<f16,32>")

@@ -96,6 +96,9 @@ def test_plan_covers_the_16bit_grid():
         for n in (16, 64, 256):
             for k in (8, 16, 40, 64, 256):
                 p = kami.plan(m, n, k, "bf16")
+                if (m, n, k) == (16, 16, 16):  # planner rule: warp-level HMMA 1D, p = 1
+                    assert p["kernel"] == "warp_ca" and p["algo"] == "1d" and p["p"] == 1
+                    p = kami.plan(m, n, k, "bf16", algo="1d")  # 1D with p = 0: tcgen05
                 assert p["kernel"] == "tcgen05" and p["stages"] >= 2, (m, n, k)
 
 

@@ -48,7 +48,7 @@ def run_and_sample(dtype, m, n, k, batch, dist="unif", algo="auto"):
     return worst, kami.last_kernel()
 
 
-@pytest.mark.parametrize("wl", ["f16-32", "f16-64", "f16-128", "lr-8", "lr-16", "lr-32", "f64-16", "f64-32",
+@pytest.mark.parametrize("wl", ["f16-16", "f16-32", "f16-64", "f16-128", "lr-8", "lr-16", "lr-32", "f64-16", "f64-32",
                                 "f64-64"])
 def test_fullsize_sampled(wl):
     dtype, m, n, k, batch, _ = WORKLOADS[wl]

@@ -72,7 +72,7 @@ TC_SHAPES = [
 @pytest.mark.parametrize("layout", ["row", "col"])
 def test_tc16_unif(shape, dtype, layout):
     m, n, k, batch = shape
-    check(m, n, k, batch, dtype, layout, "unif")
+    check(m, n, k, batch, dtype, layout, "unif", algo="1d")  # 1D with p = 0: the tcgen05 kernel for every shape
     assert kami.last_kernel().startswith("kami_tc16_1d_kernel")
 
 
@@ -81,7 +81,17 @@ def test_tc16_unif(shape, dtype, layout):
 def test_tc16_int_bit_exact(shape, dtype):
     m, n, k, batch = shape
     for layout in ("row", "col"):
-        check(m, n, k, batch, dtype, layout, "int", seed=1)
+        check(m, n, k, batch, dtype, layout, "int", seed=1, algo="1d")
+        assert kami.last_kernel().startswith("kami_tc16_1d_kernel")
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_auto_16cubed_picks_warp_hmma(dtype):
+    """AUTO at 16^3 (configs[0]) routes to the warp-level HMMA 1D (planner rule), both layouts."""
+    for layout in ("row", "col"):
+        check(16, 16, 16, 1029, dtype, layout, "int", seed=1)
+        assert kami.last_kernel() == f"kami_warp_ca_1d<{dtype},16>"
+    check(16, 16, 16, 1029, dtype, "row", "unif")
 
 
 def test_tc16_seeds_and_single():
@@ -94,12 +104,12 @@ def test_tc16_seeds_and_single():
 WARP_CASES = [(dt, s, a) for dt in ("f64",) for s in (16, 32, 64) for a in ("1d", "2d", "3d", "nonca")]
 WARP_CASES += [(dt, 32, a) for dt in ("f16", "bf16") for a in ("1d", "2d", "nonca")]
 WARP_CASES += [(dt, 64, a) for dt in ("f16", "bf16") for a in ("1d", "2d", "3d", "nonca")]
-WARP_CASES += [("f16", 128, "1d"), ("f16", 128, "2d"), ("f64", 8, "1d")]
+WARP_CASES += [("f16", 128, "1d"), ("f16", 128, "2d"), ("f64", 8, "1d"), ("f16", 16, "1d"), ("bf16", 16, "1d")]
 
 
 def warp_p(dtype, s, algo):
     # 16-bit 1D with p = 0 means the tcgen05 kernel; name the warp count explicitly
-    return {32: 2, 64: 4, 128: 8}[s] if (dtype != "f64" and algo == "1d") else 0
+    return {16: 1, 32: 2, 64: 4, 128: 8}[s] if (dtype != "f64" and algo == "1d") else 0
 
 
 @pytest.mark.parametrize("dtype,s,algo", WARP_CASES, ids=lambda x: str(x))

@@ -17,7 +17,7 @@ def _tol(dtype, k):
 
 
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
-@pytest.mark.parametrize("shape", [(16, 16, 16), (64, 64, 64), (48, 80, 40), (256, 256, 8), (192, 64, 256),
+@pytest.mark.parametrize("shape", [(16, 16, 16), (32, 32, 32), (64, 64, 64), (48, 80, 40), (256, 256, 8), (192, 64, 256),
                                    (128, 256, 24), (32, 16, 256)])
 def test_pointer_array_all_sizes(dtype, shape):
     m, n, k = shape
@@ -32,7 +32,9 @@ def test_pointer_array_all_sizes(dtype, shape):
         pc = torch.tensor([dC[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
         kami.gemm_batched(m, n, k, batch, dtype, layout, pa, pb, pc)
         torch.cuda.synchronize()
-        assert kami.last_kernel().startswith("kami_tc16_vb_kernel")
+        # square orders 16 / 32 go to the warp-level HMMA 1D (dispatch rule), the rest to tcgen05
+        want = "kami_warp_ca_1d" if (m == n == k and m <= 32) else "kami_tc16_vb_kernel"
+        assert kami.last_kernel().startswith(want), kami.last_kernel()
         Cref, S = oracle.gemm(m, n, k, batch, dtype, layout, ki.as_bits(A), ki.as_bits(B), with_scale=True)
         got_bits = oracle.to_row_major(ki.as_bits(dC.cpu()), batch, m, n, layout)
         if dist == "int":
