@@ -88,6 +88,7 @@ struct alignas(64) Tc16Params {
   CUtensorMap tmA;  // 3-D (k, m, batch), box (Wk, rowsA, G)
   CUtensorMap tmB;  // 4-D (Wn, k, n/Wn, batch), box (Wn, Wk, n/Wn, G)
   CUtensorMap tmC;  // 4-D (Wc, m, n/Wc, batch), box (Wc, rows_tile, n/Wc, G)
+  CUtensorMap tmCa; // split stores: same tensor, box (Wc, rows_tile, 1, 1) = one 64-column atom
   long long batch;
   long long units;
   int m, n, k;
@@ -113,6 +114,7 @@ struct alignas(64) Tc16Params {
   int wn_b, wk_b;           // atom widths in bytes
   void* Cg;                 // FP32 output: direct stores
   int scale;  // 0: C = AB, 1: C = alpha AB, 2: C = alpha AB + beta C (C read)
+  int split_store;  // G == U == 1, 64-column atoms, n >= 128: one TMA store per atom as it is written
 };
 
 template <int kIn>
@@ -220,7 +222,7 @@ __device__ __forceinline__ void emit8_f32_global(float* dst, const uint32_t* v, 
 
 // kUpd: the C-update epilogue (alpha != 1 or beta != 0); the plain C = AB
 // instantiation carries none of its code.
-template <int kIn, int kOut, bool kUpd>
+template <int kIn, int kOut, bool kUpd, bool kSplit>
 __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const __grid_constant__ Tc16Params p) {
   constexpr bool kXpose = kIn == IN_TF32;
   constexpr bool kDirect = kOut == OUT_F32;
@@ -249,6 +251,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     ptx::prefetch_tmap(&p.tmA);
     ptx::prefetch_tmap(&p.tmB);
     ptx::prefetch_tmap(&p.tmC);
+    if (kSplit) ptx::prefetch_tmap(&p.tmCa);
     for (int s = 0; s < p.stages; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
@@ -406,7 +409,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       const bool valid0 = row_ok && (p.G > 1 || mt * 128 + L < p.m);
       // the TMA store that last read staging buffer cb must be done reading
       if (!kDirect && leader) {
-        if (p.c_bufs == 2) ptx::bulk_wait_read<1>();
+        if (p.c_bufs == 2 && !kSplit) ptx::bulk_wait_read<1>();
         else ptx::bulk_wait_read<0>();
         if (kUpd && p.scale == 2) {  // C update: bring the old C tile into the staging buffer
           uint64_t* cf = &cfull[wg * 2 + cb];
@@ -421,6 +424,50 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       if (leader && wg == 0 && u == u0) KAMI_TS(5);
       if (kUpd && !kDirect && p.scale == 2) ptx::mbar_wait(&cfull[wg * 2 + cb], cpos.ph);
       const uint32_t cbase = c_smem + cb * p.c_buf_bytes;
+      if constexpr (kSplit && !kDirect) {
+        // one 64-column atom per chunk; every warp walks every chunk (the
+        // per-atom named barriers need all four), the accumulator is released
+        // as soon as its last TMEM load has landed, and each atom's TMA store
+        // is issued as soon as it is staged, so the store engine starts on
+        // atom 0 while atoms 1.. are still being converted
+        const bool active = col_hi > col_lo;
+        const bool valid = valid0 && (e0 + g < p.batch);
+        const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
+        uint8_t* cbuf = smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes;
+        for (int c0 = 0; c0 < p.n; c0 += 64) {
+          uint32_t v[64];
+          if (active) {
+            ptx::tmem_ld_32x32b_x32(t_row + c0, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+            ptx::tmem_ld_32x32b_x32(t_row + c0 + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+          }
+          ptx::tmem_wait_ld();
+          if (c0 + 64 >= p.n) {  // accumulator a may be overwritten by the next MMA chain
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive(&tempty[a]);
+          }
+          const uint32_t atom = (uint32_t)(c0 >> 6);
+          if (valid) {
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+              emit8<kOut, kUpd>(cbase, rowbase + atom * atom_stride + (uint32_t)(8 * q) * ESO, p.c_swz_bits,
+                                &v[8 * q], p);
+          }
+          ptx::fence_proxy_async_smem();
+          ptx::named_bar_sync(bar_id, kEpiThreads);
+          if (leader) {
+            ptx::tma_store_4d(&p.tmCa, cbuf + atom * atom_stride, 0, mt * 128, (int)atom, (int)e0);
+            ptx::bulk_commit();
+          }
+        }
+        a += 2;
+        if (a >= (uint32_t)p.acc_bufs) {
+          a -= p.acc_bufs;
+          aph ^= 1;
+        }
+        cpos.next(p.c_bufs);
+        continue;
+      }
       for (int j = 0; j < p.U; ++j) {
       const bool valid = valid0 && (e0 + j * p.G + g < p.batch);
       float* crow = nullptr;
@@ -524,16 +571,16 @@ int out_es(int out) { return out == OUT_F32 ? 4 : 2; }
 
 constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 
-// Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo,U"
+// Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo,U,split"
 // (0 / -1 = planner default; promo = TMA L2 promotion 0 none, 1 64B, 2 128B, 3 256B;
-// U = sub-tiles per unit).  Unset in production.
+// U = sub-tiles per unit; split = -1 disables per-atom C stores).  Unset in production.
 struct TcTune {
-  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0;
+  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0;
 };
 const TcTune& tc_tune() {
   static const TcTune t = [] {
     TcTune r;
-    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U);
+    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split);
     return r;
   }();
   return t;
@@ -541,12 +588,18 @@ const TcTune& tc_tune() {
 
 template <int kIn, int kOut>
 void launch_kernel(const Tc16Params& p, unsigned grid, size_t smem, cudaStream_t stream, const char* name) {
-  if (p.scale) {
-    cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    kami_tc16_1d_kernel<kIn, kOut, true><<<grid, threads_for(kIn), smem, stream>>>(p);
+  if (p.scale) {  // the update form always stores whole units
+    cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)smem);
+    kami_tc16_1d_kernel<kIn, kOut, true, false><<<grid, threads_for(kIn), smem, stream>>>(p);
+  } else if (kOut != OUT_F32 && p.split_store) {
+    cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)smem);
+    kami_tc16_1d_kernel<kIn, kOut, false, true><<<grid, threads_for(kIn), smem, stream>>>(p);
   } else {
-    cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    kami_tc16_1d_kernel<kIn, kOut, false><<<grid, threads_for(kIn), smem, stream>>>(p);
+    cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         (int)smem);
+    kami_tc16_1d_kernel<kIn, kOut, false, false><<<grid, threads_for(kIn), smem, stream>>>(p);
   }
   set_last_kernel(name);
 }
@@ -732,6 +785,16 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
             swz_mode_for(wn_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
+  // Per-atom C stores (kSplit instantiation) for one-entry tiles with >= 2
+  // 64-column atoms: the store engine starts on atom 0 while the rest is
+  // converted and the accumulator is released early (bf16 16x192x16 0.27 ->
+  // 0.52 of roofline, 192^3 0.66 -> 0.70, 256^3 0.82 -> 0.87, 32x256x64 0.89 ->
+  // 0.95).  Not for full 128-row tiles with k <= 16 (C-store dominated low-rank:
+  // lr-8 0.90 -> 0.84, lr-16 0.92 -> 0.85 measured), profiles/r1/split_store_r1.txt.
+  p.split_store = (out_kind != OUT_F32 && s.G == 1 && s.U == 1 && s.Wc == 64 && n % 64 == 0 && n >= 128 &&
+                   !(s.rows_tile == 128 && k <= 16) && beta == 0.0f && alpha == 1.0f && tc_tune().split >= 0)
+                      ? 1
+                      : 0;
   {  // C: (Wc, m, n/Wc, batch)
     cuuint64_t dims[4] = {(cuuint64_t)s.Wc, (cuuint64_t)m, (cuuint64_t)(n / s.Wc), (cuuint64_t)batch};
     cuuint64_t strides[3] = {(cuuint64_t)n * eso, (cuuint64_t)wc_b, (cuuint64_t)m * n * eso};
@@ -739,6 +802,11 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
     cuuint32_t es[4] = {1, 1, 1, 1};
     if (enc(&p.tmC, dto, 4, C, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz_mode_for(wc_b),
             CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
+    cuuint32_t box1[4] = {(cuuint32_t)s.Wc, (cuuint32_t)s.rows_tile, 1, 1};
+    if (p.split_store && enc(&p.tmCa, dto, 4, C, dims, strides, box1, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                             swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
 

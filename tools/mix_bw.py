@@ -52,6 +52,9 @@ ops = {
     "add_2r1w": (lambda: torch.add(a, b, out=c), 3),
     "addcmul_3r1w": (lambda: torch.addcmul(a, b, d, out=c), 4),
     "sum_read": (lambda: torch.sum(a, dtype=torch.float32), 1),
+    "fill_0r1w": (lambda: c.fill_(1.5), 1),
+    # 1 read : 8 writes (the low-rank k = 16 mix): a 1/8-size source broadcast into c
+    "bcast_1r8w": (lambda: c.view(8, N // 8).copy_(a[: N // 8].view(1, N // 8).expand(8, N // 8)), 1.125),
 }
 out = {}
 for name, (fn, nbuf) in ops.items():
