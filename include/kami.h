@@ -91,7 +91,14 @@ kami_status_t kami_gemm(int m, int n, int k, int64_t batch, kami_dtype_t dtype, 
 
 /* Pointer-array batched GEMM (cuBLAS *gemmBatched convention): A_array,
  * B_array, C_array are DEVICE arrays of `batch` DEVICE pointers, each
- * 16-byte aligned, each pointing at one packed matrix in `layout`. */
+ * 16-byte aligned, each pointing at one packed matrix in `layout`.  Same
+ * operation, sizes, types and errors as kami_gemm_strided_batched (PAPER.md
+ * L523: batched functions "aligned to" cuBLAS / MAGMA); entries may lie
+ * anywhere in the device's address space, C entries must not overlap.  A
+ * misaligned entry pointer cannot be detected before launch (the arrays are
+ * device memory): its result is undefined.  16-bit types run on the same
+ * tcgen05 kernel as the strided form, fed by TMA boxes over an address-space
+ * view of each entry. */
 kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
                                 const void* const* A_array, const void* const* B_array, void* const* C_array,
                                 kami_stream_t stream);

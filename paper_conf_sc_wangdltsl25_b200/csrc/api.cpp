@@ -7,6 +7,7 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdint>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <vector>
@@ -80,6 +81,17 @@ RowProblem to_row(int m, int n, int k, kami_layout_t layout, const void* A, cons
   return {n, m, k, B, A, Ba, Aa};
 }
 
+// Experiment knob for A/B runs (unset in production): KAMI_PTR_ROUTE = tma | vb | warp
+// forces the kernel 16-bit pointer arrays take (1 / 2 / 3; 0 = planner rule).
+int ptr_route() {
+  static const int r = [] {
+    const char* e = getenv("KAMI_PTR_ROUTE");
+    if (!e) return 0;
+    return !strcmp(e, "tma") ? 1 : !strcmp(e, "vb") ? 2 : !strcmp(e, "warp") ? 3 : 0;
+  }();
+  return r;
+}
+
 kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, kami_algo_t algo, int p, void* C,
                        void* const* Ca, cudaStream_t stream, double alpha = 1.0, double beta = 0.0) {
   const bool update = alpha != 1.0 || beta != 0.0;
@@ -89,18 +101,27 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
     return tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), rp.A, rp.B, C, (float)alpha,
                             (float)beta, stream, 0);
   }
-  // 16-bit pointer arrays: the LDG-fed tcgen05 kernel covers the whole size
-  // grid; square orders 16 and 32 go to the warp-level HMMA 1D instead, which
-  // is faster there (f16 x 65 536: 16^3 4.4 -> 22.0, 32^3 26.5 -> 47.9 TFLOP/s;
-  // tcgen05 wins from 64^3 on, profiles/r1/ptr_ab_r1.txt)
+  // 16-bit pointer arrays: the TMA tcgen05 kernel over address-space views
+  // (tc16.cu kPtr; f16 x 65 536: 32^3 58.0, 64^3 140.3, 128^3 280.9, 256x256x16
+  // 77.7 TFLOP/s vs 26.6 / 109.5 / 279.4 / 56.1 on the LDG-fed kernel), except
+  // k = 8 mod 16 (LDG-fed, see tc16.cu) and 16^3, where the warp-level HMMA
+  // 1D is faster (21.7 vs 10.9 TFLOP/s), profiles/r1/ptr_ab_r1.txt
+  const int route = ptr_route();
   const bool ptr_warp = Ca && is16(dtype) && algo == KAMI_ALGO_AUTO && rp.m == rp.n && rp.n == rp.k &&
-                        rp.m <= 32 && warp_ca_default_p(rp.m, rp.n, rp.k, dtype, 1) != 0;
-  if (ptr_warp && !update)
+                        rp.m <= 16 && warp_ca_default_p(rp.m, rp.n, rp.k, dtype, 1) != 0;
+  if (((ptr_warp && route == 0) || route == 3) && !update)
     return warp_ca_launch(rp.m, rp.n, rp.k, batch, dtype, 1, warp_ca_default_p(rp.m, rp.n, rp.k, dtype, 1), rp.A,
                           rp.B, C, rp.Aa, rp.Ba, Ca, stream);
-  if (Ca && is16(dtype) && algo == KAMI_ALGO_AUTO)
+  if (Ca && is16(dtype) && algo == KAMI_ALGO_AUTO) {
+    // the TMA kernel over address-space views (tc16.cu kPtr), else the LDG-fed one
+    if (route != 2) {
+      kami_status_t st = tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), nullptr,
+                                          nullptr, nullptr, 1.0f, 0.0f, stream, 0, rp.Aa, rp.Ba, Ca);
+      if (st != KAMI_ERROR_NOT_SUPPORTED) return st;
+    }
     return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, rp.m, rp.n, rp.k, nullptr, nullptr, nullptr, rp.m, rp.n,
                           rp.Aa, rp.Ba, Ca, stream);
+  }
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;

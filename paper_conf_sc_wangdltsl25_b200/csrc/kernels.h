@@ -33,8 +33,11 @@ kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const
 // in_kind: 0 f16, 1 bf16, 2 tf32, 3 e4m3, 4 e5m2; out_kind: 0 f16, 1 bf16, 2 f32.
 // C = alpha A B + beta C (C is read iff beta != 0).
 kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kind, Tc16Shape* s);
+// Aa/Ba/Ca != nullptr: device pointer arrays (kami_gemm_batched; f16/bf16, C = AB only), A/B/C unused.
 kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind, int out_kind, const void* A,
-                               const void* B, void* C, float alpha, float beta, cudaStream_t stream, int max_ctas);
+                               const void* B, void* C, float alpha, float beta, cudaStream_t stream, int max_ctas,
+                               const void* const* Aa = nullptr, const void* const* Ba = nullptr,
+                               void* const* Ca = nullptr);
 
 // ------------------------------------------------ warp-level CA (literal KAMI)
 // algo: 1 = 1D, 2 = 2D, 3 = 3D, 4 = non-CA tiled.  dtype: KAMI_DTYPE_*.

@@ -115,7 +115,32 @@ struct alignas(64) Tc16Params {
   void* Cg;                 // FP32 output: direct stores
   int scale;  // 0: C = AB, 1: C = alpha AB, 2: C = alpha AB + beta C (C read)
   int split_store;  // G == U == 1, 64-column atoms, n >= 128: one TMA store per atom as it is written
+  // pointer arrays (kPtr): entry e's matrices at Aa[e], Ba[e], Ca[e]; the tensor
+  // maps are address-space views (view_coords) and every entry is its own box
+  const void* const* Aa;
+  const void* const* Ba;
+  void* const* Ca;
+  uint32_t a_entry, b_entry, c_entry;  // shared-memory bytes of one entry's A / B / C box
+  uint32_t entry_tx, entry_tx_t;       // TMA bytes of one entry's A + B boxes per k-chunk (full / tail m-tile)
+  int m_tail;                          // m > 128, m % 128 != 0: the last m-tile uses tmAt / tmCt / tmCat
+  CUtensorMap tmAt, tmCt, tmCat;       // pointer arrays: boxes of m % 128 rows for the last m-tile
 };
+
+// Pointer arrays on TMA.  A tensor map cannot follow a pointer array, but all
+// entries live in one virtual address space: the pointer-array maps describe
+// that space as a tensor whose two outer dimensions are (16-byte offset mod
+// 2^28, 2^28-byte offset) from kViewBase, so the box of the entry at byte
+// address q has outer coordinates ((q - kViewBase) / 16 mod 2^24,
+// (q - kViewBase) / 2^28).  Entries are 16-byte aligned (kami.h), the view
+// covers 2^48 bytes, and the inner dimensions are the entry's own (k, m) /
+// (Wn, k, n/Wn) / (Wc, m, n/Wc), so the usual out-of-bounds fill (k tail,
+// rows past m) and store clipping still apply per entry.
+constexpr unsigned long long kViewBase = 256;
+__device__ __forceinline__ void view_coords(const void* q, int& lo, int& hi) {
+  const unsigned long long off = reinterpret_cast<unsigned long long>(q) - kViewBase;
+  lo = (int)((off >> 4) & 0xFFFFFFull);
+  hi = (int)(off >> 28);
+}
 
 template <int kIn>
 __device__ __forceinline__ void umma(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
@@ -222,7 +247,7 @@ __device__ __forceinline__ void emit8_f32_global(float* dst, const uint32_t* v, 
 
 // kUpd: the C-update epilogue (alpha != 1 or beta != 0); the plain C = AB
 // instantiation carries none of its code.
-template <int kIn, int kOut, bool kUpd, bool kSplit>
+template <int kIn, int kOut, bool kUpd, bool kSplit, bool kPtr = false>
 __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const __grid_constant__ Tc16Params p) {
   constexpr bool kXpose = kIn == IN_TF32;
   constexpr bool kDirect = kOut == OUT_F32;
@@ -274,7 +299,60 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
 
   const uint32_t smem_base = ptx::smem_u32(smem);
 
-  if (warp == 0) {
+  if (kPtr && warp == 0) {
+    // ------------------------------------------- producer, pointer arrays
+    // lane i < G U owns entry e0 + i of each unit: it holds that entry's A / B
+    // view coordinates (fetched one unit ahead, so the pointer loads are off
+    // the critical path) and issues its two TMA boxes; lane 0 does the ring
+    // bookkeeping for the unit's valid entries.
+    RingPos r;
+    UnitIter ui(blockIdx.x, gridDim.x, p.m_tiles);
+    const void* qa = nullptr;
+    const void* qb = nullptr;
+    {
+      const long long e = (long long)(ui.grp * p.GU) + lane;
+      if (lane < p.GU && e < p.batch) {
+        qa = p.Aa[e];
+        qb = p.Ba[e];
+      }
+    }
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
+      const long long e0 = ui.grp * p.GU;
+      const long long left = p.batch - e0;
+      const int nvalid = left < p.GU ? (int)left : p.GU;
+      int alo, ahi, blo, bhi;
+      view_coords(qa, alo, ahi);
+      view_coords(qb, blo, bhi);
+      const int mt = ui.mt;
+      ui.next();
+      const void* na = nullptr;
+      const void* nb = nullptr;
+      if (u + gridDim.x < p.units) {  // next unit's pointers
+        const long long e = (long long)(ui.grp * p.GU) + lane;
+        if (lane < p.GU && e < p.batch) {
+          na = p.Aa[e];
+          nb = p.Ba[e];
+        }
+      }
+      const bool tail = p.m_tail && mt == p.m_tiles - 1;
+      const CUtensorMap* tma = tail ? &p.tmAt : &p.tmA;
+      const uint32_t tx = (uint32_t)nvalid * (tail ? p.entry_tx_t : p.entry_tx);
+      for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
+        if (lane == 0) {
+          ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
+          ptx::mbar_arrive_expect_tx(&full[r.s], tx);
+        }
+        __syncwarp();
+        if (lane < nvalid) {
+          uint8_t* sa = smem + r.s * p.stage_bytes;
+          ptx::tma_load_4d(sa + lane * p.a_entry, tma, &full[r.s], kc * p.Wk, mt * 128, alo, ahi);
+          ptx::tma_load_5d(sa + p.a_region + lane * p.b_entry, &p.tmB, &full[r.s], 0, kc * p.Wk, 0, blo, bhi);
+        }
+      }
+      qa = na;
+      qb = nb;
+    }
+  } else if (warp == 0) {
     // ------------------------------------------------------------ producer
     if (lane == 0) {
       RingPos r;
@@ -402,13 +480,28 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       aph = 1;
     }
     RingPos cpos;
+    // pointer arrays: lane i < G U of the leader warp stores entry e0 + i of the
+    // unit (its own bulk groups); its C view coordinates are fetched one unit ahead
+    const bool storer = kPtr ? (((warp & 3) == 2) && lane < p.GU) : leader;
+    const void* qc = nullptr;
+    if (kPtr && storer && u0 < p.units && ui.grp * p.GU + lane < p.batch) qc = p.Ca[ui.grp * p.GU + lane];
     for (long long u = u0; u < p.units; u += 2ll * gridDim.x, ui.next()) {
       const int mt = ui.mt;
       const long long e0 = ui.grp * p.GU;
       const uint32_t cb = cpos.s;
       const bool valid0 = row_ok && (p.G > 1 || mt * 128 + L < p.m);
+      int clo = 0, chi = 0;
+      bool cstore = false;
+      if constexpr (kPtr) {
+        cstore = storer && e0 + lane < p.batch;
+        view_coords(qc, clo, chi);
+        UnitIter nx = ui;
+        nx.next();
+        qc = nullptr;
+        if (storer && u + 2ll * gridDim.x < p.units && nx.grp * p.GU + lane < p.batch) qc = p.Ca[nx.grp * p.GU + lane];
+      }
       // the TMA store that last read staging buffer cb must be done reading
-      if (!kDirect && leader) {
+      if (!kDirect && storer) {
         if (p.c_bufs == 2 && !kSplit) ptx::bulk_wait_read<1>();
         else ptx::bulk_wait_read<0>();
         if (kUpd && p.scale == 2) {  // C update: bring the old C tile into the staging buffer
@@ -455,8 +548,11 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
           }
           ptx::fence_proxy_async_smem();
           ptx::named_bar_sync(bar_id, kEpiThreads);
-          if (leader) {
-            ptx::tma_store_4d(&p.tmCa, cbuf + atom * atom_stride, 0, mt * 128, (int)atom, (int)e0);
+          if (kPtr ? cstore : leader) {
+            if constexpr (kPtr)
+              ptx::tma_store_5d(p.m_tail && mt == p.m_tiles - 1 ? &p.tmCat : &p.tmCa, cbuf + atom * atom_stride, 0,
+                                mt * 128, (int)atom, clo, chi);
+            else ptx::tma_store_4d(&p.tmCa, cbuf + atom * atom_stride, 0, mt * 128, (int)atom, (int)e0);
             ptx::bulk_commit();
           }
         }
@@ -521,13 +617,19 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       // make the generic-proxy smem writes visible to the TMA engine
       ptx::fence_proxy_async_smem();
       ptx::named_bar_sync(bar_id, kEpiThreads);
-      if (leader) {
+      if constexpr (kPtr) {
+        if (cstore) {
+          ptx::tma_store_5d(p.m_tail && mt == p.m_tiles - 1 ? &p.tmCt : &p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes + lane * p.c_entry, 0,
+                            mt * 128, 0, clo, chi);
+          ptx::bulk_commit();
+        }
+      } else if (leader) {
         ptx::tma_store_4d(&p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mt * 128, 0, (int)e0);
         ptx::bulk_commit();
         if (wg == 0) KAMI_TS(6);
       }
     }
-    if (!kDirect && leader) ptx::bulk_wait<0>();
+    if (!kDirect && storer) ptx::bulk_wait<0>();
     if (leader && wg == 0) KAMI_TS(7);
   }
 
@@ -588,6 +690,21 @@ const TcTune& tc_tune() {
 
 template <int kIn, int kOut>
 void launch_kernel(const Tc16Params& p, unsigned grid, size_t smem, cudaStream_t stream, const char* name) {
+  if constexpr (kIn <= IN_BF16) {
+    if (p.Aa) {  // pointer arrays (C = AB only)
+      if (p.split_store) {
+        cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false, true, true>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        kami_tc16_1d_kernel<kIn, kOut, false, true, true><<<grid, threads_for(kIn), smem, stream>>>(p);
+      } else {
+        cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false, false, true>,
+                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        kami_tc16_1d_kernel<kIn, kOut, false, false, true><<<grid, threads_for(kIn), smem, stream>>>(p);
+      }
+      set_last_kernel(kIn == IN_BF16 ? "kami_tc16_1d_kernel<bf16,ptr>" : "kami_tc16_1d_kernel<f16,ptr>");
+      return;
+    }
+  }
   if (p.scale) {  // the update form always stores whole units
     cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, true, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                          (int)smem);
@@ -680,7 +797,10 @@ kami_status_t tc16_plan_shape(int m, int n, int k, Tc16Shape* s) {
 }
 
 kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind, int out_kind, const void* A,
-                               const void* B, void* C, float alpha, float beta, cudaStream_t stream, int max_ctas) {
+                               const void* B, void* C, float alpha, float beta, cudaStream_t stream, int max_ctas,
+                               const void* const* Aa, const void* const* Ba, void* const* Ca) {
+  const bool ptr = Aa != nullptr;
+  if (ptr && (in_kind > IN_BF16 || alpha != 1.0f || beta != 0.0f || !Ba || !Ca)) return KAMI_ERROR_NOT_SUPPORTED;
   Tc16Shape s;
   kami_status_t st = tc16_plan_shape_kind(m, n, k, in_kind, out_kind, &s);
   if (st != KAMI_SUCCESS) return st;
@@ -767,6 +887,46 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
                                                         : CU_TENSOR_MAP_DATA_TYPE_FLOAT32;
   const CUtensorMapL2promotion promo =
       tc_tune().promo < 0 ? CU_TENSOR_MAP_L2_PROMOTION_L2_256B : (CUtensorMapL2promotion)tc_tune().promo;
+  p.Aa = Aa;
+  p.Ba = Ba;
+  p.Ca = Ca;
+  p.a_entry = (uint32_t)(rowsA * wk_b);
+  p.b_entry = (uint32_t)(n * wk_b);
+  p.c_entry = (uint32_t)(n * s.rows_tile * eso);
+  p.entry_tx = p.tx_bytes / (uint32_t)(G * U);
+  // pointer arrays: address-space views (view_coords), one entry per box
+  void* const vbase = reinterpret_cast<void*>(kViewBase);
+  const cuuint64_t vlo = 1ull << 24, vhi = 1ull << 20, vstride_hi = 1ull << 28;
+  // Pointer-array boxes never leave their entry: on sm_100a a TMA box that is
+  // partly out of bounds of an address-space view faults (measured: every k
+  // tail, 64x64x40, 64x64x8, 48x80x40), where the strided maps zero-fill.  So
+  // a k tail (k = 8 mod 16, the MMA K step is 16) is left to the LDG-fed
+  // kernel, which zero-fills in its producer, and the last m-tile of
+  // m > 128, m % 128 != 0 gets maps whose boxes have exactly m % 128 rows.
+  if (ptr && (k % s.Wk) != 0) return KAMI_ERROR_NOT_SUPPORTED;
+  p.m_tail = (ptr && s.G == 1 && m > 128 && (m % 128) != 0) ? 1 : 0;
+  const int rows_t = m % 128;
+  p.entry_tx_t = (uint32_t)(wk_b * rows_t + wk_b * n);
+  if (ptr) {
+    for (int t = 0; t <= p.m_tail; ++t) {  // A: (k, m, 16 B offset, 2^28 B offset)
+      cuuint64_t dims[4] = {(cuuint64_t)k, (cuuint64_t)m, vlo, vhi};
+      cuuint64_t strides[3] = {(cuuint64_t)k * esi, 16, vstride_hi};
+      cuuint32_t box[4] = {(cuuint32_t)s.Wk, (cuuint32_t)(t ? rows_t : rowsA), 1, 1};
+      cuuint32_t es[4] = {1, 1, 1, 1};
+      if (enc(t ? &p.tmAt : &p.tmA, dti, 4, vbase, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+              swz_mode_for(wk_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return KAMI_ERROR_NOT_SUPPORTED;  // view rejected: caller falls back
+    }
+    {  // B: (Wn, k, n/Wn, 16 B offset, 2^28 B offset)
+      cuuint64_t dims[5] = {(cuuint64_t)s.Wn, (cuuint64_t)k, (cuuint64_t)(n / s.Wn), vlo, vhi};
+      cuuint64_t strides[4] = {(cuuint64_t)n * esi, (cuuint64_t)wn_b, 16, vstride_hi};
+      cuuint32_t box[5] = {(cuuint32_t)s.Wn, (cuuint32_t)s.Wk, (cuuint32_t)(n / s.Wn), 1, 1};
+      cuuint32_t es[5] = {1, 1, 1, 1, 1};
+      if (enc(&p.tmB, dti, 5, vbase, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz_mode_for(wn_b), promo,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return KAMI_ERROR_NOT_SUPPORTED;  // view rejected: caller falls back
+    }
+  } else {
   {  // A: (k, m, batch)
     cuuint64_t dims[3] = {(cuuint64_t)k, (cuuint64_t)m, (cuuint64_t)batch};
     cuuint64_t strides[2] = {(cuuint64_t)k * esi, (cuuint64_t)m * k * esi};
@@ -785,6 +945,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
             swz_mode_for(wn_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
+  }  // strided
   // Per-atom C stores (kSplit instantiation) for one-entry tiles with >= 2
   // 64-column atoms: the store engine starts on atom 0 while the rest is
   // converted and the accumulator is released early (bf16 16x192x16 0.27 ->
@@ -795,7 +956,23 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
                    !(s.rows_tile == 128 && k <= 16) && beta == 0.0f && alpha == 1.0f && tc_tune().split >= 0)
                       ? 1
                       : 0;
-  {  // C: (Wc, m, n/Wc, batch)
+  if (ptr) {  // C: (Wc, m, n/Wc, 16 B offset, 2^28 B offset)
+    for (int t = 0; t <= p.m_tail; ++t) {
+      const cuuint32_t rows = (cuuint32_t)(t ? rows_t : s.rows_tile);
+      cuuint64_t dims[5] = {(cuuint64_t)s.Wc, (cuuint64_t)m, (cuuint64_t)(n / s.Wc), vlo, vhi};
+      cuuint64_t strides[4] = {(cuuint64_t)n * eso, (cuuint64_t)wc_b, 16, vstride_hi};
+      cuuint32_t box[5] = {(cuuint32_t)s.Wc, rows, (cuuint32_t)(n / s.Wc), 1, 1};
+      cuuint32_t es[5] = {1, 1, 1, 1, 1};
+      if (enc(t ? &p.tmCt : &p.tmC, dto, 5, vbase, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+              swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return KAMI_ERROR_NOT_SUPPORTED;
+      cuuint32_t box1[5] = {(cuuint32_t)s.Wc, rows, 1, 1, 1};
+      if (p.split_store && enc(t ? &p.tmCat : &p.tmCa, dto, 5, vbase, dims, strides, box1, es,
+                               CU_TENSOR_MAP_INTERLEAVE_NONE, swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return KAMI_ERROR_NOT_SUPPORTED;
+    }
+  } else {  // C: (Wc, m, n/Wc, batch)
     cuuint64_t dims[4] = {(cuuint64_t)s.Wc, (cuuint64_t)m, (cuuint64_t)(n / s.Wc), (cuuint64_t)batch};
     cuuint64_t strides[3] = {(cuuint64_t)n * eso, (cuuint64_t)wc_b, (cuuint64_t)m * n * eso};
     cuuint32_t box[4] = {(cuuint32_t)s.Wc, (cuuint32_t)s.rows_tile, (cuuint32_t)(n / s.Wc), (cuuint32_t)(G * U)};

@@ -1,5 +1,6 @@
-"""Pointer-array and variable-size batches (PAPER.md L523
-"supports various matrix orders in a batch") on the LDG-fed tcgen05 kernel,
+"""Pointer-array batches (kami_gemm_batched: the TMA tcgen05 kernel over
+address-space views) and variable-size batches (PAPER.md L523
+"supports various matrix orders in a batch": the LDG-fed tcgen05 kernel),
 against the oracle entry by entry."""
 import numpy as np
 import pytest
@@ -10,6 +11,12 @@ import oracle
 import paper_conf_sc_wangdltsl25_b200 as kami
 
 pytestmark = pytest.mark.gpu
+
+
+def _ptr_kernel(dtype, k):
+    # k = 8 mod 16 (a K tail inside the MMA's 16-element step) goes to the LDG-fed kernel,
+    # which zero-fills it; everything else to the TMA kernel over address-space views
+    return f"kami_tc16_vb_kernel<{dtype}>" if k % 16 else f"kami_tc16_1d_kernel<{dtype},ptr>"
 
 
 def _tol(dtype, k):
@@ -32,8 +39,9 @@ def test_pointer_array_all_sizes(dtype, shape):
         pc = torch.tensor([dC[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
         kami.gemm_batched(m, n, k, batch, dtype, layout, pa, pb, pc)
         torch.cuda.synchronize()
-        # square orders 16 / 32 go to the warp-level HMMA 1D (dispatch rule), the rest to tcgen05
-        want = "kami_warp_ca_1d" if (m == n == k and m <= 32) else "kami_tc16_vb_kernel"
+        # square order 16 goes to the warp-level HMMA 1D (dispatch rule), the rest to the
+        # TMA tcgen05 kernel over address-space views
+        want = "kami_warp_ca_1d" if (m == n == k and m <= 16) else _ptr_kernel(dtype, k)
         assert kami.last_kernel().startswith(want), kami.last_kernel()
         Cref, S = oracle.gemm(m, n, k, batch, dtype, layout, ki.as_bits(A), ki.as_bits(B), with_scale=True)
         got_bits = oracle.to_row_major(ki.as_bits(dC.cpu()), batch, m, n, layout)
@@ -42,6 +50,50 @@ def test_pointer_array_all_sizes(dtype, shape):
         else:
             got = oracle.decode(got_bits.reshape(-1), dtype).reshape(batch, m, n)
             assert oracle.normalised_error(got, Cref, S) <= _tol(dtype, k)
+
+
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+@pytest.mark.parametrize("shape", [(64, 64, 64), (48, 80, 40), (256, 256, 16), (192, 128, 64), (16, 192, 16),
+                                   (64, 64, 8), (64, 64, 40), (128, 128, 200), (32, 64, 24)])
+def test_pointer_array_scattered_addresses(dtype, shape):
+    """Entries at arbitrary 16-byte-aligned addresses: inside one buffer at offsets that are
+    not multiples of the entry size, and in separate allocations more than 2^28 bytes apart
+    (both coordinates of the address-space view), pointers shuffled, ragged last unit."""
+    m, n, k = shape
+    batch = 37
+    es = 2
+    A, B = ki.operands(m, n, k, batch, dtype, "int", seed=21)
+    g = torch.Generator().manual_seed(5)
+    # A: one buffer, entry i at a random 16-byte-aligned offset (non-overlapping)
+    gaps = (torch.randint(0, 9, (batch,), generator=g) * 16).tolist()
+    a_off, pos = [], 0
+    for i in range(batch):
+        pos += gaps[i]
+        a_off.append(pos)
+        pos += m * k * es
+    bufA = torch.zeros(pos // es + 8, dtype=A.dtype, device="cuda")
+    Av = A.view(batch, -1)
+    for i in range(batch):
+        bufA[a_off[i] // es: a_off[i] // es + m * k] = Av[i].cuda()
+    # B and C: separate allocations with a > 2^28-byte spacer between the halves
+    Bv = B.view(batch, -1)
+    dB = [Bv[i].cuda().clone() for i in range(batch // 2)]
+    dC = [torch.zeros(m * n, dtype=A.dtype, device="cuda") for _ in range(batch // 2)]
+    spacer = torch.empty(300 << 20, dtype=torch.uint8, device="cuda")
+    dB += [Bv[i].cuda().clone() for i in range(batch // 2, batch)]
+    dC += [torch.zeros(m * n, dtype=A.dtype, device="cuda") for _ in range(batch // 2, batch)]
+    perm = torch.randperm(batch, generator=g).tolist()
+    pa = torch.tensor([bufA.data_ptr() + a_off[i] for i in perm], dtype=torch.int64, device="cuda")
+    pb = torch.tensor([dB[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
+    pc = torch.tensor([dC[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
+    kami.gemm_batched(m, n, k, batch, dtype, "row", pa, pb, pc)
+    torch.cuda.synchronize()
+    assert kami.last_kernel() == _ptr_kernel(dtype, k), kami.last_kernel()
+    del spacer
+    Cref = oracle.gemm(m, n, k, batch, dtype, "row", ki.as_bits(A), ki.as_bits(B))
+    want = oracle.round_to(Cref, dtype).reshape(batch, m, n)
+    got = np.stack([ki.as_bits(c.cpu()).reshape(m, n) for c in dC])
+    assert np.array_equal(got, want)
 
 
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
