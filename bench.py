@@ -176,7 +176,14 @@ def dist_init():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    if world > 1:
+    if world > 1 and os.environ.get("KAMI_BENCH_SHARED_GPU") == "1":
+        # test mode only (never the measured run): N ranks on one GPU, so the
+        # multi-rank path (shards, barriers, max over ranks, stats gather) can
+        # be exercised on a 1-GPU box; NCCL refuses two ranks on one device, so
+        # the stats travel over gloo
+        torch.cuda.set_device(local % torch.cuda.device_count())
+        dist.init_process_group("gloo")
+    elif world > 1:
         torch.cuda.set_device(local)
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     else:
@@ -299,7 +306,7 @@ def main():
     kernel = kami.last_kernel()
 
     # clocks sampled during a ~1.5 s sustained burst plus the timed region
-    sampler = ClockSampler(local)
+    sampler = ClockSampler(torch.cuda.current_device())
     sampler.start()
     t_end = time.time() + 1.5
     while time.time() < t_end:
@@ -350,7 +357,8 @@ def main():
 
     # checksum of the last output (sampled verification happens in tests/)
     csum = float(C.double().sum().item())
-    stats = torch.tensor([t_ms, csum, float(batch)], dtype=torch.float64, device="cuda")
+    coll_dev = "cpu" if world > 1 and dist.get_backend() == "gloo" else "cuda"
+    stats = torch.tensor([t_ms, csum, float(batch)], dtype=torch.float64, device=coll_dev)
     if world > 1:
         gathered = [torch.zeros_like(stats) for _ in range(world)]
         dist.all_gather(gathered, stats)  # the only collective: per-rank stats over NCCL
@@ -374,7 +382,7 @@ def main():
         for _ in range(e_steps):
             kami.gemm_strided_batched_host(m, n, k, batch, dtype, "row", hA, hB, hC)
         e_dt = (time.perf_counter() - t0) / e_steps
-        et = torch.tensor([e_dt], dtype=torch.float64, device="cuda")
+        et = torch.tensor([e_dt], dtype=torch.float64, device=coll_dev)
         if world > 1:
             dist.all_reduce(et, op=dist.ReduceOp.MAX)
         e2e = {"value": flops * world / float(et.item()) / 1e12, "unit": "TFLOP/s",
