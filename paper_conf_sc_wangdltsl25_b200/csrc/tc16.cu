@@ -502,7 +502,15 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       }
       // the TMA store that last read staging buffer cb must be done reading
       if (!kDirect && storer) {
-        if (p.c_bufs == 2 && !kSplit) ptx::bulk_wait_read<1>();
+        // per-atom stores (kSplit) into a single staging buffer: only atom 0 of
+        // the unit that last used it must be read out here (A groups per unit,
+        // so A - 1 newer groups may still be in flight); each later atom waits
+        // for its own slot inside the atom loop (bf16 192^3: 298 -> 317
+        // TFLOP/s).  With two buffers (small tiles) waiting for everything is
+        // faster (bf16 16x192x16: 26.5 vs 23.2 with per-atom waits: more stores
+        // queued on the TMA unit delay the next units' loads).
+        if (kSplit && p.c_bufs == 1) ptx::bulk_wait_read_n((p.n >> 6) - 1);
+        else if (p.c_bufs == 2 && !kSplit) ptx::bulk_wait_read<1>();
         else ptx::bulk_wait_read<0>();
         if (kUpd && p.scale == 2) {  // C update: bring the old C tile into the staging buffer
           uint64_t* cf = &cfull[wg * 2 + cb];
@@ -547,6 +555,9 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
                                 &v[8 * q], p);
           }
           ptx::fence_proxy_async_smem();
+          // single buffer: the next atom's slot (its store of the previous unit)
+          // must be read out before the barrier releases the warps onto it
+          if (storer && p.c_bufs == 1 && c0 + 64 < p.n) ptx::bulk_wait_read_n((p.n >> 6) - 2);
           ptx::named_bar_sync(bar_id, kEpiThreads);
           if (kPtr ? cstore : leader) {
             if constexpr (kPtr)
@@ -953,7 +964,8 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   // 0.95).  Not for full 128-row tiles with k <= 16 (C-store dominated low-rank:
   // lr-8 0.90 -> 0.84, lr-16 0.92 -> 0.85 measured), profiles/r1/split_store_r1.txt.
   p.split_store = (out_kind != OUT_F32 && s.G == 1 && s.U == 1 && s.Wc == 64 && n % 64 == 0 && n >= 128 &&
-                   !(s.rows_tile == 128 && k <= 16) && beta == 0.0f && alpha == 1.0f && tc_tune().split >= 0)
+                   (!(s.rows_tile == 128 && k <= 16) || tc_tune().split > 0) && beta == 0.0f && alpha == 1.0f &&
+                   tc_tune().split >= 0)
                       ? 1
                       : 0;
   if (ptr) {  // C: (Wc, m, n/Wc, 16 B offset, 2^28 B offset)
