@@ -785,11 +785,15 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
     // sustained HBM throughput DROPS (measured, profiles/r1/stage_sweep_r1.txt:
     // f16 64^3 119 -> 137 TFLOP/s, f16 128^3 245 -> 283 going from 5 / 4 stages
     // of 32 KB to 3); shapes with smaller stages are insensitive.
-    const int cap = (96 * 1024) / (int)s->stage_bytes;
+    // At least 3 stages where they fit: stages of > 32 KB (n > 128, k >= 64)
+    // would otherwise get 2 (bf16 192^3: 318 -> 344-352 TFLOP/s with 3; 256^3
+    // and 192x256x192 unchanged, profiles/r1/stage_ab_r1.txt).
+    int cap = (96 * 1024) / (int)s->stage_bytes;
+    if (cap < 3) cap = 3;
     if (tc_tune().stages > 0) {
       if (st > tc_tune().stages) st = tc_tune().stages;
     } else if (st > cap) {
-      st = cap < 2 ? 2 : cap;
+      st = cap;
     }
     s->stages = st;
     s->smem_bytes = s->stages * s->stage_bytes + 2 * s->c_bufs * s->c_buf_bytes + 1024 + 1024;
