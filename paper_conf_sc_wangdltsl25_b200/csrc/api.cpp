@@ -131,7 +131,16 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
     return tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), rp.A, rp.B, C, (float)alpha,
                             (float)beta, stream, 0);
   }
-  if (plan.kernel == 2) return dmma_tma_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream, alpha, beta);
+  if (plan.kernel == 2) {
+    if (Ca) {  // pointer arrays: the TMA view, else the register-resident family
+      kami_status_t st = dmma_tma_launch(rp.m, rp.n, rp.k, batch, nullptr, nullptr, nullptr, stream, 1.0, 0.0,
+                                         rp.Aa, rp.Ba, Ca);
+      if (st != KAMI_ERROR_NOT_SUPPORTED || update) return st;
+      if (planner_choose(rp.m, rp.n, rp.k, dtype, KAMI_ALGO_2D, 0, true, &plan) != KAMI_SUCCESS) return st;
+    } else {
+      return dmma_tma_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream, alpha, beta);
+    }
+  }
   if (update) return KAMI_ERROR_NOT_SUPPORTED;  // the warp-level family has no update form
   return warp_ca_launch(rp.m, rp.n, rp.k, batch, dtype, (int)plan.algo, plan.p, rp.A, rp.B, C, rp.Aa, rp.Ba, Ca,
                         stream);

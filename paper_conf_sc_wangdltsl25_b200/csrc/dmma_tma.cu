@@ -43,11 +43,37 @@ struct DmmaTmaCfg {
 
 struct DmmaTmaParams {
   CUtensorMap tmA;  // 4-D (16, m, k/16, batch), box (16, m, k/16, 1), SW128
+                    // pointer arrays: 5-D (16, m, k/16, view lo, view hi), box (16, m, k/16, 1, 1)
   const double* B;
   double* C;
   long long batch;
   double alpha, beta;  // C = alpha A B + beta C (C read iff beta != 0)
+  // pointer arrays (kPtr; kami_gemm_batched): entry e at Aa[e], Ba[e], Ca[e]
+  const void* const* Aa;
+  const double* const* Ba;
+  double* const* Ca;
 };
+
+// Address-space view of the pointer-array A map (same scheme as tc16.cu): the
+// entry at byte address q is the box at outer coordinates
+// ((q - kViewBase) / 16 mod 2^24, (q - kViewBase) / 2^28).  The box is the
+// whole entry (16, m, k/16), never partly out of bounds.
+constexpr unsigned long long kViewBase = 256;
+__device__ __forceinline__ void view_coords(const void* q, int& lo, int& hi) {
+  const unsigned long long off = reinterpret_cast<unsigned long long>(q) - kViewBase;
+  lo = (int)((off >> 4) & 0xFFFFFFull);
+  hi = (int)(off >> 28);
+}
+template <bool kPtr>
+__device__ __forceinline__ void load_a_entry(void* dst, const DmmaTmaParams& prm, uint64_t* bar, long long e) {
+  if constexpr (kPtr) {
+    int lo, hi;
+    view_coords(prm.Aa[e], lo, hi);
+    ptx::tma_load_5d(dst, &prm.tmA, bar, 0, 0, 0, lo, hi);
+  } else {
+    ptx::tma_load_4d(dst, &prm.tmA, bar, 0, 0, 0, (int)e);
+  }
+}
 
 // B_w fragments of k-steps [K0, K1) of one entry (k = t, n = g of each 8x8 block).
 // volatile asm keeps the loads where the schedule puts them relative to the MMAs.
@@ -86,7 +112,7 @@ __device__ __forceinline__ void mma_steps(double (&c)[FM][FN][2], const double (
 }
 
 // kUpd: C = alpha A B + beta C epilogue; the plain instantiation has none of it.
-template <int M, int N, int K, int P, int TEAMS, bool kUpd, bool kRot>
+template <int M, int N, int K, int P, int TEAMS, bool kUpd, bool kRot, bool kPtr = false>
 __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(const __grid_constant__ DmmaTmaParams prm) {
   using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -112,29 +138,41 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
   uint64_t* tfull = full + team * 2;
   if (issuer && first < prm.batch) {  // prologue: A of the first entry
     ptx::mbar_arrive_expect_tx(&tfull[0], Cfg::A_BYTES);
-    ptx::tma_load_4d(abuf, &prm.tmA, &tfull[0], 0, 0, 0, (int)first);
+    load_a_entry<kPtr>(abuf, prm, &tfull[0], first);
   }
+  // entry e's B / C: packed strided, or the pointer arrays (B pointer carried
+  // one entry ahead, so the entry's loads never wait on a pointer fetch)
+  auto b_of = [&](long long e) -> const double* {
+    if constexpr (kPtr) return prm.Ba[e];
+    else return prm.B + e * (long long)K * N;
+  };
+  auto c_of = [&](long long e) -> double* {
+    if constexpr (kPtr) return prm.Ca[e];
+    else return prm.C + e * (long long)M * N;
+  };
+  const double* Bcur = first < prm.batch ? b_of(first) : nullptr;
   constexpr int H = Cfg::FK / 2;
   double b[Cfg::FK][Cfg::FN];
   // kRot: B_w rotates through the registers half an entry ahead -- the first
   // k-half of entry e+1 is loaded into the slots of entry e's first k-half as
   // soon as those MMAs have issued, so the next entry starts without an L2
   // round trip and no extra registers are needed.
-  if (kRot && first < prm.batch)
-    load_b_steps<N, Cfg::FN, 0, H>(b, prm.B + first * (long long)K * N + w * Cfg::NP, t, g);
+  if (kRot && first < prm.batch) load_b_steps<N, Cfg::FN, 0, H>(b, Bcur + w * Cfg::NP, t, g);
   uint32_t it = 0;
   for (long long e = first; e < prm.batch; e += nteams, ++it) {
     const uint32_t s = it & 1;
     const long long en = e + nteams;
+    const double* Bnext = en < prm.batch ? b_of(en) : nullptr;
+    double* const Ce = c_of(e);
     // all warps of the team finished reading buffer s^1 (entry it-1) at the
     // barrier that ended the previous iteration: refill it with entry it+1
     if (issuer && en < prm.batch) {
       ptx::mbar_arrive_expect_tx(&tfull[s ^ 1], Cfg::A_BYTES);
-      ptx::tma_load_4d(abuf + (s ^ 1) * Cfg::A_BYTES, &prm.tmA, &tfull[s ^ 1], 0, 0, 0, (int)en);
-      ptx::prefetch_l2_bulk(prm.B + en * (long long)K * N, (uint32_t)(K * N * 8));
+      load_a_entry<kPtr>(abuf + (s ^ 1) * Cfg::A_BYTES, prm, &tfull[s ^ 1], en);
+      ptx::prefetch_l2_bulk(Bnext, (uint32_t)(K * N * 8));
     }
     // GMem2Reg: this warp's B_w (k x n/p) as DMMA B fragments (k = t, n = g)
-    const double* Bg = prm.B + e * (long long)K * N + w * Cfg::NP;
+    const double* Bg = Bcur + w * Cfg::NP;
     if (kRot) {
       load_b_steps<N, Cfg::FN, H, Cfg::FK>(b, Bg, t, g);
     } else {
@@ -151,11 +189,10 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
     ptx::mbar_wait(&tfull[s], (it >> 1) & 1);
     const uint32_t a_s = ptx::smem_u32(abuf + s * Cfg::A_BYTES);
     mma_steps<M, Cfg::FM, Cfg::FN, 0, H>(c, b, a_s, t, g);
-    if (kRot && en < prm.batch)
-      load_b_steps<N, Cfg::FN, 0, H>(b, prm.B + en * (long long)K * N + w * Cfg::NP, t, g);
+    if (kRot && en < prm.batch) load_b_steps<N, Cfg::FN, 0, H>(b, Bnext + w * Cfg::NP, t, g);
     mma_steps<M, Cfg::FM, Cfg::FN, H, Cfg::FK>(c, b, a_s, t, g);
     // Reg2GMem: C_w, lane holds (row g, cols 2t, 2t+1) of each 8x8 block
-    double* Cg = prm.C + e * (long long)M * N + w * Cfg::NP;
+    double* Cg = Ce + w * Cfg::NP;
 #pragma unroll
     for (int i = 0; i < Cfg::FM; ++i)
 #pragma unroll
@@ -174,32 +211,50 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
         ptx::st_global_v2_f64(dst, r0, r1);
       }
     ptx::named_bar_sync(bar, P * 32);  // buffer s free for entry it+2
+    Bcur = Bnext;
   }
 }
 
 template <int M, int N, int K, int P, int TEAMS, bool kRot = false>
 kami_status_t launch(long long batch, const void* A, const void* B, void* C, cudaStream_t stream, const char* name,
-                     double alpha, double beta) {
+                     double alpha, double beta, const void* const* Aa, const void* const* Ba, void* const* Ca) {
   using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
   PFN_encodeTiled enc = get_encode_tiled();
   if (!enc) return KAMI_ERROR_CUDA;
+  const bool ptr = Aa != nullptr;
+  if (ptr && (alpha != 1.0 || beta != 0.0 || !Ba || !Ca)) return KAMI_ERROR_NOT_SUPPORTED;
   DmmaTmaParams prm;
   memset(&prm, 0, sizeof(prm));
-  cuuint64_t dims[4] = {16, (cuuint64_t)M, (cuuint64_t)(K / 16), (cuuint64_t)batch};
-  cuuint64_t strides[3] = {(cuuint64_t)K * 8, 128, (cuuint64_t)M * K * 8};
-  cuuint32_t box[4] = {16, (cuuint32_t)M, (cuuint32_t)(K / 16), 1};
-  cuuint32_t es[4] = {1, 1, 1, 1};
-  if (enc(&prm.tmA, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<void*>(A), dims, strides, box, es,
-          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-    return KAMI_ERROR_CUDA;
+  if (ptr) {  // address-space view, one whole entry per box
+    cuuint64_t dims[5] = {16, (cuuint64_t)M, (cuuint64_t)(K / 16), 1ull << 24, 1ull << 20};
+    cuuint64_t strides[4] = {(cuuint64_t)K * 8, 128, 16, 1ull << 28};
+    cuuint32_t box[5] = {16, (cuuint32_t)M, (cuuint32_t)(K / 16), 1, 1};
+    cuuint32_t es[5] = {1, 1, 1, 1, 1};
+    if (enc(&prm.tmA, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 5, reinterpret_cast<void*>(kViewBase), dims, strides, box,
+            es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_NOT_SUPPORTED;
+  } else {
+    cuuint64_t dims[4] = {16, (cuuint64_t)M, (cuuint64_t)(K / 16), (cuuint64_t)batch};
+    cuuint64_t strides[3] = {(cuuint64_t)K * 8, 128, (cuuint64_t)M * K * 8};
+    cuuint32_t box[4] = {16, (cuuint32_t)M, (cuuint32_t)(K / 16), 1};
+    cuuint32_t es[4] = {1, 1, 1, 1};
+    if (enc(&prm.tmA, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<void*>(A), dims, strides, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
+  }
   prm.B = static_cast<const double*>(B);
   prm.C = static_cast<double*>(C);
+  prm.Aa = Aa;
+  prm.Ba = reinterpret_cast<const double* const*>(Ba);
+  prm.Ca = reinterpret_cast<double* const*>(Ca);
   prm.batch = batch;
   prm.alpha = alpha;
   prm.beta = beta;
-  auto fn = (alpha != 1.0 || beta != 0.0) ? kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, true, kRot>
-                                          : kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, false, kRot>;
+  auto fn = ptr ? kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, false, kRot, true>
+            : (alpha != 1.0 || beta != 0.0) ? kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, true, kRot>
+                                            : kami_dmma_tma_1d_kernel<M, N, K, P, TEAMS, false, kRot>;
   if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM) != cudaSuccess)
     return KAMI_ERROR_CUDA;
   int dev = 0, sms = 148, per_sm = 1;
@@ -212,7 +267,9 @@ kami_status_t launch(long long batch, const void* A, const void* B, void* C, cud
   const long long need = (batch + TEAMS - 1) / TEAMS;
   if (grid > need) grid = need;
   fn<<<(unsigned)grid, Cfg::THREADS, Cfg::SMEM, stream>>>(prm);
-  set_last_kernel(name);
+  set_last_kernel(ptr ? (M == 64 ? "kami_dmma_tma_1d<64,ptr>" : M == 32 ? "kami_dmma_tma_1d<32,ptr>"
+                                                                         : "kami_dmma_tma_1d<16,ptr>")
+                      : name);
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
 }
 
@@ -224,26 +281,27 @@ bool dmma_tma_supported(int m, int n, int k) { return m == n && n == k && (m == 
 // (64^3 default rotates B half an entry ahead: 25.3 -> 26.1 TF/s, profiles/r1/dmma_tma_sweep_r1.txt;
 // at 16^3 / 32^3 it made no difference and the plain form stays)
 kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
-                              cudaStream_t stream, double alpha, double beta) {
+                              cudaStream_t stream, double alpha, double beta, const void* const* Aa,
+                              const void* const* Ba, void* const* Ca) {
   static const int cfg = [] {
     const char* e = getenv("KAMI_DMMA_TMA_CFG");
     return e ? atoi(e) : 0;
   }();
   if (m == 64 && n == 64 && k == 64) {
-    if (cfg == 1) return launch<64, 64, 64, 8, 2>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,p8>", alpha, beta);
-    if (cfg == 4) return launch<64, 64, 64, 4, 3>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,norot>", alpha, beta);
-    return launch<64, 64, 64, 4, 3, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<64>", alpha, beta);
+    if (cfg == 1) return launch<64, 64, 64, 8, 2>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,p8>", alpha, beta, Aa, Ba, Ca);
+    if (cfg == 4) return launch<64, 64, 64, 4, 3>(batch, A, B, C, stream, "kami_dmma_tma_1d<64,norot>", alpha, beta, Aa, Ba, Ca);
+    return launch<64, 64, 64, 4, 3, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<64>", alpha, beta, Aa, Ba, Ca);
   }
   if (m == 32 && n == 32 && k == 32) {
-    if (cfg == 3) return launch<32, 32, 32, 4, 8, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,rot>", alpha, beta);
-    if (cfg == 1) return launch<32, 32, 32, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,p2>", alpha, beta);
-    if (cfg == 2) return launch<32, 32, 32, 4, 6>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,t6>", alpha, beta);
-    return launch<32, 32, 32, 4, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32>", alpha, beta);
+    if (cfg == 3) return launch<32, 32, 32, 4, 8, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,rot>", alpha, beta, Aa, Ba, Ca);
+    if (cfg == 1) return launch<32, 32, 32, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,p2>", alpha, beta, Aa, Ba, Ca);
+    if (cfg == 2) return launch<32, 32, 32, 4, 6>(batch, A, B, C, stream, "kami_dmma_tma_1d<32,t6>", alpha, beta, Aa, Ba, Ca);
+    return launch<32, 32, 32, 4, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<32>", alpha, beta, Aa, Ba, Ca);
   }
   if (m == 16 && n == 16 && k == 16) {
-    if (cfg == 3) return launch<16, 16, 16, 2, 8, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,rot>", alpha, beta);
-    if (cfg == 1) return launch<16, 16, 16, 1, 16>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,p1>", alpha, beta);
-    return launch<16, 16, 16, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<16>", alpha, beta);
+    if (cfg == 3) return launch<16, 16, 16, 2, 8, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,rot>", alpha, beta, Aa, Ba, Ca);
+    if (cfg == 1) return launch<16, 16, 16, 1, 16>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,p1>", alpha, beta, Aa, Ba, Ca);
+    return launch<16, 16, 16, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<16>", alpha, beta, Aa, Ba, Ca);
   }
   return KAMI_ERROR_NOT_SUPPORTED;
 }

@@ -54,8 +54,11 @@ kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t 
 
 // ------------------------------------------- FP64 1D with TMA-fed broadcast
 bool dmma_tma_supported(int m, int n, int k);
+// Aa/Ba/Ca != nullptr: device pointer arrays (kami_gemm_batched, C = AB only), A/B/C unused.
 kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
-                              cudaStream_t stream, double alpha = 1.0, double beta = 0.0);
+                              cudaStream_t stream, double alpha = 1.0, double beta = 0.0,
+                              const void* const* Aa = nullptr, const void* const* Ba = nullptr,
+                              void* const* Ca = nullptr);
 
 // ------------------------- 16-bit pointer-array / variable-size (tc16_vb.cu)
 // dm/dn/dk: device arrays of per-entry sizes, or nullptr for uniform m, n, k.

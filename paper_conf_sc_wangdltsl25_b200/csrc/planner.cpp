@@ -131,8 +131,9 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
     *out = r;
     return KAMI_SUCCESS;
   }
-  // FP64 1D with the broadcast operand fed by TMA (dmma_tma.cu)
-  const bool tma_ok = !is16 && !pointer_array && dmma_tma_supported(m, n, k);
+  // FP64 1D with the broadcast operand fed by TMA (dmma_tma.cu; pointer arrays
+  // through an address-space view of each entry)
+  const bool tma_ok = !is16 && dmma_tma_supported(m, n, k);
   if (algo == KAMI_ALGO_1D_TMA) {
     if (!tma_ok || (p != 0 && p != 4)) return KAMI_ERROR_NOT_SUPPORTED;
     r.algo = KAMI_ALGO_1D_TMA;

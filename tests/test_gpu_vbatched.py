@@ -96,6 +96,36 @@ def test_pointer_array_scattered_addresses(dtype, shape):
     assert np.array_equal(got, want)
 
 
+@pytest.mark.parametrize("s", [16, 32, 64])
+@pytest.mark.parametrize("layout", ["row", "col"])
+def test_pointer_array_f64_tma_view(s, layout):
+    """FP64 pointer arrays on the DMMA kernel with TMA-fed broadcast operand (address-space
+    view of each entry's A): scattered, shuffled entries in two allocations > 2^28 B apart,
+    a batch that leaves teams with unequal entry counts; within the FP64 tolerance."""
+    batch = 203
+    A, B = ki.operands(s, s, s, batch, "f64", "unif", seed=22)
+    Av, Bv = A.view(batch, -1), B.view(batch, -1)
+    half = batch // 2
+    dA = [Av[i].cuda().clone() for i in range(half)]
+    dB = [Bv[i].cuda().clone() for i in range(half)]
+    dC = [torch.zeros(s * s, dtype=torch.float64, device="cuda") for _ in range(half)]
+    spacer = torch.empty(300 << 20, dtype=torch.uint8, device="cuda")
+    dA += [Av[i].cuda().clone() for i in range(half, batch)]
+    dB += [Bv[i].cuda().clone() for i in range(half, batch)]
+    dC += [torch.zeros(s * s, dtype=torch.float64, device="cuda") for _ in range(half, batch)]
+    perm = torch.randperm(batch, generator=torch.Generator().manual_seed(3)).tolist()
+    pa = torch.tensor([dA[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
+    pb = torch.tensor([dB[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
+    pc = torch.tensor([dC[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
+    kami.gemm_batched(s, s, s, batch, "f64", layout, pa, pb, pc)
+    torch.cuda.synchronize()
+    assert kami.last_kernel() == f"kami_dmma_tma_1d<{s},ptr>", kami.last_kernel()
+    del spacer
+    Cref, S = oracle.gemm(s, s, s, batch, "f64", layout, A.numpy(), B.numpy(), with_scale=True)
+    got = oracle.to_row_major(np.stack([c.cpu().numpy() for c in dC]).reshape(-1), batch, s, s, layout)
+    assert oracle.normalised_error(got.reshape(batch, s, s), Cref, S) <= s * 2.0 ** -52
+
+
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 @pytest.mark.parametrize("layout", ["row", "col"])
 def test_vbatched_mixed_orders(dtype, layout):
