@@ -169,6 +169,16 @@ def cpu_baseline(dtype, m, n, k, target_s=12.0, max_entries=None):
             "seconds": dt, "entries": n_entries}
 
 
+PAPER_CONTEXT = {
+    "note": "KAMI (SC'25) prints no absolute batched TFLOP/s (Fig. 12 is an image); other hardware, not a target",
+    "batched_fp64_gh200": "avg 31.60x vs MAGMA 2.9, 340.37x vs cuBLAS 12.8 at batch 1000 (orders 16-128; P:L525)",
+    "block_level_fp64_gh200": "cuBLASDx 64x64 31 TFLOP/s = 46% of the 67 TF peak (P:L90, P:L95)",
+    "block_level_fp16_rtx5090": "KAMI-1D/2D/3D 64x64 469.80/470.57/449.07 TFLOP/s (P:L484)",
+    "hardware": "NVIDIA GH200 (FP16 990 TF, FP64 67 TF), RTX 5090 (FP16 462 TF), AMD 7900 XTX, Intel Max 1100 "
+                "(PAPER.md L49, Table 3); the non-NVIDIA results are reported as speedups only",
+}
+
+
 def dist_init():
     import torch
     import torch.distributed as dist
@@ -427,6 +437,8 @@ def main():
     }
     if e2e:
         line["e2e"] = e2e
+    # the paper's own numbers, other hardware: context only (vs_baseline stays null)
+    line["paper_context"] = PAPER_CONTEXT
     if not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(dtype, m, n, k)
     print(json.dumps(line), flush=True)
