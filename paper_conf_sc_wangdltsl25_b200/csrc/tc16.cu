@@ -790,6 +790,17 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
     // and 192x256x192 unchanged, profiles/r1/stage_ab_r1.txt).
     int cap = (96 * 1024) / (int)s->stage_bytes;
     if (cap < 3) cap = 3;
+    // Units that write at least as many bytes as they read (FP8 in / FP16 out,
+    // thin-k tiles) run best with <= 4 stages: e4m3 / e5m2 64^3 175 -> 200
+    // TFLOP/s going from 6 to 4; thin-k shapes unchanged; input-dominated
+    // small tiles (bf16 16x16x64) want the deeper ring (-5% at 4),
+    // profiles/r1/stage4_ab_r1.txt.
+    {
+      const long long rt = s->rows_tile;
+      const long long in_b = (long long)s->G * s->U * (rt * k + (long long)k * n) * esi;
+      const long long out_b = (long long)s->G * s->U * rt * n * eso;
+      if (out_b >= in_b && cap > 4) cap = 4;
+    }
     if (tc_tune().stages > 0) {
       if (st > tc_tune().stages) st = tc_tune().stages;
     } else if (st > cap) {
