@@ -93,6 +93,7 @@ struct alignas(64) Tc16Params {
   long long units;
   int m, n, k;
   int G, m_tiles, rows_tile;
+  int slot;                  // TMEM lanes / A-tile rows per packed entry (m, or 32 for thin m, see plan)
   int k_chunks, Wk, Wn, Wc;  // atom widths in ELEMENTS of their operand
   int ksteps_full, ksteps_last;
   int N_mma;
@@ -449,11 +450,11 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     int g, r, col_lo, col_hi;
     bool row_ok;
     if (p.G > 1) {
-      g = L / p.m;
-      r = L - g * p.m;
-      row_ok = g < p.G;
-      const int glo = (sp * 32) / p.m;
-      int ghi = (sp * 32 + 31) / p.m;
+      g = L / p.slot;
+      r = L - g * p.slot;
+      row_ok = g < p.G && r < p.m;
+      const int glo = (sp * 32) / p.slot;
+      int ghi = (sp * 32 + 31) / p.slot;
       if (ghi > p.G - 1) ghi = p.G - 1;
       col_lo = glo * p.n;
       col_hi = glo < p.G ? (ghi + 1) * p.n : col_lo;
@@ -684,16 +685,17 @@ int out_es(int out) { return out == OUT_F32 ? 4 : 2; }
 
 constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 
-// Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo,U,split"
+// Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo,U,split,slot"
 // (0 / -1 = planner default; promo = TMA L2 promotion 0 none, 1 64B, 2 128B, 3 256B;
-// U = sub-tiles per unit; split = -1 disables per-atom C stores).  Unset in production.
+// U = sub-tiles per unit; split = -1 disables per-atom C stores, 1 forces them where
+// possible; slot = -1 disables thin-m slots).  Unset in production.
 struct TcTune {
-  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0;
+  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0, slot = 0;
 };
 const TcTune& tc_tune() {
   static const TcTune t = [] {
     TcTune r;
-    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split);
+    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split, &r.slot);
     return r;
   }();
   return t;
@@ -744,6 +746,12 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   }
   s->m_tiles = (s->G > 1 || m <= 128) ? 1 : (m + 127) / 128;
   s->rows_tile = m < 128 ? m : 128;
+  // Thin m packed 2 or 4 to a tile would sit in one or two TMEM sub-partitions
+  // (lanes 0..G m), leaving the other epilogue warps idle: give each entry a
+  // 32-lane slot instead (the A box is 32 rows; TMA zero-fills rows m..31),
+  // so every entry has its own sub-partition and warp.  Strided maps only
+  // (pointer-array boxes must stay inside their entry).
+  s->slot = (m == 16 && (s->G == 2 || s->G == 4) && tc_tune().slot >= 0) ? 32 : s->rows_tile;
   const int kgran = 32 / esi;  // elements per 32-byte MMA K step
   const int kpad = (k + kgran - 1) / kgran * kgran;
   const int wk_b = pick_atom_bytes(kpad * esi), wn_b = pick_atom_bytes(n * esi), wc_b = pick_atom_bytes(n * eso);
@@ -768,7 +776,7 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   }
   if (tc_tune().U > 0) s->U = tc_tune().U;
   for (;; s->U /= 2) {  // fall back to fewer sub-tiles if the ring does not fit
-    const int rowsA = s->G > 1 ? m : s->rows_tile;
+    const int rowsA = s->slot;
     const uint32_t a_region = align_up((uint32_t)((s->U - 1) * s->G * rowsA + 128) * wk_b, 1024);
     const uint32_t b_region = align_up((uint32_t)(s->U * s->N_mma) * wk_b, 1024);
     // TF32: + the raw N-major B slot the transposer reads
@@ -868,7 +876,9 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   p.b_sbo = 8 * wn_b;                      // 8 K-rows of one N-atom
   p.b_lbo = s.Wk * wn_b;                   // next N-atom
   p.b_kstep = (uint32_t)(kgran / 8) * p.b_sbo;  // one 32-byte K step of B rows
-  const int U = s.U, G = s.G, rowsA = s.rows_tile;
+  if (ptr) s.slot = s.rows_tile;  // view boxes never reach past the entry
+  const int U = s.U, G = s.G, rowsA = s.slot;
+  p.slot = s.slot;
   p.U = U;
   p.GU = G * U;
   p.a_region = align_up((uint32_t)((U - 1) * G * rowsA + 128) * wk_b, 1024);

@@ -52,6 +52,7 @@ def check(m, n, k, batch, dtype, layout, dist, algo="auto", p=0, seed=0):
 # --------------------------------------------------------------- tcgen05 family
 TC_SHAPES = [
     (16, 16, 16, 1029),   # G = 8 entries per MMA tile, ragged batch tail
+    (16, 64, 16, 203),    # thin m, G = 4: 32-lane slots (one TMEM sub-partition per entry), U = 2
     (32, 32, 32, 301),    # G = 4
     (64, 64, 64, 257),    # G = 2 (headline shape)
     (128, 128, 128, 33),  # G = 1, two k-chunks
@@ -63,6 +64,7 @@ TC_SHAPES = [
     (192, 192, 192, 3),   # 3 k-chunks, partial second m-tile
     (256, 256, 256, 2),   # largest order
     (16, 256, 64, 20),    # G = 1 with 16 live rows
+    (16, 128, 40, 37),    # thin m, G = 2 slots, k tail
     (128, 16, 16, 17),    # narrowest N
 ]
 
@@ -76,7 +78,8 @@ def test_tc16_unif(shape, dtype, layout):
     assert kami.last_kernel().startswith("kami_tc16_1d_kernel")
 
 
-@pytest.mark.parametrize("shape", TC_SHAPES[:6] + [(256, 256, 16, 3)], ids=lambda s: "x".join(map(str, s)))
+@pytest.mark.parametrize("shape", TC_SHAPES[:7] + [(256, 256, 16, 3), (16, 128, 40, 37)],
+                         ids=lambda s: "x".join(map(str, s)))
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 def test_tc16_int_bit_exact(shape, dtype):
     m, n, k, batch = shape
