@@ -94,6 +94,7 @@ struct alignas(64) Tc16Params {
   int m, n, k;
   int G, m_tiles, rows_tile;
   int slot;                  // TMEM lanes / A-tile rows per packed entry (m, or 32 for thin m, see plan)
+  int colrep;                // thin m, one entry per tile: A replicated into colrep 32-lane slots (plan)
   int k_chunks, Wk, Wn, Wc;  // atom widths in ELEMENTS of their operand
   int ksteps_full, ksteps_last;
   int N_mma;
@@ -366,6 +367,8 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
           uint8_t* sa = smem + r.s * p.stage_bytes;
           uint8_t* sb = sa + p.a_region;
           ptx::tma_load_3d(sa, &p.tmA, &full[r.s], kc * p.Wk, ui.mt * 128, e0);
+          for (int j = 1; j < p.colrep; ++j)  // the same A box into 32-lane slot j
+            ptx::tma_load_3d(sa + j * 32 * p.wk_b, &p.tmA, &full[r.s], kc * p.Wk, ui.mt * 128, e0);
           ptx::tma_load_4d(kXpose ? sa + p.b_raw_off : sb, &p.tmB, &full[r.s], 0, kc * p.Wk, 0, e0);
           if (u == blockIdx.x && kc == 0) KAMI_TS(2);
         }
@@ -458,6 +461,14 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       if (ghi > p.G - 1) ghi = p.G - 1;
       col_lo = glo * p.n;
       col_hi = glo < p.G ? (ghi + 1) * p.n : col_lo;
+    } else if (p.colrep) {
+      // thin m, replicated A: sub-partition sp holds every column of the entry
+      // in its lanes; its warp drains only the 64-column block sp
+      g = 0;
+      r = lane;
+      row_ok = lane < p.m;
+      col_lo = 64 * sp;
+      col_hi = sp < p.colrep ? min(64 * sp + 64, p.n) : col_lo;
     } else {
       g = 0;
       r = L;
@@ -490,7 +501,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       const int mt = ui.mt;
       const long long e0 = ui.grp * p.GU;
       const uint32_t cb = cpos.s;
-      const bool valid0 = row_ok && (p.G > 1 || mt * 128 + L < p.m);
+      const bool valid0 = row_ok && (p.G > 1 || mt * 128 + r < p.m);  // r = L except replicated tiles
       int clo = 0, chi = 0;
       bool cstore = false;
       if constexpr (kPtr) {
@@ -752,6 +763,17 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   // so every entry has its own sub-partition and warp.  Strided maps only
   // (pointer-array boxes must stay inside their entry).
   s->slot = (m == 16 && (s->G == 2 || s->G == 4) && tc_tune().slot >= 0) ? 32 : s->rows_tile;
+  // One thin entry per tile (m <= 32, n > 192): all of C sits in sub-partition
+  // 0 and one warp drained it.  The A box is loaded into ceil(n/64) 32-lane
+  // slots instead (a few hundred bytes each), so every sub-partition holds the
+  // whole product and epilogue warp j drains its 64-column block j.  The MMA
+  // is unchanged (it always spans 128 lanes).  Measured (profiles/r1/
+  // colrep_ab_r1.txt): bf16 16x256x16 0.56 -> 0.66 of roofline, 16x256x32
+  // 0.83 -> 0.95, 32x256x16 0.84 -> 0.90; n = 192 (3 blocks) and k >= 64 are
+  // as fast or faster with the per-atom split stores, so they keep those.
+  s->colrep = (s->G == 1 && m <= 32 && n > 192 && k <= 32 && s->m_tiles == 1 && tc_tune().slot >= 0)
+                  ? (n + 63) / 64
+                  : 0;
   const int kgran = 32 / esi;  // elements per 32-byte MMA K step
   const int kpad = (k + kgran - 1) / kgran * kgran;
   const int wk_b = pick_atom_bytes(kpad * esi), wn_b = pick_atom_bytes(n * esi), wc_b = pick_atom_bytes(n * eso);
@@ -822,6 +844,7 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
     if (s->acc_bufs > kMaxAcc) s->acc_bufs = kMaxAcc;
     if (st >= 2 || s->U == 1) break;
   }
+  if (s->U != 1) s->colrep = 0;  // replication is defined for one entry per unit
   s->units = 0;
   return s->stages >= 2 ? KAMI_SUCCESS : KAMI_ERROR_NOT_SUPPORTED;
 }
@@ -879,6 +902,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   if (ptr) s.slot = s.rows_tile;  // view boxes never reach past the entry
   const int U = s.U, G = s.G, rowsA = s.slot;
   p.slot = s.slot;
+  p.colrep = ptr ? 0 : s.colrep;
   p.U = U;
   p.GU = G * U;
   p.a_region = align_up((uint32_t)((U - 1) * G * rowsA + 128) * wk_b, 1024);
@@ -899,6 +923,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   }
   p.stage_bytes = s.stage_bytes;
   p.tx_bytes = (uint32_t)(wk_b * rowsA * G * U) + (uint32_t)(wk_b * n * G * U);
+  if (p.colrep > 1) p.tx_bytes += (uint32_t)((p.colrep - 1) * wk_b * rowsA);  // replicated A boxes (G = U = 1)
   p.c_tx_bytes = (uint32_t)(G * U * n * s.rows_tile * eso);
   p.stages = s.stages;
   p.acc_cols = s.acc_cols;
@@ -988,7 +1013,9 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   // 0.52 of roofline, 192^3 0.66 -> 0.70, 256^3 0.82 -> 0.87, 32x256x64 0.89 ->
   // 0.95).  Not for full 128-row tiles with k <= 16 (C-store dominated low-rank:
   // lr-8 0.90 -> 0.84, lr-16 0.92 -> 0.85 measured), profiles/r1/split_store_r1.txt.
-  p.split_store = (out_kind != OUT_F32 && s.G == 1 && s.U == 1 && s.Wc == 64 && n % 64 == 0 && n >= 128 &&
+  // (replicated thin-m tiles store from all four warps at once: no per-atom split)
+  p.split_store = (out_kind != OUT_F32 && !p.colrep && s.G == 1 && s.U == 1 && s.Wc == 64 && n % 64 == 0 &&
+                   n >= 128 &&
                    (!(s.rows_tile == 128 && k <= 16) || tc_tune().split > 0) && beta == 0.0f && alpha == 1.0f &&
                    tc_tune().split >= 0)
                       ? 1

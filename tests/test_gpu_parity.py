@@ -65,6 +65,8 @@ TC_SHAPES = [
     (256, 256, 256, 2),   # largest order
     (16, 256, 64, 20),    # G = 1 with 16 live rows
     (16, 128, 40, 37),    # thin m, G = 2 slots, k tail
+    (16, 256, 16, 45),    # thin m, G = 1: A replicated into 4 slots, one 64-column block per warp
+    (32, 240, 24, 29),    # thin m, G = 1, 4 slots, last block 48 columns, k tail
     (128, 16, 16, 17),    # narrowest N
 ]
 
@@ -78,7 +80,8 @@ def test_tc16_unif(shape, dtype, layout):
     assert kami.last_kernel().startswith("kami_tc16_1d_kernel")
 
 
-@pytest.mark.parametrize("shape", TC_SHAPES[:7] + [(256, 256, 16, 3), (16, 128, 40, 37)],
+@pytest.mark.parametrize("shape", TC_SHAPES[:7] + [(256, 256, 16, 3), (16, 128, 40, 37), (16, 256, 16, 45),
+                                                  (32, 240, 24, 29)],
                          ids=lambda s: "x".join(map(str, s)))
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 def test_tc16_int_bit_exact(shape, dtype):
