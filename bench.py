@@ -435,6 +435,10 @@ def main():
         "clocks": sampler.summary(),
         "checksum": float(allst[:, 1].sum()),
     }
+    if world > 1:  # per-rank device times (the job time is their max)
+        tms = [float(x) for x in allst[:, 0]]
+        line["ranks"] = {"time_ms": tms, "spread": max(tms) / min(tms) if min(tms) > 0 else None,
+                         "checksums": [float(x) for x in allst[:, 1]]}
     if e2e:
         line["e2e"] = e2e
     # the paper's own numbers, other hardware: context only (vs_baseline stays null)

@@ -46,4 +46,6 @@ def test_two_ranks_one_line_whole_job():
     flops = 2.0 * 32 ** 3 * d["config"]["global_batch"] * d["steps"]
     assert abs(d["value"] - flops / (d["ms_per_step"] * d["steps"] * 1e-3) / 1e12) <= 1e-6 * d["value"]
     assert d["e2e"]["value"] > 0
+    assert len(d["ranks"]["time_ms"]) == 2 and d["ranks"]["spread"] >= 1.0
+    assert abs(max(d["ranks"]["time_ms"]) - d["ms_per_step"] * d["steps"]) <= 1e-6 * d["ms_per_step"] * d["steps"]
 
