@@ -23,6 +23,7 @@ struct Tc16Shape {
   int G, m_tiles, rows_tile, Wk, Wn, Wc, k_chunks, N_mma;
   int slot;    // A-tile rows / TMEM lanes per packed entry
   int colrep;  // thin m, G = 1: number of 32-lane slots the A box is replicated into (0 = off)
+  int write_heavy;  // a unit writes at least as many bytes as it reads
   int U;  // MMA sub-tiles per unit (G U entries per unit)
   uint32_t stage_bytes, c_buf_bytes;
   int c_bufs, stages, acc_cols, acc_bufs;

@@ -124,6 +124,7 @@ struct alignas(64) Tc16Params {
   void* const* Ca;
   uint32_t a_entry, b_entry, c_entry;  // shared-memory bytes of one entry's A / B / C box
   uint32_t entry_tx, entry_tx_t;       // TMA bytes of one entry's A + B boxes per k-chunk (full / tail m-tile)
+  int l2hint;                          // 1: C stores evict_first in L2, 2: also the A loads (experiment)
   int m_tail;                          // m > 128, m % 128 != 0: the last m-tile uses tmAt / tmCt / tmCat
   CUtensorMap tmAt, tmCt, tmCat;       // pointer arrays: boxes of m % 128 rows for the last m-tile
 };
@@ -357,6 +358,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
   } else if (warp == 0) {
     // ------------------------------------------------------------ producer
     if (lane == 0) {
+      const uint64_t pol = ptx::policy_evict_first();
       RingPos r;
       UnitIter ui(blockIdx.x, gridDim.x, p.m_tiles);
       for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ui.next()) {
@@ -366,7 +368,8 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
           ptx::mbar_arrive_expect_tx(&full[r.s], p.tx_bytes);
           uint8_t* sa = smem + r.s * p.stage_bytes;
           uint8_t* sb = sa + p.a_region;
-          ptx::tma_load_3d(sa, &p.tmA, &full[r.s], kc * p.Wk, ui.mt * 128, e0);
+          if (p.l2hint >= 2) ptx::tma_load_3d_hint(sa, &p.tmA, &full[r.s], kc * p.Wk, ui.mt * 128, e0, pol);
+          else ptx::tma_load_3d(sa, &p.tmA, &full[r.s], kc * p.Wk, ui.mt * 128, e0);
           for (int j = 1; j < p.colrep; ++j)  // the same A box into 32-lane slot j
             ptx::tma_load_3d(sa + j * 32 * p.wk_b, &p.tmA, &full[r.s], kc * p.Wk, ui.mt * 128, e0);
           ptx::tma_load_4d(kXpose ? sa + p.b_raw_off : sb, &p.tmB, &full[r.s], 0, kc * p.Wk, 0, e0);
@@ -495,6 +498,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     // pointer arrays: lane i < G U of the leader warp stores entry e0 + i of the
     // unit (its own bulk groups); its C view coordinates are fetched one unit ahead
     const bool storer = kPtr ? (((warp & 3) == 2) && lane < p.GU) : leader;
+    const uint64_t cpol = ptx::policy_evict_first();
     const void* qc = nullptr;
     if (kPtr && storer && u0 < p.units && ui.grp * p.GU + lane < p.batch) qc = p.Ca[ui.grp * p.GU + lane];
     for (long long u = u0; u < p.units; u += 2ll * gridDim.x, ui.next()) {
@@ -575,6 +579,8 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
             if constexpr (kPtr)
               ptx::tma_store_5d(p.m_tail && mt == p.m_tiles - 1 ? &p.tmCat : &p.tmCa, cbuf + atom * atom_stride, 0,
                                 mt * 128, (int)atom, clo, chi);
+            else if (p.l2hint)
+              ptx::tma_store_4d_hint(&p.tmCa, cbuf + atom * atom_stride, 0, mt * 128, (int)atom, (int)e0, cpol);
             else ptx::tma_store_4d(&p.tmCa, cbuf + atom * atom_stride, 0, mt * 128, (int)atom, (int)e0);
             ptx::bulk_commit();
           }
@@ -647,7 +653,11 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
           ptx::bulk_commit();
         }
       } else if (leader) {
-        ptx::tma_store_4d(&p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mt * 128, 0, (int)e0);
+        if (p.l2hint)
+          ptx::tma_store_4d_hint(&p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mt * 128, 0,
+                                 (int)e0, cpol);
+        else
+          ptx::tma_store_4d(&p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mt * 128, 0, (int)e0);
         ptx::bulk_commit();
         if (wg == 0) KAMI_TS(6);
       }
@@ -699,14 +709,16 @@ constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 // Experiment knobs (tools/tc_tune.py), read once: KAMI_TC_TUNE="stages,cbufs,grid,promo,U,split,slot"
 // (0 / -1 = planner default; promo = TMA L2 promotion 0 none, 1 64B, 2 128B, 3 256B;
 // U = sub-tiles per unit; split = -1 disables per-atom C stores, 1 forces them where
-// possible; slot = -1 disables thin-m slots).  Unset in production.
+// possible; slot = -1 disables thin-m slots; hint = -1 no L2 policy, 1 C evict_first,
+// 2 C and A evict_first, 0 planner rule).  Unset in production.
 struct TcTune {
-  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0, slot = 0;
+  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0, slot = 0, hint = 0;
 };
 const TcTune& tc_tune() {
   static const TcTune t = [] {
     TcTune r;
-    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split, &r.slot);
+    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split, &r.slot,
+                 &r.hint);
     return r;
   }();
   return t;
@@ -829,7 +841,8 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
       const long long rt = s->rows_tile;
       const long long in_b = (long long)s->G * s->U * (rt * k + (long long)k * n) * esi;
       const long long out_b = (long long)s->G * s->U * rt * n * eso;
-      if (out_b >= in_b && cap > 4) cap = 4;
+      s->write_heavy = out_b >= in_b ? 1 : 0;
+      if (s->write_heavy && cap > 4) cap = 4;
     }
     if (tc_tune().stages > 0) {
       if (st > tc_tune().stages) st = tc_tune().stages;
@@ -936,6 +949,11 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   p.alpha = alpha;
   p.beta = beta;
   p.scale = beta != 0.0f ? 2 : (alpha != 1.0f ? 1 : 0);
+  // Units that write at least what they read store C with an L2 evict_first
+  // policy (streamed, never re-read): f16 lr-16 82 -> 90 TFLOP/s (0.88 -> 0.97
+  // of roofline), lr-32 +0.5 %; read-dominated tiles are left alone (f16 64^3
+  // was 6 % slower with it), profiles/r1/hint_ab_r1.txt.
+  p.l2hint = tc_tune().hint > 0 ? tc_tune().hint : (tc_tune().hint < 0 ? 0 : s.write_heavy);
   const long long groups = (batch + G * U - 1) / (G * U);
   p.units = groups * s.m_tiles;
 
