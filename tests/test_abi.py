@@ -102,6 +102,17 @@ def test_plan_covers_the_16bit_grid():
                 assert p["kernel"] == "tcgen05" and p["stages"] >= 2, (m, n, k)
 
 
+def test_plan_ring_depth_rules():
+    """tcgen05 ring depth (DESIGN.md 4.1 'Stages and bytes in flight'): ~96 KB of TMA loads in
+    flight, at least 3 stages where shared memory allows, at most 4 for write-heavy units."""
+    assert kami.plan(64, 64, 64, "f16")["stages"] == 3          # 32 KB stages under the 96 KB cap
+    assert kami.plan(192, 192, 192, "bf16")["stages"] == 3      # 40 KB stages: raised from 2 to 3
+    assert kami.plan(256, 256, 256, "bf16")["stages"] == 2      # 48 KB stages + 128 KB staging: 2 fit
+    assert kami.plan(64, 64, 64, "e4m3")["stages"] == 4         # FP8 in / FP16 out: write-heavy cap
+    assert kami.plan(256, 256, 16, "f16")["stages"] == 4        # low-rank: write-heavy cap (was 8)
+    assert kami.plan(16, 16, 256, "bf16")["stages"] >= 3        # read-heavy small tiles keep a deep ring
+
+
 GOLD = json.load(open(os.path.join(ROOT, "tests", "golden", "cost_model_examples.json")))
 
 
