@@ -39,7 +39,13 @@ constexpr uint32_t kCRow = 128 * 2 + 16;              // padded staging row (128
 constexpr uint32_t kCBuf = 128 * kCRow;               // one warpgroup's C staging (34 KB)
 constexpr int kSmemLimit = 232448;
 
-struct VbParams {
+struct alignas(64) VbParams {
+  // SpMM with n % 64 == 0: dense B arrives by TMA (4-D (64, k, n/64, batch), box
+  // (64, 64, n/64, G), 128-byte swizzle = the N-major atoms the copies build)
+  // and the producer warpgroup copies only the sparse A
+  CUtensorMap tmB;
+  int b_tma;
+  uint32_t b_tx;
   const void* const* A;
   const void* const* B;
   void* const* C;
@@ -136,7 +142,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < p.stages; ++s) {
-      ptx::mbar_init(&full[s], 128);
+      ptx::mbar_init(&full[s], 128 + (p.b_tma ? 1 : 0));  // + the B TMA's expect_tx arrival
       ptx::mbar_init(&empty[s], 1);
     }
     for (int a = 0; a < p.acc_bufs; ++a) {
@@ -274,7 +280,12 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         }
         // B: per entry 64 k-rows x n/8 chunks at columns [g n, g n + n) of the
         // N-major tile (atoms of 64 columns x 64 k-rows)
-        if (nc8_shift >= 0 && nc8 <= 128) {
+        if (p.b_tma) {  // one TMA box: G entries x 64 k-rows x n (zero-filled past k / batch)
+          if (tid == 0) {
+            ptx::mbar_arrive_expect_tx(&full[s], p.b_tx);
+            ptx::tma_load_4d(smem + s * p.stage_bytes + kAReg, &p.tmB, &full[s], 0, kc * 64, 0, (int)U.e0);
+          }
+        } else if (nc8_shift >= 0 && nc8 <= 128) {
           const int j = tid & (nc8 - 1), kr0 = tid >> nc8_shift, kstep = 128 >> nc8_shift;
           for (int g = 0; g < U.ng; ++g) {
             const uint16_t* B = b_tab[g];
@@ -518,6 +529,20 @@ kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf
   p.batch = batch;
   p.G = packing(m, n);
   p.bsr = 1;
+  if (n % 64 == 0) {  // dense B by TMA (the producer then copies only A's nonzero blocks)
+    PFN_encodeTiled enc = get_encode_tiled();
+    if (!enc) return KAMI_ERROR_CUDA;
+    cuuint64_t dims[4] = {64, (cuuint64_t)k, (cuuint64_t)(n / 64), (cuuint64_t)batch};
+    cuuint64_t strides[3] = {(cuuint64_t)n * 2, 128, (cuuint64_t)k * n * 2};
+    cuuint32_t box[4] = {64, 64, (cuuint32_t)(n / 64), (cuuint32_t)p.G};
+    cuuint32_t es[4] = {1, 1, 1, 1};
+    if (enc(&p.tmB, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4,
+            const_cast<void*>(B), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
+    p.b_tma = 1;
+    p.b_tx = (uint32_t)(8192 * (n / 64) * p.G);
+  }
   p.max_nnzb = max_nnzb;
   p.rowptr = row_ptr;
   p.colblk = col_blk;
