@@ -24,6 +24,7 @@ struct Tc16Shape {
   int slot;    // A-tile rows / TMEM lanes per packed entry
   int colrep;  // thin m, G = 1: number of 32-lane slots the A box is replicated into (0 = off)
   int write_heavy;  // a unit writes at least as many bytes as it reads
+  int tpack;        // 128 < m <= 192, n <= 128: two entries' tail rows share a tile (3 units per pair)
   int U;  // MMA sub-tiles per unit (G U entries per unit)
   uint32_t stage_bytes, c_buf_bytes;
   int c_bufs, stages, acc_cols, acc_bufs;
@@ -35,7 +36,8 @@ kami_status_t tc16_launch(int m, int n, int k, long long batch, bool bf16, const
                           cudaStream_t stream, int max_ctas);
 // in_kind: 0 f16, 1 bf16, 2 tf32, 3 e4m3, 4 e5m2; out_kind: 0 f16, 1 bf16, 2 f32.
 // C = alpha A B + beta C (C is read iff beta != 0).
-kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kind, Tc16Shape* s);
+// no_tp: no tail packing (pointer arrays, the C-update form)
+kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kind, Tc16Shape* s, bool no_tp = false);
 // Aa/Ba/Ca != nullptr: device pointer arrays (kami_gemm_batched; f16/bf16, C = AB only), A/B/C unused.
 kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind, int out_kind, const void* A,
                                const void* B, void* C, float alpha, float beta, cudaStream_t stream, int max_ctas,

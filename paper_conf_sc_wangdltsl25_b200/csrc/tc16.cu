@@ -125,6 +125,12 @@ struct alignas(64) Tc16Params {
   uint32_t a_entry, b_entry, c_entry;  // shared-memory bytes of one entry's A / B / C box
   uint32_t entry_tx, entry_tx_t;       // TMA bytes of one entry's A + B boxes per k-chunk (full / tail m-tile)
   int l2hint;                          // 1: C stores evict_first in L2, 2: also the A loads (experiment)
+  // tail packing (kTP; 128 < m <= 192, n <= 128): units come in threes per
+  // pair of entries -- head(e), head(e+1), then both entries' last m - 128
+  // rows packed block-diagonally into one tile (64-lane slots, N = 2n)
+  int tpack;
+  uint32_t tx_tail, idesc_tail;
+  CUtensorMap tmAt2, tmBt2, tmCt2;     // boxes (Wk, 64, 2), (Wn, Wk, n/Wn, 2), (Wc, 64, n/Wc, 2)
   int m_tail;                          // m > 128, m % 128 != 0: the last m-tile uses tmAt / tmCt / tmCat
   CUtensorMap tmAt, tmCt, tmCat;       // pointer arrays: boxes of m % 128 rows for the last m-tile
 };
@@ -250,7 +256,7 @@ __device__ __forceinline__ void emit8_f32_global(float* dst, const uint32_t* v, 
 
 // kUpd: the C-update epilogue (alpha != 1 or beta != 0); the plain C = AB
 // instantiation carries none of its code.
-template <int kIn, int kOut, bool kUpd, bool kSplit, bool kPtr = false>
+template <int kIn, int kOut, bool kUpd, bool kSplit, bool kPtr = false, bool kTP = false>
 __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const __grid_constant__ Tc16Params p) {
   constexpr bool kXpose = kIn == IN_TF32;
   constexpr bool kDirect = kOut == OUT_F32;
@@ -363,6 +369,23 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       UnitIter ui(blockIdx.x, gridDim.x, p.m_tiles);
       for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ui.next()) {
         const int e0 = (int)(ui.grp * p.GU);
+        if constexpr (kTP) {  // head(2 grp), head(2 grp + 1), packed tail pair
+          const int e2 = (int)(ui.grp * 2);
+          const bool tl = ui.mt == 2;
+          for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
+            ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
+            ptx::mbar_arrive_expect_tx(&full[r.s], tl ? p.tx_tail : p.tx_bytes);
+            uint8_t* sa = smem + r.s * p.stage_bytes;
+            if (tl) {
+              ptx::tma_load_3d(sa, &p.tmAt2, &full[r.s], kc * p.Wk, 128, e2);
+              ptx::tma_load_4d(sa + p.a_region, &p.tmBt2, &full[r.s], 0, kc * p.Wk, 0, e2);
+            } else {
+              ptx::tma_load_3d(sa, &p.tmA, &full[r.s], kc * p.Wk, 0, e2 + ui.mt);
+              ptx::tma_load_4d(sa + p.a_region, &p.tmB, &full[r.s], 0, kc * p.Wk, 0, e2 + ui.mt);
+            }
+          }
+          continue;
+        }
         for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
           ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
           ptx::mbar_arrive_expect_tx(&full[r.s], p.tx_bytes);
@@ -385,10 +408,12 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     const uint64_t adesc0 = ptx::make_smem_desc(smem_base, 16, p.a_sbo, p.a_layout);
     const uint64_t bdesc0 = ptx::make_smem_desc(smem_base + p.a_region, p.b_lbo, p.b_sbo, p.b_layout);
     const uint32_t stage16 = p.stage_bytes >> 4, bstep16 = p.b_kstep >> 4;
-    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ra.next(p.acc_bufs)) {
+    UnitIter mui(blockIdx.x, gridDim.x, p.m_tiles);  // (kTP: the unit type)
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ra.next(p.acc_bufs), mui.next()) {
       ptx::mbar_wait(&tempty[ra.s], ra.ph ^ 1);
       ptx::tc_fence_after();
       const uint32_t d_tmem = tmem_base + ra.s * p.acc_cols;
+      const uint32_t idesc = (kTP && mui.mt == 2) ? p.idesc_tail : p.idesc;
       for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
         ptx::mbar_wait(kXpose ? &bready[r.s] : &full[r.s], r.ph);
         ptx::tc_fence_after();
@@ -401,7 +426,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
             for (int ks = 0; ks < nsteps; ++ks) {
               // A: K-major, one K step = 32 bytes further along the swizzled row;
               // B: N-major, one K step = 32/es K rows further (TF32: K-major, 32 bytes)
-              umma<kIn>(d_tmem + j * p.N_mma, adj + 2 * ks, bdj + bstep16 * ks, p.idesc, (kc | ks) != 0);
+              umma<kIn>(d_tmem + j * p.N_mma, adj + 2 * ks, bdj + bstep16 * ks, idesc, (kc | ks) != 0);
             }
           }
           ptx::umma_commit(&empty[r.s]);  // stage s may be refilled once these MMAs retire
@@ -483,6 +508,13 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     const uint32_t row_bytes = (uint32_t)p.Wc * ESO;
     const uint32_t atom_stride = (uint32_t)p.rows_tile * row_bytes;
     const uint32_t rowbase = (uint32_t)(g * (p.n / p.Wc) * p.rows_tile + r) * row_bytes;
+    // kTP tail tiles: two entries' last t = m - 128 rows in 64-lane slots, N = 2n
+    const int t_rows = p.m - 128;
+    const int tg = L >> 6, tr = L & 63;
+    const bool t_row_ok = tr < t_rows;
+    const int t_col_lo = tg * p.n, t_col_hi = ((sp * 32) & 63) < t_rows ? t_col_lo + p.n : t_col_lo;
+    const uint32_t t_atom_stride = 64u * row_bytes;
+    const uint32_t t_rowbase = (uint32_t)(tg * (p.n / p.Wc) * 64 + tr) * row_bytes;
     const int wc_shift = 31 - __clz(p.Wc);
     const uint32_t c_smem = smem_base + p.c_off + (uint32_t)wg * p.c_bufs * p.c_buf_bytes;
     // this warpgroup's units: u0 + 2j gridDim; accumulators wg, wg + 2, ... (mod acc_bufs);
@@ -503,9 +535,16 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
     if (kPtr && storer && u0 < p.units && ui.grp * p.GU + lane < p.batch) qc = p.Ca[ui.grp * p.GU + lane];
     for (long long u = u0; u < p.units; u += 2ll * gridDim.x, ui.next()) {
       const int mt = ui.mt;
-      const long long e0 = ui.grp * p.GU;
       const uint32_t cb = cpos.s;
-      const bool valid0 = row_ok && (p.G > 1 || mt * 128 + r < p.m);  // r = L except replicated tiles
+      // per-unit geometry (kTP: head units are one entry's rows 0..127, tail
+      // units the packed last rows of two entries)
+      const bool tl = kTP && mt == 2;
+      const long long e0 = kTP ? ui.grp * 2 + (tl ? 0 : mt) : ui.grp * p.GU;
+      const int mrow = kTP ? (tl ? 128 : 0) : mt * 128;  // first C row of the unit's tile
+      const int q_g = tl ? tg : g, q_lo = tl ? t_col_lo : col_lo, q_hi = tl ? t_col_hi : col_hi;
+      const int q_my_lo = tl ? tg * p.n : my_lo, q_my_hi = q_my_lo + p.n;
+      const uint32_t q_rowbase = tl ? t_rowbase : rowbase, q_astride = tl ? t_atom_stride : atom_stride;
+      const bool valid0 = tl ? t_row_ok : (row_ok && (p.G > 1 || kTP || mt * 128 + r < p.m));  // r = L except replicated tiles
       int clo = 0, chi = 0;
       bool cstore = false;
       if constexpr (kPtr) {
@@ -594,16 +633,16 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
         continue;
       }
       for (int j = 0; j < p.U; ++j) {
-      const bool valid = valid0 && (e0 + j * p.G + g < p.batch);
+      const bool valid = valid0 && (e0 + j * p.G + q_g < p.batch);
       float* crow = nullptr;
       if constexpr (kDirect)
         crow = reinterpret_cast<float*>(p.Cg) + ((e0 + j * p.G + g) * p.m + mt * 128 + r) * (long long)p.n;
       const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols + j * p.N_mma;
-      const uint32_t rowbase_j = rowbase + (uint32_t)(j * p.G * (p.n / p.Wc)) * atom_stride;
-      for (int c0 = col_lo; c0 < col_hi; c0 += 64) {
+      const uint32_t rowbase_j = q_rowbase + (uint32_t)(j * p.G * (p.n / p.Wc)) * q_astride;
+      for (int c0 = q_lo; c0 < q_hi; c0 += 64) {
         uint32_t v[64];
         // issue both TMEM loads, then one wait (never read past col_hi)
-        const int left = col_hi - c0;
+        const int left = q_hi - c0;
         if (left >= 64) {
           ptx::tmem_ld_32x32b_x32(t_row + c0, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
           ptx::tmem_ld_32x32b_x32(t_row + c0 + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
@@ -619,14 +658,14 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
 #pragma unroll
         for (int q = 0; q < 8; ++q) {
           const int col = c0 + 8 * q;
-          if (valid && col >= my_lo && col < my_hi && col < col_hi) {
-            const uint32_t jc = (uint32_t)(col - my_lo);
+          if (valid && col >= q_my_lo && col < q_my_hi && col < q_hi) {
+            const uint32_t jc = (uint32_t)(col - q_my_lo);
             if constexpr (kDirect) {
               emit8_f32_global<kUpd>(crow + jc, &v[8 * q], p);
             } else {
               const uint32_t atom = jc >> wc_shift;
               const uint32_t ce = jc & (uint32_t)(p.Wc - 1);
-              emit8<kOut, kUpd>(cbase, rowbase_j + atom * atom_stride + ce * ESO, p.c_swz_bits, &v[8 * q], p);
+              emit8<kOut, kUpd>(cbase, rowbase_j + atom * q_astride + ce * ESO, p.c_swz_bits, &v[8 * q], p);
             }
           }
         }
@@ -653,11 +692,12 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
           ptx::bulk_commit();
         }
       } else if (leader) {
+        const CUtensorMap* tmc = tl ? &p.tmCt2 : &p.tmC;
         if (p.l2hint)
-          ptx::tma_store_4d_hint(&p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mt * 128, 0,
-                                 (int)e0, cpol);
+          ptx::tma_store_4d_hint(tmc, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mrow, 0, (int)e0,
+                                 cpol);
         else
-          ptx::tma_store_4d(&p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mt * 128, 0, (int)e0);
+          ptx::tma_store_4d(tmc, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes, 0, mrow, 0, (int)e0);
         ptx::bulk_commit();
         if (wg == 0) KAMI_TS(6);
       }
@@ -712,13 +752,13 @@ constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 // possible; slot = -1 disables thin-m slots; hint = -1 no L2 policy, 1 C evict_first,
 // 2 C and A evict_first, 0 planner rule).  Unset in production.
 struct TcTune {
-  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0, slot = 0, hint = 0;
+  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0, slot = 0, hint = 0, tp = 0;
 };
 const TcTune& tc_tune() {
   static const TcTune t = [] {
     TcTune r;
-    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split, &r.slot,
-                 &r.hint);
+    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split, &r.slot,
+                 &r.hint, &r.tp);
     return r;
   }();
   return t;
@@ -727,6 +767,13 @@ const TcTune& tc_tune() {
 template <int kIn, int kOut>
 void launch_kernel(const Tc16Params& p, unsigned grid, size_t smem, cudaStream_t stream, const char* name) {
   if constexpr (kIn <= IN_BF16) {
+    if (p.tpack) {  // tail packing (strided C = AB only)
+      cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false, false, false, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      kami_tc16_1d_kernel<kIn, kOut, false, false, false, true><<<grid, threads_for(kIn), smem, stream>>>(p);
+      set_last_kernel(kIn == IN_BF16 ? "kami_tc16_1d_kernel<bf16,tailpack>" : "kami_tc16_1d_kernel<f16,tailpack>");
+      return;
+    }
     if (p.Aa) {  // pointer arrays (C = AB only)
       if (p.split_store) {
         cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false, true, true>,
@@ -759,7 +806,7 @@ void launch_kernel(const Tc16Params& p, unsigned grid, size_t smem, cudaStream_t
 
 }  // namespace
 
-kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kind, Tc16Shape* s) {
+kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kind, Tc16Shape* s, bool no_tp) {
   const int esi = in_es(in_kind), eso = out_es(out_kind);
   s->G = 1;
   if (m <= 128) {
@@ -769,6 +816,11 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   }
   s->m_tiles = (s->G > 1 || m <= 128) ? 1 : (m + 127) / 128;
   s->rows_tile = m < 128 ? m : 128;
+  // Tail packing: for 128 < m <= 192 the last m-tile holds only m - 128 <= 64
+  // rows, so two entries' tails share one tile (block-diagonal, N = 2n <= 256):
+  // 1.5 units per entry instead of 2 (three units per pair: head, head, tail)
+  s->tpack = (m > 128 && m <= 192 && n <= 128 && in_kind <= IN_BF16 && !no_tp && tc_tune().tp >= 0) ? 1 : 0;
+  if (s->tpack) s->m_tiles = 3;
   // Thin m packed 2 or 4 to a tile would sit in one or two TMEM sub-partitions
   // (lanes 0..G m), leaving the other epilogue warps idle: give each entry a
   // 32-lane slot instead (the A box is 32 rows; TMA zero-fills rows m..31),
@@ -794,7 +846,7 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   s->Wn = wn_b / esi;
   s->Wc = wc_b / eso;
   s->k_chunks = (kpad + s->Wk - 1) / s->Wk;
-  s->N_mma = s->G > 1 ? s->G * n : n;
+  s->N_mma = s->G > 1 ? s->G * n : (s->tpack ? 2 * n : n);
   // Sub-tiles per unit: small tiles are bound by the per-unit fixed cost of
   // the single-thread producer / MMA roles and the epilogue barriers, so
   // U MMA tiles (G U entries) share one unit until a unit moves >= 32 KB
@@ -805,10 +857,23 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
     const long long rt = s->rows_tile;
     const long long tile_bytes =
         (long long)s->G * (rt * k * esi + (long long)k * n * esi + rt * n * eso);
-    while (s->U < 4 && tile_bytes * s->U < 32 * 1024 && 2 * s->U * s->N_mma <= 256 && s->G * 2 * s->U <= 256)
+    const int n_mma = s->tpack ? n : s->N_mma;  // (sub-tiles are decided on the unpacked tile)
+    while (s->U < 4 && tile_bytes * s->U < 32 * 1024 && 2 * s->U * n_mma <= 256 && s->G * 2 * s->U <= 256)
       s->U *= 2;
   }
   if (tc_tune().U > 0) s->U = tc_tune().U;
+  // Tail packing needs one entry per head unit; narrow tiles small enough for
+  // sub-tiles (n <= 32 and U > 1) stay with U entries per m-tile, which is
+  // faster there (bf16 192x16x16 0.53 vs 0.35 packed, 192x32x16 0.64 vs 0.53),
+  // while packing wins from n = 64 or once the tile is big (192x64x16 0.78 ->
+  // 0.88, 192x128x16 0.75 -> 0.97, 192x16x128 0.66 -> 0.89, 192x128x128 0.95
+  // -> 1.05; profiles/r1/tp_ab_r1.txt).
+  if (s->tpack && s->U > 1 && n <= 32) {
+    s->tpack = 0;
+    s->m_tiles = (m + 127) / 128;
+    s->N_mma = n;
+  }
+  if (s->tpack) s->U = 1;
   for (;; s->U /= 2) {  // fall back to fewer sub-tiles if the ring does not fit
     const int rowsA = s->slot;
     const uint32_t a_region = align_up((uint32_t)((s->U - 1) * s->G * rowsA + 128) * wk_b, 1024);
@@ -872,7 +937,8 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   const bool ptr = Aa != nullptr;
   if (ptr && (in_kind > IN_BF16 || alpha != 1.0f || beta != 0.0f || !Ba || !Ca)) return KAMI_ERROR_NOT_SUPPORTED;
   Tc16Shape s;
-  kami_status_t st = tc16_plan_shape_kind(m, n, k, in_kind, out_kind, &s);
+  // (tail packing: strided C = AB only)
+  kami_status_t st = tc16_plan_shape_kind(m, n, k, in_kind, out_kind, &s, ptr || alpha != 1.0f || beta != 0.0f);
   if (st != KAMI_SUCCESS) return st;
   PFN_encodeTiled enc = get_encode_tiled();
   if (!enc) return KAMI_ERROR_CUDA;
@@ -913,6 +979,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   p.b_lbo = s.Wk * wn_b;                   // next N-atom
   p.b_kstep = (uint32_t)(kgran / 8) * p.b_sbo;  // one 32-byte K step of B rows
   if (ptr) s.slot = s.rows_tile;  // view boxes never reach past the entry
+  p.tpack = s.tpack;
   const int U = s.U, G = s.G, rowsA = s.slot;
   p.slot = s.slot;
   p.colrep = ptr ? 0 : s.colrep;
@@ -954,8 +1021,14 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   // of roofline), lr-32 +0.5 %; read-dominated tiles are left alone (f16 64^3
   // was 6 % slower with it), profiles/r1/hint_ab_r1.txt.
   p.l2hint = tc_tune().hint > 0 ? tc_tune().hint : (tc_tune().hint < 0 ? 0 : s.write_heavy);
-  const long long groups = (batch + G * U - 1) / (G * U);
+  const long long groups = s.tpack ? (batch + 1) / 2 : (batch + G * U - 1) / (G * U);
   p.units = groups * s.m_tiles;
+  if (s.tpack) {
+    p.tx_bytes = (uint32_t)(wk_b * 128 + wk_b * n);            // head: one entry's 128 rows
+    p.tx_tail = (uint32_t)(2 * (wk_b * 64 + wk_b * n));         // tail: two entries' 64-row slots
+    p.idesc_tail = p.idesc;                                     // N = 2n
+    p.idesc = ptx::make_idesc_f16(in_kind == IN_BF16 ? 1 : 0, 128, n, 0, 1);  // head: N = n
+  }
 
   const CUtensorMapDataType dti = in_kind == IN_BF16   ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16
                                   : in_kind == IN_F16  ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
@@ -1024,6 +1097,22 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
             swz_mode_for(wn_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
+  if (s.tpack) {  // tail tiles: rows 128.. of two entries (64-row slots), both entries' B
+    cuuint64_t da[3] = {(cuuint64_t)k, (cuuint64_t)m, (cuuint64_t)batch};
+    cuuint64_t sa_[2] = {(cuuint64_t)k * esi, (cuuint64_t)m * k * esi};
+    cuuint32_t ba[3] = {(cuuint32_t)s.Wk, 64, 2};
+    cuuint32_t es3[3] = {1, 1, 1};
+    if (enc(&p.tmAt2, dti, 3, const_cast<void*>(A), da, sa_, ba, es3, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            swz_mode_for(wk_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
+    cuuint64_t db[4] = {(cuuint64_t)s.Wn, (cuuint64_t)k, (cuuint64_t)(n / s.Wn), (cuuint64_t)batch};
+    cuuint64_t sb_[3] = {(cuuint64_t)n * esi, (cuuint64_t)wn_b, (cuuint64_t)k * n * esi};
+    cuuint32_t bb[4] = {(cuuint32_t)s.Wn, (cuuint32_t)s.Wk, (cuuint32_t)(n / s.Wn), 2};
+    cuuint32_t es4[4] = {1, 1, 1, 1};
+    if (enc(&p.tmBt2, dti, 4, const_cast<void*>(B), db, sb_, bb, es4, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            swz_mode_for(wn_b), promo, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
+  }
   }  // strided
   // Per-atom C stores (kSplit instantiation) for one-entry tiles with >= 2
   // 64-column atoms: the store engine starts on atom 0 while the rest is
@@ -1032,7 +1121,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   // 0.95).  Not for full 128-row tiles with k <= 16 (C-store dominated low-rank:
   // lr-8 0.90 -> 0.84, lr-16 0.92 -> 0.85 measured), profiles/r1/split_store_r1.txt.
   // (replicated thin-m tiles store from all four warps at once: no per-atom split)
-  p.split_store = (out_kind != OUT_F32 && !p.colrep && s.G == 1 && s.U == 1 && s.Wc == 64 && n % 64 == 0 &&
+  p.split_store = (out_kind != OUT_F32 && !p.colrep && !p.tpack && s.G == 1 && s.U == 1 && s.Wc == 64 && n % 64 == 0 &&
                    n >= 128 &&
                    (!(s.rows_tile == 128 && k <= 16) || tc_tune().split > 0) && beta == 0.0f && alpha == 1.0f &&
                    tc_tune().split >= 0)
@@ -1066,6 +1155,11 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
     if (p.split_store && enc(&p.tmCa, dto, 4, C, dims, strides, box1, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                              swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE,
                              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
+    cuuint32_t boxt[4] = {(cuuint32_t)s.Wc, 64, (cuuint32_t)(n / s.Wc), 2};  // tail tiles (rows >= m clipped)
+    if (s.tpack && enc(&p.tmCt2, dto, 4, C, dims, strides, boxt, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                       swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE,
+                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
 

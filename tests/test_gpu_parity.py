@@ -66,6 +66,9 @@ TC_SHAPES = [
     (16, 256, 64, 20),    # G = 1 with 16 live rows
     (16, 128, 40, 37),    # thin m, G = 2 slots, k tail
     (16, 256, 16, 45),    # thin m, G = 1: A replicated into 4 slots, one 64-column block per warp
+    (192, 64, 64, 7),     # tail packing: head, head, packed tails; odd batch (last pair half empty)
+    (144, 128, 24, 10),   # tail packing with 16-row tails, N = 256, k tail
+    (160, 16, 16, 33),    # tail packing, narrowest N
     (32, 240, 24, 29),    # thin m, G = 1, 4 slots, last block 48 columns, k tail
     (128, 16, 16, 17),    # narrowest N
 ]
@@ -81,7 +84,7 @@ def test_tc16_unif(shape, dtype, layout):
 
 
 @pytest.mark.parametrize("shape", TC_SHAPES[:7] + [(256, 256, 16, 3), (16, 128, 40, 37), (16, 256, 16, 45),
-                                                  (32, 240, 24, 29)],
+                                                  (32, 240, 24, 29), (192, 64, 64, 7), (144, 128, 24, 10)],
                          ids=lambda s: "x".join(map(str, s)))
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 def test_tc16_int_bit_exact(shape, dtype):
