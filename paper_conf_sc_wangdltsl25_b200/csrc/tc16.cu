@@ -129,6 +129,8 @@ struct alignas(64) Tc16Params {
   // pair of entries -- head(e), head(e+1), then both entries' last m - 128
   // rows packed block-diagonally into one tile (64-lane slots, N = 2n)
   int tpack;
+  int warp_store;                      // kWS: every epilogue warp stores its own 32-row slabs (tmCw)
+  CUtensorMap tmCw;                    // box (Wc, 32, 1, 1)
   uint32_t tx_tail, idesc_tail;
   CUtensorMap tmAt2, tmBt2, tmCt2;     // boxes (Wk, 64, 2), (Wn, Wk, n/Wn, 2), (Wc, 64, n/Wc, 2)
   int m_tail;                          // m > 128, m % 128 != 0: the last m-tile uses tmAt / tmCt / tmCat
@@ -256,7 +258,7 @@ __device__ __forceinline__ void emit8_f32_global(float* dst, const uint32_t* v, 
 
 // kUpd: the C-update epilogue (alpha != 1 or beta != 0); the plain C = AB
 // instantiation carries none of its code.
-template <int kIn, int kOut, bool kUpd, bool kSplit, bool kPtr = false, bool kTP = false>
+template <int kIn, int kOut, bool kUpd, bool kSplit, bool kPtr = false, bool kTP = false, bool kWS = false>
 __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const __grid_constant__ Tc16Params p) {
   constexpr bool kXpose = kIn == IN_TF32;
   constexpr bool kDirect = kOut == OUT_F32;
@@ -555,6 +557,62 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
         qc = nullptr;
         if (storer && u + 2ll * gridDim.x < p.units && nx.grp * p.GU + lane < p.batch) qc = p.Ca[nx.grp * p.GU + lane];
       }
+      if constexpr (kWS) {
+        // Per-warp C stores (one entry per tile, 64-column atoms): each warp
+        // stages its own 32 rows of every atom (colrep tiles: its own atom) and
+        // stores them with its own TMA box as soon as they are written -- no
+        // warpgroup barrier; a warp only waits for its own previous stores to
+        // leave shared memory before reusing its slab.
+        const uint32_t cbase = c_smem + cb * p.c_buf_bytes;
+        uint8_t* cbuf = smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes;
+        const bool active = col_hi > col_lo;
+        const bool valid = valid0 && e0 < p.batch;
+        if (lane == 0) ptx::bulk_wait_read<0>();
+        __syncwarp();
+        ptx::mbar_wait(&tfull[a], aph);
+        ptx::tc_fence_after();
+        const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + a * p.acc_cols;
+        for (int c0 = col_lo; c0 < col_hi; c0 += 64) {
+          uint32_t v[64];
+          const int left = col_hi - c0;
+          if (left >= 64) {
+            ptx::tmem_ld_32x32b_x32(t_row + c0, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+            ptx::tmem_ld_32x32b_x32(t_row + c0 + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+          } else {
+            ptx::tmem_ld_32x32b_x32(t_row + c0, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
+          }
+          ptx::tmem_wait_ld();
+          const uint32_t atom = (uint32_t)(c0 >> 6);
+          if (valid) {
+#pragma unroll
+            for (int q = 0; q < 8; ++q)
+              if (8 * q < left)
+                emit8<kOut, kUpd>(cbase, rowbase + atom * atom_stride + (uint32_t)(8 * q) * ESO, p.c_swz_bits,
+                                  &v[8 * q], p);
+          }
+          ptx::fence_proxy_async_smem();
+          __syncwarp();
+          if (lane == 0 && active) {
+            const int row0 = p.colrep ? 0 : 32 * sp;  // colrep: the warp's atom holds every row
+            const uint32_t off = atom * atom_stride + (uint32_t)(p.colrep ? 0 : 32 * sp) * row_bytes;
+            if (p.l2hint)
+              ptx::tma_store_4d_hint(&p.tmCw, cbuf + off, 0, mt * 128 + row0, (int)atom, (int)e0, cpol);
+            else
+              ptx::tma_store_4d(&p.tmCw, cbuf + off, 0, mt * 128 + row0, (int)atom, (int)e0);
+            ptx::bulk_commit();
+          }
+        }
+        ptx::tc_fence_before();  // accumulator a may be overwritten by the next MMA chain
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&tempty[a]);
+        a += 2;
+        if (a >= (uint32_t)p.acc_bufs) {
+          a -= p.acc_bufs;
+          aph ^= 1;
+        }
+        cpos.next(p.c_bufs);
+        continue;
+      }
       // the TMA store that last read staging buffer cb must be done reading
       if (!kDirect && storer) {
         // per-atom stores (kSplit) into a single staging buffer: only atom 0 of
@@ -702,7 +760,7 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
         if (wg == 0) KAMI_TS(6);
       }
     }
-    if (!kDirect && storer) ptx::bulk_wait<0>();
+    if (!kDirect && (kWS ? lane == 0 : storer)) ptx::bulk_wait<0>();
     if (leader && wg == 0) KAMI_TS(7);
   }
 
@@ -752,13 +810,13 @@ constexpr int kSmemLimit = 232448;  // 227 KB opt-in per CTA
 // possible; slot = -1 disables thin-m slots; hint = -1 no L2 policy, 1 C evict_first,
 // 2 C and A evict_first, 0 planner rule).  Unset in production.
 struct TcTune {
-  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0, slot = 0, hint = 0, tp = 0;
+  int stages = 0, cbufs = 0, grid = 0, promo = -1, U = 0, split = 0, slot = 0, hint = 0, tp = 0, ws = 0;
 };
 const TcTune& tc_tune() {
   static const TcTune t = [] {
     TcTune r;
-    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split, &r.slot,
-                 &r.hint, &r.tp);
+    if (const char* e = getenv("KAMI_TC_TUNE")) sscanf(e, "%d,%d,%d,%d,%d,%d,%d,%d,%d,%d", &r.stages, &r.cbufs, &r.grid, &r.promo, &r.U, &r.split, &r.slot,
+                 &r.hint, &r.tp, &r.ws);
     return r;
   }();
   return t;
@@ -767,6 +825,13 @@ const TcTune& tc_tune() {
 template <int kIn, int kOut>
 void launch_kernel(const Tc16Params& p, unsigned grid, size_t smem, cudaStream_t stream, const char* name) {
   if constexpr (kIn <= IN_BF16) {
+    if (p.warp_store) {  // per-warp C stores (strided C = AB, one entry per tile)
+      cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false, false, false, false, true>,
+                           cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      kami_tc16_1d_kernel<kIn, kOut, false, false, false, false, true><<<grid, threads_for(kIn), smem, stream>>>(p);
+      set_last_kernel(kIn == IN_BF16 ? "kami_tc16_1d_kernel<bf16,warpstore>" : "kami_tc16_1d_kernel<f16,warpstore>");
+      return;
+    }
     if (p.tpack) {  // tail packing (strided C = AB only)
       cudaFuncSetAttribute(kami_tc16_1d_kernel<kIn, kOut, false, false, false, true>,
                            cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -1156,6 +1221,22 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
                              swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE,
                              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
+    // Per-warp stores for replicated thin-m tiles (each warp owns one atom):
+    // bf16 16x256x16 33.4 -> 35.2 TFLOP/s.  On wide one-entry tiles they tie
+    // with the per-atom split stores (192^3 -2 % .. +5 %, 256^3 / 128x256x32 /
+    // lr-32 within 1 % across two boxes) and lose on the full-tile k <= 16
+    // low-rank shapes (lr-16 80 vs 84-92), so those keep their stores,
+    // profiles/r1/ws_ab_r1.txt.  Knob ws: 1 forces where possible, -1 disables.
+    const bool ws_ok = !ptr && !s.tpack && s.G == 1 && s.U == 1 && s.Wc == 64 && n % 64 == 0 && in_kind <= IN_BF16 &&
+                       alpha == 1.0f && beta == 0.0f && (s.colrep || s.rows_tile % 32 == 0);
+    p.warp_store = (ws_ok && (tc_tune().ws > 0 || (tc_tune().ws == 0 && s.colrep))) ? 1 : 0;
+    if (p.warp_store) {
+      p.split_store = 0;
+      cuuint32_t boxw[4] = {(cuuint32_t)s.Wc, 32, 1, 1};
+      if (enc(&p.tmCw, dto, 4, C, dims, strides, boxw, es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz_mode_for(wc_b),
+              CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return KAMI_ERROR_CUDA;
+    }
     cuuint32_t boxt[4] = {(cuuint32_t)s.Wc, 64, (cuuint32_t)(n / s.Wc), 2};  // tail tiles (rows >= m clipped)
     if (s.tpack && enc(&p.tmCt2, dto, 4, C, dims, strides, boxt, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                        swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE,
