@@ -900,7 +900,12 @@ kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kin
   // colrep_ab_r1.txt): bf16 16x256x16 0.56 -> 0.66 of roofline, 16x256x32
   // 0.83 -> 0.95, 32x256x16 0.84 -> 0.90; n = 192 (3 blocks) and k >= 64 are
   // as fast or faster with the per-atom split stores, so they keep those.
-  s->colrep = (s->G == 1 && m <= 32 && n > 192 && k <= 32 && s->m_tiles == 1 && tc_tune().slot >= 0)
+  // With per-warp stores (below) n = 192 at k = 16 and the n % 64 != 0 shapes
+  // (no per-atom split stores there) gain too: 16x192x16 0.51 -> 0.52,
+  // 32x192x16 0.77 -> 0.80, 16x144x16 0.22 -> 0.38; 32x192x32 keeps the split
+  // stores (0.97 vs 0.90-0.96).
+  const bool rep_n = (k <= 16 && n > 128) || (k <= 32 && (n > 192 || n % 64 != 0));
+  s->colrep = (s->G == 1 && m <= 32 && n > 128 && rep_n && s->m_tiles == 1 && tc_tune().slot >= 0)
                   ? (n + 63) / 64
                   : 0;
   const int kgran = 32 / esi;  // elements per 32-byte MMA K step

@@ -70,6 +70,8 @@ TC_SHAPES = [
     (144, 128, 24, 10),   # tail packing with 16-row tails, N = 256, k tail
     (160, 16, 16, 33),    # tail packing, narrowest N
     (32, 240, 24, 29),    # thin m, G = 1, 4 slots, last block 48 columns, k tail
+    (16, 144, 16, 31),    # thin m, G = 1, replicated A with 16-column atoms (no per-warp stores)
+    (32, 192, 16, 23),    # thin m, G = 1, 3 slots, per-warp stores
     (128, 16, 16, 17),    # narrowest N
 ]
 
