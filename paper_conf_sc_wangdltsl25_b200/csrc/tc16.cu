@@ -713,8 +713,8 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
           ptx::tmem_ld_32x32b_x16(t_row + c0, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
         }
         ptx::tmem_wait_ld();
-#pragma unroll
-        for (int q = 0; q < 8; ++q) {
+        // only the 8-column groups this block has (narrow tiles: 2 or 4, not 8)
+        auto emit_q = [&](int q) {
           const int col = c0 + 8 * q;
           if (valid && col >= q_my_lo && col < q_my_hi && col < q_hi) {
             const uint32_t jc = (uint32_t)(col - q_my_lo);
@@ -726,6 +726,16 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
               emit8<kOut, kUpd>(cbase, rowbase_j + atom * q_astride + ce * ESO, p.c_swz_bits, &v[8 * q], p);
             }
           }
+        };
+        if (left <= 16) {
+          emit_q(0);
+          emit_q(1);
+        } else if (left <= 32) {
+#pragma unroll
+          for (int q = 0; q < 4; ++q) emit_q(q);
+        } else {
+#pragma unroll
+          for (int q = 0; q < 8; ++q) emit_q(q);
         }
       }
       }  // sub-tiles
