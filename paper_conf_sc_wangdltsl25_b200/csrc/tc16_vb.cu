@@ -167,52 +167,65 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     RingPos rs;
     uint32_t it = 0;  // stages issued (trace index)
     UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
-    // the next unit's sizes and entry pointers are fetched one unit ahead:
-    // their global-load latency (the pointer arrays live in HBM) hides behind
-    // this unit's copy issue instead of stalling the table hand-over
-    Unit Un;
-    const uint16_t *pa_n = nullptr, *pb_n = nullptr;
+    // The sizes and entry pointers of a unit are fetched TWO units ahead into
+    // alternating register slots: their global-load latency (the pointer and
+    // size arrays live in HBM; ~1.5-2k cycles under load, more than one small
+    // unit's copy issue -- tools/trace_vb.py mix) hides behind two units of
+    // copy issue.  The loop body is instantiated once per slot so a slot whose
+    // loads are in flight is never copied.
+    // With one entry per unit (G == 1, no SpMM) every thread loads the entry's
+    // pointers itself (one broadcast address per warp), so no shared table or
+    // table barrier is needed.
+    const bool one = p.G == 1 && !p.bsr;
     // SpMM: the next unit's block structure is fetched ahead too, without the
     // row_ptr -> col_blk dependency: every col_blk slot of the unit's entries
     // (<= 2 per thread: G mb kb <= 256) and every row_ptr value (<= 17)
     const int mbk = p.bsr ? p.m / 16 : 0, rpn = mbk + 1;
-    int cb_n[2] = {-1, -1}, rp_n = 0;
-    auto fetch = [&]() {
-      unit_fill(p, ui.grp, ui.mt, Un);
-      if (tid < Un.ng) {
-        pa_n = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[Un.e0 + tid]);
-        pb_n = p.bsr ? p.Bs + (Un.e0 + tid) * (long long)p.k * p.n : reinterpret_cast<const uint16_t*>(p.B[Un.e0 + tid]);
+    struct PSlot {
+      Unit U;
+      const uint16_t *pa, *pb;
+      int cb[2], rp;
+    };
+    auto fetch = [&](PSlot& S) {
+      unit_fill(p, ui.grp, ui.mt, S.U);
+      S.pa = S.pb = nullptr;
+      S.cb[0] = S.cb[1] = -1;
+      S.rp = 0;
+      if (one || tid < S.U.ng) {
+        const long long e = S.U.e0 + (one ? 0 : tid);
+        S.pa = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[e]);
+        S.pb = p.bsr ? p.Bs + e * (long long)p.k * p.n : reinterpret_cast<const uint16_t*>(p.B[e]);
       }
       if (p.bsr) {
 #pragma unroll
         for (int q = 0; q < 2; ++q) {
           const int idx = tid + 128 * q;
-          cb_n[q] = idx < Un.ng * p.max_nnzb ? __ldg(p.colblk + Un.e0 * (long long)p.max_nnzb + idx) : -1;
+          S.cb[q] = idx < S.U.ng * p.max_nnzb ? __ldg(p.colblk + S.U.e0 * (long long)p.max_nnzb + idx) : -1;
         }
-        if (tid < Un.ng * rpn) rp_n = __ldg(p.rowptr + Un.e0 * (long long)rpn + tid);
+        if (tid < S.U.ng * rpn) S.rp = __ldg(p.rowptr + S.U.e0 * (long long)rpn + tid);
       }
-    };
-    if ((long long)blockIdx.x < p.units) fetch();
-    for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
-      const Unit U = Un;
-      const uint16_t *pa = pa_n, *pb = pb_n;
-      const int cb0 = cb_n[0], cb1 = cb_n[1], rpv = rp_n;
       ui.next();
-      if (u + gridDim.x < p.units) fetch();
-      if (U.mt * 128 >= U.m) continue;
+    };
+    auto body = [&](const PSlot& S) {
+      const Unit& U = S.U;
+      const uint16_t *pa = S.pa, *pb = S.pb;
+      const int cb0 = S.cb[0], cb1 = S.cb[1], rpv = S.rp;
+      if (U.mt * 128 >= U.m) return;
       const int m = U.m, n = U.n, k = U.k, G = p.G;
       const int kchunks = (k + 63) / 64;
       const int rows = G > 1 ? U.ng * m : min(128, m - U.mt * 128);  // live tile rows
-      ptx::named_bar_sync(3, 128);  // previous unit's items issued: tables reusable
-      if (tid < U.ng) {
-        a_tab[tid] = pa;
-        b_tab[tid] = pb;
+      if (!one) {
+        ptx::named_bar_sync(3, 128);  // previous unit's items issued: tables reusable
+        if (tid < U.ng) {
+          a_tab[tid] = pa;
+          b_tab[tid] = pb;
+        }
+        if (p.bsr) {
+          blk_tab[tid] = -1;
+          if (tid < U.ng * rpn) rp_tab[tid] = rpv;
+        }
+        ptx::named_bar_sync(3, 128);
       }
-      if (p.bsr) {
-        blk_tab[tid] = -1;
-        if (tid < U.ng * rpn) rp_tab[tid] = rpv;
-      }
-      ptx::named_bar_sync(3, 128);
       if (p.bsr) {
         // block lookup table of this tile: tile block row -> global block slot.
         // Slot idx = g max_nnzb + j of entry g lies in block row br with
@@ -270,7 +283,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
                 ptx::cp_async_16(dst0 + (tbase + q - r0) * 128, src, ok ? 16 : 0);
               }
             } else {
-              const uint16_t* A = a_tab[g];
+              const uint16_t* A = one ? pa : a_tab[g];
               const uint16_t* src = A + (long long)(ebase + r0) * k + gc;
               const long long step = (long long)rstep * k;
               for (int q = r0; q < cnt; q += rstep, src += step)
@@ -288,7 +301,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         } else if (nc8_shift >= 0 && nc8 <= 128) {
           const int j = tid & (nc8 - 1), kr0 = tid >> nc8_shift, kstep = 128 >> nc8_shift;
           for (int g = 0; g < U.ng; ++g) {
-            const uint16_t* B = b_tab[g];
+            const uint16_t* B = one ? pb : b_tab[g];
             const int cc = g * nc8 + j;  // 16-byte chunk column in the tile
             const uint32_t dcol = sb + (cc >> 3) * 8192;
             const uint16_t* src = B + (long long)(kc * 64 + kr0) * n + j * 8;
@@ -305,7 +318,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
             const int kr = rem / nc8, j = rem - kr * nc8;
             const int gk = kc * 64 + kr;
             const bool ok = gk < k;
-            const uint16_t* B = b_tab[g];
+            const uint16_t* B = one ? pb : b_tab[g];
             const uint16_t* src = ok ? B + (long long)gk * n + j * 8 : B;
             const int cc = g * nc8 + j;
             ptx::cp_async_16(sb + (cc >> 3) * 8192 + kr * 128 + (((cc & 7) ^ (kr & 7)) << 4), src, ok ? 16 : 0);
@@ -317,6 +330,25 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         ptx::cp_async_mbar_arrive_noinc(&full[s]);
         if (p.dbg & 4) trace(1, it);
       }
+    };
+    const long long g1 = gridDim.x, g2 = 2 * g1;
+    long long u = blockIdx.x;
+    PSlot S0, S1;
+    if (u < p.units) fetch(S0);
+    if (u + g1 < p.units) fetch(S1);
+    while (u < p.units) {
+      {
+        const PSlot c = S0;
+        if (u + g2 < p.units) fetch(S0);
+        body(c);
+      }
+      if ((u += g1) >= p.units) break;
+      {
+        const PSlot c = S1;
+        if (u + g2 < p.units) fetch(S1);
+        body(c);
+      }
+      u += g1;
     }
     ptx::cp_async_wait<0>();  // nothing may be in flight when the CTA exits
   } else if (warp == 4) {

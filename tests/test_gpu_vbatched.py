@@ -160,3 +160,36 @@ def test_vbatched_rejects():
         kami.gemm_vbatched(4, 16, 16, 16, 300, 16, 16, "f16", "row", 16, 16, 16)  # max_m off the grid
     with pytest.raises(kami.KamiError):
         kami.gemm_vbatched(4, 16, 16, 16, 64, 64, 64, "f64", "row", 16, 16, 16)  # fp64 not supported
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_vbatched_many_units_ring_wraps(dtype):
+    """Mixed orders at a batch large enough that every persistent CTA runs
+    tens of units: the variable-size stage ring (tc16_vb.cu, VRing) wraps many
+    times, releases chunks out of slot order and reuses all of its slots."""
+    rng = np.random.default_rng(21)
+    orders = np.array([16, 32, 48, 64, 128, 192, 256])
+    batch = 1200
+    sizes = [(int(rng.choice(orders)), int(rng.choice(orders)), int(rng.choice([8, 16, 40, 64, 136, 256])))
+             for _ in range(batch)]
+    ops = [ki.operands(m, n, k, 1, dtype, "unif", seed=22, entry0=e) for e, (m, n, k) in enumerate(sizes)]
+    offA = np.concatenate([[0], np.cumsum([a.numel() for a, _ in ops])])
+    offB = np.concatenate([[0], np.cumsum([b.numel() for _, b in ops])])
+    offC = np.concatenate([[0], np.cumsum([m * n for m, n, _ in sizes])])
+    dA = torch.cat([a for a, _ in ops]).cuda()
+    dB = torch.cat([b for _, b in ops]).cuda()
+    dC = torch.full((int(offC[-1]),), float("nan"), dtype=dA.dtype, device="cuda")
+    es = dA.element_size()
+    dm, dn, dk = (torch.tensor([s[i] for s in sizes], dtype=torch.int32, device="cuda") for i in range(3))
+    pa = torch.tensor(dA.data_ptr() + offA[:-1] * es, dtype=torch.int64, device="cuda")
+    pb = torch.tensor(dB.data_ptr() + offB[:-1] * es, dtype=torch.int64, device="cuda")
+    pc = torch.tensor(dC.data_ptr() + offC[:-1] * es, dtype=torch.int64, device="cuda")
+    kami.gemm_vbatched(batch, dm, dn, dk, 256, 256, 256, dtype, "row", pa, pb, pc)
+    torch.cuda.synchronize()
+    assert kami.last_kernel().startswith("kami_tc16_vb_kernel")
+    Cb = ki.as_bits(dC.cpu())
+    for e, ((m, n, k), (A, B)) in enumerate(zip(sizes, ops)):
+        Cref, S = oracle.gemm(m, n, k, 1, dtype, "row", ki.as_bits(A), ki.as_bits(B), with_scale=True)
+        got = oracle.decode(Cb[offC[e]:offC[e + 1]], dtype)
+        assert oracle.normalised_error(got.reshape(1, m, n), Cref, S) <= _tol(dtype, k), (e, m, n, k)
