@@ -23,6 +23,7 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <numeric>
 
 #include "kernels.h"
 #include "ptx.cuh"
@@ -530,7 +531,14 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const long long grid = p.units < sms ? p.units : sms;
+  long long grid = p.units < sms ? p.units : sms;
+  // Mixed sizes: units u = entry * mtiles + mt are strided by the grid, so a
+  // grid that shares a factor with mtiles pins every CTA to one m-tile index
+  // (148 CTAs, mtiles = 2: even CTAs take every entry's first tile, odd CTAs
+  // only the second tiles of m > 128 entries -- a ~3 : 1 imbalance).  A grid
+  // coprime to mtiles walks each CTA through all m-tile indices.
+  if (p.dm && p.mtiles > 1)
+    while (grid > 1 && std::gcd(grid, (long long)p.mtiles) != 1) --grid;
   fn<<<(unsigned)grid, kVbThreads, smem, stream>>>(p);
   set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
                         : (bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>"));
