@@ -48,6 +48,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <numeric>
 
 #include "kernels.h"
 #include "ptx.cuh"
@@ -1263,7 +1264,19 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   long long grid = p.units < sms ? p.units : sms;
-  if (tc_tune().grid > 0 && tc_tune().grid < grid) grid = tc_tune().grid;
+  // Units u = group * m_tiles + mt are strided by the grid, so a grid sharing a
+  // factor with m_tiles pins every CTA to one m-tile index.  When the last
+  // m-tile (m % 128 rows) costs clearly less than a full one, that leaves the
+  // CTAs of the full tiles on the critical path: 148 -> 147 CTAs for bf16
+  // 192x192x32 112.6 -> 128.7, 192x192x64 186.6 -> 210.6, 192x256x128 329 ->
+  // 345 TFLOP/s; at a cost ratio >= 0.8 (224x128x64) or k = 16 (192x256x16)
+  // the lost SM weighs more (-2 %).  profiles/r1/grid_ab_r1.txt (tc_tune.py).
+  if (tc_tune().grid == 0 && !s.tpack && p.m_tiles > 1 && m % 128 != 0 && k >= 32) {
+    const double full = 128.0 * (k + n) + (double)k * n, last = (double)(m % 128) * (k + n) + (double)k * n;
+    if (last < 0.8 * full)
+      while (grid > 1 && std::gcd(grid, (long long)p.m_tiles) != 1) --grid;
+  }
+  if (tc_tune().grid > 0 && tc_tune().grid < p.units) grid = tc_tune().grid;  // knob overrides (A/B)
   if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
   const size_t smem = s.smem_bytes;
   const unsigned g = (unsigned)grid;
