@@ -9,7 +9,7 @@ index) through a counter-based SplitMix64 hash, so
     (multi-GPU shards generate only their own entries, SURVEY.md Sec. 8(e));
   * the same torch code runs on CPU (oracle inputs) and on CUDA (bench inputs,
     no host->device copy of gigabytes) and yields bit-identical values
-    (checked on the GPU by tests/test_gpu_inputs.py).
+    (checked on the GPU by tests/test_gpu_parity.py::test_gpu_generator_matches_cpu).
 
 Value recipes (the paper never states its value
 distribution, Sec. 5.1 -- reading R17):

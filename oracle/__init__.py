@@ -161,8 +161,12 @@ def to_row_major(X: np.ndarray, batch: int, R: int, C: int, layout: str) -> np.n
 
 def normalised_error(c_gpu: np.ndarray, c_ref: np.ndarray, s: np.ndarray) -> float:
     """max |C_gpu - C_ref| / S with S = sum_l |a||b| (north_star).  Where S == 0
-    the GPU value must be exactly 0, otherwise the error is reported as inf."""
+    the GPU value must be exactly 0, otherwise the error is reported as inf; a
+    NaN anywhere in C_gpu is reported as inf.  Pinned by
+    tests/test_oracle_checker.py."""
     c_gpu = np.asarray(c_gpu, dtype=np.float64)
+    if np.any(np.isnan(c_gpu)):  # a NaN is never within any tolerance (max() would drop it)
+        return float("inf")
     diff = np.abs(c_gpu - c_ref)
     zero = s == 0
     if np.any(zero & (c_gpu != 0)):
