@@ -208,6 +208,26 @@ const char* kami_last_kernel(void);
 
 int kami_version(void); /* (MAJOR << 16) | MINOR */
 
+/* Diagnostic: the FP64 DMMA roofline denominator measured on this device.
+ * Runs an mma.sync.m8n8k4.f64 loop (the FP64 hot path's instruction) on
+ * 4 CTAs per SM, launch after launch on `stream`, for at least min_ms
+ * (0 <= min_ms <= 60000) and synchronizes.  *burst = the fastest launch
+ * (TFLOP/s, a kernel timed alone), *sustained = the median launch of the
+ * second half of the run (clock under the power cap).  Allocates and frees
+ * 64 bytes of device memory.  KAMI_ERROR_INVALID_VALUE for null outputs or
+ * min_ms out of range; KAMI_ERROR_CUDA if a launch fails. */
+kami_status_t kami_probe_dmma_peak(double min_ms, double* burst, double* sustained, kami_stream_t stream);
+
+/* Test / diagnostic knob: cap the number of CTAs of every persistent kernel
+ * launched afterwards by this process (0 = no cap, the default).  With a cap
+ * of c, each CTA of a batch of u work units runs ceil(u / c) of them, so the
+ * parity tests exercise the pipelines' steady state (ring wrap-around,
+ * mbarrier phase flips, TMEM accumulator and C staging reuse) at small batch
+ * sizes.  Results do not depend on the cap; only the speed does.  Not
+ * thread-safe with respect to concurrent launches on other threads.
+ * Returns KAMI_ERROR_INVALID_VALUE for max_ctas < 0.  No device work. */
+kami_status_t kami_set_grid_cap(int max_ctas);
+
 #ifdef __cplusplus
 }
 #endif

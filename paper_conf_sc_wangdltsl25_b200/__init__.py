@@ -14,7 +14,8 @@ import os
 
 __all__ = [
     "KamiError", "lib", "gemm", "gemm_batched", "gemm_strided_batched", "gemm_strided_batched_host",
-    "plan", "paper_cost", "last_kernel", "DTYPE", "LAYOUT", "ALGO", "SO_PATH",
+    "plan", "paper_cost", "last_kernel", "probe_dmma_peak", "set_grid_cap", "grid_cap", "DTYPE", "LAYOUT", "ALGO",
+    "SO_PATH",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -32,7 +33,8 @@ EXPORTS = [
     "kami_gemm", "kami_gemm_batched", "kami_gemm_strided_batched", "kami_gemm_strided_batched_ex",
     "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
     "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level", "kami_gemm_vbatched",
-    "kami_spmm_bsr_strided_batched", "kami_gemm_strided_batched_axpby",
+    "kami_spmm_bsr_strided_batched", "kami_gemm_strided_batched_axpby", "kami_probe_dmma_peak",
+    "kami_set_grid_cap",
 ]
 
 
@@ -73,6 +75,11 @@ def lib() -> ctypes.CDLL:
     L.kami_gemm_strided_batched_axpby.argtypes = [i, i, i, i64, i, i, ctypes.c_double, vp, vp, ctypes.c_double, vp,
                                                   st]
     L.kami_release_workspace.argtypes = []
+    L.kami_probe_dmma_peak.argtypes = [ctypes.c_double, ctypes.POINTER(ctypes.c_double),
+                                       ctypes.POINTER(ctypes.c_double), st]
+    L.kami_probe_dmma_peak.restype = ctypes.c_int
+    L.kami_set_grid_cap.argtypes = [i]
+    L.kami_set_grid_cap.restype = ctypes.c_int
     L.kami_plan.argtypes = [i, i, i, i, i, i, i, ctypes.POINTER(KamiPlan)]
     d = ctypes.c_double
     L.kami_paper_cost.argtypes = [i, d, d, d, d, d, d, d, d, d, d, d, ctypes.POINTER(ctypes.c_double)]
@@ -239,6 +246,35 @@ def paper_cost(variant, m, n, k, p, s_e, L_sm, B_sm, theta_r, theta_w, O_tc, n_t
     _check(lib().kami_paper_cost(_enum(ALGO, variant, "variant"), m, n, k, p, s_e, L_sm, B_sm, theta_r, theta_w,
                                  O_tc, n_tc, out), "kami_paper_cost")
     return tuple(out)
+
+
+def probe_dmma_peak(min_ms=200.0, stream=None):
+    """FP64 DMMA peak measured on the current device: (burst, sustained) TFLOP/s."""
+    b, s_ = ctypes.c_double(), ctypes.c_double()
+    _check(lib().kami_probe_dmma_peak(float(min_ms), ctypes.byref(b), ctypes.byref(s_), _stream(stream)),
+           "kami_probe_dmma_peak")
+    return b.value, s_.value
+
+
+def set_grid_cap(max_ctas: int):
+    """Test knob: cap every persistent kernel's grid (0 = no cap)."""
+    _check(lib().kami_set_grid_cap(int(max_ctas)), "kami_set_grid_cap")
+
+
+class grid_cap:
+    """Context manager: ``with kami.grid_cap(4): ...`` runs the enclosed calls
+    with at most 4 CTAs per persistent kernel (steady-state parity tests)."""
+
+    def __init__(self, max_ctas: int):
+        self.max_ctas = max_ctas
+
+    def __enter__(self):
+        set_grid_cap(self.max_ctas)
+        return self
+
+    def __exit__(self, *exc):
+        set_grid_cap(0)
+        return False
 
 
 def last_kernel() -> str:

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cmath>
 #include <cstdint>
 #include <cstdlib>
@@ -20,6 +21,8 @@ namespace kami {
 
 static thread_local const char* g_last_kernel = "";
 void set_last_kernel(const char* name) { g_last_kernel = name; }
+static std::atomic<int> g_grid_cap{0};
+int grid_cap() { return g_grid_cap.load(std::memory_order_relaxed); }
 
 PFN_encodeTiled get_encode_tiled() {
   static PFN_encodeTiled fn = nullptr;
@@ -298,5 +301,11 @@ const char* kami_status_string(kami_status_t s) {
 const char* kami_last_kernel(void) { return g_last_kernel; }
 
 int kami_version(void) { return (KAMI_VERSION_MAJOR << 16) | KAMI_VERSION_MINOR; }
+
+kami_status_t kami_set_grid_cap(int max_ctas) {
+  if (max_ctas < 0) return KAMI_ERROR_INVALID_VALUE;
+  g_grid_cap.store(max_ctas, std::memory_order_relaxed);
+  return KAMI_SUCCESS;
+}
 
 }  // extern "C"

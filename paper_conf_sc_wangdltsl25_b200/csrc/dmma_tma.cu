@@ -115,6 +115,7 @@ __device__ __forceinline__ void mma_steps(double (&c)[FM][FN][2], const double (
 template <int M, int N, int K, int P, int TEAMS, bool kUpd, bool kRot, bool kPtr = false>
 __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(const __grid_constant__ DmmaTmaParams prm) {
   using Cfg = DmmaTmaCfg<M, N, K, P, TEAMS>;
+  static_assert(TEAMS < 16, "named barrier ids 1 + team must stay within bar.sync's 0..15");
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-byte aligned base; pointer arithmetic on the __shared__ array keeps
   // the address space, so table reads compile to LDS rather than generic loads
@@ -266,6 +267,7 @@ kami_status_t launch(long long batch, const void* A, const void* B, void* C, cud
   long long grid = (long long)sms * per_sm;
   const long long need = (batch + TEAMS - 1) / TEAMS;
   if (grid > need) grid = need;
+  grid = apply_grid_cap(grid);
   fn<<<(unsigned)grid, Cfg::THREADS, Cfg::SMEM, stream>>>(prm);
   set_last_kernel(ptr ? (M == 64 ? "kami_dmma_tma_1d<64,ptr>" : M == 32 ? "kami_dmma_tma_1d<32,ptr>"
                                                                          : "kami_dmma_tma_1d<16,ptr>")
@@ -300,7 +302,7 @@ kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* 
   }
   if (m == 16 && n == 16 && k == 16) {
     if (cfg == 3) return launch<16, 16, 16, 2, 8, true>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,rot>", alpha, beta, Aa, Ba, Ca);
-    if (cfg == 1) return launch<16, 16, 16, 1, 16>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,p1>", alpha, beta, Aa, Ba, Ca);
+    if (cfg == 1) return launch<16, 16, 16, 1, 15>(batch, A, B, C, stream, "kami_dmma_tma_1d<16,p1>", alpha, beta, Aa, Ba, Ca);
     return launch<16, 16, 16, 2, 8>(batch, A, B, C, stream, "kami_dmma_tma_1d<16>", alpha, beta, Aa, Ba, Ca);
   }
   return KAMI_ERROR_NOT_SUPPORTED;

@@ -92,6 +92,13 @@ extern "C" kami_status_t kami_gemm_strided_batched_host(int m, int n, int k, int
   const char* hA = static_cast<const char*>(A);
   const char* hB = static_cast<const char*>(B);
   char* hC = static_cast<char*>(C);
+  // On any error below, earlier chunks' copies may still be running on the
+  // workspace streams against the caller's host buffers: drain both streams
+  // before returning, so the caller may free or reuse them.
+  auto fail = [&](kami_status_t code) {
+    for (int j = 0; j < 2; ++j) cudaStreamSynchronize(g_ws.st[j]);
+    return code;
+  };
   int64_t i = 0;
   for (int64_t e0 = 0; e0 < batch; e0 += chunk, ++i) {
     const int64_t ne = (batch - e0) < chunk ? (batch - e0) : chunk;
@@ -100,11 +107,14 @@ extern "C" kami_status_t kami_gemm_strided_batched_host(int m, int n, int k, int
     char* dA = static_cast<char*>(g_ws.buf[slot]);
     char* dB = dA + round_up((size_t)chunk * ea, 256);
     char* dC = dB + round_up((size_t)chunk * eb, 256);
-    if (cudaMemcpyAsync(dA, hA + e0 * ea, ne * ea, cudaMemcpyHostToDevice, s) != cudaSuccess) return KAMI_ERROR_CUDA;
-    if (cudaMemcpyAsync(dB, hB + e0 * eb, ne * eb, cudaMemcpyHostToDevice, s) != cudaSuccess) return KAMI_ERROR_CUDA;
+    if (cudaMemcpyAsync(dA, hA + e0 * ea, ne * ea, cudaMemcpyHostToDevice, s) != cudaSuccess)
+      return fail(KAMI_ERROR_CUDA);
+    if (cudaMemcpyAsync(dB, hB + e0 * eb, ne * eb, cudaMemcpyHostToDevice, s) != cudaSuccess)
+      return fail(KAMI_ERROR_CUDA);
     st = kami_gemm_strided_batched(m, n, k, ne, dtype, layout, dA, dB, dC, reinterpret_cast<kami_stream_t>(s));
-    if (st != KAMI_SUCCESS) return st;
-    if (cudaMemcpyAsync(hC + e0 * ec, dC, ne * ec, cudaMemcpyDeviceToHost, s) != cudaSuccess) return KAMI_ERROR_CUDA;
+    if (st != KAMI_SUCCESS) return fail(st);
+    if (cudaMemcpyAsync(hC + e0 * ec, dC, ne * ec, cudaMemcpyDeviceToHost, s) != cudaSuccess)
+      return fail(KAMI_ERROR_CUDA);
   }
   for (int j = 0; j < 2; ++j)
     if (cudaStreamSynchronize(g_ws.st[j]) != cudaSuccess) return KAMI_ERROR_CUDA;

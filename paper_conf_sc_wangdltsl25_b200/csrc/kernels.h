@@ -17,6 +17,12 @@ typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_
                                     CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 PFN_encodeTiled get_encode_tiled();
 void set_last_kernel(const char* name);
+// kami_set_grid_cap (tests): every persistent launcher clamps its grid to this (0 = no cap)
+int grid_cap();
+inline long long apply_grid_cap(long long grid) {
+  const int c = grid_cap();
+  return (c > 0 && grid > c) ? c : grid;
+}
 
 // ---------------------------------------------------------------- tcgen05
 struct Tc16Shape {

@@ -134,8 +134,8 @@ struct alignas(64) Tc16Params {
   CUtensorMap tmCw;                    // box (Wc, 32, 1, 1)
   uint32_t tx_tail, idesc_tail;
   CUtensorMap tmAt2, tmBt2, tmCt2;     // boxes (Wk, 64, 2), (Wn, Wk, n/Wn, 2), (Wc, 64, n/Wc, 2)
-  int m_tail;                          // m > 128, m % 128 != 0: the last m-tile uses tmAt / tmCt / tmCat
-  CUtensorMap tmAt, tmCt, tmCat;       // pointer arrays: boxes of m % 128 rows for the last m-tile
+  int m_tail;                          // m > 128, m % 128 != 0: the last m-tile uses tmAt / tmCat
+  CUtensorMap tmAt, tmCat;             // pointer arrays: boxes of m % 128 rows for the last m-tile
 };
 
 // Pointer arrays on TMA.  A tensor map cannot follow a pointer array, but all
@@ -756,8 +756,16 @@ __global__ void __launch_bounds__(threads_for(kIn), 1) kami_tc16_1d_kernel(const
       ptx::named_bar_sync(bar_id, kEpiThreads);
       if constexpr (kPtr) {
         if (cstore) {
-          ptx::tma_store_5d(p.m_tail && mt == p.m_tiles - 1 ? &p.tmCt : &p.tmC, smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes + lane * p.c_entry, 0,
-                            mt * 128, 0, clo, chi);
+          uint8_t* cent = smem + p.c_off + (wg * p.c_bufs + cb) * p.c_buf_bytes + lane * p.c_entry;
+          if (p.m_tail && mt == p.m_tiles - 1) {
+            // last m-tile of m > 128, m % 128 != 0: the staging tile keeps the
+            // full tile's atom stride (128 rows per atom) while a box of m % 128
+            // rows reads its smem densely, so store one 64-column atom at a time
+            for (int at = 0; at < p.n / p.Wc; ++at)
+              ptx::tma_store_5d(&p.tmCat, cent + (uint32_t)at * atom_stride, 0, mt * 128, at, clo, chi);
+          } else {
+            ptx::tma_store_5d(&p.tmC, cent, 0, mt * 128, 0, clo, chi);
+          }
           ptx::bulk_commit();
         }
       } else if (leader) {
@@ -1215,11 +1223,13 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
       cuuint64_t strides[4] = {(cuuint64_t)n * eso, (cuuint64_t)wc_b, 16, vstride_hi};
       cuuint32_t box[5] = {(cuuint32_t)s.Wc, rows, (cuuint32_t)(n / s.Wc), 1, 1};
       cuuint32_t es[5] = {1, 1, 1, 1, 1};
-      if (enc(t ? &p.tmCt : &p.tmC, dto, 5, vbase, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
-              swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      if (!t && enc(&p.tmC, dto, 5, vbase, dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                    swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
         return KAMI_ERROR_NOT_SUPPORTED;
       cuuint32_t box1[5] = {(cuuint32_t)s.Wc, rows, 1, 1, 1};
-      if (p.split_store && enc(t ? &p.tmCat : &p.tmCa, dto, 5, vbase, dims, strides, box1, es,
+      // per-atom maps: split stores, and every tail m-tile (its staging keeps
+      // the full tile's atom stride, so it is stored atom by atom)
+      if ((p.split_store || t) && enc(t ? &p.tmCat : &p.tmCa, dto, 5, vbase, dims, strides, box1, es,
                                CU_TENSOR_MAP_INTERLEAVE_NONE, swz_mode_for(wc_b), CU_TENSOR_MAP_L2_PROMOTION_NONE,
                                CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
         return KAMI_ERROR_NOT_SUPPORTED;
@@ -1278,6 +1288,7 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
   }
   if (tc_tune().grid > 0 && tc_tune().grid < p.units) grid = tc_tune().grid;  // knob overrides (A/B)
   if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;
+  grid = apply_grid_cap(grid);
   const size_t smem = s.smem_bytes;
   const unsigned g = (unsigned)grid;
   switch (in_kind) {

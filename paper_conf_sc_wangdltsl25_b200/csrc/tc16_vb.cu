@@ -540,6 +540,7 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   // (uniform sizes with a short last m-tile, m % 128 != 0, likewise)
   if (p.mtiles > 1 && (p.dm || max_m % 128 != 0))
     while (grid > 1 && std::gcd(grid, (long long)p.mtiles) != 1) --grid;
+  grid = apply_grid_cap(grid);
   fn<<<(unsigned)grid, kVbThreads, smem, stream>>>(p);
   set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
                         : (bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>"));

@@ -764,6 +764,7 @@ kami_status_t warp_ca_launch(int m, int n, int k, long long batch, kami_dtype_t 
   long long grid = reps > 1 ? ctas_needed : (long long)sms * per_sm;
   if (grid > ctas_needed) grid = ctas_needed;
   if (grid < 1) grid = 1;
+  if (reps == 1) grid = apply_grid_cap(grid);  // (block-level mode: one CTA per team set)
   static const int prefetch = [] {
     const char* e = getenv("KAMI_L2_PREFETCH");
     return e ? atoi(e) : 1;

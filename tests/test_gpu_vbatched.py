@@ -55,7 +55,8 @@ def test_pointer_array_all_sizes(dtype, shape):
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 @pytest.mark.parametrize("shape", [(64, 64, 64), (48, 80, 40), (256, 256, 16), (192, 128, 64), (16, 192, 16),
                                    (64, 64, 8), (64, 64, 40), (128, 128, 200), (32, 64, 24),
-                                   (192, 32, 16), (144, 16, 32)])  # m-tails with U > 1 sub-tiles
+                                   (192, 32, 16), (144, 16, 32),  # m-tails with U > 1 sub-tiles
+                                   (192, 128, 16), (160, 96, 32), (144, 48, 64)])  # multi-atom m-tails
 def test_pointer_array_scattered_addresses(dtype, shape):
     """Entries at arbitrary 16-byte-aligned addresses: inside one buffer at offsets that are
     not multiples of the entry size, and in separate allocations more than 2^28 bytes apart
