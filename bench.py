@@ -79,11 +79,25 @@ def load_peaks():
     return 6650.0, 1590.0, "fallback (B200_PROFILING.md)"
 
 
+_FP64_PEAK = {}
+
+
 def fp64_peak_tflops():
-    """FP64 DMMA roofline denominator.  No measured figure exists in
-    MEASURED_PEAKS.json; DESIGN.md derives 37 TF/s (B200 datasheet FP64 tensor
-    ~ the DMMA issue rate x 148 SMs x clock), stated as 'nominal'."""
-    return 37.0
+    """FP64 DMMA roofline denominator, MEASURED on this device by the library's
+    probe (kami_probe_dmma_peak: an mma.sync.m8n8k4.f64 loop on every SM for
+    >= 300 ms; MEASURED_PEAKS.json has no FP64 figure).  The sustained rate
+    (second half of the run, clock under the power cap) is the denominator for
+    kernels timed inside a long step; falls back to the 37 TF/s nominal figure
+    (148 SMs x 1965 MHz x the DMMA issue rate) if the probe cannot run."""
+    if not _FP64_PEAK:
+        try:
+            import paper_conf_sc_wangdltsl25_b200 as kami
+
+            burst, sus = kami.probe_dmma_peak(300.0)
+            _FP64_PEAK.update(value=sus, burst=burst, source="measured (kami_probe_dmma_peak, sustained)")
+        except Exception as e:  # pragma: no cover
+            _FP64_PEAK.update(value=37.0, burst=None, source=f"nominal 37 TF/s (probe failed: {e})")
+    return _FP64_PEAK["value"]
 
 
 class ClockSampler:
@@ -141,8 +155,27 @@ class ClockSampler:
                 "gpu_temp_c": med(10), "mem_temp_c": med(11)}
 
 
+def host_cpu_info():
+    """CPU model, logical CPUs (nproc) and the affinity mask size (the threads
+    the oracle may actually use) -- BASELINE.md 4 / SURVEY.md 8(d)."""
+    model = None
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                model = line.split(":", 1)[1].strip()
+                break
+    except OSError:
+        pass
+    try:
+        aff = len(os.sched_getaffinity(0))
+    except AttributeError:  # pragma: no cover
+        aff = os.cpu_count()
+    return {"cpu_model": model, "nproc": os.cpu_count(), "affinity": aff}
+
+
 def cpu_baseline(dtype, m, n, k, target_s=12.0, max_entries=None):
-    """Time the oracle (as it stands) on this host's cores on a bounded sample."""
+    """Time the oracle (as it stands) on this host's cores on a bounded sample,
+    plus a 1-thread rate on a smaller sample (per-core baseline)."""
     import kami_inputs as ki
     import oracle
 
@@ -164,9 +197,18 @@ def cpu_baseline(dtype, m, n, k, target_s=12.0, max_entries=None):
     oracle.gemm(m, n, k, n_entries, dtype, "row", a, b, nthreads=cores)
     dt = time.perf_counter() - t0
     tflops = 2.0 * per_entry_mac * n_entries / dt / 1e12
-    return {"value": tflops, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
-            "sample": f"first {n_entries} entries of the workload (seed 0), FP64 triple loop, {dt:.1f} s",
-            "seconds": dt, "entries": n_entries}
+    # one thread on ~1/8 of the time budget
+    n1 = max(1, min(n_entries, int(n_entries / cores * (target_s / 8) / max(dt, 1e-6))))
+    t0 = time.perf_counter()
+    oracle.gemm(m, n, k, n1, dtype, "row", a[: n1 * m * k], b[: n1 * k * n], nthreads=1)
+    dt1 = time.perf_counter() - t0
+    out = {"value": tflops, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
+           "sample": f"first {n_entries} entries of the workload (seed 0), FP64 triple loop, {dt:.1f} s",
+           "seconds": dt, "entries": n_entries,
+           "one_thread": {"value": 2.0 * per_entry_mac * n1 / dt1 / 1e12, "unit": "TFLOP/s", "entries": n1,
+                          "seconds": dt1}}
+    out.update(host_cpu_info())
+    return out
 
 
 PAPER_CONTEXT = {
@@ -234,8 +276,9 @@ def run_reference(args):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
         "scaling": "weak", "vs_baseline": None, "dtype": dtype, "data": "synthetic",
         "config": dict(workload_config(args, dtype, m, n, k, batch, cfg), timing="host wall clock"),
-        "cpu_baseline": {"value": value, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{sample} entries of the workload per step (of {batch}), FP64 triple loop"},
+        "cpu_baseline": dict({"value": value, "unit": "TFLOP/s", "cores": cores, "kind": "oracle",
+                              "sample": f"{sample} entries of the workload per step (of {batch}), FP64 triple loop"},
+                             **host_cpu_info()),
         "e2e": {"value": value, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -244,7 +287,8 @@ def run_reference(args):
 def workload_config(args, dtype, m, n, k, batch, cfg):
     return {"workload": f"{dtype} strided-batched GEMM m={m} n={n} k={k} batch={batch}/GPU row-major "
                         f"(BASELINE.json configs[{cfg}])",
-            "m": m, "n": n, "k": k, "batch_per_gpu": batch, "global_batch": batch * args.gpus,
+            "m": m, "n": n, "k": k, "batch_per_gpu": batch, "global_batch": getattr(args, "global_batch", batch),
+            "scaling": getattr(args, "scaling", "weak"),
             "layout": "row", "algo": args.algo, "p": args.p, "inputs": "unif [-1,1) RNE to dtype, counter-based SplitMix64",
             "l2": "inputs larger than L2 (126 MB)" if batch * op_bytes(dtype, m, n, k) >= 126e6
                   else f"inputs rotated over {int(-(-3 * 126e6 // (batch * op_bytes(dtype, m, n, k))))} distinct "
@@ -267,6 +311,8 @@ def main():
     ap.add_argument("--p", type=int, default=0, help="warps per entry (0 = planner default)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="weak: the workload batch per GPU; strong: the workload batch split over the GPUs")
     ap.add_argument("--timing", default="graph", choices=["graph", "b2b", "events"],
                     help="graph: K steps in one CUDA graph between two events; b2b: K launches back to back "
                          "between two events; events: one event pair per launch, summed")
@@ -282,8 +328,20 @@ def main():
     import kami_inputs as ki
     import paper_conf_sc_wangdltsl25_b200 as kami
 
+    from paper_conf_sc_wangdltsl25_b200 import dist as kdist
+
     world, rank, local = dist_init()
-    dtype, m, n, k, batch, cfg = parse_workload(args.workload)
+    dtype, m, n, k, wl_batch, cfg = parse_workload(args.workload)
+    # this rank's contiguous slice of the global batch (dist.py):
+    # weak scaling = the workload batch per GPU, strong = the workload batch in total
+    if args.scaling == "strong":
+        lo, hi = kdist.shard_range(wl_batch, rank, world)
+        global_batch = wl_batch
+    else:
+        lo, hi = kdist.weak_range(wl_batch, rank)
+        global_batch = wl_batch * world
+    batch = hi - lo
+    args.global_batch = global_batch
     update = "upd" in args.workload
     esi, eso = ES_IN.get(dtype, 2), ES_OUT.get(dtype, 2)
     alg_bytes = batch * op_bytes(dtype, m, n, k, update)
@@ -294,7 +352,7 @@ def main():
     R = 1 if alg_bytes >= 126e6 else int(-(-3 * 126e6 // alg_bytes))
     sets = []
     for r_ in range(R):
-        entry0 = (rank * R + r_) * batch
+        entry0 = lo + r_ * global_batch  # set 0 = this rank's entries of the global batch
         A, B = ki.operands(m, n, k, batch, dtype, "unif", seed=0, entry0=entry0, device="cuda")
         C = torch.zeros(batch * m * n, dtype=ki.TORCH_DTYPES[ki.OUT_DTYPE[dtype]], device="cuda")
         sets.append((A, B, C))
@@ -374,18 +432,16 @@ def main():
     else:
         t_ms = ev0.elapsed_time(ev1)  # device time of the K timed steps
 
-    # checksum of the last output (sampled verification happens in tests/)
-    csum = float(C.double().sum().item())
+    # world-size-invariant checksum of this rank's outputs (set 0 = its entries
+    # [lo, hi) of the global batch; parity itself is checked in tests/), then
+    # the only collective: an all_gather of the tiny per-rank record (dist.py)
+    csum = kdist.position_checksum(C, lo, batch, m * n)
     coll_dev = "cpu" if world > 1 and dist.get_backend() == "gloo" else "cuda"
-    stats = torch.tensor([t_ms, csum, float(batch)], dtype=torch.float64, device=coll_dev)
-    if world > 1:
-        gathered = [torch.zeros_like(stats) for _ in range(world)]
-        dist.all_gather(gathered, stats)  # the only collective: per-rank stats over NCCL
-        allst = torch.stack(gathered).cpu()
-    else:
-        allst = stats.cpu().unsqueeze(0)
-    t_max_ms = float(allst[:, 0].max())
-    total_entries = float(allst[:, 2].sum())
+    recs = kdist.gather_records(kdist.RankRecord(time_ms=t_ms, checksum=float(csum), entries=float(batch)),
+                                device=coll_dev)
+    agg = kdist.aggregate(recs)
+    t_max_ms = agg["time_ms"]
+    total_entries = agg["entries"]
 
     # end-to-end: the C-ABI host entry point, host<->device copies inside the timed region
     e2e = None
@@ -418,7 +474,8 @@ def main():
     value = flops * total_entries / batch * args.steps / (t_max_ms * 1e-3) / 1e12
     avg_launch_s = (t_ms / args.steps) * 1e-3
     achieved_gbs = alg_bytes / avg_launch_s / 1e9
-    tensor_peak = {"f64": fp64_peak_tflops(), "tf32": 1125.0, "e4m3": 4500.0, "e5m2": 4500.0}.get(dtype, 2250.0)
+    tensor_peak = fp64_peak_tflops() if dtype == "f64" else {"tf32": 1125.0, "e4m3": 4500.0, "e5m2": 4500.0}.get(
+        dtype, 2250.0)
     roof_tf = min(hbm * 1e9 * flops / alg_bytes, tensor_peak * 1e12) / 1e12
     bound = "hbm"
     if dtype == "f64" and fp64_peak_tflops() * 1e12 < hbm * 1e9 * flops / alg_bytes:
@@ -429,25 +486,29 @@ def main():
     else:
         ach = flops / avg_launch_s / 1e12
         roofline = {"bound": "tensor", "achieved": ach, "peak": fp64_peak_tflops(), "unit": "TFLOP/s",
-                    "frac": ach / fp64_peak_tflops(), "peak_source": "nominal FP64 DMMA (DESIGN.md)"}
+                    "frac": ach / fp64_peak_tflops(), "peak_source": _FP64_PEAK["source"],
+                    "peak_burst": _FP64_PEAK["burst"]}
     roofline["traffic"] = traffic_from_profiles(args.workload)
     roofline["kernel"] = kernel
     roofline["roofline_tflops_per_gpu"] = roof_tf
     roofline["frac_of_roofline_tflops"] = (value / world) / roof_tf
     line = {
         "metric": METRIC, "value": value, "unit": "TFLOP/s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": t_max_ms / args.steps, "higher_is_better": True, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": t_max_ms / args.steps, "higher_is_better": True,
+        "scaling": args.scaling,
         "vs_baseline": None, "dtype": dtype, "data": "synthetic",
         "config": workload_config(args, dtype, m, n, k, batch, cfg),
         "roofline": roofline,
         "gpu_launches": args.steps,
         "clocks": sampler.summary(),
-        "checksum": float(allst[:, 1].sum()),
+        # position-weighted checksum of every output bit pattern, exactly additive
+        # over shards: identical for any world size / scaling mode on the same
+        # global entries (dist.position_checksum)
+        "checksum": agg["position_checksum"],
     }
     if world > 1:  # per-rank device times (the job time is their max)
-        tms = [float(x) for x in allst[:, 0]]
-        line["ranks"] = {"time_ms": tms, "spread": max(tms) / min(tms) if min(tms) > 0 else None,
-                         "checksums": [float(x) for x in allst[:, 1]]}
+        line["ranks"] = {"time_ms": [r.time_ms for r in recs], "spread": agg["spread"],
+                         "entries": [int(r.entries) for r in recs], "checksums": [int(r.checksum) for r in recs]}
     if e2e:
         line["e2e"] = e2e
     # the paper's own numbers, other hardware: context only (vs_baseline stays null)

@@ -79,7 +79,19 @@ typedef enum {
   KAMI_ALGO_2D = 2,
   KAMI_ALGO_3D = 3,
   KAMI_ALGO_NONCA = 4,
-  KAMI_ALGO_1D_TMA = 5
+  KAMI_ALGO_1D_TMA = 5,
+  /* 16-bit only, tcgen05 with the LOCAL operand resident in tensor memory
+   * (Table 1: local storage never passes through shared
+   * memory): A is loaded global -> registers -> TMEM, only B is broadcast
+   * through shared memory.  m, n multiples of 16 in
+   * [16, 128], k a multiple of 8 in [8, 256]; NOT_SUPPORTED otherwise. */
+  KAMI_ALGO_1D_TMEM = 6,
+  /* as 1D_TMEM with the k-chunks split into cbrt(p) = 2 k-layers (Alg. 3,
+   * L338-380), each layer's A rows written by its own loader warpgroup, and
+   * the layer partials summed inside ONE TMEM accumulator (the Alg. 3
+   * reduction costs no shared-memory traffic).  Needs every k-chunk to hold
+   * an even number of K = 16 steps (k a multiple of 32 in practice). */
+  KAMI_ALGO_3D_TMEM = 7
 } kami_algo_t;
 
 /* Opaque CUDA stream; binary compatible with cudaStream_t. */
@@ -185,7 +197,8 @@ kami_status_t kami_gemm_block_level(int m, int n, int k, int64_t batch, kami_dty
 typedef struct {
   kami_algo_t algo;      /* chosen schedule                                 */
   int p;                 /* warps (or tensor-core sub-partitions) per entry */
-  int kernel;            /* 0 = tcgen05 16-bit, 1 = warp-level DMMA/HMMA, 2 = FP64 DMMA with TMA broadcast */
+  int kernel;            /* 0 = tcgen05 16-bit (SS), 1 = warp-level DMMA/HMMA, 2 = FP64 DMMA with TMA
+                            broadcast, 3 = tcgen05 16-bit with A resident in TMEM (TS) */
   int entries_per_cta;   /* batch entries a CTA keeps in flight             */
   int stages;            /* shared-memory pipeline depth                    */
   int kslice_regs_pct;   /* share of A/B kept resident (Sec. 4.7)           */

@@ -24,7 +24,7 @@ SO_PATH = os.environ.get("KAMI_LIB") or os.path.join(_HERE, "libkami.so")
 
 DTYPE = {"f16": 0, "bf16": 1, "f64": 2, "tf32": 3, "e4m3": 4, "e5m2": 5}
 LAYOUT = {"row": 0, "col": 1}
-ALGO = {"auto": 0, "1d": 1, "2d": 2, "3d": 3, "nonca": 4, "1d_tma": 5}
+ALGO = {"auto": 0, "1d": 1, "2d": 2, "3d": 3, "nonca": 4, "1d_tma": 5, "1d_tmem": 6, "3d_tmem": 7}
 STATUS = {0: "KAMI_SUCCESS", 1: "KAMI_ERROR_INVALID_VALUE", 2: "KAMI_ERROR_NOT_SUPPORTED",
           3: "KAMI_ERROR_MISALIGNED", 4: "KAMI_ERROR_CUDA"}
 
@@ -235,7 +235,7 @@ def plan(m, n, k, dtype, layout="row", algo="auto", p=0) -> dict:
     _check(lib().kami_plan(m, n, k, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
                            _enum(ALGO, algo, "algo"), p, ctypes.byref(out)), "kami_plan")
     inv = {v: k for k, v in ALGO.items()}
-    return {"algo": inv[out.algo], "p": out.p, "kernel": {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma"}[out.kernel],
+    return {"algo": inv[out.algo], "p": out.p, "kernel": {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma", 3: "tcgen05_ts"}[out.kernel],
             "entries_per_cta": out.entries_per_cta, "stages": out.stages, "kslice_regs_pct": out.kslice_regs_pct,
             "t_all_cycles": out.t_all_cycles}
 

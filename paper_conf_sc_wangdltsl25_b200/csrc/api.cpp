@@ -63,7 +63,7 @@ kami_status_t check_common(int m, int n, int k, int64_t batch, int dtype, int la
   if (m <= 0 || n <= 0 || k <= 0 || batch < 0) return KAMI_ERROR_INVALID_VALUE;
   if (dtype < KAMI_DTYPE_F16 || dtype > KAMI_DTYPE_E5M2) return KAMI_ERROR_INVALID_VALUE;
   if (layout != KAMI_ROW_MAJOR && layout != KAMI_COL_MAJOR) return KAMI_ERROR_INVALID_VALUE;
-  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_1D_TMA) return KAMI_ERROR_INVALID_VALUE;
+  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_3D_TMEM) return KAMI_ERROR_INVALID_VALUE;
   return check_sizes(m, n, k, (kami_dtype_t)dtype);
 }
 
@@ -128,6 +128,11 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
+  if (plan.kernel == 3) {  // tcgen05 with A resident in TMEM (strided C = A B only)
+    if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
+    return tc16_ts_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, plan.algo == KAMI_ALGO_3D_TMEM ? 2 : 1,
+                          rp.A, rp.B, C, stream);
+  }
   if (plan.kernel == 1 && update && is16(dtype) && algo == KAMI_ALGO_AUTO && !Ca)
     plan.kernel = 0;  // the update form (C read) exists on tcgen05 only
   if (plan.kernel == 0) {
@@ -248,7 +253,7 @@ kami_status_t kami_gemm_block_level(int m, int n, int k, int64_t batch, kami_dty
                                     int64_t* cycles, kami_stream_t stream) {
   kami_status_t st = check_common(m, n, k, batch, dtype, layout, algo);
   if (st != KAMI_SUCCESS) return st;
-  if (p < 0 || reps < 1 || algo == KAMI_ALGO_1D_TMA) return KAMI_ERROR_INVALID_VALUE;
+  if (p < 0 || reps < 1 || algo == KAMI_ALGO_1D_TMA || algo >= KAMI_ALGO_1D_TMEM) return KAMI_ERROR_INVALID_VALUE;
   if (batch == 0) return KAMI_SUCCESS;
   if (!A || !B || !C) return KAMI_ERROR_INVALID_VALUE;
   if (!aligned16(A) || !aligned16(B) || !aligned16(C)) return KAMI_ERROR_MISALIGNED;

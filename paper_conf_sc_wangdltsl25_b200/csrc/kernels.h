@@ -50,6 +50,19 @@ kami_status_t tc16_launch_kind(int m, int n, int k, long long batch, int in_kind
                                const void* const* Aa = nullptr, const void* const* Ba = nullptr,
                                void* const* Ca = nullptr);
 
+// ------------------------------- tcgen05 with A resident in TMEM (tc16_ts.cu)
+struct TsShape {
+  int G, N_mma, Wk, Wn, Wc, k_chunks, ksteps_full, ksteps_last;
+  int layers, item_cols, slot_cols, a_slots, loader_wgs, acc_cols;
+  uint32_t stage_bytes, c_buf_bytes;
+  int c_bufs, stages;
+  uint32_t smem_bytes;
+};
+// layers: 1 = KAMI_ALGO_1D_TMEM, 2 = KAMI_ALGO_3D_TMEM
+kami_status_t tc16_ts_plan(int m, int n, int k, int layers, TsShape* s);
+kami_status_t tc16_ts_launch(int m, int n, int k, long long batch, bool bf16, int layers, const void* A,
+                             const void* B, void* C, cudaStream_t stream);
+
 // ------------------------------------------------ warp-level CA (literal KAMI)
 // algo: 1 = 1D, 2 = 2D, 3 = 3D, 4 = non-CA tiled.  dtype: KAMI_DTYPE_*.
 // Entry pointers: if A_arr != nullptr they are device arrays of per-entry

@@ -131,6 +131,23 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
     *out = r;
     return KAMI_SUCCESS;
   }
+  // tcgen05 with the local operand (A) resident in TMEM: explicit request
+  if (algo == KAMI_ALGO_1D_TMEM || algo == KAMI_ALGO_3D_TMEM) {
+    if ((dtype != KAMI_DTYPE_F16 && dtype != KAMI_DTYPE_BF16) || pointer_array || (p != 0 && p != 4 && p != 8))
+      return KAMI_ERROR_NOT_SUPPORTED;
+    TsShape ts;
+    kami_status_t st = tc16_ts_plan(m, n, k, algo == KAMI_ALGO_3D_TMEM ? 2 : 1, &ts);
+    if (st != KAMI_SUCCESS) return st == KAMI_ERROR_INVALID_VALUE ? KAMI_ERROR_NOT_SUPPORTED : st;
+    r.algo = algo;
+    r.p = algo == KAMI_ALGO_3D_TMEM ? 8 : 4;
+    r.kernel = 3;
+    r.entries_per_cta = ts.G * ts.stages;
+    r.stages = ts.stages;
+    r.kslice_regs_pct = 0;
+    r.t_all_cycles = b200_cost(algo == KAMI_ALGO_3D_TMEM ? 3 : 1, m, n, k, algo == KAMI_ALGO_3D_TMEM ? 8 : 4, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
   // FP64 1D with the broadcast operand fed by TMA (dmma_tma.cu; pointer arrays
   // through an address-space view of each entry)
   const bool tma_ok = !is16 && dmma_tma_supported(m, n, k);

@@ -74,3 +74,62 @@ def test_gloo_two_ranks_gather_and_invariance():
     assert torch.equal(got, A_full.view(torch.int16))
     tot = float(A_full.double().sum() + B_full.double().sum())
     assert abs(agg["checksum"] - tot) < 1e-9
+
+
+def test_position_checksum_additive_over_shards():
+    """The bench checksum is exactly additive over any contiguous sharding
+    (world-size invariance), and sensitive to a changed or moved entry."""
+    B, m, n = 37, 8, 16
+    C = ki.draw(9, 0, 0, B, m, n, "f16", "unif")
+    whole = kdist.position_checksum(C, 0, B, m * n)
+    for W in (1, 2, 3, 4, 8):
+        parts = []
+        for r in range(W):
+            lo, hi = kdist.shard_range(B, r, W)
+            parts.append(kdist.position_checksum(C.view(B, -1)[lo:hi], lo, hi - lo, m * n))
+        assert kdist.combine_checksums(parts) == whole
+    C2 = C.clone().view(B, -1)
+    C2[5, 3] = C2[5, 3] + 1  # one output changed
+    assert kdist.position_checksum(C2, 0, B, m * n) != whole
+    C3 = C.clone().view(B, -1)
+    C3[[4, 9]] = C3[[9, 4]]  # two entries swapped
+    assert kdist.position_checksum(C3, 0, B, m * n) != whole
+    for dt in ("f64", "f32"):
+        X = ki.draw(9, 0, 0, B, m, n, dt, "unif")
+        a = kdist.position_checksum(X, 0, B, m * n)
+        b = kdist.combine_checksums([kdist.position_checksum(X.view(B, -1)[:20], 0, 20, m * n),
+                                     kdist.position_checksum(X.view(B, -1)[20:], 20, B - 20, m * n)])
+        assert a == b
+
+
+def _bench_worker(rank, world, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        # the bench's per-rank logic, CPU stand-in for the GPU output: strong
+        # scaling shards the global batch, every rank checksums its own shard
+        B, m, n = 21, 4, 8
+        lo, hi = kdist.shard_range(B, rank, world)
+        C = ki.draw(4, 1, lo, hi - lo, m, n, "f16", "unif")
+        rec = kdist.RankRecord(time_ms=1.0 + rank, checksum=float(kdist.position_checksum(C, lo, hi - lo, m * n)),
+                               entries=float(hi - lo))
+        agg = kdist.aggregate(kdist.gather_records(rec))
+        q.put((rank, agg["position_checksum"], agg["entries"], agg["time_ms"]))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_two_ranks_strong_scaling_checksum_matches_single_process():
+    world, port = 2, _free_port()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_bench_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in ps:
+        p.start()
+    res = sorted(q.get(timeout=120) for _ in range(world))
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    single = kdist.position_checksum(ki.draw(4, 1, 0, 21, 4, 8, "f16", "unif"), 0, 21, 32)
+    assert res[0][1] == res[1][1] == single
+    assert res[0][2] == 21 and res[0][3] == 2.0
