@@ -198,7 +198,8 @@ typedef struct {
   kami_algo_t algo;      /* chosen schedule                                 */
   int p;                 /* warps (or tensor-core sub-partitions) per entry */
   int kernel;            /* 0 = tcgen05 16-bit (SS), 1 = warp-level DMMA/HMMA, 2 = FP64 DMMA with TMA
-                            broadcast, 3 = tcgen05 16-bit with A resident in TMEM (TS) */
+                            broadcast, 3 = tcgen05 16-bit with A resident in TMEM (TS), 4 = FP64 DMMA
+                            for the whole size grid (k-sliced, register residency ratio) */
   int entries_per_cta;   /* batch entries a CTA keeps in flight             */
   int stages;            /* shared-memory pipeline depth                    */
   int kslice_regs_pct;   /* share of A/B kept resident (Sec. 4.7)           */

@@ -235,7 +235,7 @@ def plan(m, n, k, dtype, layout="row", algo="auto", p=0) -> dict:
     _check(lib().kami_plan(m, n, k, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
                            _enum(ALGO, algo, "algo"), p, ctypes.byref(out)), "kami_plan")
     inv = {v: k for k, v in ALGO.items()}
-    return {"algo": inv[out.algo], "p": out.p, "kernel": {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma", 3: "tcgen05_ts"}[out.kernel],
+    return {"algo": inv[out.algo], "p": out.p, "kernel": {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma", 3: "tcgen05_ts", 4: "dmma_gen"}[out.kernel],
             "entries_per_cta": out.entries_per_cta, "stages": out.stages, "kslice_regs_pct": out.kslice_regs_pct,
             "t_all_cycles": out.t_all_cycles}
 

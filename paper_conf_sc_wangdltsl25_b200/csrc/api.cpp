@@ -54,9 +54,8 @@ kami_status_t check_sizes(int m, int n, int k, kami_dtype_t dtype) {
   if (dtype == KAMI_DTYPE_TF32) return (m % 16 || n % 16 || k % 4) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
   if (dtype == KAMI_DTYPE_E4M3 || dtype == KAMI_DTYPE_E5M2)
     return (m % 32 || n % 32 || k % 16) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
-  // FP64: the register-resident DMMA family is instantiated for these orders
-  if (m == n && n == k && (m == 8 || m == 16 || m == 32 || m == 64)) return KAMI_SUCCESS;
-  return KAMI_ERROR_NOT_SUPPORTED;
+  // FP64: multiples of 8 in [8, 256] (dmma_gen.cu covers the whole grid)
+  return (m % 8 || n % 8 || k % 8) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
 }
 
 kami_status_t check_common(int m, int n, int k, int64_t batch, int dtype, int layout, int algo) {
@@ -128,6 +127,10 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
+  if (plan.kernel == 4) {  // FP64 general sizes: k-sliced DMMA with a residency ratio (strided C = A B)
+    if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
+    return dmma_gen_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream);
+  }
   if (plan.kernel == 3) {  // tcgen05 with A resident in TMEM (strided C = A B only)
     if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
     return tc16_ts_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, plan.algo == KAMI_ALGO_3D_TMEM ? 2 : 1,

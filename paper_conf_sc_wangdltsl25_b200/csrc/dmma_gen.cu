@@ -1,0 +1,266 @@
+// dmma_gen.cu -- FP64 batched GEMM for the whole FP64 size grid (m, n, k
+// multiples of 8 in [8, 256], non-square included): KAMI-1D on the DMMA path
+// with k-slicing and a register / shared-memory RESIDENCY RATIO (PAPER.md
+// Sec. 4.7 "when the matrix order grows ... a preset fraction of the
+// local tile stays in registers and the rest is parked in shared memory";
+// Sec. 5.2.5: the best ratio depends on the order -- parking 50 % at
+// order 128 gives 1.34x, parking 75 % gives 0.71x).  SURVEY.md 8(a) row a7.
+//
+// Schedule (as dmma_tma.cu, on C^T = B^T A^T): a team of P = 4 warps owns one
+// unit = (entry, 64-column block of C).  Warp w holds its column slice
+// B_w = B[:, nb 64 + 16 w : +16] -- the LOCAL operand -- for the whole unit:
+//   k-steps [0, rs)  resident in registers (DMMA B fragments),
+//   k-steps [rs, ks) parked in the warp's private shared-memory slab (written
+//                    once per unit in fragment order, so every read is one
+//                    conflict-free LDS.64 per lane),
+// with rs = ratio * ks (ks = k / 4 DMMA k-steps; at most kRK resident).  A is
+// the broadcast operand: TM-row blocks of A (all of k) arrive by TMA in the
+// 128-byte swizzled layout (double-buffered per team, the next block's copy
+// overlaps the current block's MMAs) and all four warps read their A
+// fragments from there.  C_w blocks (TM x 16) accumulate in registers and are
+// stored straight from the fragments.  Every shape is one kernel; m, n and
+// k tails are TMA zero-fill (A) and per-fragment guards (B, C).  A's k range
+// is cut into swizzle chunks of 16 doubles (128-byte swizzle) when k % 16 == 0
+// and of 8 doubles (64-byte swizzle) otherwise, so a box never reaches past
+// its row.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdlib>
+#include <cstring>
+
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace kami {
+namespace {
+
+constexpr int kGP = 4;    // warps per team
+constexpr int kGFN = 2;   // 8-wide n-fragments per warp (16 columns)
+constexpr int kGNB = kGP * kGFN * 8;  // 64 columns per unit
+constexpr int kGTM = 32;  // A / C rows per block
+constexpr int kGFM = kGTM / 8;
+constexpr int kRK = 32;   // max resident k-steps (32 x 2 doubles = 128 registers)
+
+struct DmmaGenParams {
+  CUtensorMap tmA;  // 4-D (CE, m, k/CE, batch), box (CE, TM, k/CE, 1), CE = 16 (SW128) or 8 (SW64) doubles
+  const double* B;
+  double* C;
+  long long batch, units;
+  int m, n, k, ks, rs, nblocks, mblocks, kch;
+  int ce_shift;       // log2 of the chunk width in doubles (4: 128-byte rows, 3: 64-byte rows)
+  uint32_t swz_bits;  // 3 (SW128) or 2 (SW64)
+  uint32_t a_block_bytes, park_bytes;  // per team buffer / per warp slab
+  int teams;
+};
+
+__global__ void __launch_bounds__(kGP * 32 * 2, 1) kami_dmma_gen_kernel(const __grid_constant__ DmmaGenParams p) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int team = warp / kGP, w = warp % kGP;
+  const int g = lane >> 2, t = lane & 3;
+  // per team: A double buffer, then the four warps' parked slabs; barriers at the end
+  const uint32_t team_bytes = 2 * p.a_block_bytes + kGP * p.park_bytes;
+  uint8_t* tbase = smem + team * team_bytes;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + p.teams * team_bytes) + team * 2;
+  if (threadIdx.x == 0) {
+    ptx::prefetch_tmap(&p.tmA);
+    for (int i = 0; i < 2 * p.teams; ++i)
+      ptx::mbar_init(reinterpret_cast<uint64_t*>(smem + p.teams * team_bytes) + i, 1);
+    ptx::fence_mbar_init();
+    ptx::fence_proxy_async_smem();
+  }
+  __syncthreads();
+  if (team >= p.teams) return;
+  const long long nteams = (long long)gridDim.x * p.teams;
+  const long long first = (long long)blockIdx.x * p.teams + team;
+  const bool issuer = (w == 0 && lane == 0);
+  const uint32_t bar = 1 + team;
+  const uint32_t park = ptx::smem_u32(tbase + 2 * p.a_block_bytes + w * p.park_bytes);
+  // the team's block sequence: units u = first, first + nteams, ...; m-blocks 0.. of each
+  auto issue = [&](long long u, int mb, int s) {
+    const long long e = u / p.nblocks;
+    ptx::mbar_arrive_expect_tx(&full[s], p.a_block_bytes);
+    ptx::tma_load_4d(tbase + s * p.a_block_bytes, &p.tmA, &full[s], 0, mb * kGTM, 0, (int)e);
+  };
+  // prologue: the first two blocks
+  long long pu = first;
+  int pmb = 0;
+  if (issuer) {
+    for (int s = 0; s < 2 && pu < p.units; ++s) {
+      issue(pu, pmb, s);
+      if (++pmb == p.mblocks) {
+        pmb = 0;
+        pu += nteams;
+      }
+    }
+  }
+  double b[kRK][kGFN];
+  uint32_t it = 0;
+  for (long long u = first; u < p.units; u += nteams) {
+    const long long e = u / p.nblocks;
+    const int nb = (int)(u - e * p.nblocks);
+    const int col0 = nb * kGNB + w * (kGFN * 8);
+    const double* Bg = p.B + e * (long long)p.k * p.n;
+    // GMem2Reg: the resident k-steps of B_w; the parked ones go to this warp's slab
+#pragma unroll
+    for (int kk = 0; kk < kRK; ++kk)
+#pragma unroll
+      for (int j = 0; j < kGFN; ++j) {
+        const int col = col0 + j * 8 + g;
+        b[kk][j] = (kk < p.rs && col0 + j * 8 < p.n) ? __ldg(Bg + (kk * 4 + t) * (long long)p.n + col) : 0.0;
+      }
+    for (int kk = p.rs; kk < p.ks; ++kk)
+#pragma unroll
+      for (int j = 0; j < kGFN; ++j) {
+        const int col = col0 + j * 8 + g;
+        const double v = col0 + j * 8 < p.n ? __ldg(Bg + (kk * 4 + t) * (long long)p.n + col) : 0.0;
+        asm volatile("st.shared.f64 [%0], %1;" ::"r"(park + (uint32_t)(((kk - p.rs) * kGFN + j) * 32 + lane) * 8),
+                     "d"(v)
+                     : "memory");
+      }
+    __syncwarp();
+    for (int mb = 0; mb < p.mblocks; ++mb, ++it) {
+      const uint32_t s = it & 1;
+      double c[kGFM][kGFN][2];
+#pragma unroll
+      for (int i = 0; i < kGFM; ++i)
+#pragma unroll
+        for (int j = 0; j < kGFN; ++j) c[i][j][0] = c[i][j][1] = 0.0;
+      ptx::mbar_wait(&full[s], (it >> 1) & 1);
+      const uint32_t a_s = ptx::smem_u32(tbase + s * p.a_block_bytes);
+      const uint32_t rowb = 8u << p.ce_shift;  // bytes of one swizzled row of a chunk
+      auto step = [&](int kk, const double (&bb)[kGFN]) {
+        const int col = kk * 4 + t;
+        const uint32_t chunk_off = (uint32_t)(col >> p.ce_shift) * (kGTM * rowb);
+        const uint32_t in_row = (uint32_t)(col & ((1 << p.ce_shift) - 1)) * 8;
+#pragma unroll
+        for (int i = 0; i < kGFM; ++i) {
+          const int row = i * 8 + g;
+          double a;
+          asm volatile("ld.shared.f64 %0, [%1];"
+                       : "=d"(a)
+                       : "r"(a_s + chunk_off + ptx::swz(row * rowb + in_row, p.swz_bits)));
+#pragma unroll
+          for (int j = 0; j < kGFN; ++j)
+            asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
+                         : "+d"(c[i][j][0]), "+d"(c[i][j][1])
+                         : "d"(a), "d"(bb[j]));
+        }
+      };
+      // resident k-steps: B fragments from registers
+#pragma unroll
+      for (int kk = 0; kk < kRK; ++kk)
+        if (kk < p.rs) step(kk, b[kk]);
+      // parked k-steps: B fragments from the warp's slab (one LDS.64 per fragment)
+#pragma unroll 4
+      for (int kk = p.rs; kk < p.ks; ++kk) {
+        double bb[kGFN];
+#pragma unroll
+        for (int j = 0; j < kGFN; ++j)
+          asm volatile("ld.shared.f64 %0, [%1];"
+                       : "=d"(bb[j])
+                       : "r"(park + (uint32_t)(((kk - p.rs) * kGFN + j) * 32 + lane) * 8));
+        step(kk, bb);
+      }
+      // Reg2GMem: C_w block; lane holds (row g, cols 2t, 2t+1) of each 8x8 fragment
+      double* Cg = p.C + e * (long long)p.m * p.n;
+#pragma unroll
+      for (int i = 0; i < kGFM; ++i) {
+        const int row = mb * kGTM + i * 8 + g;
+#pragma unroll
+        for (int j = 0; j < kGFN; ++j)
+          if (row < p.m && col0 + j * 8 < p.n)
+            ptx::st_global_v2_f64(Cg + (long long)row * p.n + col0 + j * 8 + 2 * t, c[i][j][0], c[i][j][1]);
+      }
+      ptx::named_bar_sync(bar, kGP * 32);  // every warp finished reading buffer s
+      if (issuer && pu < p.units) {        // refill it with the block two ahead
+        issue(pu, pmb, s);
+        if (++pmb == p.mblocks) {
+          pmb = 0;
+          pu += nteams;
+        }
+      }
+    }
+  }
+}
+
+// Residency ratio: share of the ks k-steps of B_w kept in
+// registers.  Default: as many as fit (kRK), i.e. 100 % up to k = 128, 50 %
+// at k = 256.  KAMI_F64_RESIDENT_PCT overrides it (sweeps, tools/residency_sweep.py).
+int resident_steps(int ks) {
+  // read per call (not cached) so one process can sweep the ratio
+  const char* env = getenv("KAMI_F64_RESIDENT_PCT");
+  const int pct = env ? atoi(env) : -1;
+  int rs = pct < 0 ? ks : (ks * pct + 50) / 100;
+  if (rs > kRK) rs = kRK;
+  if (rs > ks) rs = ks;
+  if (rs < 0) rs = 0;
+  return rs;
+}
+
+uint32_t align1k(uint32_t x) { return (x + 1023) / 1024 * 1024; }
+
+}  // namespace
+
+bool dmma_gen_supported(int m, int n, int k) {
+  return m >= 8 && n >= 8 && k >= 8 && m <= 256 && n <= 256 && k <= 256 && m % 8 == 0 && n % 8 == 0 && k % 8 == 0;
+}
+
+int dmma_gen_resident_pct(int k) { return 100 * resident_steps(k / 4) / (k / 4); }
+
+kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
+                              cudaStream_t stream) {
+  if (!dmma_gen_supported(m, n, k)) return KAMI_ERROR_NOT_SUPPORTED;
+  PFN_encodeTiled enc = get_encode_tiled();
+  if (!enc) return KAMI_ERROR_CUDA;
+  DmmaGenParams p;
+  memset(&p, 0, sizeof(p));
+  p.B = static_cast<const double*>(B);
+  p.C = static_cast<double*>(C);
+  p.batch = batch;
+  p.m = m;
+  p.n = n;
+  p.k = k;
+  p.ks = k / 4;
+  p.rs = resident_steps(p.ks);
+  p.nblocks = (n + kGNB - 1) / kGNB;
+  p.mblocks = (m + kGTM - 1) / kGTM;
+  p.ce_shift = (k % 16 == 0) ? 4 : 3;
+  p.swz_bits = (k % 16 == 0) ? 3 : 2;
+  const int ce = 1 << p.ce_shift;
+  p.kch = k / ce;
+  p.units = batch * p.nblocks;
+  p.a_block_bytes = align1k((uint32_t)(kGTM * p.kch * ce * 8));
+  p.park_bytes = (uint32_t)((p.ks - p.rs) * kGFN * 32 * 8);
+  const uint32_t team_bytes = 2 * p.a_block_bytes + kGP * p.park_bytes;
+  p.teams = (team_bytes * 2 + 1024 + 64 <= 232448 - 1024) ? 2 : 1;
+  const uint32_t smem = p.teams * team_bytes + 1024 /*align*/ + 64 /*barriers*/;
+  if (smem > 232448) return KAMI_ERROR_NOT_SUPPORTED;
+  {  // A: (CE doubles, m, k/CE chunks, batch), box (CE, TM, k/CE, 1); rows past m zero-filled
+    cuuint64_t dims[4] = {(cuuint64_t)ce, (cuuint64_t)m, (cuuint64_t)p.kch, (cuuint64_t)batch};
+    cuuint64_t strides[3] = {(cuuint64_t)k * 8, (cuuint64_t)ce * 8, (cuuint64_t)m * k * 8};
+    cuuint32_t box[4] = {(cuuint32_t)ce, (cuuint32_t)kGTM, (cuuint32_t)p.kch, 1};
+    cuuint32_t es[4] = {1, 1, 1, 1};
+    if (enc(&p.tmA, CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 4, const_cast<void*>(A), dims, strides, box, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, ce == 16 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_64B,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
+  }
+  if (cudaFuncSetAttribute(kami_dmma_gen_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+      cudaSuccess)
+    return KAMI_ERROR_CUDA;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long need = (p.units + p.teams - 1) / p.teams;
+  long long grid = sms < need ? sms : need;
+  grid = apply_grid_cap(grid);
+  kami_dmma_gen_kernel<<<(unsigned)grid, kGP * 32 * 2, smem, stream>>>(p);
+  set_last_kernel("kami_dmma_gen_1d");
+  return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+}
+
+}  // namespace kami

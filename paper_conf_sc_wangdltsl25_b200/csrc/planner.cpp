@@ -151,6 +151,22 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
   // FP64 1D with the broadcast operand fed by TMA (dmma_tma.cu; pointer arrays
   // through an address-space view of each entry)
   const bool tma_ok = !is16 && dmma_tma_supported(m, n, k);
+  // FP64 off the square orders the fixed-shape kernels are instantiated for:
+  // the general k-sliced DMMA kernel with a register residency ratio
+  // (dmma_gen.cu; a7).  Explicit 1D with p = 0 selects it too.
+  const bool warp_shape = !is16 && m == n && n == k && (m == 8 || m == 16 || m == 32 || m == 64);
+  if (!is16 && !pointer_array && dmma_gen_supported(m, n, k) &&
+      ((algo == KAMI_ALGO_AUTO && !warp_shape) || (algo == KAMI_ALGO_1D && p == 0 && !warp_shape))) {
+    r.algo = KAMI_ALGO_1D;
+    r.p = 4;
+    r.kernel = 4;
+    r.entries_per_cta = 2;
+    r.stages = 2;
+    r.kslice_regs_pct = dmma_gen_resident_pct(k);
+    r.t_all_cycles = b200_cost(1, n, m, k, 4, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
   if (algo == KAMI_ALGO_1D_TMA) {
     if (!tma_ok || (p != 0 && p != 4)) return KAMI_ERROR_NOT_SUPPORTED;
     r.algo = KAMI_ALGO_1D_TMA;

@@ -51,7 +51,8 @@ FAKE = 0x10000  # never dereferenced: every case below fails validation first
     ((24, 16, 16, 1, 0, 0), UNSUP),        # 16-bit m not a multiple of 16
     ((16, 16, 12, 1, 0, 0), UNSUP),        # 16-bit k not a multiple of 8
     ((272, 16, 16, 1, 0, 0), UNSUP),       # > 256
-    ((48, 48, 48, 1, 2, 0), UNSUP),        # fp64 outside the instantiated orders
+    ((44, 48, 48, 1, 2, 0), UNSUP),        # fp64 m not a multiple of 8
+    ((48, 48, 20, 1, 2, 0), UNSUP),        # fp64 k not a multiple of 8
 ])
 def test_rejects_before_launch(args, code):
     L = kami.lib()

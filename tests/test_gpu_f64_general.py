@@ -1,0 +1,62 @@
+"""FP64 over the whole size grid (m, n, k multiples of 8 in [8, 256], non-square
+included) on the k-sliced DMMA kernel with a register / shared-memory
+residency ratio (dmma_gen.cu; Sec. 4.7,
+Sec. 5.2.5), against the oracle: max |C - C_ref| / S <= k 2^-52
+(DESIGN.md "Tolerances"), integer inputs bit-exact."""
+import os
+
+import numpy as np
+import pytest
+
+import paper_conf_sc_wangdltsl25_b200 as kami
+from test_gpu_parity import check
+
+pytestmark = pytest.mark.gpu
+
+GEN_SHAPES = [
+    (128, 128, 128, 37),  # the paper's order-128 case (Sec. 5.2.5)
+    (256, 256, 256, 5),   # largest order: 4 m-blocks x 4 n-blocks, 50 % of B_w resident
+    (192, 192, 192, 7),
+    (96, 40, 72, 61),     # non-square, k % 16 = 8 (64-byte swizzled A chunks)
+    (8, 256, 8, 33),      # one 8-row fragment, wide N
+    (256, 8, 256, 9),     # one 8-column fragment, deep K
+    (48, 48, 48, 55),     # square order outside the fixed-shape kernels
+    (24, 40, 56, 77),     # small, all tails
+    (200, 136, 104, 11),  # ragged m-block and n-block
+    (64, 128, 32, 41),
+]
+
+
+@pytest.mark.parametrize("shape", GEN_SHAPES, ids=lambda s: "x".join(map(str, s)))
+def test_f64_general(shape):
+    m, n, k, batch = shape
+    for layout, dist, seed in (("row", "unif", 1), ("col", "unif", 2), ("row", "int", 3)):
+        check(m, n, k, batch, "f64", layout, dist, seed=seed)
+        assert kami.last_kernel() == "kami_dmma_gen_1d", kami.last_kernel()
+
+
+@pytest.mark.parametrize("pct", [100, 75, 50, 25, 0])
+@pytest.mark.parametrize("shape", [(128, 128, 128, 19), (64, 96, 256, 23)], ids=lambda s: "x".join(map(str, s)))
+def test_f64_residency_ratios(pct, shape):
+    """Every residency ratio gives the same result (only where B_w lives changes)."""
+    m, n, k, batch = shape
+    os.environ["KAMI_F64_RESIDENT_PCT"] = str(pct)
+    try:
+        check(m, n, k, batch, "f64", "row", "unif", seed=4)
+        check(m, n, k, batch, "f64", "row", "int", seed=5)
+        assert kami.plan(m, n, k, "f64")["kslice_regs_pct"] <= max(pct, 0) + 1
+    finally:
+        del os.environ["KAMI_F64_RESIDENT_PCT"]
+
+
+def test_f64_general_steady_state():
+    with kami.grid_cap(3):
+        check(128, 128, 128, 29, "f64", "row", "unif", seed=6)
+        check(96, 40, 72, 97, "f64", "col", "int", seed=7)
+        check(256, 256, 256, 4, "f64", "row", "unif", seed=8)
+
+
+def test_f64_plan_reports_residency():
+    p = kami.plan(256, 256, 256, "f64")
+    assert p["kernel"] == "dmma_gen" and p["kslice_regs_pct"] == 50
+    assert kami.plan(128, 128, 128, "f64")["kslice_regs_pct"] == 100
