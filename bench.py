@@ -64,10 +64,12 @@ def op_bytes(dtype, m, n, k, update=False):
 def parse_workload(name):
     if name in WORKLOADS:
         return WORKLOADS[name]
-    if name.startswith("bf16-"):  # bf16-<m>x<n>x<k>[:batch]
-        spec, _, b = name[5:].partition(":")
+    dt, _, rest = name.partition("-")
+    if dt in ("bf16", "f16", "f64") and "x" in rest:  # <dtype>-<m>x<n>x<k>[:batch]
+        spec, _, b = rest.partition(":")
         m, n, k = (int(x) for x in spec.split("x"))
-        return ("bf16", m, n, k, int(b) if b else 125000, 4)
+        default = {"bf16": (125000, 4), "f16": (65536, 1), "f64": (32768, 2)}[dt]
+        return (dt, m, n, k, int(b) if b else default[0], default[1])
     raise SystemExit(f"unknown workload {name}")
 
 

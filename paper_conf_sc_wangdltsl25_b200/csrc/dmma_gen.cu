@@ -42,6 +42,8 @@ constexpr int kGNB = kGP * kGFN * 8;  // 64 columns per unit
 constexpr int kGTM = 32;  // A / C rows per block
 constexpr int kGFM = kGTM / 8;
 constexpr int kRK = 32;   // max resident k-steps (32 x 2 doubles = 128 registers)
+constexpr int kRKSmall = 8;  // k <= 32: 16 registers of B, four teams per SM
+constexpr int kGenSmem = 232448;
 
 struct DmmaGenParams {
   CUtensorMap tmA;  // 4-D (CE, m, k/CE, batch), box (CE, TM, k/CE, 1), CE = 16 (SW128) or 8 (SW64) doubles
@@ -55,7 +57,9 @@ struct DmmaGenParams {
   int teams;
 };
 
-__global__ void __launch_bounds__(kGP * 32 * 2, 1) kami_dmma_gen_kernel(const __grid_constant__ DmmaGenParams p) {
+template <int RK>
+__global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
+    kami_dmma_gen_kernel(const __grid_constant__ DmmaGenParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -97,7 +101,7 @@ __global__ void __launch_bounds__(kGP * 32 * 2, 1) kami_dmma_gen_kernel(const __
       }
     }
   }
-  double b[kRK][kGFN];
+  double b[RK][kGFN];
   uint32_t it = 0;
   for (long long u = first; u < p.units; u += nteams) {
     const long long e = u / p.nblocks;
@@ -106,7 +110,7 @@ __global__ void __launch_bounds__(kGP * 32 * 2, 1) kami_dmma_gen_kernel(const __
     const double* Bg = p.B + e * (long long)p.k * p.n;
     // GMem2Reg: the resident k-steps of B_w; the parked ones go to this warp's slab
 #pragma unroll
-    for (int kk = 0; kk < kRK; ++kk)
+    for (int kk = 0; kk < RK; ++kk)
 #pragma unroll
       for (int j = 0; j < kGFN; ++j) {
         const int col = col0 + j * 8 + g;
@@ -152,7 +156,7 @@ __global__ void __launch_bounds__(kGP * 32 * 2, 1) kami_dmma_gen_kernel(const __
       };
       // resident k-steps: B fragments from registers
 #pragma unroll
-      for (int kk = 0; kk < kRK; ++kk)
+      for (int kk = 0; kk < RK; ++kk)
         if (kk < p.rs) step(kk, b[kk]);
       // parked k-steps: B fragments from the warp's slab (one LDS.64 per fragment)
 #pragma unroll 4
@@ -190,18 +194,40 @@ __global__ void __launch_bounds__(kGP * 32 * 2, 1) kami_dmma_gen_kernel(const __
 // Residency ratio: share of the ks k-steps of B_w kept in
 // registers.  Default: as many as fit (kRK), i.e. 100 % up to k = 128, 50 %
 // at k = 256.  KAMI_F64_RESIDENT_PCT overrides it (sweeps, tools/residency_sweep.py).
-int resident_steps(int ks) {
+uint32_t align1k(uint32_t x) { return (x + 1023) / 1024 * 1024; }
+
+// Plan of one launch: resident k-steps, register template, teams per CTA and
+// shared-memory bytes.  The parked slabs must fit next to the A double buffer:
+// a ratio that parks more than fits is raised to the smallest that fits.
+struct GenPlan {
+  int rk, rs, teams, ce_shift;
+  uint32_t a_block_bytes, park_bytes, smem;
+};
+GenPlan gen_plan(int m, int n, int k) {
+  GenPlan g;
+  const int ks = k / 4;
+  g.ce_shift = (k % 16 == 0) ? 4 : 3;
+  g.rk = ks <= kRKSmall ? kRKSmall : kRK;
   // read per call (not cached) so one process can sweep the ratio
   const char* env = getenv("KAMI_F64_RESIDENT_PCT");
   const int pct = env ? atoi(env) : -1;
   int rs = pct < 0 ? ks : (ks * pct + 50) / 100;
-  if (rs > kRK) rs = kRK;
+  if (rs > g.rk) rs = g.rk;
   if (rs > ks) rs = ks;
   if (rs < 0) rs = 0;
-  return rs;
+  g.a_block_bytes = align1k((uint32_t)(kGTM * k * 8));
+  const int slab_step = kGFN * 32 * 8;  // bytes per parked k-step per warp
+  const int room = (kGenSmem - 1024 - 64 - 2 * (int)g.a_block_bytes) / (kGP * slab_step);
+  if (ks - rs > room) rs = ks - room;
+  g.rs = rs;
+  g.park_bytes = (uint32_t)((ks - rs) * slab_step);
+  const uint32_t team_bytes = 2 * g.a_block_bytes + kGP * g.park_bytes;
+  const int max_teams = g.rk == kRK ? 2 : 4;
+  g.teams = 1;
+  while (g.teams < max_teams && (g.teams + 1) * team_bytes + 1024 + 64 <= (uint32_t)kGenSmem) ++g.teams;
+  g.smem = g.teams * team_bytes + 1024 /*align*/ + 64 /*barriers*/;
+  return g;
 }
-
-uint32_t align1k(uint32_t x) { return (x + 1023) / 1024 * 1024; }
 
 }  // namespace
 
@@ -209,7 +235,7 @@ bool dmma_gen_supported(int m, int n, int k) {
   return m >= 8 && n >= 8 && k >= 8 && m <= 256 && n <= 256 && k <= 256 && m % 8 == 0 && n % 8 == 0 && k % 8 == 0;
 }
 
-int dmma_gen_resident_pct(int k) { return 100 * resident_steps(k / 4) / (k / 4); }
+int dmma_gen_resident_pct(int k) { return 100 * gen_plan(k, k, k).rs / (k / 4); }
 
 kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
                               cudaStream_t stream) {
@@ -225,20 +251,20 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
   p.n = n;
   p.k = k;
   p.ks = k / 4;
-  p.rs = resident_steps(p.ks);
+  const GenPlan gp = gen_plan(m, n, k);
+  if (gp.smem > (uint32_t)kGenSmem) return KAMI_ERROR_NOT_SUPPORTED;
+  p.rs = gp.rs;
   p.nblocks = (n + kGNB - 1) / kGNB;
   p.mblocks = (m + kGTM - 1) / kGTM;
-  p.ce_shift = (k % 16 == 0) ? 4 : 3;
-  p.swz_bits = (k % 16 == 0) ? 3 : 2;
+  p.ce_shift = gp.ce_shift;
+  p.swz_bits = gp.ce_shift == 4 ? 3 : 2;
   const int ce = 1 << p.ce_shift;
   p.kch = k / ce;
   p.units = batch * p.nblocks;
-  p.a_block_bytes = align1k((uint32_t)(kGTM * p.kch * ce * 8));
-  p.park_bytes = (uint32_t)((p.ks - p.rs) * kGFN * 32 * 8);
-  const uint32_t team_bytes = 2 * p.a_block_bytes + kGP * p.park_bytes;
-  p.teams = (team_bytes * 2 + 1024 + 64 <= 232448 - 1024) ? 2 : 1;
-  const uint32_t smem = p.teams * team_bytes + 1024 /*align*/ + 64 /*barriers*/;
-  if (smem > 232448) return KAMI_ERROR_NOT_SUPPORTED;
+  p.a_block_bytes = gp.a_block_bytes;
+  p.park_bytes = gp.park_bytes;
+  p.teams = gp.teams;
+  const uint32_t smem = gp.smem;
   {  // A: (CE doubles, m, k/CE chunks, batch), box (CE, TM, k/CE, 1); rows past m zero-filled
     cuuint64_t dims[4] = {(cuuint64_t)ce, (cuuint64_t)m, (cuuint64_t)p.kch, (cuuint64_t)batch};
     cuuint64_t strides[3] = {(cuuint64_t)k * 8, (cuuint64_t)ce * 8, (cuuint64_t)m * k * 8};
@@ -249,8 +275,8 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
-  if (cudaFuncSetAttribute(kami_dmma_gen_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
-      cudaSuccess)
+  auto fn = gp.rk == kRK ? kami_dmma_gen_kernel<kRK> : kami_dmma_gen_kernel<kRKSmall>;
+  if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
     return KAMI_ERROR_CUDA;
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
@@ -258,7 +284,7 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
   const long long need = (p.units + p.teams - 1) / p.teams;
   long long grid = sms < need ? sms : need;
   grid = apply_grid_cap(grid);
-  kami_dmma_gen_kernel<<<(unsigned)grid, kGP * 32 * 2, smem, stream>>>(p);
+  fn<<<(unsigned)grid, kGP * 32 * (gp.rk == kRK ? 2 : 4), smem, stream>>>(p);
   set_last_kernel("kami_dmma_gen_1d");
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
 }

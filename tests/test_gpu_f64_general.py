@@ -44,7 +44,11 @@ def test_f64_residency_ratios(pct, shape):
     try:
         check(m, n, k, batch, "f64", "row", "unif", seed=4)
         check(m, n, k, batch, "f64", "row", "int", seed=5)
-        assert kami.plan(m, n, k, "f64")["kslice_regs_pct"] <= max(pct, 0) + 1
+        got = kami.plan(m, n, k, "f64")["kslice_regs_pct"]
+        if k == 128:  # fits as requested
+            assert got == pct, got
+        else:  # k = 256: at most 32 of 64 k-steps in registers, parking limited by shared memory
+            assert 25 <= got <= 50, got
     finally:
         del os.environ["KAMI_F64_RESIDENT_PCT"]
 

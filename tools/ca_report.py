@@ -44,6 +44,13 @@ CASES["f16-128_w1d"] = ("f16", 128, "1d", 8, 4096)
 CASES["f16-128_2d"] = ("f16", 128, "2d", 16, 4096)
 CASES["f16-64_tc16"] = ("f16", 64, "tc16", 4, 8192)
 CASES["f16-128_tc16"] = ("f16", 128, "tc16", 4, 4096)
+# round 2: tcgen05 with A resident in TMEM (TS form), 1D and 3D k-layers
+CASES["f16-64_ts1d"] = ("f16", 64, "tc16ts", 4, 8192)
+CASES["f16-64_ts3d"] = ("f16", 64, "tc16ts", 8, 8192)
+CASES["f16-128_ts1d"] = ("f16", 128, "tc16ts", 4, 4096)
+CASES["f16-128_ts3d"] = ("f16", 128, "tc16ts", 8, 4096)
+CASES["f16-32_ts1d"] = ("f16", 32, "tc16ts", 4, 8192)
+CASES["f16-32_tc16"] = ("f16", 32, "tc16", 4, 8192)
 
 
 def closed_form(dtype, s, algo, p):
@@ -65,6 +72,8 @@ def closed_form(dtype, s, algo, p):
         return (m * k + k * n) * se + (wn * m * k + wm * k * n) * se
     if algo == "tc16":  # TMA writes A,B once; UMMA reads A,B once; epilogue stages C (write) + TMA store (read)
         return 2 * (m * k + k * n) * se + 2 * m * n * se
+    if algo == "tc16ts":  # A: global -> registers -> TMEM (no SMEM); B: TMA write + UMMA read; C staged
+        return 2 * k * n * se + 2 * m * n * se
     return None
 
 
@@ -98,8 +107,9 @@ def main(rnd="r1"):
         tma_out = d.get("l1tex__m_l1tex2xbar_write_bytes_mem_global_op_tma_st.sum", 0)
         mmas = 2.0 * s ** 3 / 4096 * batch
         per_entry = (ld + st) / batch
-        if algo == "tc16":  # async-proxy traffic is not LSU traffic: TMA writes + analytic UMMA reads
-            umma_reads = 2 * s * s * 2 * batch
+        if algo in ("tc16", "tc16ts"):  # async-proxy traffic is not LSU traffic: TMA bytes + analytic UMMA reads
+            # (SS form: the tensor core reads A and B from SMEM once per entry; TS form: only B)
+            umma_reads = (2 if algo == "tc16" else 1) * s * s * 2 * batch
             per_entry = (ld + st + tma_in + tma_out + umma_reads) / batch
         cf = closed_form(dtype, s, algo, p)
         wf_ld = d.get("l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum", 0)
