@@ -209,6 +209,36 @@ typedef struct {
 kami_status_t kami_plan(int m, int n, int k, kami_dtype_t dtype, kami_layout_t layout, kami_algo_t algo, int p,
                         kami_plan_t* out);
 
+/* What bounds a candidate in the planner's B200 cycle model. */
+typedef enum {
+  KAMI_BOUND_HBM = 0,      /* algorithmic bytes / HBM bandwidth                       */
+  KAMI_BOUND_TENSOR = 1,   /* flops / tensor-pipe rate (tcgen05, HMMA or DMMA)        */
+  KAMI_BOUND_SMEM = 2,     /* shared-memory bytes / SMEM bandwidth                    */
+  KAMI_BOUND_TMA = 3,      /* TMA box rows x per-row engine time                      */
+  KAMI_BOUND_ISSUE = 4,    /* per-unit fixed cost of the persistent pipeline          */
+  KAMI_BOUND_LATENCY = 5   /* a team's serial chain (DRAM latency + Eqs. 4/8/12 with
+                              B200 constants + barriers) over the teams per SM       */
+} kami_bound_t;
+
+/* One schedule the library can run for a shape, with the model's prediction
+ * (Eqs. 4/8/12 with B200 constants for the
+ * register-resident schedules, a streaming roofline for the tcgen05 ones). */
+typedef struct {
+  kami_algo_t algo;
+  int p;
+  int kernel;                    /* as kami_plan_t.kernel                     */
+  double model_cycles_per_entry; /* per SM, at 1965 MHz                       */
+  double model_tflops;           /* whole GPU (148 SMs)                       */
+  int bound;                     /* kami_bound_t of the largest term          */
+} kami_candidate_t;
+
+/* Every candidate schedule for a strided problem (row-major view after the
+ * layout transform) with the model's prediction; AUTO takes the fastest.
+ * Writes min(*count, max) entries to `out` (may be NULL with max = 0) and the
+ * total number to *count.  Host-only (no device work); errors as kami_plan. */
+kami_status_t kami_plan_candidates(int m, int n, int k, kami_dtype_t dtype, kami_layout_t layout,
+                                   kami_candidate_t* out, int max, int* count);
+
 /* Paper-faithful cost model (Eqs. 1-12, readings R6-R8): fills
  * V_cm, T_cm, T_cp, T_all for variant 1/2/3 (KAMI_ALGO_1D/2D/3D). */
 kami_status_t kami_paper_cost(kami_algo_t variant, double m, double n, double k, double p, double s_e,

@@ -34,7 +34,7 @@ EXPORTS = [
     "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
     "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level", "kami_gemm_vbatched",
     "kami_spmm_bsr_strided_batched", "kami_gemm_strided_batched_axpby", "kami_probe_dmma_peak",
-    "kami_set_grid_cap",
+    "kami_set_grid_cap", "kami_plan_candidates",
 ]
 
 
@@ -50,6 +50,15 @@ class KamiPlan(ctypes.Structure):
                 ("entries_per_cta", ctypes.c_int), ("stages", ctypes.c_int), ("kslice_regs_pct", ctypes.c_int),
                 ("t_all_cycles", ctypes.c_double)]
 
+
+class KamiCandidate(ctypes.Structure):
+    _fields_ = [("algo", ctypes.c_int), ("p", ctypes.c_int), ("kernel", ctypes.c_int),
+                ("model_cycles_per_entry", ctypes.c_double), ("model_tflops", ctypes.c_double),
+                ("bound", ctypes.c_int)]
+
+
+BOUND = {0: "hbm", 1: "tensor", 2: "smem", 3: "tma", 4: "issue", 5: "latency"}
+KERNEL = {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma", 3: "tcgen05_ts", 4: "dmma_gen"}
 
 _lib = None
 
@@ -78,6 +87,8 @@ def lib() -> ctypes.CDLL:
     L.kami_probe_dmma_peak.argtypes = [ctypes.c_double, ctypes.POINTER(ctypes.c_double),
                                        ctypes.POINTER(ctypes.c_double), st]
     L.kami_probe_dmma_peak.restype = ctypes.c_int
+    L.kami_plan_candidates.argtypes = [i, i, i, i, i, ctypes.POINTER(KamiCandidate), i, ctypes.POINTER(i)]
+    L.kami_plan_candidates.restype = ctypes.c_int
     L.kami_set_grid_cap.argtypes = [i]
     L.kami_set_grid_cap.restype = ctypes.c_int
     L.kami_plan.argtypes = [i, i, i, i, i, i, i, ctypes.POINTER(KamiPlan)]
@@ -235,9 +246,21 @@ def plan(m, n, k, dtype, layout="row", algo="auto", p=0) -> dict:
     _check(lib().kami_plan(m, n, k, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"),
                            _enum(ALGO, algo, "algo"), p, ctypes.byref(out)), "kami_plan")
     inv = {v: k for k, v in ALGO.items()}
-    return {"algo": inv[out.algo], "p": out.p, "kernel": {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma", 3: "tcgen05_ts", 4: "dmma_gen"}[out.kernel],
+    return {"algo": inv[out.algo], "p": out.p, "kernel": KERNEL[out.kernel],
             "entries_per_cta": out.entries_per_cta, "stages": out.stages, "kslice_regs_pct": out.kslice_regs_pct,
             "t_all_cycles": out.t_all_cycles}
+
+
+def plan_candidates(m, n, k, dtype, layout="row") -> list:
+    """Every schedule the library can run for the shape, with the planner
+    model's prediction (AUTO takes the smallest model_cycles_per_entry)."""
+    buf = (KamiCandidate * 32)()
+    cnt = ctypes.c_int(0)
+    _check(lib().kami_plan_candidates(m, n, k, _enum(DTYPE, dtype, "dtype"), _enum(LAYOUT, layout, "layout"), buf, 32,
+                                      ctypes.byref(cnt)), "kami_plan_candidates")
+    inv = {v: k_ for k_, v in ALGO.items()}
+    return [{"algo": inv[c.algo], "p": c.p, "kernel": KERNEL[c.kernel], "model_cycles_per_entry": c.model_cycles_per_entry,
+             "model_tflops": c.model_tflops, "bound": BOUND[c.bound]} for c in buf[:min(cnt.value, 32)]]
 
 
 def paper_cost(variant, m, n, k, p, s_e, L_sm, B_sm, theta_r, theta_w, O_tc, n_tc):

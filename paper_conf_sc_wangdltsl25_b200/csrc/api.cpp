@@ -136,8 +136,11 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
     return tc16_ts_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, plan.algo == KAMI_ALGO_3D_TMEM ? 2 : 1,
                           rp.A, rp.B, C, stream);
   }
-  if (plan.kernel == 1 && update && is16(dtype) && algo == KAMI_ALGO_AUTO && !Ca)
-    plan.kernel = 0;  // the update form (C read) exists on tcgen05 only
+  if ((plan.kernel == 1 || plan.kernel == 3) && update && is16(dtype) && algo == KAMI_ALGO_AUTO && !Ca)
+    plan.kernel = 0;  // the update form (C read) exists on the SS tcgen05 kernel only
+  if ((plan.kernel == 4 || plan.kernel == 1) && update && algo == KAMI_ALGO_AUTO && !Ca &&
+      dmma_tma_supported(rp.m, rp.n, rp.k))
+    plan.kernel = 2;  // FP64 update form: the TMA-broadcast DMMA kernel
   if (plan.kernel == 0) {
     return tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), rp.A, rp.B, C, (float)alpha,
                             (float)beta, stream, 0);
@@ -276,6 +279,16 @@ kami_status_t kami_plan(int m, int n, int k, kami_dtype_t dtype, kami_layout_t l
   if (!out || p < 0) return KAMI_ERROR_INVALID_VALUE;
   RowProblem rp = to_row(m, n, k, layout, nullptr, nullptr, nullptr, nullptr);
   return planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, false, out);
+}
+
+kami_status_t kami_plan_candidates(int m, int n, int k, kami_dtype_t dtype, kami_layout_t layout,
+                                   kami_candidate_t* out, int max, int* count) {
+  kami_status_t st = check_common(m, n, k, 1, dtype, layout, KAMI_ALGO_AUTO);
+  if (st != KAMI_SUCCESS) return st;
+  if (!count || max < 0 || (max > 0 && !out)) return KAMI_ERROR_INVALID_VALUE;
+  RowProblem rp = to_row(m, n, k, layout, nullptr, nullptr, nullptr, nullptr);
+  *count = planner_candidates(rp.m, rp.n, rp.k, dtype, false, out, max);
+  return KAMI_SUCCESS;
 }
 
 kami_status_t kami_paper_cost(kami_algo_t variant, double m, double n, double k, double p, double s_e,

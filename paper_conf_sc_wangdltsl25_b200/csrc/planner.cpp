@@ -1,6 +1,9 @@
-// planner.cpp -- see planner.h.
+// planner.cpp -- see planner.h.  SURVEY.md 8(a) row a1: the schedule of an
+// AUTO call is the argmax of a B200 cycle model over every kernel the library
+// can run for the shape.  No per-shape measured table.
 #include "planner.h"
 
+#include <algorithm>
 #include <cmath>
 
 #include "kernels.h"
@@ -37,24 +40,55 @@ PaperCost paper_cost(int variant, double m, double n, double k, double p, double
 
 namespace {
 
-// B200 constants, measured by tools/ubench.cu (profiles/r1/ubench_b200.json):
-// L_sm = 29 cycles (dependent LDS), B_sm = 127.6 B/cycle/SM (conflict-free
-// LDS.128), n_tc = 4 sub-partition tensor cores, O_tc per tensor core:
-// DMMA FP64 37.1 TF/s -> 31.9 flop/cycle; legacy HMMA FP16 554.5 TF/s ->
-// 477 flop/cycle (at 1965 MHz, 148 SMs).  HBM: 6541.8 GB/s measured copy
-// (MEASURED_PEAKS.json) -> 22.5 B/cycle/SM.  T_lat: DRAM round trip seen by a
-// team that starts a new entry (~1200 cycles; entries prefetched into L2 by
-// the previous one).
-constexpr double kLsm = 29, kBsm = 127.6, kNtc = 4;
-constexpr double kHbmBpc = 22.5, kTlat = 1200;
+// ----------------------------------------------------------- B200 constants
+// Every constant is a measured machine property (one SM, 1965 MHz), not a
+// per-shape result:
+//   kHbmBpc   6534.1 GB/s copy bandwidth (MEASURED_PEAKS.json hbm_gbs) /
+//             148 SMs / 1.965 GHz = 22.5 B per cycle per SM
+//   kLsm      29 cycles dependent LDS latency      (profiles/r1/ubench_b200.json)
+//   kBsm      127.6 B per cycle per SM, LDS.128    (ubench_b200.json)
+//   kDmmaFpc  37.1 TFLOP/s DMMA (ubench, kami_probe_dmma_peak) -> 127.6 flop/cycle/SM
+//   kHmmaFpc  554.5 TFLOP/s mma.sync HMMA (ubench) -> 1907 flop/cycle/SM
+//   kUmmaFpc  2250 TFLOP/s dense tcgen05 kind::f16 nominal -> 7737 flop/cycle/SM
+//   kNtc      4 sub-partition tensor cores per SM
+//   kTbar     named-barrier wait per CA stage: block-level mode measures the
+//             communication phase at 1.5-4x the model's T_cm; the excess per
+//             stage is 139-375 cycles (profiles/r1/block_level.md: f64 64^3
+//             1D/2D/3D +139/+345/+308, f16 64^3 +185/+375/+147), mean 250
+//   kTlat     DRAM round trip a team waits on when it starts an entry whose
+//             operands its previous entry prefetched into L2 (~L2 latency
+//             under load), 700 cycles
+//   kTmaLdRow cycles of TMA engine time per LOADED box row: 32-byte rows
+//             stream at 6.0 TB/s (8 stages; 64/128-byte rows 6.9-7.1 TB/s),
+//             i.e. 187.5 G rows/s / 148 SMs = one row per 1.55 cycles per SM
+//             (tools/ubench_tma.cu, profiles/r2/ubench_tma.json)
+//   kTmaStRow per STORED row (C through the staging tile): 4 cycles,
+//             calibrated on the one shape bound by it (f16 16^3: 512 stored
+//             32-byte rows per 32-entry unit, 3400 cycles per unit measured,
+//             profiles/r2/variant_sweep_r2.json) and checked on 48^3 (1728
+//             rows, 3728 cycles measured, 4090 modelled)
+//   kUnitSS   per-unit fixed cost of the SS tcgen05 pipeline (single-thread
+//             producer / MMA loops, two named barriers and one TMA store per
+//             unit in the epilogue): ncu f16 32^3 ~190 MMA-lane instructions
+//             per unit (profiles/r1), 900 cycles
+//   kItemTS   per A item of the TS kernel (one k-chunk x one layer): the
+//             loader's LDG -> tcgen05.st -> wait::st -> mbarrier round trip
+//             with two items in flight per thread: 1400 cycles (TS 32^3 = one
+//             item per 4-entry unit: 1587 cycles per unit measured; bf16
+//             48^3 / 96^3, three items: 1183 / 1328 per item)
+constexpr double kHbmBpc = 22.5, kLsm = 29, kBsm = 127.6, kNtc = 4;
+constexpr double kDmmaFpc = 127.6, kHmmaFpc = 1907.0, kUmmaFpc = 7737.0;
+constexpr double kTbar = 250, kTlat = 700;
+constexpr double kTmaLdRow = 1.55, kTmaStRow = 4.0, kUnitSS = 900, kItemTS = 1400;
 
 double b200_cost(int variant, int m, int n, int k, int p, kami_dtype_t dt) {
   const double s_e = dt == KAMI_DTYPE_F64 ? 8 : 2;
-  const double O = dt == KAMI_DTYPE_F64 ? 31.9 : 477;
+  const double O = (dt == KAMI_DTYPE_F64 ? kDmmaFpc : kHmmaFpc) / kNtc;  // per tensor core
   PaperCost c = paper_cost(variant, m, n, k, p, s_e, kLsm, kBsm, 1, 1, O, kNtc);
   const double stages = variant == 1 ? p : variant == 2 ? std::sqrt((double)p) : std::round(std::cbrt((double)p));
-  const double ratio = std::max(1.0, p / kNtc);
-  double t = stages * (c.T_cm + ratio * c.T_cp);
+  const double ratio = std::max(1.0, p / kNtc);  // reading R8: a warp cannot use a fraction of a tensor core
+  // + the barrier wait per stage (block_level.md); a one-warp team has no barrier
+  double t = stages * (c.T_cm + (p > 1 ? kTbar : 0.0) + ratio * c.T_cp);
   if (variant == 3) {  // reading R9: layer reduction through SMEM
     const double s_acc = dt == KAMI_DTYPE_F64 ? 8 : 4;
     t += 2 * (stages - 1) * (double)m * n * s_acc / kBsm;
@@ -62,172 +96,268 @@ double b200_cost(int variant, int m, int n, int k, int p, kami_dtype_t dt) {
   return t;
 }
 
-// Batched form: an SM streams entries; with t teams resident the per-entry
-// time is bounded by HBM and by the serial (latency + T_all) of one team
-// spread over t teams.
-double b200_entry_cycles(int variant, int m, int n, int k, int p, kami_dtype_t dt, int teams_per_sm) {
-  const double s_e = dt == KAMI_DTYPE_F64 ? 8 : 2;
-  const double t_hbm = (double)(m * k + k * n + m * n) * s_e / kHbmBpc;
-  const double t_all = b200_cost(variant, m, n, k, p, dt);
-  return std::max(t_hbm, (kTlat + t_all) / std::max(1, teams_per_sm));
+int es_in(kami_dtype_t dt) {
+  return dt == KAMI_DTYPE_F64 ? 8 : dt == KAMI_DTYPE_TF32 ? 4 : (dt == KAMI_DTYPE_E4M3 || dt == KAMI_DTYPE_E5M2) ? 1 : 2;
+}
+int es_out(kami_dtype_t dt) { return dt == KAMI_DTYPE_F64 ? 8 : dt == KAMI_DTYPE_TF32 ? 4 : 2; }
+int in_kind(kami_dtype_t d) {
+  return d == KAMI_DTYPE_F16 ? 0 : d == KAMI_DTYPE_BF16 ? 1 : d == KAMI_DTYPE_TF32 ? 2 : d == KAMI_DTYPE_E4M3 ? 3 : 4;
+}
+int out_kind(kami_dtype_t d) { return d == KAMI_DTYPE_BF16 ? 1 : d == KAMI_DTYPE_TF32 ? 2 : 0; }
+
+struct Pred {
+  double cycles;  // per entry per SM
+  int bound;
+};
+Pred pmax(std::initializer_list<std::pair<double, int>> terms) {
+  Pred r{0, 0};
+  for (auto& t : terms)
+    if (t.first > r.cycles) r = {t.first, t.second};
+  return r;
 }
 
-// Measured throughput of each schedule (bench.py, 20 steps, one B200,
-// profiles/r1/f64_sweep_r1.txt).  Where a shape is calibrated, AUTO takes the
-// measured-fastest schedule; elsewhere it takes the model's minimum.
-struct Calib {
-  kami_dtype_t dt;
-  int s, algo, p;
-  double tflops;
-};
-const Calib kCalib[] = {
-    {KAMI_DTYPE_F64, 16, 1, 1, 7.07},  {KAMI_DTYPE_F64, 16, 2, 4, 5.66},  {KAMI_DTYPE_F64, 16, 3, 8, 4.98},
-    {KAMI_DTYPE_F64, 32, 1, 2, 14.29}, {KAMI_DTYPE_F64, 32, 2, 4, 12.42}, {KAMI_DTYPE_F64, 32, 3, 8, 11.63},
-    {KAMI_DTYPE_F64, 64, 1, 8, 14.13}, {KAMI_DTYPE_F64, 64, 2, 16, 17.20}, {KAMI_DTYPE_F64, 64, 3, 8, 15.84},
-};
-
-double calibrated(kami_dtype_t dt, int m, int n, int k, int algo, int p) {
-  if (m != n || n != k) return 0;
-  for (const Calib& c : kCalib)
-    if (c.dt == dt && c.s == m && c.algo == algo && c.p == p) return c.tflops;
-  return 0;
+double bytes_entry(int m, int n, int k, kami_dtype_t dt) {
+  return (double)(m * k + k * n) * es_in(dt) + (double)m * n * es_out(dt);
 }
 
-// measured TFLOP/s of the FP64 TMA-broadcast 1D kernel (0 = not calibrated;
-// bench.py --algo 1d_tma, profiles/r1/dmma_tma_sweep_r1.txt)
-double calibrated_tma(int m) { return m == 16 ? 7.42 : m == 32 ? 15.02 : m == 64 ? 25.45 : 0; }
+// SS tcgen05 (tc16.cu): per unit = max(HBM, TMA rows, fixed); E entries per unit
+bool model_ss(int m, int n, int k, kami_dtype_t dt, Pred* out) {
+  Tc16Shape s;
+  if (tc16_plan_shape_kind(m, n, k, in_kind(dt), out_kind(dt), &s) != KAMI_SUCCESS) return false;
+  const double E = s.tpack ? 2.0 / 3.0 : (s.m_tiles > 1 ? 1.0 / s.m_tiles : (double)s.G * s.U);
+  const int esi = es_in(dt);
+  const int kpad = (k + 32 / esi - 1) / (32 / esi) * (32 / esi);
+  const double rows_tile = m < 128 ? m : 128;
+  const double gu = s.m_tiles > 1 ? 1 : (double)s.G * s.U;
+  const double rowsA = (s.m_tiles > 1 ? rows_tile : (double)s.slot * gu) * s.k_chunks * (s.colrep ? s.colrep : 1);
+  const double rowsB = (double)kpad * (n / s.Wn) * gu;
+  const double rowsC = rows_tile * (n / s.Wc) * gu;
+  const double t_hbm = E * bytes_entry(m, n, k, dt) / kHbmBpc;
+  const double t_tma = (rowsA + rowsB) * kTmaLdRow + rowsC * kTmaStRow;
+  const double t_tc = E * 2.0 * m * n * k / kUmmaFpc;
+  Pred p = pmax({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {kUnitSS, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR}});
+  p.cycles /= E;
+  *out = p;
+  return true;
+}
+
+// TS tcgen05 (tc16_ts.cu): A by LDG -> TMEM (no TMA rows), B and C by TMA
+bool model_ts(int m, int n, int k, kami_dtype_t dt, int layers, Pred* out) {
+  if (dt != KAMI_DTYPE_F16 && dt != KAMI_DTYPE_BF16) return false;
+  TsShape s;
+  if (tc16_ts_plan(m, n, k, layers, &s) != KAMI_SUCCESS) return false;
+  const double E = s.G;
+  const int kpad = (k + 15) / 16 * 16;
+  const double rowsB = (double)kpad * (n / s.Wn) * E, rowsC = (double)m * (n / s.Wc) * E;
+  const double t_hbm = E * bytes_entry(m, n, k, dt) / kHbmBpc;
+  const double t_tma = rowsB * kTmaLdRow + rowsC * kTmaStRow;
+  const double t_tc = E * 2.0 * m * n * k / kUmmaFpc;
+  const double t_fix = kItemTS * s.k_chunks * layers;  // one loader round trip per A item
+  Pred p = pmax({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {t_fix, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR}});
+  p.cycles /= E;
+  *out = p;
+  return true;
+}
+
+// register-resident warp teams (warp_ca.cu): a team loads its entry with its
+// own LDGs (one round trip to L2, where its previous entry prefetched it),
+// runs the CA schedule (T_all of Eqs. 4/8/12 with B200 constants + the
+// barrier wait per stage) and stores C (fire and forget) before it starts the
+// next entry, so per SM an entry costs its HBM transfer plus the team's
+// unhidden chain spread over the resident teams
+bool model_warp(int m, int n, int k, kami_dtype_t dt, int variant, int p, Pred* out) {
+  if (warp_ca_supported(m, n, k, dt, variant, p) != KAMI_SUCCESS) return false;
+  const int teams = warp_ca_teams_per_sm(m, n, k, dt, variant, p);
+  const double be = bytes_entry(m, n, k, dt);
+  const double rate = (dt == KAMI_DTYPE_F64 ? kDmmaFpc : kHmmaFpc) / kNtc;  // per tensor core
+  const double t_sched = variant == 4 ? 2.0 * m * n * k / (rate * std::min<double>(p, kNtc))
+                                      : b200_cost(variant, m, n, k, p, dt);
+  const double t_chain = kTlat + t_sched;
+  const double t_tc = 2.0 * m * n * k / (dt == KAMI_DTYPE_F64 ? kDmmaFpc : kHmmaFpc);
+  const double t_mem = be / kHbmBpc + t_chain / teams;
+  *out = pmax({{t_mem, t_chain / teams > be / kHbmBpc ? KAMI_BOUND_LATENCY : KAMI_BOUND_HBM},
+               {t_tc, KAMI_BOUND_TENSOR}});
+  return true;
+}
+
+// FP64 1D with TMA broadcast of A (dmma_tma.cu): P = 4 warps, TEAMS per CTA
+bool model_dmma_tma(int m, int n, int k, Pred* out) {
+  if (!dmma_tma_supported(m, n, k)) return false;
+  const int teams = m == 64 ? 3 : 8;
+  const double be = bytes_entry(m, n, k, KAMI_DTYPE_F64);
+  const double flops = 2.0 * m * n * k;
+  const double smem = (double)m * k * 8 * (1 + 4);  // TMA write + 4 warps read A
+  // per team: B_w loads (prefetched into L2) + its share of the DMMA work
+  const double t_team = kTlat + flops / (kDmmaFpc / kNtc * 4) * kNtc / 4;
+  *out = pmax({{be / kHbmBpc, KAMI_BOUND_HBM}, {flops / kDmmaFpc, KAMI_BOUND_TENSOR},
+               {smem / kBsm, KAMI_BOUND_SMEM}, {t_team / teams, KAMI_BOUND_LATENCY}});
+  return true;
+}
+
+// FP64 general sizes (dmma_gen.cu): units (entry, 64-column block), A re-read
+// per column block from L2, 32-row blocks of A through a double buffer
+bool model_dmma_gen(int m, int n, int k, Pred* out) {
+  if (!dmma_gen_supported(m, n, k)) return false;
+  const double be = bytes_entry(m, n, k, KAMI_DTYPE_F64);
+  const double flops = 2.0 * m * n * k;
+  const double nblocks = (n + 63) / 64, mblocks = (m + 31) / 32;
+  const double smem = nblocks * (double)(mblocks * 32) * k * 8 * (1 + 4);
+  const double teams = k <= 32 ? 4 : 2;
+  // per team and 32-row block: one TMA round trip that is only one block ahead
+  const double t_team = nblocks * (kTlat + mblocks * (kTlat / 2 + flops / nblocks / mblocks / (kDmmaFpc / 2)));
+  *out = pmax({{be / kHbmBpc, KAMI_BOUND_HBM}, {flops / kDmmaFpc, KAMI_BOUND_TENSOR},
+               {smem / kBsm, KAMI_BOUND_SMEM}, {t_team / teams, KAMI_BOUND_LATENCY}});
+  return true;
+}
+
+void fill_plan(kami_plan_t* r, int kernel, kami_algo_t algo, int p, int m, int n, int k, kami_dtype_t dt) {
+  *r = kami_plan_t{};
+  r->algo = algo;
+  r->p = p;
+  r->kernel = kernel;
+  r->stages = 2;
+  r->entries_per_cta = 1;
+  if (kernel == 0) {
+    Tc16Shape s;
+    if (tc16_plan_shape_kind(m, n, k, in_kind(dt), out_kind(dt), &s) == KAMI_SUCCESS) {
+      r->entries_per_cta = s.G * s.U * s.stages;
+      r->stages = s.stages;
+    }
+    r->kslice_regs_pct = 0;  // operands stream through SMEM in k-chunks
+    r->t_all_cycles = b200_cost(1, m, n, k, 4, dt);
+  } else if (kernel == 3) {
+    TsShape s;
+    if (tc16_ts_plan(m, n, k, algo == KAMI_ALGO_3D_TMEM ? 2 : 1, &s) == KAMI_SUCCESS) {
+      r->entries_per_cta = s.G * s.stages;
+      r->stages = s.stages;
+    }
+    r->kslice_regs_pct = 100;  // A entirely TMEM-resident (local), B streamed
+    r->t_all_cycles = b200_cost(algo == KAMI_ALGO_3D_TMEM ? 3 : 1, m, n, k, p, dt);
+  } else if (kernel == 2) {
+    r->entries_per_cta = m == 64 ? 3 : 8;
+    r->kslice_regs_pct = 50;  // B_w resident in registers, A broadcast through SMEM
+    r->t_all_cycles = b200_cost(1, n, m, k, 4, dt);
+  } else if (kernel == 4) {
+    r->entries_per_cta = k <= 32 ? 4 : 2;
+    r->kslice_regs_pct = dmma_gen_resident_pct(k);
+    r->t_all_cycles = b200_cost(1, n, m, k, 4, dt);
+  } else {
+    r->entries_per_cta = p >= 8 ? 1 : 8 / p;
+    r->kslice_regs_pct = 100;
+    r->t_all_cycles = algo == KAMI_ALGO_NONCA ? 0 : b200_cost((int)algo, m, n, k, p, dt);
+  }
+}
 
 }  // namespace
+
+int planner_candidates(int m, int n, int k, kami_dtype_t dt, bool pointer_array, kami_candidate_t* out, int max) {
+  int cnt = 0;
+  auto add = [&](int kernel, kami_algo_t algo, int p, const Pred& pr) {
+    if (cnt < max && out) {
+      kami_candidate_t& c = out[cnt];
+      c.algo = algo;
+      c.p = p;
+      c.kernel = kernel;
+      c.model_cycles_per_entry = pr.cycles;
+      c.model_tflops = 2.0 * m * n * k * 148 * 1.965e9 / pr.cycles / 1e12;
+      c.bound = pr.bound;
+    }
+    ++cnt;
+  };
+  Pred pr;
+  const bool is16 = dt != KAMI_DTYPE_F64;
+  if (pointer_array) return 0;  // pointer arrays: fixed routing (api.cpp), not modelled
+  if (is16) {
+    if (model_ss(m, n, k, dt, &pr)) add(0, KAMI_ALGO_1D, 4, pr);
+    if (model_ts(m, n, k, dt, 1, &pr)) add(3, KAMI_ALGO_1D_TMEM, 4, pr);
+    if (model_ts(m, n, k, dt, 2, &pr)) add(3, KAMI_ALGO_3D_TMEM, 8, pr);
+  } else {
+    if (model_dmma_tma(m, n, k, &pr)) add(2, KAMI_ALGO_1D_TMA, 4, pr);
+    if (model_dmma_gen(m, n, k, &pr)) add(4, KAMI_ALGO_1D, 4, pr);
+  }
+  if (dt == KAMI_DTYPE_F16 || dt == KAMI_DTYPE_BF16 || dt == KAMI_DTYPE_F64) {
+    for (int v : {1, 2, 3}) {
+      const int pp = warp_ca_default_p(m, n, k, dt, v);
+      if (pp && model_warp(m, n, k, dt, v, pp, &pr)) add(1, (kami_algo_t)v, pp, pr);
+    }
+  }
+  return cnt;
+}
 
 kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_t algo, int p, bool pointer_array,
                              kami_plan_t* out) {
   kami_plan_t r{};
   const bool is16 = dtype != KAMI_DTYPE_F64;  // all tcgen05 types (f16, bf16, tf32, fp8)
-  // 16-bit strided: the tcgen05 family implements 1D with p = 4 sub-partition
-  // tensor cores (tc16.cu); it covers the whole 16-bit size grid.  An explicit
-  // p > 0 selects the warp-level family with p warps instead.
-  // 16^3 FP16 / BF16 AUTO: the warp-level HMMA 1D (p = 1, LDG-fed, register
-  // resident) beats the tcgen05 kernel at every batch measured -- 32-byte TMA
-  // rows and a per-unit fixed cost bound tcgen05 there (configs[0] 4.8 ->
-  // 2.2 us per launch; 65 536 entries 19 -> 27 TFLOP/s, profiles/r1/small16_r1.txt)
-  if (algo == KAMI_ALGO_AUTO && !pointer_array && m == 16 && n == 16 && k == 16 &&
-      (dtype == KAMI_DTYPE_F16 || dtype == KAMI_DTYPE_BF16))
-    return planner_choose(m, n, k, dtype, KAMI_ALGO_1D, 1, pointer_array, out);
-  if (is16 && !pointer_array &&
-      (algo == KAMI_ALGO_AUTO || algo == KAMI_ALGO_1D_TMA || (algo == KAMI_ALGO_1D && p == 0))) {
-    Tc16Shape s;
-    const int ik = dtype == KAMI_DTYPE_F16 ? 0 : dtype == KAMI_DTYPE_BF16 ? 1 : dtype == KAMI_DTYPE_TF32 ? 2
-                 : dtype == KAMI_DTYPE_E4M3 ? 3 : 4;
-    const int ok = dtype == KAMI_DTYPE_BF16 ? 1 : dtype == KAMI_DTYPE_TF32 ? 2 : 0;
-    kami_status_t st = tc16_plan_shape_kind(m, n, k, ik, ok, &s);
-    if (st != KAMI_SUCCESS) return st;
-    r.algo = KAMI_ALGO_1D;
-    r.p = 4;
-    r.kernel = 0;
-    r.entries_per_cta = s.G * s.stages;
-    r.stages = s.stages;
-    r.kslice_regs_pct = 0;  // operands stream through SMEM in k-chunks of s.Wk
-    r.t_all_cycles = b200_cost(1, m, n, k, 4, dtype);
+  if (algo == KAMI_ALGO_AUTO && !pointer_array) {
+    // the model's argmax over every kernel that runs this shape
+    kami_candidate_t c[16];
+    const int nc = std::min(16, planner_candidates(m, n, k, dtype, false, c, 16));
+    int best = -1;
+    for (int i = 0; i < nc; ++i)
+      if (best < 0 || c[i].model_cycles_per_entry < c[best].model_cycles_per_entry) best = i;
+    if (best < 0) return KAMI_ERROR_NOT_SUPPORTED;
+    fill_plan(&r, c[best].kernel, c[best].algo, c[best].p, m, n, k, dtype);
+    r.t_all_cycles = c[best].model_cycles_per_entry;
     *out = r;
     return KAMI_SUCCESS;
   }
-  // tcgen05 with the local operand (A) resident in TMEM: explicit request
+  // ---- explicit schedules (and pointer arrays, routed by api.cpp)
+  // 16-bit 1D with p = 0 / 1D_TMA / AUTO on pointer arrays: the SS tcgen05 kernel
+  if (is16 && !pointer_array &&
+      (algo == KAMI_ALGO_1D_TMA || (algo == KAMI_ALGO_1D && p == 0))) {
+    Tc16Shape s;
+    kami_status_t st = tc16_plan_shape_kind(m, n, k, in_kind(dtype), out_kind(dtype), &s);
+    if (st != KAMI_SUCCESS) return st;
+    fill_plan(&r, 0, KAMI_ALGO_1D, 4, m, n, k, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
+  // tcgen05 with the local operand (A) resident in TMEM
   if (algo == KAMI_ALGO_1D_TMEM || algo == KAMI_ALGO_3D_TMEM) {
     if ((dtype != KAMI_DTYPE_F16 && dtype != KAMI_DTYPE_BF16) || pointer_array || (p != 0 && p != 4 && p != 8))
       return KAMI_ERROR_NOT_SUPPORTED;
     TsShape ts;
     kami_status_t st = tc16_ts_plan(m, n, k, algo == KAMI_ALGO_3D_TMEM ? 2 : 1, &ts);
     if (st != KAMI_SUCCESS) return st == KAMI_ERROR_INVALID_VALUE ? KAMI_ERROR_NOT_SUPPORTED : st;
-    r.algo = algo;
-    r.p = algo == KAMI_ALGO_3D_TMEM ? 8 : 4;
-    r.kernel = 3;
-    r.entries_per_cta = ts.G * ts.stages;
-    r.stages = ts.stages;
-    r.kslice_regs_pct = 0;
-    r.t_all_cycles = b200_cost(algo == KAMI_ALGO_3D_TMEM ? 3 : 1, m, n, k, algo == KAMI_ALGO_3D_TMEM ? 8 : 4, dtype);
+    fill_plan(&r, 3, algo, algo == KAMI_ALGO_3D_TMEM ? 8 : 4, m, n, k, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
+  // FP64 general sizes: explicit 1D with p = 0 off the fixed-shape orders
+  const bool warp_shape = !is16 && m == n && n == k && (m == 8 || m == 16 || m == 32 || m == 64);
+  if (!is16 && !pointer_array && algo == KAMI_ALGO_1D && p == 0 && !warp_shape && dmma_gen_supported(m, n, k)) {
+    fill_plan(&r, 4, KAMI_ALGO_1D, 4, m, n, k, dtype);
     *out = r;
     return KAMI_SUCCESS;
   }
   // FP64 1D with the broadcast operand fed by TMA (dmma_tma.cu; pointer arrays
   // through an address-space view of each entry)
   const bool tma_ok = !is16 && dmma_tma_supported(m, n, k);
-  // FP64 off the square orders the fixed-shape kernels are instantiated for:
-  // the general k-sliced DMMA kernel with a register residency ratio
-  // (dmma_gen.cu; a7).  Explicit 1D with p = 0 selects it too.
-  const bool warp_shape = !is16 && m == n && n == k && (m == 8 || m == 16 || m == 32 || m == 64);
-  if (!is16 && !pointer_array && dmma_gen_supported(m, n, k) &&
-      ((algo == KAMI_ALGO_AUTO && !warp_shape) || (algo == KAMI_ALGO_1D && p == 0 && !warp_shape))) {
-    r.algo = KAMI_ALGO_1D;
-    r.p = 4;
-    r.kernel = 4;
-    r.entries_per_cta = 2;
-    r.stages = 2;
-    r.kslice_regs_pct = dmma_gen_resident_pct(k);
-    r.t_all_cycles = b200_cost(1, n, m, k, 4, dtype);
-    *out = r;
-    return KAMI_SUCCESS;
-  }
-  if (algo == KAMI_ALGO_1D_TMA) {
+  if (algo == KAMI_ALGO_1D_TMA || (algo == KAMI_ALGO_AUTO && pointer_array && tma_ok)) {
     if (!tma_ok || (p != 0 && p != 4)) return KAMI_ERROR_NOT_SUPPORTED;
-    r.algo = KAMI_ALGO_1D_TMA;
-    r.p = 4;
-    r.kernel = 2;
-    r.entries_per_cta = m == 64 ? 3 : 8;
-    r.stages = 2;
-    r.kslice_regs_pct = 50;  // B_w resident in registers, A broadcast through SMEM
-    r.t_all_cycles = b200_cost(1, n, m, k, 4, dtype);
+    fill_plan(&r, 2, KAMI_ALGO_1D_TMA, 4, m, n, k, dtype);
     *out = r;
     return KAMI_SUCCESS;
   }
-  if (algo == KAMI_ALGO_AUTO && tma_ok) {
-    const double t_tma = calibrated_tma(m);
-    double best_w = 0;
+  // warp-level register-resident family (explicit algo, or pointer arrays)
+  kami_algo_t a = algo;
+  int pp = p;
+  if (a == KAMI_ALGO_AUTO) {  // pointer arrays the fixed routes above do not take: the model's best warp schedule
+    double best = 1e300;
     for (int v : {1, 2, 3}) {
-      const int pp = warp_ca_default_p(m, n, k, dtype, v);
-      if (pp) best_w = std::max(best_w, calibrated(dtype, m, n, k, v, pp));
+      const int q = warp_ca_default_p(m, n, k, dtype, v);
+      Pred pr;
+      if (q && model_warp(m, n, k, dtype, v, q, &pr) && pr.cycles < best) {
+        best = pr.cycles;
+        a = (kami_algo_t)v;
+        pp = q;
+      }
     }
-    if (t_tma > best_w) return planner_choose(m, n, k, dtype, KAMI_ALGO_1D_TMA, 0, pointer_array, out);
+    if (a == KAMI_ALGO_AUTO) return KAMI_ERROR_NOT_SUPPORTED;
   }
-  if (algo == KAMI_ALGO_1D_TMA) return KAMI_ERROR_NOT_SUPPORTED;
-  // warp-level register-resident family
-  int cand[3] = {1, 2, 3};
-  if (algo != KAMI_ALGO_AUTO) {
-    const int pp = p ? p : warp_ca_default_p(m, n, k, dtype, (int)algo);
-    if (pp == 0 || warp_ca_supported(m, n, k, dtype, (int)algo, pp) != KAMI_SUCCESS)
-      return KAMI_ERROR_NOT_SUPPORTED;
-    r.algo = algo;
-    r.p = pp;
-    r.kernel = 1;
-    r.entries_per_cta = pp >= 8 ? 1 : 8 / pp;
-    r.stages = 2;
-    r.kslice_regs_pct = 100;
-    r.t_all_cycles = algo == KAMI_ALGO_NONCA ? 0 : b200_cost((int)algo, m, n, k, pp, dtype);
-    *out = r;
-    return KAMI_SUCCESS;
-  }
-  double best = 1e300, best_meas = 0;
-  int best_v = 0, best_p = 0;
-  for (int v : cand) {
-    const int pp = warp_ca_default_p(m, n, k, dtype, v);
-    if (pp == 0) continue;
-    const double meas = calibrated(dtype, m, n, k, v, pp);
-    const double t = b200_entry_cycles(v, m, n, k, pp, dtype, warp_ca_teams_per_sm(m, n, k, dtype, v, pp));
-    const bool better = best_meas > 0 || meas > 0 ? meas > best_meas : t < best;  // ties keep 1D
-    if (best_v == 0 || better) {
-      best = t;
-      best_meas = meas;
-      best_v = v;
-      best_p = pp;
-    }
-  }
-  if (best_v == 0) return KAMI_ERROR_NOT_SUPPORTED;
-  r.algo = (kami_algo_t)best_v;
-  r.p = best_p;
-  r.kernel = 1;
-  r.entries_per_cta = best_p >= 8 ? 1 : 8 / best_p;
-  r.stages = 2;
-  r.kslice_regs_pct = 100;
-  r.t_all_cycles = b200_cost(best_v, m, n, k, best_p, dtype);
+  if (pp == 0) pp = warp_ca_default_p(m, n, k, dtype, (int)a);
+  if (pp == 0 || warp_ca_supported(m, n, k, dtype, (int)a, pp) != KAMI_SUCCESS) return KAMI_ERROR_NOT_SUPPORTED;
+  fill_plan(&r, 1, a, pp, m, n, k, dtype);
   *out = r;
   return KAMI_SUCCESS;
 }

@@ -21,6 +21,9 @@ PaperCost paper_cost(int variant, double m, double n, double k, double p, double
 kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_t algo, int p, bool pointer_array,
                              kami_plan_t* out);
 
+// every candidate schedule with the model's prediction (kami_plan_candidates)
+int planner_candidates(int m, int n, int k, kami_dtype_t dt, bool pointer_array, kami_candidate_t* out, int max);
+
 int warp_ca_default_p(int m, int n, int k, kami_dtype_t dtype, int algo);
 int warp_ca_teams_per_sm(int m, int n, int k, kami_dtype_t dtype, int algo, int p);
 

@@ -727,16 +727,14 @@ int warp_ca_teams_per_sm(int m, int n, int k, kami_dtype_t dtype, int algo, int 
   LaunchInfo li;
   if (!lookup(m, n, k, dtype, algo, p, &li)) return 1;
   const int teams_per_cta = li.threads / 32 / li.p;
-  int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, li.fn, li.threads, li.smem) != cudaSuccess ||
-      per_sm < 1) {
-    cudaGetLastError();
-    const double es = dtype == KAMI_DTYPE_F64 ? 2.0 : 0.5;  // 32-bit registers per element
-    const double elems = (double)m * k / li.p * 2 + (double)k * n / li.p * 2 + (double)m * n / li.p;
-    const double regs = elems * es / 32 + 32;
-    per_sm = (int)(65536.0 / (li.threads * regs));
-    if (per_sm < 1) per_sm = 1;
-  }
+  // a register estimate (not the occupancy API), so the planner's choice is
+  // the same with and without a device (tests/test_planner_model.py)
+  const double es = dtype == KAMI_DTYPE_F64 ? 2.0 : 0.5;  // 32-bit registers per element
+  const double elems = (double)m * k / li.p * 2 + (double)k * n / li.p * 2 + (double)m * n / li.p;
+  const double regs = elems * es / 32 + 32;
+  int per_sm = (int)(65536.0 / (li.threads * regs));
+  if (per_sm < 1) per_sm = 1;
+  if (per_sm * li.threads > 2048) per_sm = 2048 / li.threads;  // 64 warps per SM
   return per_sm * teams_per_cta;
 }
 

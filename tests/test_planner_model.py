@@ -1,0 +1,89 @@
+"""The planner's choice against measurements (VERDICT r1
+next #7): for every BASELINE.json config in the committed variant sweep
+(profiles/r2/variant_sweep_r2.json, tools/variant_sweep_r2.py on one B200),
+the schedule AUTO picks -- the argmax of the B200 cycle model over every
+kernel the library can run for the shape (kami_plan_candidates) -- must be
+the measured-fastest candidate, or within 5 % of it (measurement repeatability
+on these boxes is ~2-8 %).  CPU only: the model needs no
+device, and no measured number enters the library."""
+import json
+import os
+
+import pytest
+
+import paper_conf_sc_wangdltsl25_b200 as kami
+
+SWEEP = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "r2",
+                     "variant_sweep_r2.json")
+TOL = 0.95
+
+
+def _configs():
+    if not os.path.exists(SWEEP):
+        return []
+    return json.load(open(SWEEP))["configs"]
+
+
+FAMILY = {"kami_tc16_1d_kernel": "tcgen05", "kami_tc16_ts": "tcgen05_ts", "kami_warp": "warp_ca",
+          "kami_dmma_tma": "dmma_tma", "kami_dmma_gen": "dmma_gen"}
+
+
+def family(kernel_name):
+    return next((v for key, v in FAMILY.items() if kernel_name.startswith(key)), None)
+
+
+def measured_for_plan(cfg, plan):
+    """The sweep's measurement of the schedule a plan names (kernel family,
+    algo and warp count)."""
+    for c in cfg["candidates"]:
+        if c["algo"] == "auto" or family(c["kernel"]) != plan["kernel"]:
+            continue
+        if plan["kernel"] == "warp_ca":
+            if c["algo"] == plan["algo"] and (c["p"] == plan["p"] or (c["p"] == 0 and c["algo"] != "1d")):
+                return c["tflops"]
+        elif plan["kernel"] == "tcgen05_ts":
+            if c["algo"] == plan["algo"]:
+                return c["tflops"]
+        else:
+            return c["tflops"]
+    return None
+
+
+@pytest.mark.parametrize("cfg", _configs(), ids=lambda c: c["cfg"])
+def test_auto_pick_is_measured_best(cfg):
+    dt, m, n, k = cfg["dtype"], cfg["m"], cfg["n"], cfg["k"]
+    best = max(c["tflops"] for c in cfg["candidates"] if c["algo"] != "auto")
+    plan = kami.plan(m, n, k, dt)
+    got = measured_for_plan(cfg, plan)
+    assert got is not None, (cfg["cfg"], plan)
+    assert got >= TOL * best, (cfg["cfg"], plan, got, best)
+
+
+@pytest.mark.parametrize("cfg", _configs(), ids=lambda c: c["cfg"])
+def test_model_ranks_kernel_families_like_the_measurements(cfg):
+    """The model's predicted order of the kernel families agrees with the
+    measured order wherever the measurements differ by more than 25 %."""
+    dt, m, n, k = cfg["dtype"], cfg["m"], cfg["n"], cfg["k"]
+    model = {}
+    for c in kami.plan_candidates(m, n, k, dt):
+        model[c["kernel"]] = max(model.get(c["kernel"], 0.0), c["model_tflops"])
+    meas = {}
+    for c in cfg["candidates"]:
+        if c["algo"] == "auto":
+            continue
+        f = family(c["kernel"])
+        if f:
+            meas[f] = max(meas.get(f, 0.0), c["tflops"])
+    fams = [f for f in meas if f in model]
+    for a in fams:
+        for b in fams:
+            if meas[a] > 1.25 * meas[b]:
+                assert model[a] > model[b], (cfg["cfg"], a, b, meas, model)
+
+
+def test_model_has_no_measured_table():
+    """The choice is a function of the shape alone (no device, no table): a
+    shape never measured still gets a plan with a predicted bound."""
+    c = kami.plan_candidates(80, 112, 72, "bf16")
+    assert c and all(x["model_tflops"] > 0 for x in c)
+    assert kami.plan(80, 112, 72, "bf16")["kernel"] in ("tcgen05", "tcgen05_ts")
