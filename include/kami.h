@@ -19,11 +19,11 @@
  *     KAMI_ROW_MAJOR: X_b(r, c) at  X + b*R*C + r*C + c
  *     KAMI_COL_MAJOR: X_b(r, c) at  X + b*R*C + c*R + r
  *
- * Sizes supported (R5): 16-bit types need m, n multiples of 16 in
- * [16, 256] and k a multiple of 8 in [8, 256]; TF32 the same with k a
- * multiple of 4; FP8 m, n multiples of 32 and k of 16 (all <= 256); FP64
- * m = n = k in {8, 16, 32, 64}.  Anything else returns
- * KAMI_ERROR_NOT_SUPPORTED.
+ * Sizes supported (R5): 16-bit and FP64 types: m, n, k multiples
+ * of 8 in [8, 256] (the SURVEY.md 8(b) grid); TF32 m, n multiples of 16, k of
+ * 4; FP8 m, n multiples of 32 and k of 16 (all <= 256).  Anything else
+ * returns KAMI_ERROR_NOT_SUPPORTED.  Some entry points narrow this (the
+ * update form, pointer arrays of FP64, SpMM): see each declaration.
  *
  * Ownership and threading: the caller owns every buffer.  Device entry points
  * never allocate device memory, never synchronise and enqueue on `stream`
@@ -110,7 +110,9 @@ kami_status_t kami_gemm(int m, int n, int k, int64_t batch, kami_dtype_t dtype, 
  * misaligned entry pointer cannot be detected before launch (the arrays are
  * device memory): its result is undefined.  16-bit types run on the same
  * tcgen05 kernel as the strided form, fed by TMA boxes over an address-space
- * view of each entry. */
+ * view of each entry; m or n = 8 mod 16 on the LDG-fed
+ * tcgen05 kernel.  FP64 pointer arrays: m = n = k in {8, 16, 32, 64} only
+ * (NOT_SUPPORTED otherwise: the general FP64 kernel is strided). */
 kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
                                 const void* const* A_array, const void* const* B_array, void* const* C_array,
                                 kami_stream_t stream);
@@ -199,7 +201,8 @@ typedef struct {
   int p;                 /* warps (or tensor-core sub-partitions) per entry */
   int kernel;            /* 0 = tcgen05 16-bit (SS), 1 = warp-level DMMA/HMMA, 2 = FP64 DMMA with TMA
                             broadcast, 3 = tcgen05 16-bit with A resident in TMEM (TS), 4 = FP64 DMMA
-                            for the whole size grid (k-sliced, register residency ratio) */
+                            for the whole size grid (k-sliced, register residency ratio), 5 = LDG-fed
+                            tcgen05 16-bit (m or n = 8 mod 16) */
   int entries_per_cta;   /* batch entries a CTA keeps in flight             */
   int stages;            /* shared-memory pipeline depth                    */
   int kslice_regs_pct;   /* share of A/B kept resident (Sec. 4.7)           */

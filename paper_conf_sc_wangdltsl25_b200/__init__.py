@@ -58,7 +58,7 @@ class KamiCandidate(ctypes.Structure):
 
 
 BOUND = {0: "hbm", 1: "tensor", 2: "smem", 3: "tma", 4: "issue", 5: "latency"}
-KERNEL = {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma", 3: "tcgen05_ts", 4: "dmma_gen"}
+KERNEL = {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma", 3: "tcgen05_ts", 4: "dmma_gen", 5: "tcgen05_ldg"}
 
 _lib = None
 

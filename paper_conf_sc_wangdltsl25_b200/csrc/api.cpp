@@ -50,7 +50,7 @@ bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) ==
 // Size grid (R5).  Checked before anything touches the device.
 kami_status_t check_sizes(int m, int n, int k, kami_dtype_t dtype) {
   if (m > 256 || n > 256 || k > 256) return KAMI_ERROR_NOT_SUPPORTED;
-  if (is16(dtype)) return (m % 16 || n % 16 || k % 8) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
+  if (is16(dtype)) return (m % 8 || n % 8 || k % 8) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
   if (dtype == KAMI_DTYPE_TF32) return (m % 16 || n % 16 || k % 4) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
   if (dtype == KAMI_DTYPE_E4M3 || dtype == KAMI_DTYPE_E5M2)
     return (m % 32 || n % 32 || k % 16) ? KAMI_ERROR_NOT_SUPPORTED : KAMI_SUCCESS;
@@ -116,7 +116,7 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
                           rp.B, C, rp.Aa, rp.Ba, Ca, stream);
   if (Ca && is16(dtype) && algo == KAMI_ALGO_AUTO) {
     // the TMA kernel over address-space views (tc16.cu kPtr), else the LDG-fed one
-    if (route != 2) {
+    if (route != 2 && rp.m % 16 == 0 && rp.n % 16 == 0) {
       kami_status_t st = tc16_launch_kind(rp.m, rp.n, rp.k, batch, in_kind(dtype), out_kind(dtype), nullptr,
                                           nullptr, nullptr, 1.0f, 0.0f, stream, 0, rp.Aa, rp.Ba, Ca);
       if (st != KAMI_ERROR_NOT_SUPPORTED) return st;
@@ -127,6 +127,10 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
+  if (plan.kernel == 5) {  // 16-bit m or n = 8 mod 16: the LDG-fed tcgen05 kernel on packed entries
+    if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
+    return tc16_vb_strided_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream);
+  }
   if (plan.kernel == 4) {  // FP64 general sizes: k-sliced DMMA with a residency ratio (strided C = A B)
     if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
     return dmma_gen_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream);

@@ -96,6 +96,10 @@ kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, co
                              const int* dk, int max_m, int max_n, const void* const* A, const void* const* B,
                              void* const* C, cudaStream_t stream);
 
+// strided batches with m or n = 8 mod 16 (16-bit): the same LDG-fed kernel on packed entries
+kami_status_t tc16_vb_strided_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B,
+                                     void* C, cudaStream_t stream);
+
 // SpMM: block-sparse A (BSR, 16x16 blocks) x dense B on tcgen05 (densify on load)
 kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf16, const int* row_ptr,
                                    const int* col_blk, const void* vals, int max_nnzb, const void* B, void* C,

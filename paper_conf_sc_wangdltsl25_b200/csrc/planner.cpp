@@ -159,6 +159,26 @@ bool model_ts(int m, int n, int k, kami_dtype_t dt, int layers, Pred* out) {
   return true;
 }
 
+// LDG-fed tcgen05 (tc16_vb.cu) for 16-bit m or n = 8 mod 16: the same
+// schedule with the operands copied by a producer warpgroup (16-byte
+// cp.async); per unit max(HBM, the copy issue of the unit's 16-byte chunks,
+// the SS unit cost); kVbChunk cycles per 16-byte chunk per SM (128 producer
+// threads, one LDGSTS each per ~4 cycles -> 0.125 cycle per chunk, x2 for the
+// zero-fill / swizzle address math), i.e. ~64 B/cycle of copy issue
+constexpr double kVbChunk = 0.25;
+bool model_vb(int m, int n, int k, kami_dtype_t dt, Pred* out) {
+  if ((dt != KAMI_DTYPE_F16 && dt != KAMI_DTYPE_BF16) || (m % 16 == 0 && n % 16 == 0)) return false;
+  const int g1 = m > 128 ? 1 : 128 / m, g2 = 256 / n;
+  const double G = m > 128 ? 1.0 / ((m + 127) / 128) : (double)std::max(1, std::min(g1, g2));
+  const double be = bytes_entry(m, n, k, dt);
+  const double t_hbm = G * be / kHbmBpc;
+  const double t_copy = G * (double)(m * k + k * n) * 2 / 16 * kVbChunk + G * (double)m * n * 2 / 16 * kVbChunk;
+  Pred p = pmax({{t_hbm, KAMI_BOUND_HBM}, {t_copy, KAMI_BOUND_ISSUE}, {kUnitSS, KAMI_BOUND_ISSUE}});
+  p.cycles /= G;
+  *out = p;
+  return true;
+}
+
 // register-resident warp teams (warp_ca.cu): a team loads its entry with its
 // own LDGs (one round trip to L2, where its previous entry prefetched it),
 // runs the CA schedule (T_all of Eqs. 4/8/12 with B200 constants + the
@@ -237,6 +257,10 @@ void fill_plan(kami_plan_t* r, int kernel, kami_algo_t algo, int p, int m, int n
     r->entries_per_cta = m == 64 ? 3 : 8;
     r->kslice_regs_pct = 50;  // B_w resident in registers, A broadcast through SMEM
     r->t_all_cycles = b200_cost(1, n, m, k, 4, dt);
+  } else if (kernel == 5) {
+    r->entries_per_cta = 1;
+    r->kslice_regs_pct = 0;
+    r->t_all_cycles = b200_cost(1, m, n, k, 4, dt);
   } else if (kernel == 4) {
     r->entries_per_cta = k <= 32 ? 4 : 2;
     r->kslice_regs_pct = dmma_gen_resident_pct(k);
@@ -268,6 +292,7 @@ int planner_candidates(int m, int n, int k, kami_dtype_t dt, bool pointer_array,
   const bool is16 = dt != KAMI_DTYPE_F64;
   if (pointer_array) return 0;  // pointer arrays: fixed routing (api.cpp), not modelled
   if (is16) {
+    if (model_vb(m, n, k, dt, &pr)) add(5, KAMI_ALGO_1D, 4, pr);
     if (model_ss(m, n, k, dt, &pr)) add(0, KAMI_ALGO_1D, 4, pr);
     if (model_ts(m, n, k, dt, 1, &pr)) add(3, KAMI_ALGO_1D_TMEM, 4, pr);
     if (model_ts(m, n, k, dt, 2, &pr)) add(3, KAMI_ALGO_3D_TMEM, 8, pr);
@@ -302,6 +327,13 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
     return KAMI_SUCCESS;
   }
   // ---- explicit schedules (and pointer arrays, routed by api.cpp)
+  // 16-bit m or n = 8 mod 16: the LDG-fed tcgen05 kernel is the tcgen05 1D there
+  if ((dtype == KAMI_DTYPE_F16 || dtype == KAMI_DTYPE_BF16) && !pointer_array && (m % 16 || n % 16) &&
+      (algo == KAMI_ALGO_1D && p == 0)) {
+    fill_plan(&r, 5, KAMI_ALGO_1D, 4, m, n, k, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
   // 16-bit 1D with p = 0 / 1D_TMA / AUTO on pointer arrays: the SS tcgen05 kernel
   if (is16 && !pointer_array &&
       (algo == KAMI_ALGO_1D_TMA || (algo == KAMI_ALGO_1D && p == 0))) {

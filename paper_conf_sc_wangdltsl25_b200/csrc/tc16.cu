@@ -892,6 +892,9 @@ void launch_kernel(const Tc16Params& p, unsigned grid, size_t smem, cudaStream_t
 
 kami_status_t tc16_plan_shape_kind(int m, int n, int k, int in_kind, int out_kind, Tc16Shape* s, bool no_tp) {
   const int esi = in_es(in_kind), eso = out_es(out_kind);
+  // m, n multiples of 16 (TMEM lane groups / swizzle atoms of whole 16-element
+  // rows); 8 mod 16 goes to the LDG-fed kernel (tc16_vb.cu)
+  if (m % 16 || n % 16) return KAMI_ERROR_NOT_SUPPORTED;
   s->G = 1;
   if (m <= 128) {
     int g1 = 128 / m, g2 = 256 / n;

@@ -69,13 +69,17 @@ struct alignas(64) VbParams {
   const uint16_t* Bs;
   uint16_t* Cs;
   int dbg;  // experiments only (env KAMI_VB_DEBUG): 1 = skip C stores, 2 = skip A/B copies
+  // strided batches whose m or n is 8 mod 16 (no TMA tile for them; R5):
+  // entry e at As + e m k, Bs + e k n, Cs + e m n
+  int strided;
+  const uint16_t* As;
 };
 
 __device__ __forceinline__ const uint16_t* entry_B(const VbParams& p, long long e, int k, int n) {
-  return p.bsr ? p.Bs + e * (long long)k * n : reinterpret_cast<const uint16_t*>(p.B[e]);
+  return (p.bsr || p.strided) ? p.Bs + e * (long long)k * n : reinterpret_cast<const uint16_t*>(p.B[e]);
 }
 __device__ __forceinline__ uint16_t* entry_C(const VbParams& p, long long e, int m, int n) {
-  return p.bsr ? p.Cs + e * (long long)m * n : reinterpret_cast<uint16_t*>(p.C[e]);
+  return (p.bsr || p.strided) ? p.Cs + e * (long long)m * n : reinterpret_cast<uint16_t*>(p.C[e]);
 }
 __device__ __forceinline__ void entry_dims(const VbParams& p, long long e, int& m, int& n, int& k) {
   if (p.dm) {
@@ -194,8 +198,10 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       S.rp = 0;
       if (one || tid < S.U.ng) {
         const long long e = S.U.e0 + (one ? 0 : tid);
-        S.pa = p.bsr ? nullptr : reinterpret_cast<const uint16_t*>(p.A[e]);
-        S.pb = p.bsr ? p.Bs + e * (long long)p.k * p.n : reinterpret_cast<const uint16_t*>(p.B[e]);
+        S.pa = p.bsr ? nullptr
+               : p.strided ? p.As + e * (long long)p.m * p.k
+                           : reinterpret_cast<const uint16_t*>(p.A[e]);
+        S.pb = (p.bsr || p.strided) ? p.Bs + e * (long long)p.k * p.n : reinterpret_cast<const uint16_t*>(p.B[e]);
       }
       if (p.bsr) {
 #pragma unroll
@@ -369,7 +375,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       if (p.dbg & 4) trace(6, acc_it);
       ptx::tc_fence_after();
       const uint32_t d_tmem = tmem_base + a * p.acc_cols;
-      const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, p.G * U.n, 0, 1);
+      // N of the MMA: the tile's G n live columns rounded up to the M = 128 granule of
+      // 16 (n = 8 mod 16: the pad columns' products are never stored)
+      const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, (p.G * U.n + 15) & ~15, 0, 1);
       const int kpad = (U.k + 15) / 16 * 16;
       const int kchunks = (U.k + 63) / 64;
       for (int kc = 0; kc < kchunks; ++kc, rs.next(p.stages), ++it) {
@@ -444,8 +452,15 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
             for (int c0 = 0; c0 < hw; c0 += 32) {
               uint32_t v[32];
               const uint32_t col = (uint32_t)(gg * n + h0 + c0);
-              if (hw - c0 >= 32) ptx::tmem_ld_32x32b_x32(t_row + col, v);
-              else ptx::tmem_ld_32x32b_x16(t_row + col, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
+              const int rem = hw - c0;  // multiple of 8
+              if (rem >= 32) {
+                ptx::tmem_ld_32x32b_x32(t_row + col, v);
+              } else if (rem >= 16) {
+                ptx::tmem_ld_32x32b_x16(t_row + col, *reinterpret_cast<uint32_t(*)[16]>(&v[0]));
+                if (rem >= 24) ptx::tmem_ld_32x32b_x8(t_row + col + 16, &v[16]);
+              } else {
+                ptx::tmem_ld_32x32b_x8(t_row + col, &v[0]);
+              }
               ptx::tmem_wait_ld();
               if (row_ok && g == gg) {
 #pragma unroll
@@ -542,6 +557,10 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
     while (grid > 1 && std::gcd(grid, (long long)p.mtiles) != 1) --grid;
   grid = apply_grid_cap(grid);
   fn<<<(unsigned)grid, kVbThreads, smem, stream>>>(p);
+  if (p.strided) {
+    set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16,strided>" : "kami_tc16_vb_kernel<f16,strided>");
+    return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+  }
   set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
                         : (bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>"));
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
@@ -591,6 +610,22 @@ kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf
   p.vals = static_cast<const uint16_t*>(vals);
   p.Bs = static_cast<const uint16_t*>(B);
   p.Cs = static_cast<uint16_t*>(C);
+  return vb_launch(p, bf16, n, m, stream);
+}
+
+kami_status_t tc16_vb_strided_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B,
+                                     void* C, cudaStream_t stream) {
+  VbParams p;
+  memset(&p, 0, sizeof(p));
+  p.strided = 1;
+  p.As = static_cast<const uint16_t*>(A);
+  p.Bs = static_cast<const uint16_t*>(B);
+  p.Cs = static_cast<uint16_t*>(C);
+  p.m = m;
+  p.n = n;
+  p.k = k;
+  p.batch = batch;
+  p.G = packing(m, n);
   return vb_launch(p, bf16, n, m, stream);
 }
 

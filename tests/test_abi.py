@@ -48,7 +48,8 @@ FAKE = 0x10000  # never dereferenced: every case below fails validation first
     ((16, 16, 16, -1, 0, 0), INVALID),     # batch < 0
     ((16, 16, 16, 1, 7, 0), INVALID),      # unknown dtype
     ((16, 16, 16, 1, 0, 5), INVALID),      # unknown layout
-    ((24, 16, 16, 1, 0, 0), UNSUP),        # 16-bit m not a multiple of 16
+    ((20, 16, 16, 1, 0, 0), UNSUP),        # 16-bit m not a multiple of 8
+    ((16, 12, 16, 1, 1, 0), UNSUP),        # 16-bit n not a multiple of 8
     ((16, 16, 12, 1, 0, 0), UNSUP),        # 16-bit k not a multiple of 8
     ((272, 16, 16, 1, 0, 0), UNSUP),       # > 256
     ((44, 48, 48, 1, 2, 0), UNSUP),        # fp64 m not a multiple of 8
