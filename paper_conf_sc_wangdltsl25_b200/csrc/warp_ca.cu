@@ -693,6 +693,27 @@ bool lookup(int m, int n, int k, kami_dtype_t dtype, int algo, int p, LaunchInfo
   // FP16 / BF16 HMMA (m16n8k16): CA evidence family
   KAMI_CASE(H16, KAMI_DTYPE_F16, 16, 16, 16, 1, Sched1D, 1, "kami_warp_ca_1d<f16,16>")
   KAMI_CASE(B16, KAMI_DTYPE_BF16, 16, 16, 16, 1, Sched1D, 1, "kami_warp_ca_1d<bf16,16>")
+  // thin tiles (m or n = 16, k <= 32) where the tcgen05 unit is mostly empty:
+  // one warp per entry, register resident (BF16 sweep's slowest points)
+#define KAMI_THIN_CASES(MM, NN, KK)                                                                 \
+  KAMI_CASE(H16, KAMI_DTYPE_F16, MM, NN, KK, 1, Sched1D, 1, "kami_warp_ca_1d<f16," #MM "x" #NN "x" #KK ">") \
+  KAMI_CASE(B16, KAMI_DTYPE_BF16, MM, NN, KK, 1, Sched1D, 1, "kami_warp_ca_1d<bf16," #MM "x" #NN "x" #KK ">")
+  KAMI_THIN_CASES(16, 64, 16)
+  KAMI_THIN_CASES(16, 128, 16)
+  KAMI_THIN_CASES(16, 192, 16)
+  KAMI_THIN_CASES(16, 128, 32)
+  KAMI_THIN_CASES(32, 128, 16)
+  KAMI_THIN_CASES(64, 16, 16)
+  KAMI_THIN_CASES(128, 16, 16)
+  KAMI_THIN_CASES(192, 16, 16)
+  KAMI_THIN_CASES(128, 32, 16)
+  KAMI_THIN_CASES(16, 32, 16)
+  KAMI_THIN_CASES(32, 16, 16)
+  KAMI_THIN_CASES(16, 256, 16)
+  KAMI_THIN_CASES(256, 16, 16)
+  KAMI_THIN_CASES(16, 192, 32)
+  KAMI_THIN_CASES(192, 16, 32)
+  KAMI_THIN_CASES(16, 16, 32)
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 1, Sched1D, 2, "kami_warp_ca_1d<f16,32>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 2, Sched2D, 4, "kami_warp_ca_2d<f16,32>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 4, SchedNonCA, 4, "kami_warp_nonca<f16,32>")

@@ -43,6 +43,24 @@ CONFIGS = [
     ("c4 bf16-192", "bf16", 192, 192, 192, 20000),
     ("c4 bf16-16x128x16", "bf16", 16, 128, 16, 125000),
     ("c4 f64-128 (a7)", "f64", 128, 128, 128, 8192),
+    # the BF16 sweep's slowest r1 points (thin m / n, k <= 32)
+    ("c4 bf16-16x192x16", "bf16", 16, 192, 16, 125000),
+    ("c4 bf16-192x16x16", "bf16", 192, 16, 16, 125000),
+    ("c4 bf16-16x64x16", "bf16", 16, 64, 16, 125000),
+    ("c4 bf16-16x128x32", "bf16", 16, 128, 32, 125000),
+    ("c4 bf16-16x32x16", "bf16", 16, 32, 16, 125000),
+    ("c4 bf16-16x256x16", "bf16", 16, 256, 16, 125000),
+    ("c4 bf16-128x16x16", "bf16", 128, 16, 16, 125000),
+    ("c4 bf16-32x128x16", "bf16", 32, 128, 16, 125000),
+    ("c4 bf16-64x16x16", "bf16", 64, 16, 16, 125000),
+    ("c4 bf16-32x16x16", "bf16", 32, 16, 16, 125000),
+    ("c4 bf16-256x16x16", "bf16", 256, 16, 16, 125000),
+    ("c4 bf16-16x192x32", "bf16", 16, 192, 32, 125000),
+    ("c4 bf16-192x16x32", "bf16", 192, 16, 32, 125000),
+    ("c4 bf16-16x16x32", "bf16", 16, 16, 32, 125000),
+    ("c4 bf16-128x32x16", "bf16", 128, 32, 16, 125000),
+    ("c4 bf16-40x24x56 (8-grid)", "bf16", 40, 24, 56, 125000),
+    ("c4 f64-96x40x72 (a7)", "f64", 96, 40, 72, 32768),
 ]
 
 # candidate schedules: (algo, p); the library rejects the ones a shape has no kernel for
