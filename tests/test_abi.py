@@ -94,14 +94,19 @@ def test_plan_host_logic():
 
 
 def test_plan_covers_the_16bit_grid():
-    for m in (16, 32, 48, 64, 128, 192, 256):
-        for n in (16, 64, 256):
+    """Every shape of the 16-bit grid has a plan; AUTO is the model's pick (a
+    tcgen05 kernel or, for some thin tiles, the one-warp register-resident 1D),
+    and 1D with p = 0 always names the tcgen05 kernel of the shape."""
+    for m in (8, 16, 24, 32, 48, 64, 128, 192, 256):
+        for n in (8, 16, 40, 64, 256):
             for k in (8, 16, 40, 64, 256):
                 p = kami.plan(m, n, k, "bf16")
-                if (m, n, k) == (16, 16, 16):  # planner rule: warp-level HMMA 1D, p = 1
-                    assert p["kernel"] == "warp_ca" and p["algo"] == "1d" and p["p"] == 1
-                    p = kami.plan(m, n, k, "bf16", algo="1d")  # 1D with p = 0: tcgen05
-                assert p["kernel"] == "tcgen05" and p["stages"] >= 2, (m, n, k)
+                assert p["kernel"] in ("tcgen05", "tcgen05_ts", "tcgen05_ldg", "warp_ca"), (m, n, k, p)
+                if p["kernel"] == "warp_ca":
+                    assert p["algo"] == "1d" and p["p"] == 1, (m, n, k, p)
+                q = kami.plan(m, n, k, "bf16", algo="1d")  # 1D with p = 0: the tcgen05 family
+                want = "tcgen05" if m % 16 == 0 and n % 16 == 0 else "tcgen05_ldg"
+                assert q["kernel"] == want and q["stages"] >= 2, (m, n, k, q)
 
 
 def test_plan_ring_depth_rules():
