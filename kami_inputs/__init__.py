@@ -198,3 +198,28 @@ def bsr_operands(m: int, n: int, k: int, batch: int, dtype: str, density: float 
     vals[eidx, slot.to(torch.int64)] = v.view(-1, BLK, BLK).to(TORCH_DTYPES[dtype])
     _, B = operands(m, n, k, batch, dtype, dist, seed=seed, entry0=entry0, device=device)
     return row_ptr, col_blk, vals, B
+
+
+def block_sparse(m: int, k: int, batch: int, dtype: str, density: float = 0.5, dist: str = "unif", seed: int = 0,
+                 entry0: int = 0):
+    """The block-sparse matrices of bsr_operands as a dense block description
+    (no storage format): present [batch, m/16, k/16] bool and blocks [batch,
+    m/16, k/16, 16, 16] of ``dtype`` (zero where absent), drawn with the same
+    keys, so bsr_operands(...) and any other storage built from these hold
+    the same matrices.  CPU only."""
+    assert m % BLK == 0 and k % BLK == 0
+    mb, kb = m // BLK, k // BLK
+    nb = mb * kb
+    ids = torch.arange(batch * nb, dtype=torch.int64) + entry0 * nb
+    u = _lshr(_key(seed, 0, ids), 11).to(torch.float64) * (2.0 ** -53)
+    present = (u < density).view(batch, mb, kb)
+    el = torch.arange(BLK * BLK, dtype=torch.int64)
+    zz = _key(seed, 1, ids.unsqueeze(1) * (BLK * BLK) + el.unsqueeze(0))
+    if dist == "unif":
+        v = _lshr(zz, 11).to(torch.float64) * (2.0 ** -52) - 1.0
+    else:
+        R = int_range(k, dtype)
+        v = (torch.remainder(_lshr(zz, 33), 2 * R + 1) - R).to(torch.float64)
+    blocks = v.view(batch, mb, kb, BLK, BLK).to(TORCH_DTYPES[dtype])
+    blocks[~present] = 0
+    return present, blocks

@@ -200,6 +200,65 @@ def spmm_bsr(m: int, n: int, k: int, batch: int, dtype: str, row_ptr, col_blk, v
     return (C, S) if with_scale else C
 
 
+def morton_encode(i: int, j: int) -> int:
+    """Z-Morton code of block (row i, column j) (oracle.c, Sec. 4.6)."""
+    L = lib()
+    L.oracle_morton_encode.restype = ctypes.c_int
+    L.oracle_morton_encode.argtypes = [ctypes.c_int, ctypes.c_int]
+    return int(L.oracle_morton_encode(i, j))
+
+
+def morton_decode(z: int) -> tuple:
+    L = lib()
+    L.oracle_morton_decode.restype = None
+    L.oracle_morton_decode.argtypes = [ctypes.c_int, ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.c_int)]
+    a, b = ctypes.c_int(), ctypes.c_int()
+    L.oracle_morton_decode(z, ctypes.byref(a), ctypes.byref(b))
+    return a.value, b.value
+
+
+def zmorton_from_blocks(present: np.ndarray, blocks: np.ndarray):
+    """Z-Morton block storage of a batch of block-sparse matrices, built from
+    the dense block description: present [batch, mb, kb] bool, blocks [batch,
+    mb, kb, 16, 16] (any dtype).  Returns (nnzb [batch] int32, zcode [batch,
+    max_nnzb] int32 ascending, -1 padded, vals [batch, max_nnzb, 16, 16]) with
+    max_nnzb = mb kb.  Plain loops: the oracle's encoder, independent of the
+    library's decoder."""
+    present = np.asarray(present, dtype=bool)
+    batch, mb, kb = present.shape
+    nnzb = np.zeros(batch, dtype=np.int32)
+    zcode = np.full((batch, mb * kb), -1, dtype=np.int32)
+    vals = np.zeros((batch, mb * kb) + blocks.shape[3:], dtype=blocks.dtype)
+    for b in range(batch):
+        items = sorted((morton_encode(i, j), i, j) for i in range(mb) for j in range(kb) if present[b, i, j])
+        nnzb[b] = len(items)
+        for s, (z, i, j) in enumerate(items):
+            zcode[b, s] = z
+            vals[b, s] = blocks[b, i, j]
+    return nnzb, zcode, vals
+
+
+def spmm_zmorton(m: int, n: int, k: int, batch: int, dtype: str, nnzb, zcode, vals, B, blk: int = 16,
+                 with_scale: bool = False):
+    """C_ref = A B for A in Z-Morton block storage (decoded block by block,
+    densified, then the plain GEMM definition).  Returns [batch, m, n]."""
+    L = lib()
+    L.oracle_spmm_zmorton.restype = ctypes.c_int
+    L.oracle_spmm_zmorton.argtypes = [ctypes.c_int] * 4 + [ctypes.c_int64, ctypes.c_int] + [ctypes.c_void_p] * 3 + \
+        [ctypes.c_int] + [ctypes.c_void_p] * 3
+    nz = np.ascontiguousarray(np.asarray(nnzb), dtype=np.int32).reshape(-1)
+    zc = np.ascontiguousarray(np.asarray(zcode), dtype=np.int32).reshape(batch, -1)
+    v = _raw(np.asarray(vals).reshape(-1), dtype)
+    b = _raw(np.asarray(B).reshape(-1), dtype)
+    C = np.empty((batch, m, n), dtype=np.float64)
+    S = np.empty((batch, m, n), dtype=np.float64) if with_scale else None
+    rc = L.oracle_spmm_zmorton(m, n, k, blk, batch, DTYPES[dtype], nz.ctypes.data, zc.ctypes.data, v.ctypes.data,
+                               zc.shape[1], b.ctypes.data, C.ctypes.data, S.ctypes.data if S is not None else None)
+    if rc != 0:
+        raise ValueError(f"oracle_spmm_zmorton rejected its arguments ({rc})")
+    return (C, S) if with_scale else C
+
+
 def axpby(C_ref: np.ndarray, C_in: np.ndarray, alpha: float, beta: float) -> np.ndarray:
     """alpha * C_ref + beta * C_in in binary64 (the C-update form, DESIGN.md f4)."""
     out = np.ascontiguousarray(C_ref, dtype=np.float64).copy()

@@ -286,6 +286,65 @@ int oracle_spmm_bsr(int m, int n, int k, int blk, int64_t batch, int dtype, cons
   return rc;
 }
 
+/* ---------------------------------------- multi-level Z-Morton block order
+ * PAPER.md Sec. 4.6 L409 (Fig. 7(b)): for the 2D / 3D algorithms the dense
+ * 16 x 16 blocks of a sparse matrix are stored in a multi-level Z-Morton
+ * order.  Reading (R31): the Z curve visits, at every level, the
+ * top-left, top-right, bottom-left, bottom-right quadrant, i.e. the code of
+ * block (block row i, block column j) interleaves the bits of j (even bit
+ * positions) and i (odd positions):  z = sum_t j_t 2^(2t) + i_t 2^(2t+1).
+ * Every aligned 2^L x 2^L submatrix is then one contiguous code range, at
+ * every level L -- the "efficient submatrix indexing".  Written bit by bit. */
+int oracle_morton_encode(int i, int j) {
+  int z = 0;
+  for (int t = 0; t < 15; ++t) {
+    z |= ((j >> t) & 1) << (2 * t);
+    z |= ((i >> t) & 1) << (2 * t + 1);
+  }
+  return z;
+}
+void oracle_morton_decode(int z, int* i, int* j) {
+  int a = 0, b = 0;
+  for (int t = 0; t < 15; ++t) {
+    b |= ((z >> (2 * t)) & 1) << t;
+    a |= ((z >> (2 * t + 1)) & 1) << t;
+  }
+  *i = a;
+  *j = b;
+}
+
+/* SpMM with A in Z-Morton block storage: entry b holds nnzb[b] blocks, the
+ * j-th with Morton code zcode[b * max_nnzb + j] and values
+ * vals[(b * max_nnzb + j) * blk * blk ...] (row-major block).  A is densified
+ * (absent blocks are zero), then the plain GEMM definition. */
+int oracle_spmm_zmorton(int m, int n, int k, int blk, int64_t batch, int dtype, const int* nnzb, const int* zcode,
+                        const void* vals, int max_nnzb, const void* B, double* C, double* S) {
+  if (m <= 0 || n <= 0 || k <= 0 || blk <= 0 || batch < 0 || m % blk || k % blk) return 1;
+  double* Ad = (double*)malloc(sizeof(double) * (size_t)m * k);
+  double* Bd = (double*)malloc(sizeof(double) * (size_t)k * n);
+  if (!Ad || !Bd) return 2;
+  int rc = 0;
+  for (int64_t b = 0; b < batch && rc == 0; ++b) {
+    memset(Ad, 0, sizeof(double) * (size_t)m * k);
+    if (nnzb[b] < 0 || nnzb[b] > max_nnzb) { rc = 3; break; }
+    for (int j = 0; j < nnzb[b]; ++j) {
+      int bi, bj;
+      oracle_morton_decode(zcode[b * max_nnzb + j], &bi, &bj);
+      if ((bi + 1) * blk > m || (bj + 1) * blk > k) { rc = 3; break; }
+      for (int r = 0; r < blk; ++r)
+        for (int c = 0; c < blk; ++c)
+          Ad[(size_t)(bi * blk + r) * k + bj * blk + c] =
+              load_elem(vals, dtype, (b * max_nnzb + j) * (int64_t)blk * blk + r * blk + c);
+    }
+    for (int64_t t = 0; t < (int64_t)k * n; ++t) Bd[t] = load_elem(B, dtype, b * (int64_t)k * n + t);
+    rc = rc ? rc : oracle_gemm(m, n, k, 1, ORACLE_F64, ORACLE_ROW, Ad, Bd, C + b * (int64_t)m * n,
+                               S ? S + b * (int64_t)m * n : NULL, 1);
+  }
+  free(Ad);
+  free(Bd);
+  return rc;
+}
+
 /* ------------------------------------------------- alpha A B + beta C_in
  * The GEMM-update form the algorithms' GMem2Reg(C_i <- C) implies (Alg. 1-3
  * load C, R1/f4):  C_ref = alpha * (A B)_ref + beta * C_in, both

@@ -84,3 +84,51 @@ def test_generator_density_and_sorting():
         for i in range(8):
             cols = cb[b, rp[b, i]:rp[b, i + 1]].tolist()
             assert cols == sorted(cols) and len(set(cols)) == len(cols)
+
+
+# ------------------------------------------------ Z-Morton block storage (f3)
+# PAPER.md Sec. 4.6, Fig. 7(b): "a multi-level Z-Morton order is
+# implemented to facilitate efficient submatrix indexing" (R31).
+
+
+def test_morton_order_of_a_4x4_block_grid():
+    # the Z curve: quadrants TL, TR, BL, BR at every level, hand-written
+    want = [(0, 0), (0, 1), (1, 0), (1, 1), (0, 2), (0, 3), (1, 2), (1, 3),
+            (2, 0), (2, 1), (3, 0), (3, 1), (2, 2), (2, 3), (3, 2), (3, 3)]
+    got = sorted(((oracle.morton_encode(i, j), (i, j)) for i in range(4) for j in range(4)))
+    assert [ij for _, ij in got] == want
+    assert [z for z, _ in got] == list(range(16))
+
+
+def test_morton_round_trip_and_every_aligned_submatrix_is_one_range():
+    for i in range(16):
+        for j in range(16):
+            assert oracle.morton_decode(oracle.morton_encode(i, j)) == (i, j)
+    for L in range(5):  # 1x1 ... 16x16 aligned submatrices
+        s = 1 << L
+        for i0 in range(0, 16, s):
+            for j0 in range(0, 16, s):
+                codes = sorted(oracle.morton_encode(i, j) for i in range(i0, i0 + s) for j in range(j0, j0 + s))
+                assert codes == list(range(codes[0], codes[0] + s * s))
+
+
+@pytest.mark.parametrize("shape", [(64, 32, 48, 5), (128, 64, 256, 3), (16, 16, 16, 7), (192, 48, 96, 2)])
+@pytest.mark.parametrize("density", [0.5, 1.0, 0.0])
+def test_zmorton_spmm_equals_bsr_spmm(shape, density):
+    """The same block-sparse matrices in two independent storage formats give
+    bit-identical oracle products (and density 1 is the dense GEMM)."""
+    import kami_inputs as ki
+    m, n, k, batch = shape
+    rp, cb, v, B = ki.bsr_operands(m, n, k, batch, "f16", density=density, dist="unif", seed=3)
+    present, blocks = ki.block_sparse(m, k, batch, "f16", density=density, dist="unif", seed=3)
+    nnzb, zcode, zvals = oracle.zmorton_from_blocks(present.numpy(), ki.as_bits(blocks))
+    C1 = oracle.spmm_bsr(m, n, k, batch, "f16", rp.numpy(), cb.numpy(), ki.as_bits(v), ki.as_bits(B))
+    C2 = oracle.spmm_zmorton(m, n, k, batch, "f16", nnzb, zcode, zvals, ki.as_bits(B))
+    assert np.array_equal(C1, C2)
+    assert (nnzb == present.reshape(batch, -1).sum(1).numpy()).all()
+    if density == 1.0:
+        A = blocks.permute(0, 1, 3, 2, 4).reshape(batch, m, k)
+        Cd = oracle.gemm(m, n, k, batch, "f16", "row", ki.as_bits(A.contiguous()), ki.as_bits(B))
+        assert np.array_equal(C2, Cd)
+    if density == 0.0:
+        assert not C2.any()
