@@ -180,6 +180,22 @@ kami_status_t kami_spmm_bsr_strided_batched(int m, int n, int k, int64_t batch, 
                                             const int* row_ptr, const int* col_blk, const void* vals,
                                             int max_nnzb, const void* B, void* C, kami_stream_t stream);
 
+/* SpMM with A in multi-level Z-Morton block storage (Sec. 4.6,
+ * Fig. 7(b): the storage of the 2D / 3D algorithms, "to facilitate efficient
+ * submatrix indexing").  Entry b holds nnzb[b] dense 16 x 16 blocks; the j-th
+ * (j < nnzb[b]) is block (i, c) of A with Morton code
+ *     zcode[b*max_nnzb + j] = sum_t c_t 4^t + i_t 2 * 4^t
+ * (column bits in the even positions, row bits in the odd ones: the Z curve
+ * visits TL, TR, BL, BR at every level, so every aligned 2^L x 2^L submatrix
+ * is one contiguous code range), codes ascending, values at
+ * vals[(b*max_nnzb + j)*256 + r*16 + c'] (row-major block).  B, C dense
+ * row-major packed strided batches.  All arrays DEVICE memory.  Same sizes,
+ * types, errors and kernel as kami_spmm_bsr_strided_batched (the kernel
+ * decodes each block's position from its code). */
+kami_status_t kami_spmm_zmorton_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                                const int* nnzb, const int* zcode, const void* vals, int max_nnzb,
+                                                const void* B, void* C, kami_stream_t stream);
+
 /* Block-level (on-chip-resident) mode -- the paper's block-level experiment
  * (Sec. 5.1, Sec. 5.2, Fig. 8/9): every entry is owned by one
  * team of p warps that loads A_b and B_b once and runs the CA schedule `reps`

@@ -34,7 +34,7 @@ EXPORTS = [
     "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
     "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level", "kami_gemm_vbatched",
     "kami_spmm_bsr_strided_batched", "kami_gemm_strided_batched_axpby", "kami_probe_dmma_peak",
-    "kami_set_grid_cap", "kami_plan_candidates",
+    "kami_set_grid_cap", "kami_plan_candidates", "kami_spmm_zmorton_strided_batched",
 ]
 
 
@@ -81,6 +81,8 @@ def lib() -> ctypes.CDLL:
     L.kami_gemm_block_level.argtypes = [i, i, i, i64, i, i, i, i, i, vp, vp, vp, vp, st]
     L.kami_gemm_vbatched.argtypes = [i64, vp, vp, vp, i, i, i, i, i, vp, vp, vp, st]
     L.kami_spmm_bsr_strided_batched.argtypes = [i, i, i, i64, i, vp, vp, vp, i, vp, vp, st]
+    L.kami_spmm_zmorton_strided_batched.argtypes = [i, i, i, i64, i, vp, vp, vp, i, vp, vp, st]
+    L.kami_spmm_zmorton_strided_batched.restype = ctypes.c_int
     L.kami_gemm_strided_batched_axpby.argtypes = [i, i, i, i64, i, i, ctypes.c_double, vp, vp, ctypes.c_double, vp,
                                                   st]
     L.kami_release_workspace.argtypes = []
@@ -209,6 +211,17 @@ def spmm_bsr_strided_batched(m, n, k, batch, dtype, row_ptr, col_blk, vals, B, C
     _check(lib().kami_spmm_bsr_strided_batched(m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _ptr(row_ptr),
                                                _ptr(col_blk), _ptr(vals), max_nnzb, _ptr(B), _ptr(C),
                                                _stream(stream)), "kami_spmm_bsr_strided_batched")
+    return C
+
+
+def spmm_zmorton_strided_batched(m, n, k, batch, dtype, nnzb, zcode, vals, B, C, stream=None):
+    """Block-sparse A in Z-Morton block storage (Sec. 4.6, Fig. 7(b))
+    times dense B.  nnzb [batch] and zcode [batch, max_nnzb] int32, vals
+    [batch, max_nnzb, 16, 16], B/C packed row-major -- all device tensors."""
+    max_nnzb = zcode.shape[-1]
+    _check(lib().kami_spmm_zmorton_strided_batched(m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _ptr(nnzb),
+                                                   _ptr(zcode), _ptr(vals), max_nnzb, _ptr(B), _ptr(C),
+                                                   _stream(stream)), "kami_spmm_zmorton_strided_batched")
     return C
 
 

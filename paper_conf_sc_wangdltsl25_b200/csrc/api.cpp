@@ -258,6 +258,21 @@ kami_status_t kami_spmm_bsr_strided_batched(int m, int n, int k, int64_t batch, 
                               reinterpret_cast<cudaStream_t>(stream));
 }
 
+kami_status_t kami_spmm_zmorton_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                                const int* nnzb, const int* zcode, const void* vals, int max_nnzb,
+                                                const void* B, void* C, kami_stream_t stream) {
+  kami_status_t st = check_common(m, n, k, batch, dtype, KAMI_ROW_MAJOR, KAMI_ALGO_AUTO);
+  if (st != KAMI_SUCCESS) return st;
+  if (!is16(dtype) || k % 16 || m % 16) return KAMI_ERROR_NOT_SUPPORTED;
+  if (max_nnzb < 0 || max_nnzb > (m / 16) * (k / 16)) return KAMI_ERROR_INVALID_VALUE;
+  if (batch == 0) return KAMI_SUCCESS;
+  if (!nnzb || !zcode || !vals || !B || !C || max_nnzb == 0) return KAMI_ERROR_INVALID_VALUE;
+  if (!aligned16(vals) || !aligned16(B) || !aligned16(C)) return KAMI_ERROR_MISALIGNED;
+  if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
+  return tc16_spmm_bsr_launch(m, n, k, batch, dtype == KAMI_DTYPE_BF16, nnzb, zcode, vals, max_nnzb, B, C,
+                              reinterpret_cast<cudaStream_t>(stream), /*zorder=*/true);
+}
+
 kami_status_t kami_gemm_block_level(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
                                     kami_algo_t algo, int p, int reps, const void* A, const void* B, void* C,
                                     int64_t* cycles, kami_stream_t stream) {

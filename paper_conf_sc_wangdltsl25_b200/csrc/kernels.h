@@ -101,8 +101,9 @@ kami_status_t tc16_vb_strided_launch(int m, int n, int k, long long batch, bool 
                                      void* C, cudaStream_t stream);
 
 // SpMM: block-sparse A (BSR, 16x16 blocks) x dense B on tcgen05 (densify on load)
+// zorder: A in Z-Morton block storage (row_ptr = per-entry block counts, col_blk = Morton codes)
 kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf16, const int* row_ptr,
                                    const int* col_blk, const void* vals, int max_nnzb, const void* B, void* C,
-                                   cudaStream_t stream);
+                                   cudaStream_t stream, bool zorder = false);
 
 }  // namespace kami

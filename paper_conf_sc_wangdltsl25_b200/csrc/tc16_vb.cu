@@ -65,6 +65,11 @@ struct alignas(64) VbParams {
   int bsr, max_nnzb;
   const int* rowptr;
   const int* colblk;
+  // Z-Morton block storage (Sec. 4.6, Fig. 7(b); R31):
+  // colblk holds each stored block's Morton code (ascending), rowptr the
+  // per-entry block counts nnzb[batch]; a block's (row, column) is decoded
+  // from its code, so no row pointer walk is needed
+  int zorder;
   const uint16_t* vals;
   const uint16_t* Bs;
   uint16_t* Cs;
@@ -185,7 +190,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     // SpMM: the next unit's block structure is fetched ahead too, without the
     // row_ptr -> col_blk dependency: every col_blk slot of the unit's entries
     // (<= 2 per thread: G mb kb <= 256) and every row_ptr value (<= 17)
-    const int mbk = p.bsr ? p.m / 16 : 0, rpn = mbk + 1;
+    const int mbk = p.bsr ? p.m / 16 : 0, rpn = p.zorder ? 1 : mbk + 1;
     struct PSlot {
       Unit U;
       const uint16_t *pa, *pb;
@@ -245,8 +250,23 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
           if (col < 0) continue;
           const int g = idx / p.max_nnzb, j = idx - g * p.max_nnzb;
           const int* rpg = rp_tab + g * rpn;
+          int br;
+          if (p.zorder) {  // (row, column) from the Morton code: odd bits row, even bits column
+            if (j >= rpg[0]) continue;  // past the entry's nnzb
+            const uint32_t z = (uint32_t)col;
+            uint32_t r = 0, c = 0;
+#pragma unroll
+            for (int t = 0; t < 5; ++t) {
+              c |= ((z >> (2 * t)) & 1u) << t;
+              r |= ((z >> (2 * t + 1)) & 1u) << t;
+            }
+            br = (int)r;
+            if (br < br0 || br >= br1) continue;
+            blk_tab[(g * mbk + br - br0) * 16 + (int)c] = (int)((U.e0 + g) * p.max_nnzb + j);
+            continue;
+          }
           if (j >= rpg[mbk]) continue;  // unused tail slot
-          int br = 0;
+          br = 0;
           while (rpg[br + 1] <= j) ++br;
           if (br < br0 || br >= br1) continue;
           blk_tab[(g * mbk + br - br0) * 16 + col] = (int)((U.e0 + g) * p.max_nnzb + j);
@@ -561,6 +581,10 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
     set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16,strided>" : "kami_tc16_vb_kernel<f16,strided>");
     return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
   }
+  if (p.zorder) {
+    set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16,spmm_zmorton>" : "kami_tc16_vb_kernel<f16,spmm_zmorton>");
+    return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+  }
   set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
                         : (bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>"));
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
@@ -581,9 +605,10 @@ extern "C" int kami_debug_vb_trace(long long* out) {
 
 kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf16, const int* row_ptr,
                                    const int* col_blk, const void* vals, int max_nnzb, const void* B, void* C,
-                                   cudaStream_t stream) {
+                                   cudaStream_t stream, bool zorder) {
   VbParams p;
   memset(&p, 0, sizeof(p));
+  p.zorder = zorder ? 1 : 0;
   p.m = m;
   p.n = n;
   p.k = k;
