@@ -594,7 +594,8 @@ int packing(int m, int n) {  // entries per 128-lane tile (same rule as tc16.cu)
   if (m > 128) return 1;
   const int g1 = 128 / m, g2 = 256 / n;
   const int g = g1 < g2 ? g1 : g2;
-  return g < 1 ? 1 : g;
+  // at most 8: the per-unit entry pointer tables hold 8 (m = 8 would pack 16)
+  return g < 1 ? 1 : (g > 8 ? 8 : g);
 }
 
 }  // namespace

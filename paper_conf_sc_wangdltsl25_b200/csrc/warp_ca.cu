@@ -693,27 +693,24 @@ bool lookup(int m, int n, int k, kami_dtype_t dtype, int algo, int p, LaunchInfo
   // FP16 / BF16 HMMA (m16n8k16): CA evidence family
   KAMI_CASE(H16, KAMI_DTYPE_F16, 16, 16, 16, 1, Sched1D, 1, "kami_warp_ca_1d<f16,16>")
   KAMI_CASE(B16, KAMI_DTYPE_BF16, 16, 16, 16, 1, Sched1D, 1, "kami_warp_ca_1d<bf16,16>")
-  // thin tiles (m or n = 16, k <= 32) where the tcgen05 unit is mostly empty:
-  // one warp per entry, register resident (BF16 sweep's slowest points)
+  // thin tiles (k <= 32 with n = 16 or 32, and bf16/f16 16 x 128 x 16) where
+  // the tcgen05 unit is mostly empty: one warp per entry, register resident.
+  // Kept only where they measured faster than the tcgen05 kernel
+  // (profiles/r2/variant_sweep_r2.json); the wide ones (m = 16 with n >= 64 and
+  // k = 32, n >= 192, 32 x 128) lost to it and were removed.
 #define KAMI_THIN_CASES(MM, NN, KK)                                                                 \
   KAMI_CASE(H16, KAMI_DTYPE_F16, MM, NN, KK, 1, Sched1D, 1, "kami_warp_ca_1d<f16," #MM "x" #NN "x" #KK ">") \
   KAMI_CASE(B16, KAMI_DTYPE_BF16, MM, NN, KK, 1, Sched1D, 1, "kami_warp_ca_1d<bf16," #MM "x" #NN "x" #KK ">")
-  KAMI_THIN_CASES(16, 64, 16)
   KAMI_THIN_CASES(16, 128, 16)
-  KAMI_THIN_CASES(16, 192, 16)
-  KAMI_THIN_CASES(16, 128, 32)
-  KAMI_THIN_CASES(32, 128, 16)
+  KAMI_THIN_CASES(16, 32, 16)
+  KAMI_THIN_CASES(16, 16, 32)
+  KAMI_THIN_CASES(32, 16, 16)
   KAMI_THIN_CASES(64, 16, 16)
   KAMI_THIN_CASES(128, 16, 16)
   KAMI_THIN_CASES(192, 16, 16)
-  KAMI_THIN_CASES(128, 32, 16)
-  KAMI_THIN_CASES(16, 32, 16)
-  KAMI_THIN_CASES(32, 16, 16)
-  KAMI_THIN_CASES(16, 256, 16)
   KAMI_THIN_CASES(256, 16, 16)
-  KAMI_THIN_CASES(16, 192, 32)
   KAMI_THIN_CASES(192, 16, 32)
-  KAMI_THIN_CASES(16, 16, 32)
+  KAMI_THIN_CASES(128, 32, 16)
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 1, Sched1D, 2, "kami_warp_ca_1d<f16,32>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 2, Sched2D, 4, "kami_warp_ca_2d<f16,32>")
   KAMI_CASE(H16, KAMI_DTYPE_F16, 32, 32, 32, 4, SchedNonCA, 4, "kami_warp_nonca<f16,32>")
@@ -750,9 +747,13 @@ int warp_ca_teams_per_sm(int m, int n, int k, kami_dtype_t dtype, int algo, int 
   const int teams_per_cta = li.threads / 32 / li.p;
   // a register estimate (not the occupancy API), so the planner's choice is
   // the same with and without a device (tests/test_planner_model.py)
-  const double es = dtype == KAMI_DTYPE_F64 ? 2.0 : 0.5;  // 32-bit registers per element
-  const double elems = (double)m * k / li.p * 2 + (double)k * n / li.p * 2 + (double)m * n / li.p;
-  const double regs = elems * es / 32 + 32;
+  // registers per thread: A_i, B_i (twice, send + receive buffers of the
+  // exchange, unless p = 1) and C_i, 16-bit operands two per register, FP32 /
+  // FP64 accumulators one / two (matches ptxas within ~10 % on the built
+  // instantiations, _build/warp_ca.cu.log)
+  const bool f64 = dtype == KAMI_DTYPE_F64;
+  const double ab = ((double)m * k + (double)k * n * (li.p > 1 ? 2 : 1)) / li.p * (f64 ? 2.0 : 0.5);
+  const double regs = (ab + (double)m * n / li.p * (f64 ? 2.0 : 1.0)) / 32 + 24;
   int per_sm = (int)(65536.0 / (li.threads * regs));
   if (per_sm < 1) per_sm = 1;
   if (per_sm * li.threads > 2048) per_sm = 2048 / li.threads;  // 64 warps per SM
