@@ -45,6 +45,13 @@ constexpr int kRK = 32;   // max resident k-steps (32 x 2 doubles = 128 register
 constexpr int kRKSmall = 8;  // k <= 32: 16 registers of B, four teams per SM
 constexpr int kGenSmem = 232448;
 
+// k index lane t supplies in k-step kk: with 16-double swizzle chunks the
+// bank-conflict-free order of dmma_tma.cu (units a and a ^ 4 per k-step);
+// with 8-double chunks (64-byte swizzle) the natural order
+__device__ __forceinline__ int kcol(int kk, int t, int ce_shift) {
+  return ce_shift == 4 ? ((kk >> 2) << 4) + ((kk & 3) << 1) + (t & 1) + ((t >> 1) << 3) : kk * 4 + t;
+}
+
 struct DmmaGenParams {
   CUtensorMap tmA;  // 4-D (CE, m, k/CE, batch), box (CE, TM, k/CE, 1), CE = 16 (SW128) or 8 (SW64) doubles
   const double* B;
@@ -114,13 +121,14 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
 #pragma unroll
       for (int j = 0; j < kGFN; ++j) {
         const int col = col0 + j * 8 + g;
-        b[kk][j] = (kk < p.rs && col0 + j * 8 < p.n) ? __ldg(Bg + (kk * 4 + t) * (long long)p.n + col) : 0.0;
+        b[kk][j] = (kk < p.rs && col0 + j * 8 < p.n) ? __ldg(Bg + kcol(kk, t, p.ce_shift) * (long long)p.n + col)
+                                                      : 0.0;
       }
     for (int kk = p.rs; kk < p.ks; ++kk)
 #pragma unroll
       for (int j = 0; j < kGFN; ++j) {
         const int col = col0 + j * 8 + g;
-        const double v = col0 + j * 8 < p.n ? __ldg(Bg + (kk * 4 + t) * (long long)p.n + col) : 0.0;
+        const double v = col0 + j * 8 < p.n ? __ldg(Bg + kcol(kk, t, p.ce_shift) * (long long)p.n + col) : 0.0;
         asm volatile("st.shared.f64 [%0], %1;" ::"r"(park + (uint32_t)(((kk - p.rs) * kGFN + j) * 32 + lane) * 8),
                      "d"(v)
                      : "memory");
@@ -137,7 +145,7 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
       const uint32_t a_s = ptx::smem_u32(tbase + s * p.a_block_bytes);
       const uint32_t rowb = 8u << p.ce_shift;  // bytes of one swizzled row of a chunk
       auto step = [&](int kk, const double (&bb)[kGFN]) {
-        const int col = kk * 4 + t;
+        const int col = kcol(kk, t, p.ce_shift);
         const uint32_t chunk_off = (uint32_t)(col >> p.ce_shift) * (kGTM * rowb);
         const uint32_t in_row = (uint32_t)(col & ((1 << p.ce_shift) - 1)) * 8;
         // all FM A fragments first (their LDS latencies overlap), then the FM x FN DMMAs

@@ -75,7 +75,21 @@ __device__ __forceinline__ void load_a_entry(void* dst, const DmmaTmaParams& prm
   }
 }
 
-// B_w fragments of k-steps [K0, K1) of one entry (k = t, n = g of each 8x8 block).
+// The k index lane t supplies in DMMA k-step kk.  The 128-byte swizzle puts
+// 16-byte unit u of A row r at unit u ^ (r mod 8); an LDS.64 is served per
+// half-warp (4 rows x 4 lanes), so with the natural order (lanes t = 0..3 ->
+// columns 4 kk + t, i.e. units 2a, 2a + 1) rows r and r ^ 1 of a half-warp hit
+// the same 8 banks: 4 wavefronts per LDS.64 instead of 2 (ncu: 69.4 M
+// wavefronts for 33.5 M ideal at f64 64^3, profiles/r2).  Taking the k-step's
+// four columns from units a and a ^ 4 of the 16-column chunk (lanes t = 0, 1:
+// columns 2a, 2a + 1; t = 2, 3: 2a + 8, 2a + 9) gives the four rows of a
+// half-warp eight distinct units.  Any permutation of k applied to A and B
+// alike leaves the product unchanged.
+__device__ __forceinline__ int kperm(int kk, int t) {
+  return ((kk >> 2) << 4) + ((kk & 3) << 1) + (t & 1) + ((t >> 1) << 3);
+}
+
+// B_w fragments of k-steps [K0, K1) of one entry (k = kperm(kk, t), n = g of each 8x8 block).
 // volatile asm keeps the loads where the schedule puts them relative to the MMAs.
 template <int N, int FN, int K0, int K1, int FK>
 __device__ __forceinline__ void load_b_steps(double (&b)[FK][FN], const double* Bg, int t, int g) {
@@ -83,7 +97,7 @@ __device__ __forceinline__ void load_b_steps(double (&b)[FK][FN], const double* 
   for (int kk = K0; kk < K1; ++kk)
 #pragma unroll
     for (int j = 0; j < FN; ++j)
-      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(b[kk][j]) : "l"(Bg + (kk * 4 + t) * N + j * 8 + g));
+      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(b[kk][j]) : "l"(Bg + kperm(kk, t) * N + j * 8 + g));
 }
 
 // One k-step range of the entry: A fragments from the swizzled broadcast tile
@@ -93,7 +107,7 @@ __device__ __forceinline__ void mma_steps(double (&c)[FM][FN][2], const double (
                                           int g) {
 #pragma unroll
   for (int kk = K0; kk < K1; ++kk) {
-    const int col = kk * 4 + t;
+    const int col = kperm(kk, t);
     const uint32_t chunk_off = (uint32_t)(col >> 4) * (M * 128) + ((col & 1) << 3);
     const uint32_t unit = (uint32_t)((col & 15) >> 1);
 #pragma unroll
@@ -180,7 +194,7 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
 #pragma unroll
       for (int kk = 0; kk < Cfg::FK; ++kk)
 #pragma unroll
-        for (int j = 0; j < Cfg::FN; ++j) b[kk][j] = __ldg(Bg + (kk * 4 + t) * N + j * 8 + g);
+        for (int j = 0; j < Cfg::FN; ++j) b[kk][j] = __ldg(Bg + kperm(kk, t) * N + j * 8 + g);
     }
     double c[Cfg::FM][Cfg::FN][2];
 #pragma unroll
