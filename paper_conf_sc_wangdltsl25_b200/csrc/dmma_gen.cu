@@ -148,22 +148,19 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
         const int col = kcol(kk, t, p.ce_shift);
         const uint32_t chunk_off = (uint32_t)(col >> p.ce_shift) * (kGTM * rowb);
         const uint32_t in_row = (uint32_t)(col & ((1 << p.ce_shift) - 1)) * 8;
-        // all FM A fragments first (their LDS latencies overlap), then the FM x FN DMMAs
-        double a[kGFM];
 #pragma unroll
         for (int i = 0; i < kGFM; ++i) {
           const int row = i * 8 + g;
+          double a;
           asm volatile("ld.shared.f64 %0, [%1];"
-                       : "=d"(a[i])
+                       : "=d"(a)
                        : "r"(a_s + chunk_off + ptx::swz(row * rowb + in_row, p.swz_bits)));
-        }
-#pragma unroll
-        for (int i = 0; i < kGFM; ++i)
 #pragma unroll
           for (int j = 0; j < kGFN; ++j)
             asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
                          : "+d"(c[i][j][0]), "+d"(c[i][j][1])
-                         : "d"(a[i]), "d"(bb[j]));
+                         : "d"(a), "d"(bb[j]));
+        }
       };
       // resident k-steps: B fragments from registers
 #pragma unroll
