@@ -91,7 +91,14 @@ typedef enum {
    * the layer partials summed inside ONE TMEM accumulator (the Alg. 3
    * reduction costs no shared-memory traffic).  Needs every k-chunk to hold
    * an even number of K = 16 steps (k a multiple of 32 in practice). */
-  KAMI_ALGO_3D_TMEM = 7
+  KAMI_ALGO_3D_TMEM = 7,
+  /* 16-bit only, 192 < m <= 256: KAMI-2D across a CTA pair (tcgen05
+   * cta_group::2, M = 256): CTA r owns rows [128r, 128r+128) of A and C and
+   * columns [r n/2, (r+1) n/2) of B in its shared memory; the pair's MMA
+   * broadcasts each B column block to the other CTA's rows (Alg. 2).
+   * n a multiple of 32 in [32,256], k a multiple of 8; NOT_SUPPORTED
+   * otherwise. */
+  KAMI_ALGO_2D_PAIR = 8
 } kami_algo_t;
 
 /* Opaque CUDA stream; binary compatible with cudaStream_t. */
@@ -218,7 +225,7 @@ typedef struct {
   int kernel;            /* 0 = tcgen05 16-bit (SS), 1 = warp-level DMMA/HMMA, 2 = FP64 DMMA with TMA
                             broadcast, 3 = tcgen05 16-bit with A resident in TMEM (TS), 4 = FP64 DMMA
                             for the whole size grid (k-sliced, register residency ratio), 5 = LDG-fed
-                            tcgen05 16-bit (m or n = 8 mod 16) */
+                            tcgen05 16-bit (m or n = 8 mod 16), 6 = tcgen05 CTA pair (2D, cta_group::2) */
   int entries_per_cta;   /* batch entries a CTA keeps in flight             */
   int stages;            /* shared-memory pipeline depth                    */
   int kslice_regs_pct;   /* share of A/B kept resident (Sec. 4.7)           */

@@ -62,7 +62,7 @@ kami_status_t check_common(int m, int n, int k, int64_t batch, int dtype, int la
   if (m <= 0 || n <= 0 || k <= 0 || batch < 0) return KAMI_ERROR_INVALID_VALUE;
   if (dtype < KAMI_DTYPE_F16 || dtype > KAMI_DTYPE_E5M2) return KAMI_ERROR_INVALID_VALUE;
   if (layout != KAMI_ROW_MAJOR && layout != KAMI_COL_MAJOR) return KAMI_ERROR_INVALID_VALUE;
-  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_3D_TMEM) return KAMI_ERROR_INVALID_VALUE;
+  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_2D_PAIR) return KAMI_ERROR_INVALID_VALUE;
   return check_sizes(m, n, k, (kami_dtype_t)dtype);
 }
 
@@ -127,6 +127,10 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
+  if (plan.kernel == 6) {  // tcgen05 CTA pair (strided C = A B)
+    if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
+    return tc16_pair_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream);
+  }
   if (plan.kernel == 5) {  // 16-bit m or n = 8 mod 16: the LDG-fed tcgen05 kernel on packed entries
     if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
     return tc16_vb_strided_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream);
@@ -140,7 +144,8 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
     return tc16_ts_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, plan.algo == KAMI_ALGO_3D_TMEM ? 2 : 1,
                           rp.A, rp.B, C, stream);
   }
-  if ((plan.kernel == 1 || plan.kernel == 3) && update && is16(dtype) && algo == KAMI_ALGO_AUTO && !Ca)
+  if ((plan.kernel == 1 || plan.kernel == 3 || plan.kernel == 6) && update && is16(dtype) && algo == KAMI_ALGO_AUTO &&
+      !Ca)
     plan.kernel = 0;  // the update form (C read) exists on the SS tcgen05 kernel only
   if ((plan.kernel == 4 || plan.kernel == 1) && update && algo == KAMI_ALGO_AUTO && !Ca &&
       dmma_tma_supported(rp.m, rp.n, rp.k))

@@ -63,6 +63,11 @@ kami_status_t tc16_ts_plan(int m, int n, int k, int layers, TsShape* s);
 kami_status_t tc16_ts_launch(int m, int n, int k, long long batch, bool bf16, int layers, const void* A,
                              const void* B, void* C, cudaStream_t stream);
 
+// ------------------------ tcgen05 CTA pair, KAMI-2D over 2 SMs (tc16_pair.cu)
+bool tc16_pair_supported(int m, int n, int k);
+kami_status_t tc16_pair_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B, void* C,
+                               cudaStream_t stream);
+
 // ------------------------------------------------ warp-level CA (literal KAMI)
 // algo: 1 = 1D, 2 = 2D, 3 = 3D, 4 = non-CA tiled.  dtype: KAMI_DTYPE_*.
 // Entry pointers: if A_arr != nullptr they are device arrays of per-entry

@@ -200,6 +200,28 @@ bool model_ts(int m, int n, int k, kami_dtype_t dt, int layers, Pred* out) {
   return true;
 }
 
+// CTA pair (tc16_pair.cu): one entry per pair-unit on two SMs; per CTA the
+// unit moves its 128 rows of A and C and half of B
+bool model_pair(int m, int n, int k, kami_dtype_t dt, Pred* out) {
+  if ((dt != KAMI_DTYPE_F16 && dt != KAMI_DTYPE_BF16) || !tc16_pair_supported(m, n, k)) return false;
+  const int kpad = (k + 15) / 16 * 16;
+  const int wk = kpad * 2 % 128 == 0 ? 64 : kpad * 2 % 64 == 0 ? 32 : 16;
+  const int wn = n % 128 == 0 ? 64 : n % 64 == 0 ? 32 : 16;            // atom of the n/2-column half
+  const int wc = (2 * n) % 128 == 0 ? 64 : (2 * n) % 64 == 0 ? 32 : 16;
+  const int kchunks = (kpad + wk - 1) / wk;
+  const double t_hbm = bytes_entry(m, n, k, dt) / (2 * kHbmBpc);
+  const double rows_ld = 128.0 * kchunks + (double)kpad * ((n / 2) / wn);
+  const double rows_st = 128.0 * (n / wc);
+  const double t_tma = rows_ld * kTmaLdRow + rows_st * kTmaStRow;
+  const double t_epi = kEpiVal * n;
+  const double t_tc = 2.0 * m * n * k / (2 * kUmmaFpc);
+  Pred p = psoft({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {kUnitSS, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR},
+                  {t_epi, KAMI_BOUND_ISSUE}});
+  p.cycles *= 2;  // two SMs per entry: cycles per entry per SM
+  *out = p;
+  return true;
+}
+
 // LDG-fed tcgen05 (tc16_vb.cu) for 16-bit m or n = 8 mod 16: the same
 // schedule with the operands copied by a producer warpgroup (16-byte
 // cp.async); per unit max(HBM, the copy issue of the unit's 16-byte chunks,
@@ -300,6 +322,11 @@ void fill_plan(kami_plan_t* r, int kernel, kami_algo_t algo, int p, int m, int n
     r->entries_per_cta = m == 64 ? 3 : 8;
     r->kslice_regs_pct = 50;  // B_w resident in registers, A broadcast through SMEM
     r->t_all_cycles = b200_cost(1, n, m, k, 4, dt);
+  } else if (kernel == 6) {
+    r->entries_per_cta = 1;
+    r->stages = 4;
+    r->kslice_regs_pct = 0;
+    r->t_all_cycles = b200_cost(2, m, n, k, 8, dt);
   } else if (kernel == 5) {
     r->entries_per_cta = 1;
     r->kslice_regs_pct = 0;
@@ -339,6 +366,7 @@ int planner_candidates(int m, int n, int k, kami_dtype_t dt, bool pointer_array,
     if (model_ss(m, n, k, dt, &pr)) add(0, KAMI_ALGO_1D, 4, pr);
     if (model_ts(m, n, k, dt, 1, &pr)) add(3, KAMI_ALGO_1D_TMEM, 4, pr);
     if (model_ts(m, n, k, dt, 2, &pr)) add(3, KAMI_ALGO_3D_TMEM, 8, pr);
+    if (model_pair(m, n, k, dt, &pr)) add(6, KAMI_ALGO_2D_PAIR, 8, pr);
   } else {
     if (model_dmma_tma(m, n, k, &pr)) add(2, KAMI_ALGO_1D_TMA, 4, pr);
     if (model_dmma_gen(m, n, k, &pr)) add(4, KAMI_ALGO_1D, 4, pr);
@@ -395,6 +423,15 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
     kami_status_t st = tc16_ts_plan(m, n, k, algo == KAMI_ALGO_3D_TMEM ? 2 : 1, &ts);
     if (st != KAMI_SUCCESS) return st == KAMI_ERROR_INVALID_VALUE ? KAMI_ERROR_NOT_SUPPORTED : st;
     fill_plan(&r, 3, algo, algo == KAMI_ALGO_3D_TMEM ? 8 : 4, m, n, k, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
+  // tcgen05 CTA pair
+  if (algo == KAMI_ALGO_2D_PAIR) {
+    if ((dtype != KAMI_DTYPE_F16 && dtype != KAMI_DTYPE_BF16) || pointer_array || (p != 0 && p != 8) ||
+        !tc16_pair_supported(m, n, k))
+      return KAMI_ERROR_NOT_SUPPORTED;
+    fill_plan(&r, 6, KAMI_ALGO_2D_PAIR, 8, m, n, k, dtype);
     *out = r;
     return KAMI_SUCCESS;
   }
