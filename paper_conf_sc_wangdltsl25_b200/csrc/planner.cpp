@@ -200,6 +200,9 @@ bool model_ts(int m, int n, int k, kami_dtype_t dt, int layers, Pred* out) {
   return true;
 }
 
+// The CTA-pair kernel is selectable explicitly (KAMI_ALGO_2D_PAIR); AUTO
+// considers it once it is measured faster than the single-CTA kernel.
+constexpr bool kPairInAuto = false;
 // CTA pair (tc16_pair.cu): one entry per pair-unit on two SMs; per CTA the
 // unit moves its 128 rows of A and C and half of B
 bool model_pair(int m, int n, int k, kami_dtype_t dt, Pred* out) {
@@ -366,7 +369,7 @@ int planner_candidates(int m, int n, int k, kami_dtype_t dt, bool pointer_array,
     if (model_ss(m, n, k, dt, &pr)) add(0, KAMI_ALGO_1D, 4, pr);
     if (model_ts(m, n, k, dt, 1, &pr)) add(3, KAMI_ALGO_1D_TMEM, 4, pr);
     if (model_ts(m, n, k, dt, 2, &pr)) add(3, KAMI_ALGO_3D_TMEM, 8, pr);
-    if (model_pair(m, n, k, dt, &pr)) add(6, KAMI_ALGO_2D_PAIR, 8, pr);
+    if (kPairInAuto && model_pair(m, n, k, dt, &pr)) add(6, KAMI_ALGO_2D_PAIR, 8, pr);
   } else {
     if (model_dmma_tma(m, n, k, &pr)) add(2, KAMI_ALGO_1D_TMA, 4, pr);
     if (model_dmma_gen(m, n, k, &pr)) add(4, KAMI_ALGO_1D, 4, pr);
