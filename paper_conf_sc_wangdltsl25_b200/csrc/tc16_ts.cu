@@ -291,8 +291,76 @@ __global__ void __launch_bounds__(kTsBaseThreads + 128 * kLW, 1)
     auto advance = [&](ItemPos& x) {
       for (int j = 0; j < kLW; ++j) x.next(p, gridDim.x);
     };
-    uint32_t va[32], vb[32];
-    if (it.u < p.units) {
+    if (kLW == 1 && nld <= 4 && it.u < p.units) {  // (576-thread CTAs have no registers for it)
+      // items of <= 32 columns (16 registers): FOUR in flight per thread.
+      // With two, an item's LDG latency (~1500 cycles under load) was exposed
+      // once per item (TS 32^3: 1587 cycles per one-item unit against 1094 of
+      // HBM time).
+      auto load16 = [&](const ItemPos& x, uint32_t(&v)[16]) {
+        const long long e = x.grp * p.G + g;
+        const bool ok = row_in_tile && e < p.batch;
+        const int c0 = x.kc * p.Wk + x.l * p.item_cols;
+        const uint16_t* rowp = p.A + (e * p.m + r) * (long long)p.k + c0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          if (j < nld) {
+            uint4 w = make_uint4(0, 0, 0, 0);
+            if (ok && c0 + 8 * j < p.k) w = ldg16(rowp + 8 * j);
+            v[4 * j] = w.x;
+            v[4 * j + 1] = w.y;
+            v[4 * j + 2] = w.z;
+            v[4 * j + 3] = w.w;
+          }
+        }
+      };
+      auto store16 = [&](RingPos& sp_, const uint32_t(&v)[16]) {
+        ptx::mbar_wait(&aempty[sp_.s], sp_.ph ^ 1);
+        ptx::tc_fence_after();
+        const uint32_t ta = a_base + sp_.s * p.slot_cols;
+        if (nld == 1) tmem_st_x<4>(ta, v);
+        else if (nld == 2) tmem_st_x<8>(ta, v);
+        else tmem_st_x<16>(ta, v);
+        ptx::tmem_wait_st();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&afull[sp_.s]);
+        for (int j = 0; j < kLW; ++j) sp_.next(p.a_slots);
+      };
+      uint32_t q0[16], q1[16], q2[16], q3[16];
+      ItemPos p0 = it, p1 = p0, p2;
+      advance(p1);
+      p2 = p1;
+      advance(p2);
+      load16(p0, q0);
+      if (p1.u < p.units) load16(p1, q1);
+      if (p2.u < p.units) load16(p2, q2);
+      for (;;) {  // q0..q2 hold p0..p2 at the top of each round
+        ItemPos p3 = p2;
+        advance(p3);
+        if (p3.u < p.units) load16(p3, q3);
+        store16(rs, q0);
+        if (p1.u >= p.units) break;
+        ItemPos p4 = p3;
+        advance(p4);
+        if (p4.u < p.units) load16(p4, q0);
+        store16(rs, q1);
+        if (p2.u >= p.units) break;
+        ItemPos p5 = p4;
+        advance(p5);
+        if (p5.u < p.units) load16(p5, q1);
+        store16(rs, q2);
+        if (p3.u >= p.units) break;
+        ItemPos p6 = p5;
+        advance(p6);
+        if (p6.u < p.units) load16(p6, q2);
+        store16(rs, q3);
+        if (p4.u >= p.units) break;
+        p0 = p4;
+        p1 = p5;
+        p2 = p6;
+      }
+    } else if (it.u < p.units) {
+      uint32_t va[32], vb[32];
       load(it, va);
       // two items in flight per thread: the next item's loads are issued
       // before the current item is written to TMEM (static buffer roles)
