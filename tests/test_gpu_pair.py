@@ -46,6 +46,6 @@ def test_pair_steady_state(shape):
 def test_pair_rejects_out_of_scope():
     import torch
     A = torch.zeros(256 * 256, dtype=torch.float16, device="cuda")
-    for (m, n, k) in ((128, 128, 64), (256, 48, 64), (192, 64, 64)):
+    for (m, n, k) in ((128, 128, 64), (256, 48, 64), (112, 64, 64)):
         with pytest.raises(kami.KamiError):
             kami.gemm_strided_batched(m, n, k, 1, "f16", "row", A, A, A, algo="2d_pair")
