@@ -32,6 +32,7 @@
 
 #include "kernels.h"
 #include "ptx.cuh"
+#include "sched.cuh"
 
 namespace kami {
 namespace {
@@ -62,6 +63,7 @@ struct DmmaGenParams {
   uint32_t swz_bits;  // 3 (SW128) or 2 (SW64)
   uint32_t a_block_bytes, park_bytes;  // per team buffer / per warp slab
   int teams;
+  int nbuf;  // A blocks in flight per team (2 or 3)
 };
 
 template <int RK>
@@ -72,13 +74,13 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int team = warp / kGP, w = warp % kGP;
   const int g = lane >> 2, t = lane & 3;
-  // per team: A double buffer, then the four warps' parked slabs; barriers at the end
-  const uint32_t team_bytes = 2 * p.a_block_bytes + kGP * p.park_bytes;
+  // per team: nbuf A blocks, then the four warps' parked slabs; barriers at the end
+  const uint32_t team_bytes = p.nbuf * p.a_block_bytes + kGP * p.park_bytes;
   uint8_t* tbase = smem + team * team_bytes;
-  uint64_t* full = reinterpret_cast<uint64_t*>(smem + p.teams * team_bytes) + team * 2;
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + p.teams * team_bytes) + team * 3;
   if (threadIdx.x == 0) {
     ptx::prefetch_tmap(&p.tmA);
-    for (int i = 0; i < 2 * p.teams; ++i)
+    for (int i = 0; i < 3 * p.teams; ++i)
       ptx::mbar_init(reinterpret_cast<uint64_t*>(smem + p.teams * team_bytes) + i, 1);
     ptx::fence_mbar_init();
     ptx::fence_proxy_async_smem();
@@ -89,18 +91,18 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   const long long first = (long long)blockIdx.x * p.teams + team;
   const bool issuer = (w == 0 && lane == 0);
   const uint32_t bar = 1 + team;
-  const uint32_t park = ptx::smem_u32(tbase + 2 * p.a_block_bytes + w * p.park_bytes);
+  const uint32_t park = ptx::smem_u32(tbase + p.nbuf * p.a_block_bytes + w * p.park_bytes);
   // the team's block sequence: units u = first, first + nteams, ...; m-blocks 0.. of each
   auto issue = [&](long long u, int mb, int s) {
     const long long e = u / p.nblocks;
     ptx::mbar_arrive_expect_tx(&full[s], p.a_block_bytes);
     ptx::tma_load_4d(tbase + s * p.a_block_bytes, &p.tmA, &full[s], 0, mb * kGTM, 0, (int)e);
   };
-  // prologue: the first two blocks
+  // prologue: the first nbuf blocks
   long long pu = first;
   int pmb = 0;
   if (issuer) {
-    for (int s = 0; s < 2 && pu < p.units; ++s) {
+    for (int s = 0; s < p.nbuf && pu < p.units; ++s) {
       issue(pu, pmb, s);
       if (++pmb == p.mblocks) {
         pmb = 0;
@@ -109,10 +111,12 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
     }
   }
   double b[RK][kGFN];
-  uint32_t it = 0;
+  RingPos ab;  // A buffer ring (slot, parity)
   for (long long u = first; u < p.units; u += nteams) {
     const long long e = u / p.nblocks;
     const int nb = (int)(u - e * p.nblocks);
+    if (issuer && u + nteams < p.units)  // the next unit's B into L2 while this one computes
+      ptx::prefetch_l2_bulk(p.B + ((u + nteams) / p.nblocks) * (long long)p.k * p.n, (uint32_t)(p.k * p.n * 8));
     const int col0 = nb * kGNB + w * (kGFN * 8);
     const double* Bg = p.B + e * (long long)p.k * p.n;
     // GMem2Reg: the resident k-steps of B_w; the parked ones go to this warp's slab
@@ -134,14 +138,14 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
                      : "memory");
       }
     __syncwarp();
-    for (int mb = 0; mb < p.mblocks; ++mb, ++it) {
-      const uint32_t s = it & 1;
+    for (int mb = 0; mb < p.mblocks; ++mb, ab.next(p.nbuf)) {
+      const uint32_t s = ab.s;
       double c[kGFM][kGFN][2];
 #pragma unroll
       for (int i = 0; i < kGFM; ++i)
 #pragma unroll
         for (int j = 0; j < kGFN; ++j) c[i][j][0] = c[i][j][1] = 0.0;
-      ptx::mbar_wait(&full[s], (it >> 1) & 1);
+      ptx::mbar_wait(&full[s], ab.ph);
       const uint32_t a_s = ptx::smem_u32(tbase + s * p.a_block_bytes);
       const uint32_t rowb = 8u << p.ce_shift;  // bytes of one swizzled row of a chunk
       auto step = [&](int kk, const double (&bb)[kGFN]) {
@@ -188,7 +192,7 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
             ptx::st_global_v2_f64(Cg + (long long)row * p.n + col0 + j * 8 + 2 * t, c[i][j][0], c[i][j][1]);
       }
       ptx::named_bar_sync(bar, kGP * 32);  // every warp finished reading buffer s
-      if (issuer && pu < p.units) {        // refill it with the block two ahead
+      if (issuer && pu < p.units) {        // refill it with the block nbuf ahead
         issue(pu, pmb, s);
         if (++pmb == p.mblocks) {
           pmb = 0;
@@ -208,7 +212,7 @@ uint32_t align1k(uint32_t x) { return (x + 1023) / 1024 * 1024; }
 // shared-memory bytes.  The parked slabs must fit next to the A double buffer:
 // a ratio that parks more than fits is raised to the smallest that fits.
 struct GenPlan {
-  int rk, rs, teams, ce_shift;
+  int rk, rs, teams, ce_shift, nbuf;
   uint32_t a_block_bytes, park_bytes, smem;
 };
 GenPlan gen_plan(int m, int n, int k) {
@@ -229,11 +233,14 @@ GenPlan gen_plan(int m, int n, int k) {
   if (ks - rs > room) rs = ks - room;
   g.rs = rs;
   g.park_bytes = (uint32_t)((ks - rs) * slab_step);
-  const uint32_t team_bytes = 2 * g.a_block_bytes + kGP * g.park_bytes;
+  // three A blocks in flight when they fit next to the slabs (one more TMA
+  // round trip of slack per team), else two
+  g.nbuf = (3 * g.a_block_bytes + kGP * g.park_bytes + 1024 + 96 <= (uint32_t)kGenSmem) ? 3 : 2;
+  const uint32_t team_bytes = g.nbuf * g.a_block_bytes + kGP * g.park_bytes;
   const int max_teams = g.rk == kRK ? 2 : 4;
   g.teams = 1;
-  while (g.teams < max_teams && (g.teams + 1) * team_bytes + 1024 + 64 <= (uint32_t)kGenSmem) ++g.teams;
-  g.smem = g.teams * team_bytes + 1024 /*align*/ + 64 /*barriers*/;
+  while (g.teams < max_teams && (g.teams + 1) * team_bytes + 1024 + 96 <= (uint32_t)kGenSmem) ++g.teams;
+  g.smem = g.teams * team_bytes + 1024 /*align*/ + 96 /*barriers*/;
   return g;
 }
 
@@ -272,6 +279,7 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
   p.a_block_bytes = gp.a_block_bytes;
   p.park_bytes = gp.park_bytes;
   p.teams = gp.teams;
+  p.nbuf = gp.nbuf;
   const uint32_t smem = gp.smem;
   {  // A: (CE doubles, m, k/CE chunks, batch), box (CE, TM, k/CE, 1); rows past m zero-filled
     cuuint64_t dims[4] = {(cuuint64_t)ce, (cuuint64_t)m, (cuuint64_t)p.kch, (cuuint64_t)batch};
