@@ -118,8 +118,9 @@ kami_status_t kami_gemm(int m, int n, int k, int64_t batch, kami_dtype_t dtype, 
  * device memory): its result is undefined.  16-bit types run on the same
  * tcgen05 kernel as the strided form, fed by TMA boxes over an address-space
  * view of each entry; m or n = 8 mod 16 on the LDG-fed
- * tcgen05 kernel.  FP64 pointer arrays: m = n = k in {8, 16, 32, 64} only
- * (NOT_SUPPORTED otherwise: the general FP64 kernel is strided). */
+ * tcgen05 kernel.  FP64: m = n = k in {16, 32, 64} on the TMA-broadcast
+ * DMMA kernel, 8^3 on the warp-level one, every other shape of the grid on
+ * the k-sliced DMMA kernel with cp.async-fed A blocks. */
 kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,
                                 const void* const* A_array, const void* const* B_array, void* const* C_array,
                                 kami_stream_t stream);

@@ -135,9 +135,9 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
     if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
     return tc16_vb_strided_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream);
   }
-  if (plan.kernel == 4) {  // FP64 general sizes: k-sliced DMMA with a residency ratio (strided C = A B)
-    if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
-    return dmma_gen_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream);
+  if (plan.kernel == 4) {  // FP64 general sizes: k-sliced DMMA with a residency ratio (C = A B)
+    if (update) return KAMI_ERROR_NOT_SUPPORTED;
+    return dmma_gen_launch(rp.m, rp.n, rp.k, batch, rp.A, rp.B, C, stream, rp.Aa, rp.Ba, Ca);
   }
   if (plan.kernel == 3) {  // tcgen05 with A resident in TMEM (strided C = A B only)
     if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;

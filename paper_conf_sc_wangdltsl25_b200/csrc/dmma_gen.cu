@@ -64,9 +64,16 @@ struct DmmaGenParams {
   uint32_t a_block_bytes, park_bytes;  // per team buffer / per warp slab
   int teams;
   int nbuf;  // A blocks in flight per team (2 or 3)
+  // pointer arrays (kPtr; kami_gemm_batched): entry e at Aa[e], Ba[e], Ca[e]
+  // (device).  A blocks are copied by the team with 16-byte cp.async into the
+  // same swizzled layout the TMA box writes (rows past m zero-filled): a TMA
+  // view box could not stay inside an entry whose m is not a multiple of 32.
+  const double* const* Aa;
+  const double* const* Ba;
+  double* const* Ca;
 };
 
-template <int RK>
+template <int RK, bool kPtr>
 __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
     kami_dmma_gen_kernel(const __grid_constant__ DmmaGenParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -80,8 +87,8 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + p.teams * team_bytes) + team * 3;
   if (threadIdx.x == 0) {
     ptx::prefetch_tmap(&p.tmA);
-    for (int i = 0; i < 3 * p.teams; ++i)
-      ptx::mbar_init(reinterpret_cast<uint64_t*>(smem + p.teams * team_bytes) + i, 1);
+    for (int i = 0; i < 3 * p.teams; ++i)  // TMA: one expect_tx arrival; cp.async: the team's 128 threads
+      ptx::mbar_init(reinterpret_cast<uint64_t*>(smem + p.teams * team_bytes) + i, kPtr ? kGP * 32 : 1);
     ptx::fence_mbar_init();
     ptx::fence_proxy_async_smem();
   }
@@ -93,15 +100,33 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   const uint32_t bar = 1 + team;
   const uint32_t park = ptx::smem_u32(tbase + p.nbuf * p.a_block_bytes + w * p.park_bytes);
   // the team's block sequence: units u = first, first + nteams, ...; m-blocks 0.. of each
+  const int tid = w * 32 + lane;  // 0..127 within the team
   auto issue = [&](long long u, int mb, int s) {
     const long long e = u / p.nblocks;
-    ptx::mbar_arrive_expect_tx(&full[s], p.a_block_bytes);
-    ptx::tma_load_4d(tbase + s * p.a_block_bytes, &p.tmA, &full[s], 0, mb * kGTM, 0, (int)e);
+    if constexpr (kPtr) {  // every thread of the team: 16-byte chunks of the 32 x k block
+      const double* Ae = p.Aa[e];
+      const uint32_t dst0 = ptx::smem_u32(tbase + s * p.a_block_bytes);
+      const int cpr = p.k >> 1;  // 16-byte chunks per row
+      const uint32_t rowb = 8u << p.ce_shift;
+      for (int i = tid; i < kGTM * cpr; i += kGP * 32) {
+        const int r = i / cpr, c = i - r * cpr;  // row, chunk (two doubles)
+        const int col = 2 * c;
+        const int row = mb * kGTM + r;
+        const uint32_t off = (uint32_t)(col >> p.ce_shift) * (kGTM * rowb) +
+                             ptx::swz((uint32_t)r * rowb + (uint32_t)(col & ((1 << p.ce_shift) - 1)) * 8, p.swz_bits);
+        const bool ok = row < p.m;
+        ptx::cp_async_16(dst0 + off, ok ? Ae + (long long)row * p.k + col : Ae, ok ? 16u : 0u);
+      }
+      ptx::cp_async_mbar_arrive_noinc(&full[s]);
+    } else {
+      ptx::mbar_arrive_expect_tx(&full[s], p.a_block_bytes);
+      ptx::tma_load_4d(tbase + s * p.a_block_bytes, &p.tmA, &full[s], 0, mb * kGTM, 0, (int)e);
+    }
   };
   // prologue: the first nbuf blocks
   long long pu = first;
   int pmb = 0;
-  if (issuer) {
+  if (issuer || kPtr) {
     for (int s = 0; s < p.nbuf && pu < p.units; ++s) {
       issue(pu, pmb, s);
       if (++pmb == p.mblocks) {
@@ -115,10 +140,12 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   for (long long u = first; u < p.units; u += nteams) {
     const long long e = u / p.nblocks;
     const int nb = (int)(u - e * p.nblocks);
-    if (issuer && u + nteams < p.units)  // the next unit's B into L2 while this one computes
-      ptx::prefetch_l2_bulk(p.B + ((u + nteams) / p.nblocks) * (long long)p.k * p.n, (uint32_t)(p.k * p.n * 8));
+    if (issuer && u + nteams < p.units) {  // the next unit's B into L2 while this one computes
+      const long long en = (u + nteams) / p.nblocks;
+      ptx::prefetch_l2_bulk(kPtr ? p.Ba[en] : p.B + en * (long long)p.k * p.n, (uint32_t)(p.k * p.n * 8));
+    }
     const int col0 = nb * kGNB + w * (kGFN * 8);
-    const double* Bg = p.B + e * (long long)p.k * p.n;
+    const double* Bg = kPtr ? p.Ba[e] : p.B + e * (long long)p.k * p.n;
     // GMem2Reg: the resident k-steps of B_w; the parked ones go to this warp's slab
 #pragma unroll
     for (int kk = 0; kk < RK; ++kk)
@@ -182,7 +209,7 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
         step(kk, bb);
       }
       // Reg2GMem: C_w block; lane holds (row g, cols 2t, 2t+1) of each 8x8 fragment
-      double* Cg = p.C + e * (long long)p.m * p.n;
+      double* Cg = kPtr ? p.Ca[e] : p.C + e * (long long)p.m * p.n;
 #pragma unroll
       for (int i = 0; i < kGFM; ++i) {
         const int row = mb * kGTM + i * 8 + g;
@@ -192,7 +219,7 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
             ptx::st_global_v2_f64(Cg + (long long)row * p.n + col0 + j * 8 + 2 * t, c[i][j][0], c[i][j][1]);
       }
       ptx::named_bar_sync(bar, kGP * 32);  // every warp finished reading buffer s
-      if (issuer && pu < p.units) {        // refill it with the block nbuf ahead
+      if ((issuer || kPtr) && pu < p.units) {  // refill it with the block nbuf ahead
         issue(pu, pmb, s);
         if (++pmb == p.mblocks) {
           pmb = 0;
@@ -253,12 +280,17 @@ bool dmma_gen_supported(int m, int n, int k) {
 int dmma_gen_resident_pct(int k) { return 100 * gen_plan(k, k, k).rs / (k / 4); }
 
 kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
-                              cudaStream_t stream) {
+                              cudaStream_t stream, const void* const* Aa, const void* const* Ba, void* const* Ca) {
   if (!dmma_gen_supported(m, n, k)) return KAMI_ERROR_NOT_SUPPORTED;
+  const bool ptr = Aa != nullptr;
+  if (ptr && (!Ba || !Ca)) return KAMI_ERROR_INVALID_VALUE;
   PFN_encodeTiled enc = get_encode_tiled();
   if (!enc) return KAMI_ERROR_CUDA;
   DmmaGenParams p;
   memset(&p, 0, sizeof(p));
+  p.Aa = reinterpret_cast<const double* const*>(Aa);
+  p.Ba = reinterpret_cast<const double* const*>(Ba);
+  p.Ca = reinterpret_cast<double* const*>(Ca);
   p.B = static_cast<const double*>(B);
   p.C = static_cast<double*>(C);
   p.batch = batch;
@@ -281,7 +313,7 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
   p.teams = gp.teams;
   p.nbuf = gp.nbuf;
   const uint32_t smem = gp.smem;
-  {  // A: (CE doubles, m, k/CE chunks, batch), box (CE, TM, k/CE, 1); rows past m zero-filled
+  if (!ptr) {  // A: (CE doubles, m, k/CE chunks, batch), box (CE, TM, k/CE, 1); rows past m zero-filled
     cuuint64_t dims[4] = {(cuuint64_t)ce, (cuuint64_t)m, (cuuint64_t)p.kch, (cuuint64_t)batch};
     cuuint64_t strides[3] = {(cuuint64_t)k * 8, (cuuint64_t)ce * 8, (cuuint64_t)m * k * 8};
     cuuint32_t box[4] = {(cuuint32_t)ce, (cuuint32_t)kGTM, (cuuint32_t)p.kch, 1};
@@ -291,7 +323,8 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
-  auto fn = gp.rk == kRK ? kami_dmma_gen_kernel<kRK> : kami_dmma_gen_kernel<kRKSmall>;
+  auto fn = ptr ? (gp.rk == kRK ? kami_dmma_gen_kernel<kRK, true> : kami_dmma_gen_kernel<kRKSmall, true>)
+                : (gp.rk == kRK ? kami_dmma_gen_kernel<kRK, false> : kami_dmma_gen_kernel<kRKSmall, false>);
   if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) != cudaSuccess)
     return KAMI_ERROR_CUDA;
   int dev = 0, sms = 148;
@@ -301,7 +334,7 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
   long long grid = sms < need ? sms : need;
   grid = apply_grid_cap(grid);
   fn<<<(unsigned)grid, kGP * 32 * (gp.rk == kRK ? 2 : 4), smem, stream>>>(p);
-  set_last_kernel("kami_dmma_gen_1d");
+  set_last_kernel(ptr ? "kami_dmma_gen_1d<ptr>" : "kami_dmma_gen_1d");
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
 }
 

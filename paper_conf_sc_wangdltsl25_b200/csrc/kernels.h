@@ -92,8 +92,10 @@ kami_status_t dmma_tma_launch(int m, int n, int k, long long batch, const void* 
 // --------------- FP64, whole size grid, k-slicing + residency ratio (dmma_gen.cu)
 bool dmma_gen_supported(int m, int n, int k);
 int dmma_gen_resident_pct(int k);  // share of B_w's k-steps kept in registers (rest parked in SMEM)
+// Aa/Ba/Ca != nullptr: device pointer arrays (kami_gemm_batched), A/B/C unused
 kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* A, const void* B, void* C,
-                              cudaStream_t stream);
+                              cudaStream_t stream, const void* const* Aa = nullptr, const void* const* Ba = nullptr,
+                              void* const* Ca = nullptr);
 
 // ------------------------- 16-bit pointer-array / variable-size (tc16_vb.cu)
 // dm/dn/dk: device arrays of per-entry sizes, or nullptr for uniform m, n, k.

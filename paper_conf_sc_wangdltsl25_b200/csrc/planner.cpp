@@ -445,6 +445,12 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
     *out = r;
     return KAMI_SUCCESS;
   }
+  // FP64 pointer arrays off the fixed shapes: dmma_gen with cp.async-fed A blocks
+  if (!is16 && pointer_array && algo == KAMI_ALGO_AUTO && !warp_shape && dmma_gen_supported(m, n, k)) {
+    fill_plan(&r, 4, KAMI_ALGO_1D, 4, m, n, k, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
   // FP64 1D with the broadcast operand fed by TMA (dmma_tma.cu; pointer arrays
   // through an address-space view of each entry)
   const bool tma_ok = !is16 && dmma_tma_supported(m, n, k);

@@ -64,3 +64,34 @@ def test_f64_plan_reports_residency():
     p = kami.plan(256, 256, 256, "f64")
     assert p["kernel"] == "dmma_gen" and p["kslice_regs_pct"] == 50
     assert kami.plan(128, 128, 128, "f64")["kslice_regs_pct"] == 100
+
+
+@pytest.mark.parametrize("shape", [(128, 128, 128, 23), (96, 40, 72, 41), (200, 136, 104, 9), (24, 40, 56, 77),
+                                   (48, 48, 48, 55), (256, 256, 256, 3)], ids=lambda s: "x".join(map(str, s)))
+def test_f64_general_pointer_arrays(shape):
+    """kami_gemm_batched in FP64 off the fixed shapes (A blocks copied by the
+    team with cp.async): scattered, shuffled entries; steady state."""
+    import numpy as np
+    import torch
+
+    import kami_inputs as ki
+    import oracle
+    m, n, k, batch = shape
+    for layout, dist, seed, cap in (("row", "unif", 11, 0), ("col", "int", 12, 3)):
+        A, B = ki.operands(m, n, k, batch, "f64", dist, seed=seed)
+        dA, dB = A.cuda().view(batch, -1), B.cuda().view(batch, -1)
+        dC = torch.full((batch, m * n), float("nan"), dtype=torch.float64, device="cuda")
+        perm = torch.randperm(batch, generator=torch.Generator().manual_seed(seed)).tolist()
+        pa = torch.tensor([dA[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
+        pb = torch.tensor([dB[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
+        pc = torch.tensor([dC[i].data_ptr() for i in perm], dtype=torch.int64, device="cuda")
+        with kami.grid_cap(cap):
+            kami.gemm_batched(m, n, k, batch, "f64", layout, pa, pb, pc)
+        torch.cuda.synchronize()
+        assert kami.last_kernel() == "kami_dmma_gen_1d<ptr>", kami.last_kernel()
+        Cref, S = oracle.gemm(m, n, k, batch, "f64", layout, A.numpy(), B.numpy(), with_scale=True)
+        got = oracle.to_row_major(dC.cpu().numpy().reshape(-1), batch, m, n, layout)
+        if dist == "int":
+            assert np.array_equal(got, Cref.reshape(batch, m, n))
+        else:
+            assert oracle.normalised_error(got, Cref, S) <= k * 2.0 ** -52
