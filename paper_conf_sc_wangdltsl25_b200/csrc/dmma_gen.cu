@@ -140,7 +140,7 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   for (long long u = first; u < p.units; u += nteams) {
     const long long e = u / p.nblocks;
     const int nb = (int)(u - e * p.nblocks);
-    if (issuer && u + nteams < p.units) {  // the next unit's B into L2 while this one computes
+    if (issuer && p.nblocks == 1 && u + nteams < p.units) {  // the next unit's B into L2 while this one computes
       const long long en = (u + nteams) / p.nblocks;
       ptx::prefetch_l2_bulk(kPtr ? p.Ba[en] : p.B + en * (long long)p.k * p.n, (uint32_t)(p.k * p.n * 8));
     }
