@@ -198,8 +198,11 @@ kami_status_t kami_spmm_bsr_strided_batched(int m, int n, int k, int64_t batch, 
  * is one contiguous code range), codes ascending, values at
  * vals[(b*max_nnzb + j)*256 + r*16 + c'] (row-major block).  B, C dense
  * row-major packed strided batches.  All arrays DEVICE memory.  Same sizes,
- * types, errors and kernel as kami_spmm_bsr_strided_batched (the kernel
- * decodes each block's position from its code). */
+ * types and errors as kami_spmm_bsr_strided_batched.  m > 128 (n a multiple
+ * of 32): the 2D schedule across a CTA pair, CTA r taking block rows
+ * [8r, 8r+8) = the Morton codes [128r, 128r+128), one contiguous range of the
+ * sorted codes; otherwise the 1D kernel, which decodes each block's position
+ * from its code. */
 kami_status_t kami_spmm_zmorton_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
                                                 const int* nnzb, const int* zcode, const void* vals, int max_nnzb,
                                                 const void* B, void* C, kami_stream_t stream);

@@ -274,6 +274,12 @@ kami_status_t kami_spmm_zmorton_strided_batched(int m, int n, int k, int64_t bat
   if (!nnzb || !zcode || !vals || !B || !C || max_nnzb == 0) return KAMI_ERROR_INVALID_VALUE;
   if (!aligned16(vals) || !aligned16(B) || !aligned16(C)) return KAMI_ERROR_MISALIGNED;
   if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
+  // m > 128: the 2D schedule across a CTA pair, each CTA finding its block
+  // rows as one contiguous Morton range (tc16_pair.cu); else the 1D kernel,
+  // which decodes each block's position from its code (tc16_vb.cu)
+  if (tc16_pair_supported(m, n, k))
+    return tc16_pair_launch(m, n, k, batch, dtype == KAMI_DTYPE_BF16, nullptr, B, C,
+                            reinterpret_cast<cudaStream_t>(stream), nnzb, zcode, vals, max_nnzb);
   return tc16_spmm_bsr_launch(m, n, k, batch, dtype == KAMI_DTYPE_BF16, nnzb, zcode, vals, max_nnzb, B, C,
                               reinterpret_cast<cudaStream_t>(stream), /*zorder=*/true);
 }

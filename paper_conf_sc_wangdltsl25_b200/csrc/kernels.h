@@ -65,8 +65,10 @@ kami_status_t tc16_ts_launch(int m, int n, int k, long long batch, bool bf16, in
 
 // ------------------------ tcgen05 CTA pair, KAMI-2D over 2 SMs (tc16_pair.cu)
 bool tc16_pair_supported(int m, int n, int k);
+// zcode != nullptr: A in Z-Morton block storage (nnzb, zcode, vals as kami_spmm_zmorton_strided_batched)
 kami_status_t tc16_pair_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B, void* C,
-                               cudaStream_t stream);
+                               cudaStream_t stream, const int* nnzb = nullptr, const int* zcode = nullptr,
+                               const void* vals = nullptr, int max_nnzb = 0);
 
 // ------------------------------------------------ warp-level CA (literal KAMI)
 // algo: 1 = 1D, 2 = 2D, 3 = 3D, 4 = non-CA tiled.  dtype: KAMI_DTYPE_*.

@@ -59,6 +59,15 @@ struct alignas(64) PairParams {
   uint32_t a_bytes, stage_bytes, tx_pair;
   int stages, acc_cols;
   uint32_t c_off, c_warp_bytes, bar_off, c_swz_bits;
+  // kSparse: A in Z-Morton block storage (Sec. 4.6: the 2D
+  // algorithm's storage).  CTA r's rows [128 r, 128 r + 128) are block rows
+  // [8 r, 8 r + 8): with at most 16 block columns those blocks are exactly the
+  // Morton codes [128 r, 128 r + 128) -- one contiguous range of the sorted
+  // code array, found by binary search (the "efficient submatrix indexing")
+  const int* nnzb;
+  const int* zcode;
+  const uint16_t* vals;
+  int max_nnzb;
 };
 
 __device__ __forceinline__ uint32_t cta_rank() {
@@ -110,7 +119,18 @@ __device__ __forceinline__ void commit_pair(uint64_t* bar) {  // arrive on bar i
       : "memory");
 }
 
-template <int kBf16>
+// first index in the ascending codes zc[0, nz) whose value is >= v
+__device__ __forceinline__ int lower_bound_dev(const int* zc, int nz, int v) {
+  int lo = 0, hi = nz;
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (__ldg(zc + mid) < v) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+
+template <int kBf16, bool kSparse>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
     kami_tc16_pair_kernel(const __grid_constant__ PairParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -119,18 +139,22 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
   uint64_t* empty = full + kPMaxStages;
   uint64_t* tfull = empty + kPMaxStages;
   uint64_t* tempty = tfull + 2;  // leader's are used
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* afull = tempty + 2;  // kSparse: this CTA's A copies of stage s landed (32 cp.async lanes)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(afull + kPMaxStages);
+  int* tab = reinterpret_cast<int*>(tmem_slot + 2);  // kSparse: [8 block rows][16 block cols] -> slot
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = cta_rank();
   const long long pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
 
   if (threadIdx.x == 0) {
-    ptx::prefetch_tmap(&p.tmA);
+    if (!kSparse) ptx::prefetch_tmap(&p.tmA);
     ptx::prefetch_tmap(&p.tmB);
     ptx::prefetch_tmap(&p.tmC);
     for (int s = 0; s < p.stages; ++s) {
-      ptx::mbar_init(&full[s], 1);
+      // sparse: the leader's expect_tx (B) + the peer's relay of its A copies
+      ptx::mbar_init(&full[s], kSparse ? 2 : 1);
       ptx::mbar_init(&empty[s], 1);
+      ptx::mbar_init(&afull[s], 32);
     }
     for (int a = 0; a < 2; ++a) {
       ptx::mbar_init(&tfull[a], 1);
@@ -151,7 +175,69 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
   const uint32_t tmem_base = *tmem_slot;
   const uint32_t smem_base = ptx::smem_u32(smem);
 
-  if (warp == 0) {
+  if (kSparse && warp == 0) {
+    // ------------------------- sparse A producer + B TMA (both CTAs)
+    RingPos r;
+    const uint32_t full_leader = mapa(ptx::smem_u32(full), 0);
+    const int bcols = p.Wk >> 4;  // 16-column blocks per k-chunk
+    const uint32_t a_bits = p.a_layout == 2 ? 3 : p.a_layout == 4 ? 2 : 1;
+    const uint32_t wk_b = (uint32_t)p.Wk * 2;
+    for (long long e = pair; e < p.batch; e += npairs) {
+      // this CTA's blocks: Morton codes [128 rank, 128 rank + 128)
+      const int* zc = p.zcode + e * (long long)p.max_nnzb;
+      const int nz = __ldg(p.nnzb + e);
+      const int lo = lower_bound_dev(zc, nz, 128 * (int)rank), hi = lower_bound_dev(zc, nz, 128 * (int)rank + 128);
+#pragma unroll
+      for (int i = 0; i < 4; ++i) tab[lane + 32 * i] = -1;
+      __syncwarp();
+      for (int j = lo + lane; j < hi; j += 32) {
+        const uint32_t z = (uint32_t)__ldg(zc + j);
+        uint32_t br = 0, bc = 0;
+#pragma unroll
+        for (int t = 0; t < 4; ++t) {
+          bc |= ((z >> (2 * t)) & 1u) << t;
+          br |= ((z >> (2 * t + 1)) & 1u) << t;
+        }
+        tab[(br & 7) * 16 + bc] = j;
+      }
+      __syncwarp();
+      const uint16_t* ve = p.vals + e * (long long)p.max_nnzb * 256;
+      for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
+        ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
+        const uint32_t sa = smem_base + r.s * p.stage_bytes;
+        if (lane == 0) {
+          if (rank == 0) ptx::mbar_arrive_expect_tx(&full[r.s], p.tx_pair);
+          tma_load_4d_pair(sa + p.a_bytes, &p.tmB, full_leader + r.s * 8, 0, kc * p.Wk,
+                           (int)rank * ((p.n >> 1) / p.Wn), (int)e);
+        }
+        // GMem2Reg + Reg2SMem of the present blocks, densified into the
+        // K-major swizzled A tile (absent blocks zero-filled)
+        for (int i = lane; i < 8 * bcols * 32; i += 32) {
+          const int blk = i >> 5, ch = i & 31;
+          const int lbr = blk / bcols, lbc = blk - lbr * bcols;
+          const int slot = tab[lbr * 16 + kc * bcols + lbc];
+          const int row = lbr * 16 + (ch >> 1), hh = ch & 1;
+          const uint32_t dst = sa + ptx::swz((uint32_t)row * wk_b + (uint32_t)(lbc * 2 + hh) * 16, a_bits);
+          const bool ok = slot >= 0;
+          ptx::cp_async_16(dst, ok ? ve + (long long)slot * 256 + (ch >> 1) * 16 + hh * 8 : ve, ok ? 16u : 0u);
+        }
+        ptx::cp_async_mbar_arrive_noinc(&afull[r.s]);
+      }
+    }
+    ptx::cp_async_wait<0>();
+  } else if (kSparse && warp == 1 && rank == 1) {
+    // ------------------ relay: the peer's A copies of stage s -> leader's full[s]
+    if (lane == 0) {
+      RingPos r;
+      const uint32_t full_leader = mapa(ptx::smem_u32(full), 0);
+      for (long long e = pair; e < p.batch; e += npairs)
+        for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
+          ptx::mbar_wait(&afull[r.s], r.ph);
+          ptx::fence_proxy_async_smem();  // generic (cp.async) writes -> the tensor core's async-proxy reads
+          mbar_arrive_cluster(full_leader + r.s * 8);
+        }
+    }
+  } else if (warp == 0) {
     // ---------------------------------------------- TMA (both CTAs)
     if (lane == 0) {
       RingPos r;
@@ -180,6 +266,10 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
         const uint32_t d = tmem_base + ra.s * p.acc_cols;
         for (int kc = 0; kc < p.k_chunks; ++kc, rb.next(p.stages)) {
           ptx::mbar_wait(&full[rb.s], rb.ph);
+          if constexpr (kSparse) {  // the leader's own A copies
+            ptx::mbar_wait(&afull[rb.s], rb.ph);
+            ptx::fence_proxy_async_smem();
+          }
           ptx::tc_fence_after();
           if (lane == 0) {
             const int nst = kc == p.k_chunks - 1 ? p.ksteps_last : p.ksteps_full;
@@ -284,8 +374,11 @@ bool tc16_pair_supported(int m, int n, int k) {
 }
 
 kami_status_t tc16_pair_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B, void* C,
-                               cudaStream_t stream) {
+                               cudaStream_t stream, const int* nnzb, const int* zcode, const void* vals,
+                               int max_nnzb) {
   if (!tc16_pair_supported(m, n, k)) return KAMI_ERROR_NOT_SUPPORTED;
+  const bool sparse = zcode != nullptr;
+  if (sparse && (k % 16 || !nnzb || !vals)) return KAMI_ERROR_NOT_SUPPORTED;
   PFN_encodeTiled enc = get_encode_tiled();
   if (!enc) return KAMI_ERROR_CUDA;
   PairParams p;
@@ -312,7 +405,12 @@ kami_status_t tc16_pair_launch(int m, int n, int k, long long batch, bool bf16, 
   p.b_kstep = 2 * p.b_sbo;
   p.a_bytes = pr_align(128 * wk_b);
   p.stage_bytes = p.a_bytes + pr_align((uint32_t)(n / 2) * wk_b);
-  p.tx_pair = 2 * (uint32_t)(128 * wk_b + (n / 2) * wk_b);
+  // (sparse: only B arrives by TMA; A by the producer warps' cp.async)
+  p.tx_pair = sparse ? 2 * (uint32_t)((n / 2) * wk_b) : 2 * (uint32_t)(128 * wk_b + (n / 2) * wk_b);
+  p.nnzb = nnzb;
+  p.zcode = zcode;
+  p.vals = static_cast<const uint16_t*>(vals);
+  p.max_nnzb = max_nnzb;
   p.c_swz_bits = wc_b == 128 ? 3 : wc_b == 64 ? 2 : 1;
   p.c_warp_bytes = pr_align(32 * wc_b);  // one atom x 32 rows, double-buffered per warp
   const uint32_t c_total = 8 * 2 * p.c_warp_bytes;
@@ -326,7 +424,7 @@ kami_status_t tc16_pair_launch(int m, int n, int k, long long batch, bool bf16, 
   p.bar_off = p.c_off + c_total;
   const uint32_t smem = p.bar_off + 1024 + 1024;
   const CUtensorMapDataType dt = bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
-  {
+  if (!sparse) {
     cuuint64_t dims[3] = {(cuuint64_t)k, (cuuint64_t)m, (cuuint64_t)batch};
     cuuint64_t strides[2] = {(cuuint64_t)k * 2, (cuuint64_t)m * k * 2};
     cuuint32_t box[3] = {(cuuint32_t)p.Wk, 128, 1};
@@ -360,10 +458,12 @@ kami_status_t tc16_pair_launch(int m, int n, int k, long long batch, bool bf16, 
   if (pairs > batch) pairs = batch;
   const long long cap = apply_grid_cap(2 * pairs);
   pairs = cap / 2 > 0 ? cap / 2 : 1;
-  auto fn = bf16 ? kami_tc16_pair_kernel<1> : kami_tc16_pair_kernel<0>;
+  auto fn = sparse ? (bf16 ? kami_tc16_pair_kernel<1, true> : kami_tc16_pair_kernel<0, true>)
+                   : (bf16 ? kami_tc16_pair_kernel<1, false> : kami_tc16_pair_kernel<0, false>);
   cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   fn<<<(unsigned)(2 * pairs), kPThreads, smem, stream>>>(p);
-  set_last_kernel(bf16 ? "kami_tc16_pair_2d<bf16>" : "kami_tc16_pair_2d<f16>");
+  set_last_kernel(sparse ? (bf16 ? "kami_tc16_pair_2d<bf16,spmm_zmorton>" : "kami_tc16_pair_2d<f16,spmm_zmorton>")
+                         : (bf16 ? "kami_tc16_pair_2d<bf16>" : "kami_tc16_pair_2d<f16>"));
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
 }
 

@@ -59,7 +59,7 @@ def test_spmm_dense_equivalence():
 # ------------------------------------------- Z-Morton block storage (f3)
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 @pytest.mark.parametrize("shape", [(16, 16, 16), (64, 64, 64), (128, 128, 128), (192, 64, 256), (256, 256, 32),
-                                   (48, 80, 112)])
+                                   (48, 80, 112), (256, 256, 256), (224, 96, 160), (144, 32, 48)])
 @pytest.mark.parametrize("density", [0.5, 1.0, 0.1])
 def test_spmm_zmorton_vs_oracle(dtype, shape, density):
     """A in multi-level Z-Morton block storage (Sec. 4.6), built
@@ -77,6 +77,8 @@ def test_spmm_zmorton_vs_oracle(dtype, shape, density):
                                           torch.from_numpy(zcode).cuda(), zv.cuda(), B.cuda(), C)
         torch.cuda.synchronize()
         assert "spmm_zmorton" in kami.last_kernel()
+        if m > 128:  # the 2D schedule across a CTA pair
+            assert kami.last_kernel().startswith("kami_tc16_pair_2d"), kami.last_kernel()
         Cref, S = oracle.spmm_zmorton(m, n, k, batch, dtype, nnzb, zcode, zvals, ki.as_bits(B), with_scale=True)
         got_bits = ki.as_bits(C.cpu()).reshape(batch, m, n)
         if dist == "int":
