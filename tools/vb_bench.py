@@ -38,6 +38,37 @@ if a.mode == "spmm":
     nnzb = float(rp[:, -1].sum())
     flops = 2.0 * nnzb * 256 * n  # useful (sparse) flops
     byts = nnzb * (512 + 4) + a.batch * ((m // 16 + 1) * 4 + (k * n + m * n) * 2)
+elif a.mode == "zmorton":
+    # the same block-sparse matrices in Z-Morton block storage, built here with
+    # torch (codes = interleaved block row / column bits, sorted per entry)
+    m, n, k = (int(x) for x in a.shape.split("x"))
+    rp, cb, v, B = ki.bsr_operands(m, n, k, a.batch, a.dtype, density=a.density, device="cuda")
+    mb = m // 16
+    cnt = (rp[:, 1:] - rp[:, :-1]).long()
+    br = torch.repeat_interleave(torch.arange(mb, device="cuda").repeat(a.batch), cnt.reshape(-1))
+    nnz = rp[:, -1].long()
+    ent = torch.repeat_interleave(torch.arange(a.batch, device="cuda"), nnz)
+    slot = torch.arange(int(nnz.sum()), device="cuda") - torch.repeat_interleave(torch.cumsum(nnz, 0) - nnz, nnz)
+    bc = cb[ent, slot].long()
+    z = torch.zeros_like(br)
+    for t in range(4):
+        z |= ((bc >> t) & 1) << (2 * t)
+        z |= ((br >> t) & 1) << (2 * t + 1)
+    key = ent * 1024 + z
+    order = torch.argsort(key)
+    zc = torch.full_like(cb, -1)
+    newslot = slot  # ranks within the entry after sorting
+    ent_s, z_s, old_s = ent[order], z[order], slot[order]
+    rank = torch.arange(len(order), device="cuda") - torch.repeat_interleave(torch.cumsum(nnz, 0) - nnz, nnz)
+    zc[ent_s, rank] = z_s.int()
+    zv = torch.zeros_like(v)
+    zv[ent_s, rank] = v[ent_s, old_s]
+    nz = nnz.int()
+    C = torch.empty(a.batch * m * n, dtype=B.dtype, device="cuda")
+    run = lambda: kami.spmm_zmorton_strided_batched(m, n, k, a.batch, a.dtype, nz, zc, zv, B, C)  # noqa: E731
+    nnzb = float(nnz.sum())
+    flops = 2.0 * nnzb * 256 * n
+    byts = nnzb * (512 + 4) + a.batch * (4 + (k * n + m * n) * 2)
 elif a.mode == "ptr":
     m, n, k = (int(x) for x in a.shape.split("x"))
     A, B = ki.operands(m, n, k, a.batch, a.dtype, "unif", device="cuda")
