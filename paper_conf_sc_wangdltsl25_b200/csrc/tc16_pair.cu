@@ -131,7 +131,7 @@ __device__ __forceinline__ int lower_bound_dev(const int* zc, int nz, int v) {
 }
 
 template <int kBf16, bool kSparse>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads + (kSparse ? 128 : 0), 1)
     kami_tc16_pair_kernel(const __grid_constant__ PairParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = smem_raw + ((1024u - (ptx::smem_u32(smem_raw) & 1023u)) & 1023u);
@@ -154,7 +154,7 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
       // sparse: the leader's expect_tx (B) + the peer's relay of its A copies
       ptx::mbar_init(&full[s], kSparse ? 2 : 1);
       ptx::mbar_init(&empty[s], 1);
-      ptx::mbar_init(&afull[s], 32);
+      ptx::mbar_init(&afull[s], 128);  // kSparse: the copier warpgroup
     }
     for (int a = 0; a < 2; ++a) {
       ptx::mbar_init(&tfull[a], 1);
@@ -176,21 +176,34 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
   const uint32_t smem_base = ptx::smem_u32(smem);
 
   if (kSparse && warp == 0) {
-    // ------------------------- sparse A producer + B TMA (both CTAs)
+    // ------------------------------------- B TMA (both CTAs), sparse mode
+    if (lane == 0) {
+      RingPos r;
+      const uint32_t full_leader = mapa(ptx::smem_u32(full), 0);
+      for (long long e = pair; e < p.batch; e += npairs)
+        for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
+          ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
+          if (rank == 0) ptx::mbar_arrive_expect_tx(&full[r.s], p.tx_pair);
+          tma_load_4d_pair(smem_base + r.s * p.stage_bytes + p.a_bytes, &p.tmB, full_leader + r.s * 8, 0,
+                           kc * p.Wk, (int)rank * ((p.n >> 1) / p.Wn), (int)e);
+        }
+    }
+  } else if (kSparse && warp >= kPThreads / 32) {
+    // ------------- sparse A copier warpgroup (both CTAs): GMem2Reg + Reg2SMem
+    const int tid = threadIdx.x - kPThreads;  // 0..127
     RingPos r;
-    const uint32_t full_leader = mapa(ptx::smem_u32(full), 0);
     const int bcols = p.Wk >> 4;  // 16-column blocks per k-chunk
     const uint32_t a_bits = p.a_layout == 2 ? 3 : p.a_layout == 4 ? 2 : 1;
     const uint32_t wk_b = (uint32_t)p.Wk * 2;
     for (long long e = pair; e < p.batch; e += npairs) {
-      // this CTA's blocks: Morton codes [128 rank, 128 rank + 128)
+      // this CTA's blocks: Morton codes [128 rank, 128 rank + 128), one range
       const int* zc = p.zcode + e * (long long)p.max_nnzb;
       const int nz = __ldg(p.nnzb + e);
       const int lo = lower_bound_dev(zc, nz, 128 * (int)rank), hi = lower_bound_dev(zc, nz, 128 * (int)rank + 128);
-#pragma unroll
-      for (int i = 0; i < 4; ++i) tab[lane + 32 * i] = -1;
-      __syncwarp();
-      for (int j = lo + lane; j < hi; j += 32) {
+      ptx::named_bar_sync(3, 128);  // the previous unit's copies are all issued: the table is free
+      tab[tid] = -1;
+      ptx::named_bar_sync(3, 128);
+      for (int j = lo + tid; j < hi; j += 128) {
         const uint32_t z = (uint32_t)__ldg(zc + j);
         uint32_t br = 0, bc = 0;
 #pragma unroll
@@ -200,19 +213,15 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kPThreads, 1)
         }
         tab[(br & 7) * 16 + bc] = j;
       }
-      __syncwarp();
+      ptx::named_bar_sync(3, 128);
       const uint16_t* ve = p.vals + e * (long long)p.max_nnzb * 256;
       for (int kc = 0; kc < p.k_chunks; ++kc, r.next(p.stages)) {
         ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
         const uint32_t sa = smem_base + r.s * p.stage_bytes;
-        if (lane == 0) {
-          if (rank == 0) ptx::mbar_arrive_expect_tx(&full[r.s], p.tx_pair);
-          tma_load_4d_pair(sa + p.a_bytes, &p.tmB, full_leader + r.s * 8, 0, kc * p.Wk,
-                           (int)rank * ((p.n >> 1) / p.Wn), (int)e);
-        }
-        // GMem2Reg + Reg2SMem of the present blocks, densified into the
-        // K-major swizzled A tile (absent blocks zero-filled)
-        for (int i = lane; i < 8 * bcols * 32; i += 32) {
+        // the present blocks densified into the K-major swizzled A tile
+        // (absent blocks zero-filled); consecutive threads take consecutive
+        // 16-byte chunks of a block (contiguous 512-byte block rows)
+        for (int i = tid; i < 8 * bcols * 32; i += 128) {
           const int blk = i >> 5, ch = i & 31;
           const int lbr = blk / bcols, lbc = blk - lbr * bcols;
           const int slot = tab[lbr * 16 + kc * bcols + lbc];
@@ -461,7 +470,7 @@ kami_status_t tc16_pair_launch(int m, int n, int k, long long batch, bool bf16, 
   auto fn = sparse ? (bf16 ? kami_tc16_pair_kernel<1, true> : kami_tc16_pair_kernel<0, true>)
                    : (bf16 ? kami_tc16_pair_kernel<1, false> : kami_tc16_pair_kernel<0, false>);
   cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  fn<<<(unsigned)(2 * pairs), kPThreads, smem, stream>>>(p);
+  fn<<<(unsigned)(2 * pairs), kPThreads + (sparse ? 128 : 0), smem, stream>>>(p);
   set_last_kernel(sparse ? (bf16 ? "kami_tc16_pair_2d<bf16,spmm_zmorton>" : "kami_tc16_pair_2d<f16,spmm_zmorton>")
                          : (bf16 ? "kami_tc16_pair_2d<bf16>" : "kami_tc16_pair_2d<f16>"));
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
