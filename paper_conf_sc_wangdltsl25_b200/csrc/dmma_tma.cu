@@ -24,6 +24,7 @@
 
 #include "kernels.h"
 #include "ptx.cuh"
+#include "sched.cuh"
 
 namespace kami {
 namespace {
@@ -54,16 +55,8 @@ struct DmmaTmaParams {
   double* const* Ca;
 };
 
-// Address-space view of the pointer-array A map (same scheme as tc16.cu): the
-// entry at byte address q is the box at outer coordinates
-// ((q - kViewBase) / 16 mod 2^24, (q - kViewBase) / 2^28).  The box is the
-// whole entry (16, m, k/16), never partly out of bounds.
-constexpr unsigned long long kViewBase = 256;
-__device__ __forceinline__ void view_coords(const void* q, int& lo, int& hi) {
-  const unsigned long long off = reinterpret_cast<unsigned long long>(q) - kViewBase;
-  lo = (int)((off >> 4) & 0xFFFFFFull);
-  hi = (int)(off >> 28);
-}
+// Pointer-array A: address-space view (sched.cuh); the box is the whole entry
+// (16, m, k/16), never partly out of bounds.
 template <bool kPtr>
 __device__ __forceinline__ void load_a_entry(void* dst, const DmmaTmaParams& prm, uint64_t* bar, long long e) {
   if constexpr (kPtr) {

@@ -44,4 +44,20 @@ struct RingPos {
   }
 };
 
+// Pointer arrays on TMA (tc16.cu, dmma_tma.cu, tc16_vb.cu).  A tensor map
+// cannot follow a pointer array, but all entries live in one virtual address
+// space: a view map describes that space as a tensor whose two outer
+// dimensions are (16-byte offset mod 2^28, 2^28-byte offset) from kViewBase,
+// so the box of the entry at byte address q has outer coordinates
+// ((q - kViewBase) / 16 mod 2^24, (q - kViewBase) / 2^28).  Entries are 16-byte
+// aligned (kami.h) and the view covers 2^48 bytes; the inner dimensions are the
+// entry's own, and a box must never leave them (measured on sm_100a: a box
+// partly out of bounds of a view faults where a strided map zero-fills).
+constexpr unsigned long long kViewBase = 256;
+__device__ __forceinline__ void view_coords(const void* q, int& lo, int& hi) {
+  const unsigned long long off = reinterpret_cast<unsigned long long>(q) - kViewBase;
+  lo = (int)((off >> 4) & 0xFFFFFFull);
+  hi = (int)(off >> 28);
+}
+
 }  // namespace kami

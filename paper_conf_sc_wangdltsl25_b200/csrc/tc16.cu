@@ -138,21 +138,7 @@ struct alignas(64) Tc16Params {
   CUtensorMap tmAt, tmCat;             // pointer arrays: boxes of m % 128 rows for the last m-tile
 };
 
-// Pointer arrays on TMA.  A tensor map cannot follow a pointer array, but all
-// entries live in one virtual address space: the pointer-array maps describe
-// that space as a tensor whose two outer dimensions are (16-byte offset mod
-// 2^28, 2^28-byte offset) from kViewBase, so the box of the entry at byte
-// address q has outer coordinates ((q - kViewBase) / 16 mod 2^24,
-// (q - kViewBase) / 2^28).  Entries are 16-byte aligned (kami.h), the view
-// covers 2^48 bytes, and the inner dimensions are the entry's own (k, m) /
-// (Wn, k, n/Wn) / (Wc, m, n/Wc), so the usual out-of-bounds fill (k tail,
-// rows past m) and store clipping still apply per entry.
-constexpr unsigned long long kViewBase = 256;
-__device__ __forceinline__ void view_coords(const void* q, int& lo, int& hi) {
-  const unsigned long long off = reinterpret_cast<unsigned long long>(q) - kViewBase;
-  lo = (int)((off >> 4) & 0xFFFFFFull);
-  hi = (int)(off >> 28);
-}
+// Pointer arrays on TMA: address-space views (view_coords, sched.cuh).
 
 template <int kIn>
 __device__ __forceinline__ void umma(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {

@@ -23,6 +23,7 @@
 #include <cstdint>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <numeric>
 
 #include "kernels.h"
@@ -78,6 +79,13 @@ struct alignas(64) VbParams {
   // entry e at As + e m k, Bs + e k n, Cs + e m n
   int strided;
   const uint16_t* As;
+  // TMA views (non-SpMM modes): an entry with k % 64 == 0 has its
+  // A chunk (64 k, live tile rows) loaded by one TMA box through an
+  // address-space view (sched.cuh), and with n % 64 == 0 too its B chunk
+  // (64 n, 64 k, n / 64); the boxes land in the same 128-byte-swizzled
+  // layouts the copies build.  Other entries keep the cp.async path.
+  // vmap[(k / 64 - 1) * 16 + rows / 8 - 1]: A views; vmap[64 + (n / 64 - 1) * 4 + k / 64 - 1]: B views
+  const CUtensorMap* vmap;
 };
 
 __device__ __forceinline__ const uint16_t* entry_B(const VbParams& p, long long e, int k, int n) {
@@ -152,7 +160,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < p.stages; ++s) {
-      ptx::mbar_init(&full[s], 128 + (p.b_tma ? 1 : 0));  // + the B TMA's expect_tx arrival
+      // + thread 0's arrival: the B TMA's expect_tx (SpMM), or per stage either
+      // the view TMAs' expect_tx or a plain arrival (TMA views)
+      ptx::mbar_init(&full[s], 128 + ((p.b_tma || p.vmap) ? 1 : 0));
       ptx::mbar_init(&empty[s], 1);
     }
     for (int a = 0; a < p.acc_bufs; ++a) {
@@ -285,11 +295,30 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         // a multiple of 16; zero-filled past k): for k < 64 the copy issue --
         // the producer's bottleneck (tools/trace_vb.py) -- shrinks with k.
         const int kpad_c = min(64, ((k + 15) & ~15) - kc * 64);
+        // TMA views for this unit (uniform across the warpgroup)
+        const bool va = p.vmap != nullptr && G == 1 && (k & 63) == 0;
+        const bool vb = va && (n & 63) == 0;
+        if (p.vmap && tid == 0) {
+          if (va) {
+            int lo, hi;
+            ptx::mbar_arrive_expect_tx(&full[s], (uint32_t)rows * 128u + (vb ? (uint32_t)n * 128u : 0u));
+            view_coords(pa, lo, hi);
+            ptx::tma_load_4d(smem + s * p.stage_bytes, p.vmap + ((k >> 6) - 1) * 16 + (rows >> 3) - 1, &full[s],
+                             kc * 64, U.mt * 128, lo, hi);
+            if (vb) {
+              view_coords(pb, lo, hi);
+              ptx::tma_load_5d(smem + s * p.stage_bytes + kAReg, p.vmap + 64 + ((n >> 6) - 1) * 4 + (k >> 6) - 1,
+                               &full[s], 0, kc * 64, 0, lo, hi);
+            }
+          } else {
+            ptx::mbar_arrive(&full[s]);
+          }
+        }
         // A: thread = (16-byte chunk j, row r0 + rstep q): the chunks of a row
         // are spread over 2^cshift threads, the swizzle phase (r & 7) is fixed
         // per thread (rstep is a multiple of 8) and addresses advance by
         // constant strides.
-        {
+        if (!va) {
           const int cpa = kpad_c >> 3;  // live chunks per row: 2, 4, 6 or 8
           const int cshift = cpa <= 2 ? 1 : cpa <= 4 ? 2 : 3;
           const int j = tid & ((1 << cshift) - 1), r0 = tid >> cshift, rstep = 128 >> cshift;
@@ -320,7 +349,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         }
         // B: per entry 64 k-rows x n/8 chunks at columns [g n, g n + n) of the
         // N-major tile (atoms of 64 columns x 64 k-rows)
-        if (p.b_tma) {  // one TMA box: G entries x 64 k-rows x n (zero-filled past k / batch)
+        if (vb) {
+          // (view TMA issued above)
+        } else if (p.b_tma) {  // one TMA box: G entries x 64 k-rows x n (zero-filled past k / batch)
           if (tid == 0) {
             ptx::mbar_arrive_expect_tx(&full[s], p.b_tx);
             ptx::tma_load_4d(smem + s * p.stage_bytes + kAReg, &p.tmB, &full[s], 0, kc * 64, 0, (int)U.e0);
@@ -533,6 +564,62 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   if (warp == 4) ptx::tmem_dealloc(tmem_base, p.acc_cols * p.acc_bufs);
 }
 
+// The TMA view maps of the non-SpMM modes: they depend only on the shape class,
+// not on any pointer (the view's base is kViewBase), so one table per device
+// serves every launch.  A (k = 64 kq, rows): dims (k, 256, 2^24, 2^20), box
+// (64, rows, 1, 1); B (n = 64 nq, k = 64 kq): dims (64, k, n / 64, 2^24, 2^20),
+// box (64, 64, n / 64, 1, 1); both 128-byte swizzle.
+// Built on the first launch that is not being captured into a CUDA graph (the
+// allocation and copy are not capturable); until then the copies are used.
+const CUtensorMap* vb_view_maps(cudaStream_t stream) {
+  static std::mutex mu;
+  static const CUtensorMap* table[64] = {};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  std::lock_guard<std::mutex> lock(mu);
+  if (table[dev]) return table[dev];
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(stream, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) return nullptr;
+  PFN_encodeTiled enc = get_encode_tiled();
+  if (!enc) return nullptr;
+  CUtensorMap h[80];
+  memset(h, 0, sizeof(h));
+  void* const vbase = reinterpret_cast<void*>(kViewBase);
+  const cuuint64_t vlo = 1ull << 24, vhi = 1ull << 20, vstride_hi = 1ull << 28;
+  for (int kq = 1; kq <= 4; ++kq)
+    for (int r = 8; r <= 128; r += 8) {
+      const int k = 64 * kq;
+      cuuint64_t dims[4] = {(cuuint64_t)k, 256, vlo, vhi};
+      cuuint64_t strides[3] = {(cuuint64_t)k * 2, 16, vstride_hi};
+      cuuint32_t box[4] = {64, (cuuint32_t)r, 1, 1};
+      cuuint32_t es[4] = {1, 1, 1, 1};
+      if (enc(&h[(kq - 1) * 16 + r / 8 - 1], CU_TENSOR_MAP_DATA_TYPE_UINT16, 4, vbase, dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return nullptr;
+    }
+  for (int nq = 1; nq <= 4; ++nq)
+    for (int kq = 1; kq <= 4; ++kq) {
+      const int n = 64 * nq, k = 64 * kq;
+      cuuint64_t dims[5] = {64, (cuuint64_t)k, (cuuint64_t)nq, vlo, vhi};
+      cuuint64_t strides[4] = {(cuuint64_t)n * 2, 128, 16, vstride_hi};
+      cuuint32_t box[5] = {64, 64, (cuuint32_t)nq, 1, 1};
+      cuuint32_t es[5] = {1, 1, 1, 1, 1};
+      if (enc(&h[64 + (nq - 1) * 4 + kq - 1], CU_TENSOR_MAP_DATA_TYPE_UINT16, 5, vbase, dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return nullptr;
+    }
+  void* d = nullptr;
+  if (cudaMalloc(&d, sizeof(h)) != cudaSuccess) return nullptr;
+  if (cudaMemcpy(d, h, sizeof(h), cudaMemcpyHostToDevice) != cudaSuccess) {
+    cudaFree(d);
+    return nullptr;
+  }
+  table[dev] = static_cast<const CUtensorMap*>(d);  // process lifetime
+  return table[dev];
+}
+
 int pow2_ceil(int x) {
   int q = 32;
   while (q < x) q <<= 1;
@@ -558,6 +645,11 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   {
     const char* d = getenv("KAMI_VB_DEBUG");
     p.dbg = d ? atoi(d) : 0;
+  }
+  // TMA views (one entry per tile; KAMI_VB_VIEWS=0 disables them, A/B experiments)
+  if (!p.bsr && p.G == 1) {
+    const char* v = getenv("KAMI_VB_VIEWS");
+    if (!v || atoi(v) != 0) p.vmap = vb_view_maps(stream);
   }
   const uint32_t smem = p.bar_off + 2048 + 1024;
   auto fn = bf16 ? kami_tc16_vb_kernel<true> : kami_tc16_vb_kernel<false>;
