@@ -79,14 +79,40 @@ struct alignas(64) VbParams {
   // entry e at As + e m k, Bs + e k n, Cs + e m n
   int strided;
   const uint16_t* As;
-  // TMA views (non-SpMM modes): an entry with k % 64 == 0 has its
-  // A chunk (64 k, live tile rows) loaded by one TMA box through an
-  // address-space view (sched.cuh), and with n % 64 == 0 too its B chunk
-  // (64 n, 64 k, n / 64); the boxes land in the same 128-byte-swizzled
-  // layouts the copies build.  Other entries keep the cp.async path.
-  // vmap[(k / 64 - 1) * 16 + rows / 8 - 1]: A views; vmap[64 + (n / 64 - 1) * 4 + k / 64 - 1]: B views
+  // TMA views (non-SpMM modes with one entry per tile): an entry
+  // whose k is 16, 32 or a multiple of 64 has its A chunk (Wk = min(k, 64)
+  // columns x the tile's live rows) loaded by one TMA box through an
+  // address-space view (sched.cuh), and if n is 16, 32 or a multiple of 64
+  // too, its B chunk (Wn = min(n, 64) columns x Wk k-rows x n / Wn atoms).
+  // Boxes use the 2 Wk- / 2 Wn-byte swizzle, so the MMA descriptors follow the
+  // unit's (Wk, Wn) (vb_layout); other entries keep the cp.async path and its
+  // 128-byte layouts.  vmap[vidx(k) * 16 + rows / 8 - 1]: A views,
+  // vmap[96 + vidx(n) * 6 + vidx(k)]: B views, vidx: 16, 32, 64, 128, 192, 256 -> 0..5
   const CUtensorMap* vmap;
+  int vsmall;  // 0: views only for multiples of 64 (A/B experiments, KAMI_VB_VIEWS=2)
 };
+
+// TMA-view class of a size (16, 32 or a multiple of 64 up to 256), else -1
+__host__ __device__ __forceinline__ int vidx(int x) {
+  return x == 16 ? 0 : x == 32 ? 1 : ((x & 63) == 0 && x <= 256) ? 1 + (x >> 6) : -1;
+}
+// Shared-memory layout of one unit's stage: A rows of wa bytes (K-major,
+// wa-byte swizzle), B atoms of wb-byte rows x kr k-rows (N-major, wb-byte
+// swizzle).  The copies build (128, 128, 64); view units (min(k, 64) 2,
+// min(n, 64) 2, min(k, 64)).
+struct VbLayout {
+  bool va, vb;
+  uint32_t wa, wb, kr;
+};
+__device__ __forceinline__ VbLayout vb_layout(const VbParams& p, int n, int k) {
+  VbLayout L;
+  L.va = p.vmap != nullptr && p.G == 1 && vidx(k) >= (p.vsmall ? 0 : 2);
+  L.vb = L.va && vidx(n) >= (p.vsmall ? 0 : 2);
+  L.wa = L.va ? (uint32_t)min(k, 64) * 2u : 128u;
+  L.wb = L.vb ? (uint32_t)min(n, 64) * 2u : 128u;
+  L.kr = L.vb ? (uint32_t)min(k, 64) : 64u;
+  return L;
+}
 
 __device__ __forceinline__ const uint16_t* entry_B(const VbParams& p, long long e, int k, int n) {
   return (p.bsr || p.strided) ? p.Bs + e * (long long)k * n : reinterpret_cast<const uint16_t*>(p.B[e]);
@@ -296,19 +322,19 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         // the producer's bottleneck (tools/trace_vb.py) -- shrinks with k.
         const int kpad_c = min(64, ((k + 15) & ~15) - kc * 64);
         // TMA views for this unit (uniform across the warpgroup)
-        const bool va = p.vmap != nullptr && G == 1 && (k & 63) == 0;
-        const bool vb = va && (n & 63) == 0;
+        const VbLayout lay = vb_layout(p, n, k);
+        const bool va = lay.va, vb = lay.vb;
         if (p.vmap && tid == 0) {
           if (va) {
             int lo, hi;
-            ptx::mbar_arrive_expect_tx(&full[s], (uint32_t)rows * 128u + (vb ? (uint32_t)n * 128u : 0u));
+            ptx::mbar_arrive_expect_tx(&full[s], (uint32_t)rows * lay.wa + (vb ? lay.kr * (uint32_t)n * 2u : 0u));
             view_coords(pa, lo, hi);
-            ptx::tma_load_4d(smem + s * p.stage_bytes, p.vmap + ((k >> 6) - 1) * 16 + (rows >> 3) - 1, &full[s],
-                             kc * 64, U.mt * 128, lo, hi);
+            ptx::tma_load_4d(smem + s * p.stage_bytes, p.vmap + vidx(k) * 16 + (rows >> 3) - 1, &full[s], kc * 64,
+                             U.mt * 128, lo, hi);
             if (vb) {
               view_coords(pb, lo, hi);
-              ptx::tma_load_5d(smem + s * p.stage_bytes + kAReg, p.vmap + 64 + ((n >> 6) - 1) * 4 + (k >> 6) - 1,
-                               &full[s], 0, kc * 64, 0, lo, hi);
+              ptx::tma_load_5d(smem + s * p.stage_bytes + kAReg, p.vmap + 96 + vidx(n) * 6 + vidx(k), &full[s], 0,
+                               kc * 64, 0, lo, hi);
             }
           } else {
             ptx::mbar_arrive(&full[s]);
@@ -431,6 +457,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, (p.G * U.n + 15) & ~15, 0, 1);
       const int kpad = (U.k + 15) / 16 * 16;
       const int kchunks = (U.k + 63) / 64;
+      const VbLayout lay = vb_layout(p, U.n, U.k);
       for (int kc = 0; kc < kchunks; ++kc, rs.next(p.stages), ++it) {
         const uint32_t s = rs.s;
         ptx::mbar_wait(&full[s], rs.ph);
@@ -441,8 +468,11 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
           const uint32_t sa = smem_base + s * p.stage_bytes, sb = sa + kAReg;
           const int nsteps = (kpad - kc * 64) >= 64 ? 4 : (kpad - kc * 64) / 16;
           for (int ks = 0; ks < nsteps; ++ks) {
-            const uint64_t adesc = ptx::make_smem_desc(sa + ks * 32, 16, 1024, 2);
-            const uint64_t bdesc = ptx::make_smem_desc(sb + ks * 2048, 8192, 1024, 2);
+            // A: K-major, a K step is 32 bytes along the row; B: N-major, a K
+            // step is 16 k-rows, atoms kr k-rows apart
+            const uint64_t adesc = ptx::make_smem_desc(sa + ks * 32, 16, 8 * lay.wa, ptx::umma_layout_code(lay.wa));
+            const uint64_t bdesc = ptx::make_smem_desc(sb + ks * 16 * lay.wb, lay.kr * lay.wb, 8 * lay.wb,
+                                                       ptx::umma_layout_code(lay.wb));
             ptx::umma_f16_ss(d_tmem, adesc, bdesc, idesc, (kc | ks) != 0);
           }
           ptx::umma_commit(&empty[s]);
@@ -566,9 +596,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
 
 // The TMA view maps of the non-SpMM modes: they depend only on the shape class,
 // not on any pointer (the view's base is kViewBase), so one table per device
-// serves every launch.  A (k = 64 kq, rows): dims (k, 256, 2^24, 2^20), box
-// (64, rows, 1, 1); B (n = 64 nq, k = 64 kq): dims (64, k, n / 64, 2^24, 2^20),
-// box (64, 64, n / 64, 1, 1); both 128-byte swizzle.
+// serves every launch.  A (k, rows): dims (k, 256, 2^24, 2^20), box (Wk, rows,
+// 1, 1); B (n, k): dims (Wn, k, n / Wn, 2^24, 2^20), box (Wn, Wk, n / Wn, 1, 1);
+// Wk = min(k, 64), Wn = min(n, 64), swizzle 2 Wk / 2 Wn bytes.
 // Built on the first launch that is not being captured into a CUDA graph (the
 // allocation and copy are not capturable); until then the copies are used.
 const CUtensorMap* vb_view_maps(cudaStream_t stream) {
@@ -582,31 +612,36 @@ const CUtensorMap* vb_view_maps(cudaStream_t stream) {
   if (cudaStreamIsCapturing(stream, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) return nullptr;
   PFN_encodeTiled enc = get_encode_tiled();
   if (!enc) return nullptr;
-  CUtensorMap h[80];
+  constexpr int kMaps = 96 + 36;
+  CUtensorMap h[kMaps];
   memset(h, 0, sizeof(h));
   void* const vbase = reinterpret_cast<void*>(kViewBase);
   const cuuint64_t vlo = 1ull << 24, vhi = 1ull << 20, vstride_hi = 1ull << 28;
-  for (int kq = 1; kq <= 4; ++kq)
+  const int cls[6] = {16, 32, 64, 128, 192, 256};
+  auto swz = [](int bytes) {
+    return bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+  };
+  for (int ki = 0; ki < 6; ++ki)
     for (int r = 8; r <= 128; r += 8) {
-      const int k = 64 * kq;
+      const int k = cls[ki], wk = k < 64 ? k : 64;
       cuuint64_t dims[4] = {(cuuint64_t)k, 256, vlo, vhi};
       cuuint64_t strides[3] = {(cuuint64_t)k * 2, 16, vstride_hi};
-      cuuint32_t box[4] = {64, (cuuint32_t)r, 1, 1};
+      cuuint32_t box[4] = {(cuuint32_t)wk, (cuuint32_t)r, 1, 1};
       cuuint32_t es[4] = {1, 1, 1, 1};
-      if (enc(&h[(kq - 1) * 16 + r / 8 - 1], CU_TENSOR_MAP_DATA_TYPE_UINT16, 4, vbase, dims, strides, box, es,
-              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+      if (enc(&h[ki * 16 + r / 8 - 1], CU_TENSOR_MAP_DATA_TYPE_UINT16, 4, vbase, dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, swz(wk * 2), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
         return nullptr;
     }
-  for (int nq = 1; nq <= 4; ++nq)
-    for (int kq = 1; kq <= 4; ++kq) {
-      const int n = 64 * nq, k = 64 * kq;
-      cuuint64_t dims[5] = {64, (cuuint64_t)k, (cuuint64_t)nq, vlo, vhi};
-      cuuint64_t strides[4] = {(cuuint64_t)n * 2, 128, 16, vstride_hi};
-      cuuint32_t box[5] = {64, 64, (cuuint32_t)nq, 1, 1};
+  for (int ni = 0; ni < 6; ++ni)
+    for (int ki = 0; ki < 6; ++ki) {
+      const int n = cls[ni], k = cls[ki], wn = n < 64 ? n : 64, wk = k < 64 ? k : 64;
+      cuuint64_t dims[5] = {(cuuint64_t)wn, (cuuint64_t)k, (cuuint64_t)(n / wn), vlo, vhi};
+      cuuint64_t strides[4] = {(cuuint64_t)n * 2, (cuuint64_t)wn * 2, 16, vstride_hi};
+      cuuint32_t box[5] = {(cuuint32_t)wn, (cuuint32_t)wk, (cuuint32_t)(n / wn), 1, 1};
       cuuint32_t es[5] = {1, 1, 1, 1, 1};
-      if (enc(&h[64 + (nq - 1) * 4 + kq - 1], CU_TENSOR_MAP_DATA_TYPE_UINT16, 5, vbase, dims, strides, box, es,
-              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+      if (enc(&h[96 + ni * 6 + ki], CU_TENSOR_MAP_DATA_TYPE_UINT16, 5, vbase, dims, strides, box, es,
+              CU_TENSOR_MAP_INTERLEAVE_NONE, swz(wn * 2), CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
               CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
         return nullptr;
     }
@@ -650,6 +685,7 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   if (!p.bsr && p.G == 1) {
     const char* v = getenv("KAMI_VB_VIEWS");
     if (!v || atoi(v) != 0) p.vmap = vb_view_maps(stream);
+    p.vsmall = (v && atoi(v) == 2) ? 0 : 1;
   }
   const uint32_t smem = p.bar_off + 2048 + 1024;
   auto fn = bf16 ? kami_tc16_vb_kernel<true> : kami_tc16_vb_kernel<false>;

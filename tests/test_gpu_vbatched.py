@@ -167,8 +167,8 @@ def test_vbatched_rejects():
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 def test_vbatched_many_units_ring_wraps(dtype):
     """Mixed orders at a batch large enough that every persistent CTA runs
-    tens of units: the variable-size stage ring (tc16_vb.cu, VRing) wraps many
-    times, releases chunks out of slot order and reuses all of its slots."""
+    tens of units: the stage ring wraps many times and every TMEM accumulator
+    and C staging buffer is reused, with view (TMA) and copy units interleaved."""
     rng = np.random.default_rng(21)
     orders = np.array([16, 32, 48, 64, 128, 192, 256])
     batch = 1200
@@ -194,3 +194,52 @@ def test_vbatched_many_units_ring_wraps(dtype):
         Cref, S = oracle.gemm(m, n, k, 1, dtype, "row", ki.as_bits(A), ki.as_bits(B), with_scale=True)
         got = oracle.decode(Cb[offC[e]:offC[e + 1]], dtype)
         assert oracle.normalised_error(got.reshape(1, m, n), Cref, S) <= _tol(dtype, k), (e, m, n, k)
+
+
+def _mixed_batch(sizes, dtype, seed):
+    ops = [ki.operands(m, n, k, 1, dtype, "unif", seed=seed, entry0=e) for e, (m, n, k) in enumerate(sizes)]
+    offA = np.concatenate([[0], np.cumsum([a.numel() for a, _ in ops])])
+    offB = np.concatenate([[0], np.cumsum([b.numel() for _, b in ops])])
+    offC = np.concatenate([[0], np.cumsum([m * n for m, n, _ in sizes])])
+    dA = torch.cat([a for a, _ in ops]).cuda()
+    dB = torch.cat([b for _, b in ops]).cuda()
+    es = dA.element_size()
+    dm, dn, dk = (torch.tensor([s[i] for s in sizes], dtype=torch.int32, device="cuda") for i in range(3))
+    pa = torch.tensor(dA.data_ptr() + offA[:-1] * es, dtype=torch.int64, device="cuda")
+    pb = torch.tensor(dB.data_ptr() + offB[:-1] * es, dtype=torch.int64, device="cuda")
+
+    def run(keep=(dA, dB)):  # the closure keeps the operands alive
+        dC = torch.full((int(offC[-1]),), float("nan"), dtype=dA.dtype, device="cuda")
+        pc = torch.tensor(dC.data_ptr() + offC[:-1] * es, dtype=torch.int64, device="cuda")
+        kami.gemm_vbatched(len(sizes), dm, dn, dk, 256, 256, 256, dtype, "row", pa, pb, pc)
+        torch.cuda.synchronize()
+        return dC
+    return ops, offC, run
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_vbatched_view_classes(dtype, monkeypatch):
+    """Every TMA-view class of tc16_vb.cu (k and n in {16, 32} with 32 / 64-byte
+    swizzles, multiples of 64 with 128-byte ones), the copy path beside them
+    (k or n 8, 48), and m-tiles of 8..128 live rows (m 8, 72, 200): against the
+    oracle, and bit-identical with the views disabled (KAMI_VB_VIEWS=0, the
+    cp.async path for every entry)."""
+    sizes = [(m, n, k) for m in (8, 72, 128, 200, 256) for n in (16, 32, 48, 64, 192, 256)
+             for k in (8, 16, 32, 48, 64, 128, 192, 256)]
+    rng = np.random.default_rng(31)
+    sizes = [sizes[i] for i in rng.permutation(len(sizes))]
+    ops, offC, run = _mixed_batch(sizes, dtype, seed=32)
+    monkeypatch.setenv("KAMI_VB_VIEWS", "1")
+    C1 = ki.as_bits(run().cpu())
+    monkeypatch.setenv("KAMI_VB_VIEWS", "0")
+    C0 = ki.as_bits(run().cpu())
+    bad = {0: [], 1: []}
+    for e, ((m, n, k), (A, B)) in enumerate(zip(sizes, ops)):
+        Cref, S = oracle.gemm(m, n, k, 1, dtype, "row", ki.as_bits(A), ki.as_bits(B), with_scale=True)
+        for v, Cv in ((0, C0), (1, C1)):
+            got = oracle.decode(Cv[offC[e]:offC[e + 1]], dtype)
+            if not oracle.normalised_error(got.reshape(1, m, n), Cref, S) <= _tol(dtype, k):
+                bad[v].append((m, n, k))
+    assert not bad[0] and not bad[1], bad
+    assert np.array_equal(C0, C1)
