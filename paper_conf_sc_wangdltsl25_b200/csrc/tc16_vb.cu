@@ -90,6 +90,16 @@ struct alignas(64) VbParams {
   // vmap[96 + vidx(n) * 6 + vidx(k)]: B views, vidx: 16, 32, 64, 128, 192, 256 -> 0..5
   const CUtensorMap* vmap;
   int vsmall;  // 0: views only for multiples of 64 (A/B experiments, KAMI_VB_VIEWS=2)
+  int vprefetch;
+  int early;  // release the accumulator before the copy-out (KAMI_VB_EARLY, A/B experiments)
+  // Variable-size batches, class-sorted: a pre-pass buckets the
+  // entries by (m, n, k) and packs each bucket's entries G(m, n) to a tile like
+  // a uniform batch.  utab[u] = {first position, ng | mt << 8, class, G}; A, B,
+  // C are then the pointer arrays in bucket order (position -> entry's
+  // pointers, written by the pre-pass); *nunits = live unit count.
+  int sorted;
+  const int4* utab;
+  const int* nunits;  // prefetch the next unit's maps (KAMI_VB_PREFETCH=0 disables, A/B experiments)
 };
 
 // TMA-view class of a size (16, 32 or a multiple of 64 up to 256), else -1
@@ -106,7 +116,7 @@ struct VbLayout {
 };
 __device__ __forceinline__ VbLayout vb_layout(const VbParams& p, int n, int k) {
   VbLayout L;
-  L.va = p.vmap != nullptr && p.G == 1 && vidx(k) >= (p.vsmall ? 0 : 2);
+  L.va = p.vmap != nullptr && vidx(k) >= (p.vsmall ? 0 : 2);
   L.vb = L.va && vidx(n) >= (p.vsmall ? 0 : 2);
   L.wa = L.va ? (uint32_t)min(k, 64) * 2u : 128u;
   L.wb = L.vb ? (uint32_t)min(n, 64) * 2u : 128u;
@@ -134,7 +144,7 @@ __device__ __forceinline__ void entry_dims(const VbParams& p, long long e, int& 
 // unit -> first entry, m-tile, live entries, sizes
 struct Unit {
   long long e0;
-  int mt, ng, m, n, k;
+  int mt, ng, m, n, k, G;
 };
 // Fills U for (entry group grp, m-tile mt).  The size loads (variable-size
 // batches) are consumed one unit later by the callers, so their latency hides
@@ -145,8 +155,33 @@ __device__ __forceinline__ void unit_fill(const VbParams& p, long long grp, int 
   U.e0 = grp * p.G;
   const long long left = p.batch - U.e0;
   U.ng = left < p.G ? (int)left : p.G;
+  U.G = p.G;
   entry_dims(p, U.e0, U.m, U.n, U.k);
 }
+// class key of a size triple (multiples of 8 in [8, 256]): 5 bits each
+__host__ __device__ __forceinline__ int vb_class(int m, int n, int k) {
+  return (((m >> 3) - 1) << 10) | (((n >> 3) - 1) << 5) | ((k >> 3) - 1);
+}
+// entries per tile (block-diagonal packing), capped at the 8-entry tables
+__host__ __device__ __forceinline__ int vb_pack(int m, int n) {
+  if (m > 128) return 1;
+  const int g1 = 128 / m, g2 = 256 / n;
+  const int g = g1 < g2 ? g1 : g2;
+  return g < 1 ? 1 : (g > 8 ? 8 : g);
+}
+// sorted mode: unit u from the pre-pass table
+__device__ __forceinline__ void unit_fill_sorted(const VbParams& p, long long u, Unit& U) {
+  const int4 t = __ldg(p.utab + u);
+  U.e0 = t.x;
+  U.ng = t.y & 0xFF;
+  U.mt = t.y >> 8;
+  U.m = ((t.z >> 10) + 1) << 3;
+  U.n = (((t.z >> 5) & 31) + 1) << 3;
+  U.k = ((t.z & 31) + 1) << 3;
+  U.G = t.w;
+}
+// entry index of slot g of a unit (sorted mode: its position in bucket order)
+__device__ __forceinline__ long long unit_entry(const VbParams&, const Unit& U, int g) { return U.e0 + g; }
 
 __device__ __forceinline__ void cp_async_wait_n(int n) {
   switch (n) {
@@ -186,9 +221,11 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < p.stages; ++s) {
-      // + thread 0's arrival: the B TMA's expect_tx (SpMM), or per stage either
-      // the view TMAs' expect_tx or a plain arrival (TMA views)
-      ptx::mbar_init(&full[s], 128 + ((p.b_tma || p.vmap) ? 1 : 0));
+      // SpMM: the 128 copy threads' .noinc arrivals + the B TMA's expect_tx.
+      // Otherwise one regular arrival by producer thread 0 per stage (after
+      // the TMA issue, or after every copy thread raised the pending count
+      // with its cp.async arrival and a named barrier).
+      ptx::mbar_init(&full[s], p.bsr ? 128 + (p.b_tma ? 1 : 0) : 1);
       ptx::mbar_init(&empty[s], 1);
     }
     for (int a = 0; a < p.acc_bufs; ++a) {
@@ -203,6 +240,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   const uint32_t smem_base = ptx::smem_u32(smem);
+  const long long units = p.sorted ? (long long)*p.nunits : p.units;
 
   if (warp < 4) {
     // ------------------------------------------------ producer warpgroup
@@ -222,7 +260,8 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     // With one entry per unit (G == 1, no SpMM) every thread loads the entry's
     // pointers itself (one broadcast address per warp), so no shared table or
     // table barrier is needed.
-    const bool one = p.G == 1 && !p.bsr;
+    const bool one = p.G == 1 && !p.bsr && !p.sorted;
+    long long uf = blockIdx.x;  // sorted mode: the next unit to fetch
     // SpMM: the next unit's block structure is fetched ahead too, without the
     // row_ptr -> col_blk dependency: every col_blk slot of the unit's entries
     // (<= 2 per thread: G mb kb <= 256) and every row_ptr value (<= 17)
@@ -233,12 +272,17 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       int cb[2], rp;
     };
     auto fetch = [&](PSlot& S) {
-      unit_fill(p, ui.grp, ui.mt, S.U);
+      if (p.sorted) {
+        unit_fill_sorted(p, uf, S.U);
+        uf += gridDim.x;
+      } else {
+        unit_fill(p, ui.grp, ui.mt, S.U);
+      }
       S.pa = S.pb = nullptr;
       S.cb[0] = S.cb[1] = -1;
       S.rp = 0;
       if (one || tid < S.U.ng) {
-        const long long e = S.U.e0 + (one ? 0 : tid);
+        const long long e = one ? S.U.e0 : unit_entry(p, S.U, tid);
         S.pa = p.bsr ? nullptr
                : p.strided ? p.As + e * (long long)p.m * p.k
                            : reinterpret_cast<const uint16_t*>(p.A[e]);
@@ -259,9 +303,56 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       const uint16_t *pa = S.pa, *pb = S.pb;
       const int cb0 = S.cb[0], cb1 = S.cb[1], rpv = S.rp;
       if (U.mt * 128 >= U.m) return;
-      const int m = U.m, n = U.n, k = U.k, G = p.G;
+      const int m = U.m, n = U.n, k = U.k, G = U.G;
       const int kchunks = (k + 63) / 64;
       const int rows = G > 1 ? U.ng * m : min(128, m - U.mt * 128);  // live tile rows
+      // ---- all-TMA unit (A and B through views): warp 0 alone; lane g holds
+      // entry g's pointers, lane 0 issues every box and makes the stage's one
+      // arrival.  The other warps only follow the ring.
+      const VbLayout lay = vb_layout(p, n, k);
+      if (!p.bsr && lay.va && lay.vb && !(p.dbg & 2)) {
+        if (tid < 32) {
+          const int rows_e = G > 1 ? m : rows;
+          const uint32_t a_e = (uint32_t)rows_e * lay.wa, b_e = lay.kr * (uint32_t)n * 2u;
+          const uint32_t tx = (uint32_t)U.ng * (a_e + b_e);
+          const CUtensorMap* ma = p.vmap + vidx(k) * 16 + (rows_e >> 3) - 1;
+          const CUtensorMap* mb = p.vmap + 96 + vidx(n) * 6 + vidx(k);
+          const int arow = G > 1 ? 0 : U.mt * 128;
+          int alo = 0, ahi = 0, blo = 0, bhi = 0;
+          if (one || tid < U.ng) {
+            view_coords(pa, alo, ahi);
+            view_coords(pb, blo, bhi);
+          }
+          for (int kc = 0; kc < kchunks; ++kc, rs.next(p.stages), ++it) {
+            const uint32_t s = rs.s;
+            ptx::mbar_wait(&empty[s], rs.ph ^ 1);
+            if (p.dbg & 4) trace(0, it);
+            uint8_t* st = smem + s * p.stage_bytes;
+            if (tid == 0) ptx::mbar_arrive_expect_tx(&full[s], tx);
+#pragma unroll 1
+            for (int g = 0; g < U.ng; ++g) {
+              const int xa = __shfl_sync(0xffffffffu, alo, g), ya = __shfl_sync(0xffffffffu, ahi, g);
+              const int xb = __shfl_sync(0xffffffffu, blo, g), yb = __shfl_sync(0xffffffffu, bhi, g);
+              if (tid == 0) {
+                ptx::tma_load_4d(st + g * a_e, ma, &full[s], kc * 64, arow, xa, ya);
+                ptx::tma_load_5d(st + kAReg + g * b_e, mb, &full[s], 0, kc * 64, 0, xb, yb);
+              }
+            }
+            if (p.dbg & 4) trace(1, it);
+          }
+        } else {
+          // the other warps only advance their ring position; the next copy
+          // unit starts with a warpgroup barrier (below), so they never wait
+          // on a slot more than one lap away from warp 0 (mbarrier waits test
+          // the phase parity only: a lap ahead or behind would alias)
+          for (int kc = 0; kc < kchunks; ++kc) rs.next(p.stages);
+          it += kchunks;
+        }
+        return;
+      }
+      if (one && !p.bsr && p.vmap) {
+        ptx::named_bar_sync(3, 128);  // warp 0 has issued every earlier TMA unit (see above)
+      }
       if (!one) {
         ptx::named_bar_sync(3, 128);  // previous unit's items issued: tables reusable
         if (tid < U.ng) {
@@ -321,23 +412,18 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         // a multiple of 16; zero-filled past k): for k < 64 the copy issue --
         // the producer's bottleneck (tools/trace_vb.py) -- shrinks with k.
         const int kpad_c = min(64, ((k + 15) & ~15) - kc * 64);
-        // TMA views for this unit (uniform across the warpgroup)
-        const VbLayout lay = vb_layout(p, n, k);
-        const bool va = lay.va, vb = lay.vb;
-        if (p.vmap && tid == 0) {
-          if (va) {
+        // A through views, B copied (n off the view classes): thread 0 raises
+        // the stage's transaction count and issues one A box per entry
+        const bool va = lay.va, vb = false;
+        if (va && tid == 0) {
+          const int rows_e = G > 1 ? m : rows;
+          ptx::mbar_expect_tx(&full[s], (uint32_t)U.ng * (uint32_t)rows_e * lay.wa);
+          const CUtensorMap* ma = p.vmap + vidx(k) * 16 + (rows_e >> 3) - 1;
+          for (int g = 0; g < U.ng; ++g) {
             int lo, hi;
-            ptx::mbar_arrive_expect_tx(&full[s], (uint32_t)rows * lay.wa + (vb ? lay.kr * (uint32_t)n * 2u : 0u));
-            view_coords(pa, lo, hi);
-            ptx::tma_load_4d(smem + s * p.stage_bytes, p.vmap + vidx(k) * 16 + (rows >> 3) - 1, &full[s], kc * 64,
-                             U.mt * 128, lo, hi);
-            if (vb) {
-              view_coords(pb, lo, hi);
-              ptx::tma_load_5d(smem + s * p.stage_bytes + kAReg, p.vmap + 96 + vidx(n) * 6 + vidx(k), &full[s], 0,
-                               kc * 64, 0, lo, hi);
-            }
-          } else {
-            ptx::mbar_arrive(&full[s]);
+            view_coords(one ? pa : a_tab[g], lo, hi);
+            ptx::tma_load_4d(smem + s * p.stage_bytes + g * rows_e * lay.wa, ma, &full[s], kc * 64,
+                             G > 1 ? 0 : U.mt * 128, lo, hi);
           }
         }
         // A: thread = (16-byte chunk j, row r0 + rstep q): the chunks of a row
@@ -411,25 +497,45 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         }  // dbg & 2
         // full[s] completes when all 128 threads' copies of this stage landed;
         // the MMA warp fences generic->async proxy before reading the stage
-        ptx::cp_async_mbar_arrive_noinc(&full[s]);
+        if (p.bsr) {
+          ptx::cp_async_mbar_arrive_noinc(&full[s]);
+        } else {
+          ptx::cp_async_mbar_arrive(&full[s]);  // pending count raised until the copies land
+          ptx::named_bar_sync(3, 128);          // every thread's raise precedes the arrival
+          if (tid == 0) ptx::mbar_arrive(&full[s]);
+        }
         if (p.dbg & 4) trace(1, it);
       }
+    };
+    // the next unit's view maps are prefetched into the TMA descriptor cache
+    // while the current unit issues (a cold map costs a global-memory round
+    // trip inside the TMA issue)
+    auto prefetch_maps = [&](const PSlot& S) {
+      const Unit& V = S.U;
+      if (tid != 0 || V.mt * 128 >= V.m) return;
+      const VbLayout lay = vb_layout(p, V.n, V.k);
+      if (!lay.va) return;
+      const int rows = min(128, V.m - V.mt * 128);
+      ptx::prefetch_tmap(p.vmap + vidx(V.k) * 16 + (rows >> 3) - 1);
+      if (lay.vb) ptx::prefetch_tmap(p.vmap + 96 + vidx(V.n) * 6 + vidx(V.k));
     };
     const long long g1 = gridDim.x, g2 = 2 * g1;
     long long u = blockIdx.x;
     PSlot S0, S1;
-    if (u < p.units) fetch(S0);
-    if (u + g1 < p.units) fetch(S1);
-    while (u < p.units) {
+    if (u < units) fetch(S0);
+    if (u + g1 < units) fetch(S1);
+    while (u < units) {
       {
         const PSlot c = S0;
-        if (u + g2 < p.units) fetch(S0);
+        if (u + g2 < units) fetch(S0);
+        if (p.vprefetch && p.vmap && u + g1 < units) prefetch_maps(S1);
         body(c);
       }
-      if ((u += g1) >= p.units) break;
+      if ((u += g1) >= units) break;
       {
         const PSlot c = S1;
-        if (u + g2 < p.units) fetch(S1);
+        if (u + g2 < units) fetch(S1);
+        if (p.vprefetch && p.vmap && u + g1 < units) prefetch_maps(S0);
         body(c);
       }
       u += g1;
@@ -441,11 +547,15 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     uint32_t it = 0, acc_it = 0;  // trace indices
     UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
     Unit Un;
-    if ((long long)blockIdx.x < p.units) unit_fill(p, ui.grp, ui.mt, Un);
-    for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
+    auto fill = [&](long long v) {
+      if (p.sorted) unit_fill_sorted(p, v, Un);
+      else unit_fill(p, ui.grp, ui.mt, Un);
+    };
+    if ((long long)blockIdx.x < units) fill(blockIdx.x);
+    for (long long u = blockIdx.x; u < units; u += gridDim.x) {
       const Unit U = Un;
       ui.next();
-      if (u + gridDim.x < p.units) unit_fill(p, ui.grp, ui.mt, Un);
+      if (u + gridDim.x < units) fill(u + gridDim.x);
       if (U.mt * 128 >= U.m) continue;
       const uint32_t a = ra.s;
       ptx::mbar_wait(&tempty[a], ra.ph ^ 1);
@@ -454,7 +564,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       const uint32_t d_tmem = tmem_base + a * p.acc_cols;
       // N of the MMA: the tile's G n live columns rounded up to the M = 128 granule of
       // 16 (n = 8 mod 16: the pad columns' products are never stored)
-      const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, (p.G * U.n + 15) & ~15, 0, 1);
+      const uint32_t idesc = ptx::make_idesc_f16(kBF16 ? 1 : 0, 128, (U.G * U.n + 15) & ~15, 0, 1);
       const int kpad = (U.k + 15) / 16 * 16;
       const int kchunks = (U.k + 63) / 64;
       const VbLayout lay = vb_layout(p, U.n, U.k);
@@ -496,16 +606,17 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
     Unit Un;
     uint16_t* pc_n = nullptr;
-    auto fetch = [&]() {
-      unit_fill(p, ui.grp, ui.mt, Un);
-      if (L < Un.ng) pc_n = entry_C(p, Un.e0 + L, Un.m, Un.n);
+    auto fetch = [&](long long v) {
+      if (p.sorted) unit_fill_sorted(p, v, Un);
+      else unit_fill(p, ui.grp, ui.mt, Un);
+      if (L < Un.ng) pc_n = entry_C(p, unit_entry(p, Un, L), Un.m, Un.n);
     };
-    if ((long long)blockIdx.x < p.units) fetch();
-    for (long long u = blockIdx.x; u < p.units; u += gridDim.x) {
+    if ((long long)blockIdx.x < units) fetch(blockIdx.x);
+    for (long long u = blockIdx.x; u < units; u += gridDim.x) {
       const Unit U = Un;
       uint16_t* const pc = pc_n;
       ui.next();
-      if (u + gridDim.x < p.units) fetch();
+      if (u + gridDim.x < units) fetch(u + gridDim.x);
       if (U.mt * 128 >= U.m) continue;
       const uint32_t a = ra.s;
       const uint32_t aph = ra.ph;
@@ -513,7 +624,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       const bool mine = (int)(live & 1) == wg;
       ++live;
       if (!mine) continue;
-      const int m = U.m, n = U.n, G = p.G;
+      const int m = U.m, n = U.n, G = U.G;
       const int rows = G > 1 ? U.ng * m : min(128, m - U.mt * 128);
       // lanes -> (entry g, row); the warp's lanes may span several entries
       const int g = G > 1 ? L / m : 0;
@@ -566,6 +677,14 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
             }
           }
         }
+        if (p.early && h0 + 128 >= n) {
+          // every accumulator column is in registers / staging: release the
+          // accumulator before the copy-out, so the MMA of the unit after next
+          // overlaps this unit's stores
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive(&tempty[a]);
+        }
         ptx::named_bar_sync(1 + wg, 128);
         // copy-out: chunk index i -> (tile row i / cpr, 16-byte chunk i % cpr)
         const int cpr = hw / 8;
@@ -582,9 +701,11 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         }
         ptx::named_bar_sync(1 + wg, 128);  // staging buffer reusable
       }
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&tempty[a]);
+      if (!p.early) {
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&tempty[a]);
+      }
       if (p.dbg & 4) trace(5, live);
     }
   }
@@ -655,6 +776,164 @@ const CUtensorMap* vb_view_maps(cudaStream_t stream) {
   return table[dev];
 }
 
+// ---------------------------------------------------------------------------
+// Class-sorted variable-size batches (pre-pass).  Entries are
+// bucketed by their exact (m, n, k) (32^3 classes), each bucket is packed
+// G(m, n) entries to a tile, and the unit table lists every bucket's tiles.
+// Three small kernels on the caller's stream; positions inside a bucket come
+// from atomics, so which entries share a tile varies from run to run, but an
+// entry's result does not (block-diagonal tiles: an entry's rows and columns
+// meet only its own operands, in the same K order).
+constexpr int kClasses = 32 * 32 * 32;
+
+// The pre-pass workspace comes from the library's own stream-ordered pool,
+// which keeps its memory between calls (release threshold: unlimited), so a
+// call does not re-map pages the way the default pool does after every
+// synchronisation; the allocation is graph-capturable.
+cudaMemPool_t vb_pool() {
+  static std::mutex mu;
+  static cudaMemPool_t pools[64] = {};
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  std::lock_guard<std::mutex> lock(mu);
+  if (!pools[dev]) {
+    cudaMemPoolProps props;
+    memset(&props, 0, sizeof(props));
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = dev;
+    cudaMemPool_t pool = nullptr;
+    if (cudaMemPoolCreate(&pool, &props) != cudaSuccess) return nullptr;
+    uint64_t thr = ~0ull;
+    cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    pools[dev] = pool;
+  }
+  return pools[dev];
+}
+// sizes on the kami.h grid (multiples of 8 in [8, 256]); an entry off the grid
+// is skipped (not computed) rather than indexing past the class tables
+__device__ __forceinline__ bool vb_on_grid(int m, int n, int k) {
+  return ((m | n | k) & 7) == 0 && m >= 8 && n >= 8 && k >= 8 && m <= 256 && n <= 256 && k <= 256;
+}
+
+__global__ void vb_class_hist(long long batch, const int* dm, const int* dn, const int* dk, int* hist) {
+  for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < batch;
+       e += (long long)gridDim.x * blockDim.x) {
+    const int m = __ldg(dm + e), n = __ldg(dn + e), k = __ldg(dk + e);
+    const bool ok = vb_on_grid(m, n, k);
+    const int c = ok ? vb_class(m, n, k) : -1;
+    // warp-aggregated: one atomic per distinct class in the warp (a uniform
+    // batch would otherwise serialise every entry on one address)
+    const unsigned act = __activemask();
+    const unsigned peers = __match_any_sync(act, c);
+    if (ok && (threadIdx.x & 31) == __ffs(peers) - 1) atomicAdd(hist + c, __popc(peers));
+  }
+}
+
+// one block of 1024 threads, 32 classes each: exclusive scans of the bucket
+// sizes (entry offsets) and of the bucket unit counts (unit offsets).  Each
+// array is staged in shared memory (coalesced, 128 KB) and every thread scans
+// its 32 consecutive classes there.
+__device__ __forceinline__ int vb_class_units(int c, int cnt) {
+  if (cnt == 0) return 0;  // most classes are empty: no divisions for them
+  const int m = ((c >> 10) + 1) << 3, n = (((c >> 5) & 31) + 1) << 3;
+  const int G = vb_pack(m, n);
+  return (cnt + G - 1) / G * ((m + 127) >> 7);
+}
+__global__ void __launch_bounds__(1024) vb_class_scan(const int* hist, int* eoff, int* uoff, int* nunits) {
+  extern __shared__ int sh[];  // [kClasses]
+  __shared__ int ws_e[32], ws_u[32];
+  const int t = threadIdx.x, c0 = t * 32;
+  for (int c = t; c < kClasses; c += 1024) sh[c] = __ldg(hist + c);
+  __syncthreads();
+  int se = 0, su = 0;
+  for (int i = 0; i < 32; ++i) {
+    const int c = c0 + ((i + t) & 31);  // rotated: no bank conflicts
+    const int cnt = sh[c];
+    se += cnt;
+    su += vb_class_units(c, cnt);
+  }
+  int ie = se, iu = su;
+  for (int o = 1; o < 32; o <<= 1) {
+    const int xe = __shfl_up_sync(0xffffffffu, ie, o), xu = __shfl_up_sync(0xffffffffu, iu, o);
+    if ((t & 31) >= o) {
+      ie += xe;
+      iu += xu;
+    }
+  }
+  if ((t & 31) == 31) {
+    ws_e[t >> 5] = ie;
+    ws_u[t >> 5] = iu;
+  }
+  __syncthreads();
+  if (t < 32) {
+    int ve = ws_e[t], vu = ws_u[t];
+    for (int o = 1; o < 32; o <<= 1) {
+      const int xe = __shfl_up_sync(0xffffffffu, ve, o), xu = __shfl_up_sync(0xffffffffu, vu, o);
+      if (t >= o) {
+        ve += xe;
+        vu += xu;
+      }
+    }
+    ws_e[t] = ve;
+    ws_u[t] = vu;
+  }
+  __syncthreads();
+  const int be0 = ie - se + ((t >> 5) ? ws_e[(t >> 5) - 1] : 0);
+  const int bu0 = iu - su + ((t >> 5) ? ws_u[(t >> 5) - 1] : 0);
+  if (t == 1023) *nunits = bu0 + su;
+  for (int pass = 0; pass < 2; ++pass) {
+    __syncthreads();
+    for (int c = t; c < kClasses; c += 1024) {
+      const int cnt = __ldg(hist + c);
+      sh[c] = pass ? vb_class_units(c, cnt) : cnt;
+    }
+    __syncthreads();
+    int b = pass ? bu0 : be0;
+    for (int i = 0; i < 32; ++i) {  // in place: the exclusive offsets
+      const int v = sh[c0 + i];
+      sh[c0 + i] = b;
+      b += v;
+    }
+    __syncthreads();
+    int* out = pass ? uoff : eoff;
+    for (int c = t; c < kClasses; c += 1024) out[c] = sh[c];
+    __syncthreads();
+  }
+}
+
+// scatter: entry -> its bucket position; the first entry of every tile writes
+// the tile's units (one per m-tile)
+__global__ void vb_class_scatter(long long batch, const int* dm, const int* dn, const int* dk, const int* hist,
+                                 const int* eoff, const int* uoff, int* cursor, const void* const* A,
+                                 const void* const* B, void* const* C, const void** sA, const void** sB, void** sC,
+                                 int4* utab) {
+  for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < batch;
+       e += (long long)gridDim.x * blockDim.x) {
+    const int m = __ldg(dm + e), n = __ldg(dn + e), k = __ldg(dk + e);
+    const bool ok = vb_on_grid(m, n, k);
+    const int c = ok ? vb_class(m, n, k) : -1;
+    const unsigned act = __activemask();
+    const unsigned peers = __match_any_sync(act, c);
+    const int lane = threadIdx.x & 31, leader = __ffs(peers) - 1;
+    int base = 0;
+    if (ok && lane == leader) base = atomicAdd(cursor + c, __popc(peers));
+    base = __shfl_sync(peers, base, leader);
+    if (!ok) continue;
+    const int pos = base + __popc(peers & ((1u << lane) - 1u));
+    const int first = eoff[c] + pos;
+    sA[first] = A[e];
+    sB[first] = B[e];
+    sC[first] = C[e];
+    const int G = vb_pack(m, n);
+    if (pos % G == 0) {
+      const int cnt = hist[c], ng = cnt - pos < G ? cnt - pos : G, mt_n = (m + 127) >> 7;
+      for (int mt = 0; mt < mt_n; ++mt)
+        utab[uoff[c] + (pos / G) * mt_n + mt] = make_int4(first, ng | (mt << 8), c, G);
+    }
+  }
+}
+
 int pow2_ceil(int x) {
   int q = 32;
   while (q < x) q <<= 1;
@@ -663,7 +942,8 @@ int pow2_ceil(int x) {
 
 // n_max: widest B tile (columns) a unit can need; G entries per unit
 kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream_t stream) {
-  const int N = p.G * n_max;
+  // widest tile: G n columns (sorted mode: any class, G n <= min(8 n_max, 256))
+  const int N = p.G * n_max < 256 ? p.G * n_max : 256;
   const uint32_t b_region = (uint32_t)((N + 63) / 64) * 8192;
   p.stage_bytes = kAReg + b_region;
   p.acc_cols = pow2_ceil(N);
@@ -675,17 +955,22 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   p.stages = st;
   p.c_off = st * p.stage_bytes;
   p.bar_off = p.c_off + 2 * kCBuf;
-  p.mtiles = p.G > 1 ? 1 : (max_m + 127) / 128;
-  p.units = ((p.batch + p.G - 1) / p.G) * p.mtiles;
+  p.mtiles = (p.G > 1 && !p.sorted) ? 1 : (max_m + 127) / 128;
+  // (sorted mode: an upper bound; the kernel reads the live count)
+  p.units = p.sorted ? p.batch * p.mtiles : ((p.batch + p.G - 1) / p.G) * p.mtiles;
   {
     const char* d = getenv("KAMI_VB_DEBUG");
     p.dbg = d ? atoi(d) : 0;
+    const char* e = getenv("KAMI_VB_EARLY");
+    p.early = (e && atoi(e) == 0) ? 0 : 1;
   }
-  // TMA views (one entry per tile; KAMI_VB_VIEWS=0 disables them, A/B experiments)
-  if (!p.bsr && p.G == 1) {
+  // TMA views (KAMI_VB_VIEWS=0 disables them, A/B experiments)
+  if (!p.bsr) {
     const char* v = getenv("KAMI_VB_VIEWS");
     if (!v || atoi(v) != 0) p.vmap = vb_view_maps(stream);
     p.vsmall = (v && atoi(v) == 2) ? 0 : 1;
+    const char* pf = getenv("KAMI_VB_PREFETCH");
+    p.vprefetch = (pf && atoi(pf) == 1) ? 1 : 0;
   }
   const uint32_t smem = p.bar_off + 2048 + 1024;
   auto fn = bf16 ? kami_tc16_vb_kernel<true> : kami_tc16_vb_kernel<false>;
@@ -701,7 +986,7 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   // only the second tiles of m > 128 entries -- a ~3 : 1 imbalance).  A grid
   // coprime to mtiles walks each CTA through all m-tile indices.
   // (uniform sizes with a short last m-tile, m % 128 != 0, likewise)
-  if (p.mtiles > 1 && (p.dm || max_m % 128 != 0))
+  if (!p.sorted && p.mtiles > 1 && (p.dm || max_m % 128 != 0))
     while (grid > 1 && std::gcd(grid, (long long)p.mtiles) != 1) --grid;
   grid = apply_grid_cap(grid);
   fn<<<(unsigned)grid, kVbThreads, smem, stream>>>(p);
@@ -711,6 +996,10 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   }
   if (p.zorder) {
     set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16,spmm_zmorton>" : "kami_tc16_vb_kernel<f16,spmm_zmorton>");
+    return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+  }
+  if (p.sorted) {
+    set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16,sorted>" : "kami_tc16_vb_kernel<f16,sorted>");
     return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
   }
   set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
@@ -798,8 +1087,53 @@ kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, co
   p.n = n;
   p.k = k;
   p.batch = batch;
-  p.G = dm ? 1 : packing(m, n);  // mixed sizes cannot share a tile
-  return vb_launch(p, bf16, dm ? max_n : n, dm ? max_m : m, stream);
+  p.G = dm ? 1 : packing(m, n);  // mixed sizes share a tile only class-sorted
+  // Variable sizes: class-sorted (pre-pass + packed tiles) for batches of at
+  // least 256 entries, where the pre-pass's few microseconds are repaid;
+  // KAMI_VB_SORT=0 / 1 forces it off / on (A/B experiments, tests).
+  const char* env = getenv("KAMI_VB_SORT");
+  const bool sort = dm && batch < (1ll << 30) && (env ? atoi(env) != 0 : batch >= 256);
+  if (!sort) return vb_launch(p, bf16, dm ? max_n : n, dm ? max_m : m, stream);
+  const long long mt_max = (max_m + 127) / 128;
+  const size_t bytes =
+      sizeof(int) * (4 * (size_t)kClasses + 4) + sizeof(int4) * (size_t)(batch * mt_max) + 3 * sizeof(void*) * (size_t)batch;
+  void* ws = nullptr;
+  cudaMemPool_t pool = vb_pool();
+  if (!pool || cudaMallocFromPoolAsync(&ws, bytes, pool, stream) != cudaSuccess) return KAMI_ERROR_CUDA;
+  int* hist = static_cast<int*>(ws);
+  int* cursor = hist + kClasses;
+  int* eoff = cursor + kClasses;
+  int* uoff = eoff + kClasses;
+  int* nunits = uoff + kClasses;
+  int4* utab = reinterpret_cast<int4*>(nunits + 4);  // 16-byte aligned (4 kClasses + 4 ints)
+  const void** sA = reinterpret_cast<const void**>(utab + batch * mt_max);
+  const void** sB = sA + batch;
+  void** sC = const_cast<void**>(sB + batch);
+  kami_status_t st = KAMI_SUCCESS;
+  if (cudaMemsetAsync(hist, 0, sizeof(int) * 2 * kClasses, stream) != cudaSuccess) st = KAMI_ERROR_CUDA;
+  if (cudaFuncSetAttribute(vb_class_scan, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                           kClasses * (int)sizeof(int)) != cudaSuccess)
+    st = KAMI_ERROR_CUDA;
+  if (st == KAMI_SUCCESS) {
+    const int blocks = (int)((batch + 255) / 256 < 1184 ? (batch + 255) / 256 : 1184);
+    vb_class_hist<<<blocks, 256, 0, stream>>>(batch, dm, dn, dk, hist);
+    vb_class_scan<<<1, 1024, kClasses * sizeof(int), stream>>>(hist, eoff, uoff, nunits);
+    vb_class_scatter<<<blocks, 256, 0, stream>>>(batch, dm, dn, dk, hist, eoff, uoff, cursor, A, B, C, sA, sB, sC,
+                                                 utab);
+    if (cudaGetLastError() != cudaSuccess) st = KAMI_ERROR_CUDA;
+  }
+  if (st == KAMI_SUCCESS) {
+    p.sorted = 1;
+    p.G = 8;  // buffer sizing: the widest packed tile (G n <= min(8 max_n, 256))
+    p.utab = utab;
+    p.A = sA;
+    p.B = sB;
+    p.C = sC;
+    p.nunits = nunits;
+    st = vb_launch(p, bf16, max_n, max_m, stream);
+  }
+  cudaFreeAsync(ws, stream);  // stream-ordered: after the kernels
+  return st;
 }
 
 }  // namespace kami

@@ -222,18 +222,25 @@ def _mixed_batch(sizes, dtype, seed):
 def test_vbatched_view_classes(dtype, monkeypatch):
     """Every TMA-view class of tc16_vb.cu (k and n in {16, 32} with 32 / 64-byte
     swizzles, multiples of 64 with 128-byte ones), the copy path beside them
-    (k or n 8, 48), and m-tiles of 8..128 live rows (m 8, 72, 200): against the
-    oracle, and bit-identical with the views disabled (KAMI_VB_VIEWS=0, the
+    (k or n 8, 48), and m-tiles of 8..128 live rows (m 8, 72, 200), one entry
+    per tile and class-sorted packed tiles (KAMI_VB_SORT): against the oracle,
+    and the four (sort, views) modes bit-identical (KAMI_VB_VIEWS=0: the
     cp.async path for every entry)."""
     sizes = [(m, n, k) for m in (8, 72, 128, 200, 256) for n in (16, 32, 48, 64, 192, 256)
              for k in (8, 16, 32, 48, 64, 128, 192, 256)]
     rng = np.random.default_rng(31)
     sizes = [sizes[i] for i in rng.permutation(len(sizes))]
     ops, offC, run = _mixed_batch(sizes, dtype, seed=32)
-    monkeypatch.setenv("KAMI_VB_VIEWS", "1")
-    C1 = ki.as_bits(run().cpu())
-    monkeypatch.setenv("KAMI_VB_VIEWS", "0")
-    C0 = ki.as_bits(run().cpu())
+    outs = {}
+    for srt in ("0", "1"):
+        for views in ("0", "1"):
+            monkeypatch.setenv("KAMI_VB_SORT", srt)
+            monkeypatch.setenv("KAMI_VB_VIEWS", views)
+            outs[srt + views] = ki.as_bits(run().cpu())
+            assert kami.last_kernel().endswith("sorted>") == (srt == "1")
+    C0, C1 = outs["00"], outs["11"]
+    for key in ("01", "10"):
+        assert np.array_equal(outs[key], C0), key
     bad = {0: [], 1: []}
     for e, ((m, n, k), (A, B)) in enumerate(zip(sizes, ops)):
         Cref, S = oracle.gemm(m, n, k, 1, dtype, "row", ki.as_bits(A), ki.as_bits(B), with_scale=True)
@@ -243,3 +250,32 @@ def test_vbatched_view_classes(dtype, monkeypatch):
                 bad[v].append((m, n, k))
     assert not bad[0] and not bad[1], bad
     assert np.array_equal(C0, C1)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("dtype", ["f16", "bf16"])
+def test_vbatched_sorted_many_classes(dtype, monkeypatch):
+    """Class-sorted mode at scale: 3000 entries over the BF16-sweep orders and
+    thin / odd sizes, so buckets hold partial tiles (ng < G), every CTA runs
+    many units and packed tiles of every G (1..8) occur; parity with the
+    oracle and bit-identity with the unsorted path."""
+    rng = np.random.default_rng(41)
+    orders = [8, 16, 24, 32, 48, 64, 96, 128, 192, 256]
+    sizes = [tuple(int(x) for x in rng.choice(orders, 3)) for _ in range(3000)]
+    ops, offC, run = _mixed_batch(sizes, dtype, seed=42)
+    monkeypatch.setenv("KAMI_VB_SORT", "1")
+    Cs = ki.as_bits(run().cpu())
+    assert kami.last_kernel().endswith("sorted>")
+    monkeypatch.setenv("KAMI_VB_SORT", "0")
+    Cu = ki.as_bits(run().cpu())
+    diff = [e for e in range(len(sizes)) if not np.array_equal(Cs[offC[e]:offC[e + 1]], Cu[offC[e]:offC[e + 1]])]
+    check = sorted(set(range(0, len(sizes), 7)) | set(diff[:20]))
+    bad = []
+    for e in check:
+        (m, n, k), (A, B) = sizes[e], ops[e]
+        Cref, S = oracle.gemm(m, n, k, 1, dtype, "row", ki.as_bits(A), ki.as_bits(B), with_scale=True)
+        for name, Cv in (("sorted", Cs), ("unsorted", Cu)):
+            got = oracle.decode(Cv[offC[e]:offC[e + 1]], dtype)
+            if not oracle.normalised_error(got.reshape(1, m, n), Cref, S) <= _tol(dtype, k):
+                bad.append((name, e, m, n, k))
+    assert not bad and not diff, (bad[:20], [(e,) + sizes[e] for e in diff[:20]], len(diff))

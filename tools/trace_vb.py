@@ -15,13 +15,14 @@ os.environ["KAMI_VB_DEBUG"] = "4"
 import kami_inputs as ki  # noqa: E402
 import paper_conf_sc_wangdltsl25_b200 as kami  # noqa: E402
 
-mix = len(sys.argv) > 1 and sys.argv[1] == "mix"
+mix = len(sys.argv) > 1 and (sys.argv[1] == "mix" or sys.argv[1].startswith("u"))
+uni = int(sys.argv[1][1:]) if mix and sys.argv[1].startswith("u") else 0  # "u64": uniform 64^3 via vbatched
 m = n = k = 64 if mix else (int(sys.argv[1]) if len(sys.argv) > 1 else 64)
 batch = int(sys.argv[2]) if len(sys.argv) > 2 else 32768
 es = 2
 if mix:  # tools/vb_bench.py --mode vb recipe: orders from {16,...,256}^3
     rng = np.random.default_rng(0)
-    sz = rng.choice(np.array([16, 32, 64, 128, 192, 256]), size=(batch, 3))
+    sz = rng.choice(np.array([uni] if uni else [16, 32, 64, 128, 192, 256]), size=(batch, 3))
     mm, nn, kk = sz[:, 0], sz[:, 1], sz[:, 2]
     offA = np.concatenate([[0], np.cumsum(mm * kk)])
     offB = np.concatenate([[0], np.cumsum(kk * nn)])
@@ -65,3 +66,10 @@ for e in range(7):
         print(f"{names[e]:18s} period {np.median(np.diff(v)):.0f} cycles")
 pi = t[1, 20:60] - t[0, 20:60]
 print("producer issue time per stage (median)", np.median(pi))
+lat = t[2, 20:200] - t[1, 20:200]
+lat = lat[(t[2, 20:200] > 0) & (t[1, 20:200] > 0)]
+print("issue -> MMA start per stage (median / p90)", np.median(lat), np.percentile(lat, 90))
+wait_slot = t[0, 20:200] - t[1, 19:199]
+print("producer wait for a free slot after the previous issue (median)", np.median(wait_slot[wait_slot > -1e12]))
+n_st = int((t[1] > 0).sum())
+print("stages traced", n_st, "span cycles", int(t[1, n_st - 1] - t[1, 0]), "per stage", (t[1, n_st - 1] - t[1, 0]) / max(1, n_st - 1))

@@ -26,6 +26,8 @@ ap.add_argument("--shape", default="64x64x64")
 ap.add_argument("--batch", type=int, default=65536)
 ap.add_argument("--reps", type=int, default=10)
 ap.add_argument("--density", type=float, default=0.5)
+ap.add_argument("--orders", default="16,32,64,128,192,256", help="vb mode: the order set")
+ap.add_argument("--nmax", type=int, default=256, help="vb mode: max_n passed to the call")
 ap.add_argument("--noperm", action="store_true", help="ptr mode: pointers in entry order (no scatter)")
 a = ap.parse_args()
 hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
@@ -83,7 +85,7 @@ elif a.mode == "ptr":
     byts = (m * k + k * n + m * n) * es * a.batch
 else:
     rng = np.random.default_rng(0)
-    orders = np.array([16, 32, 64, 128, 192, 256])
+    orders = np.array([int(x) for x in a.orders.split(",")])
     sz = rng.choice(orders, size=(a.batch, 3))
     mm, nn, kk = sz[:, 0], sz[:, 1], sz[:, 2]
     es = 2
@@ -101,7 +103,7 @@ else:
     pa = torch.tensor(A.data_ptr() + offA[:-1] * es, dtype=torch.int64, device="cuda")
     pb = torch.tensor(B.data_ptr() + offB[:-1] * es, dtype=torch.int64, device="cuda")
     pc = torch.tensor(C.data_ptr() + offC[:-1] * es, dtype=torch.int64, device="cuda")
-    run = lambda: kami.gemm_vbatched(a.batch, dm, dn, dk, 256, 256, 256, a.dtype, "row", pa, pb, pc)  # noqa: E731
+    run = lambda: kami.gemm_vbatched(a.batch, dm, dn, dk, 256, a.nmax, 256, a.dtype, "row", pa, pb, pc)  # noqa: E731
     flops = float((2.0 * mm * nn * kk).sum())
     byts = float(((mm * kk + kk * nn + mm * nn) * es).sum())
 for _ in range(3):
