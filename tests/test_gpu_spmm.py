@@ -14,8 +14,8 @@ pytestmark = pytest.mark.gpu
 
 @pytest.mark.parametrize("dtype", ["f16", "bf16"])
 @pytest.mark.parametrize("shape", [(16, 16, 16), (64, 64, 64), (128, 128, 128), (192, 64, 256), (256, 256, 32),
-                                   (48, 80, 112)])
-@pytest.mark.parametrize("density", [0.5, 1.0, 0.1])
+                                   (48, 80, 112), (224, 96, 160), (32, 48, 256), (256, 16, 256)])
+@pytest.mark.parametrize("density", [0.5, 1.0, 0.1, 0.0])
 def test_spmm_vs_oracle(dtype, shape, density):
     m, n, k = shape
     batch = 19
