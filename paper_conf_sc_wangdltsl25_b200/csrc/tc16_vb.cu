@@ -46,8 +46,12 @@ struct alignas(64) VbParams {
   // (64, 64, n/64, G), 128-byte swizzle = the N-major atoms the copies build)
   // and the producer warpgroup copies only the sparse A
   CUtensorMap tmB;
+  // SpMM: A's nonzero 16 x 16 blocks by TMA, one box per block, from the
+  // block array viewed as (16, 16, batch max_nnzb) with the 32-byte swizzle
+  CUtensorMap tmA;
   int b_tma;
   uint32_t b_tx;
+  int b_wb;  // SpMM: B atom row bytes (2 Wn, Wn = 64, 32 or 16 columns)
   const void* const* A;
   const void* const* B;
   void* const* C;
@@ -110,12 +114,24 @@ __host__ __device__ __forceinline__ int vidx(int x) {
 // wa-byte swizzle), B atoms of wb-byte rows x kr k-rows (N-major, wb-byte
 // swizzle).  The copies build (128, 128, 64); view units (min(k, 64) 2,
 // min(n, 64) 2, min(k, 64)).
+// SpMM (slab): A as four 4 KB k-step slabs per stage (128 rows x 32 bytes,
+// K-major, 32-byte swizzle -- the layout a 16 x 16 block box lands in), B as
+// N-major atoms of b_wb-byte rows.
 struct VbLayout {
-  bool va, vb;
+  bool va, vb, slab;
   uint32_t wa, wb, kr;
 };
 __device__ __forceinline__ VbLayout vb_layout(const VbParams& p, int n, int k) {
   VbLayout L;
+  if (p.bsr) {
+    L.va = L.vb = false;
+    L.slab = true;
+    L.wa = 32u;
+    L.wb = (uint32_t)p.b_wb;
+    L.kr = 64u;
+    return L;
+  }
+  L.slab = false;
   L.va = p.vmap != nullptr && vidx(k) >= (p.vsmall ? 0 : 2);
   L.vb = L.va && vidx(n) >= (p.vsmall ? 0 : 2);
   L.wa = L.va ? (uint32_t)min(k, 64) * 2u : 128u;
@@ -221,7 +237,8 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < p.stages; ++s) {
-      // SpMM: the 128 copy threads' .noinc arrivals + the B TMA's expect_tx.
+      // SpMM: the 128 producer threads' arrivals (after their A boxes'
+      // expect_tx and zero stores) + the B TMA's arrive.expect_tx.
       // Otherwise one regular arrival by producer thread 0 per stage (after
       // the TMA issue, or after every copy thread raised the pending count
       // with its cp.async arrival and a named barrier).
@@ -430,7 +447,29 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         // are spread over 2^cshift threads, the swizzle phase (r & 7) is fixed
         // per thread (rstep is a multiple of 8) and addresses advance by
         // constant strides.
-        if (!va) {
+        if (p.bsr) {
+          // SpMM A (Sec. 4.6): one TMA box per nonzero
+          // 16 x 16 block, straight from the block array into its k-step slab
+          // (block row ib of the tile at ib * 512 in slab ks); the absent
+          // blocks of the tile are zeroed in shared memory -- A is densified
+          // on chip, only its nonzero blocks cross HBM.  Thread quad
+          // (ib, ks) = tid / 4 owns one block position of the stage.
+          const int nib = rows >> 4, nks = kpad_c >> 4;
+          const int slot = tid >> 2, part = tid & 3, ib = slot >> 2, ks = slot & 3;
+          if (ib < nib && ks < nks) {
+            const int idx = blk_tab[ib * 16 + kc * 4 + ks];
+            const uint32_t off = s * p.stage_bytes + (uint32_t)ks * 4096u + (uint32_t)ib * 512u;
+            if (idx >= 0) {
+              if (part == 0) {
+                ptx::mbar_expect_tx(&full[s], 512u);
+                ptx::tma_load_3d(smem + off, &p.tmA, &full[s], 0, 0, idx);
+              }
+            } else {
+#pragma unroll
+              for (int q = 0; q < 8; ++q) ptx::st_shared_v4(smem_base + off + (uint32_t)(q * 4 + part) * 16u, 0u, 0u, 0u, 0u);
+            }
+          }
+        } else if (!va) {
           const int cpa = kpad_c >> 3;  // live chunks per row: 2, 4, 6 or 8
           const int cshift = cpa <= 2 ? 1 : cpa <= 4 ? 2 : 3;
           const int j = tid & ((1 << cshift) - 1), r0 = tid >> cshift, rstep = 128 >> cshift;
@@ -441,16 +480,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
             const int tbase = G > 1 ? g * m : 0;                 // first tile row of the entry
             const int ebase = G > 1 ? 0 : U.mt * 128;            // first entry row in the tile
             const int cnt = G > 1 ? m : rows;                    // entry rows in the tile
-            if (p.bsr) {
-              for (int q = r0; q < cnt; q += rstep) {
-                const int r = tbase + q;
-                const int slot = col_ok ? blk_tab[(r >> 4) * 16 + (gc >> 4)] : -1;
-                const bool ok = slot >= 0;
-                const uint16_t* src =
-                    ok ? p.vals + ((long long)slot * 256 + ((ebase + q) & 15) * 16 + (gc & 15)) : p.vals;
-                ptx::cp_async_16(dst0 + (tbase + q - r0) * 128, src, ok ? 16 : 0);
-              }
-            } else {
+            {
               const uint16_t* A = one ? pa : a_tab[g];
               const uint16_t* src = A + (long long)(ebase + r0) * k + gc;
               const long long step = (long long)rstep * k;
@@ -498,7 +528,10 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         // full[s] completes when all 128 threads' copies of this stage landed;
         // the MMA warp fences generic->async proxy before reading the stage
         if (p.bsr) {
-          ptx::cp_async_mbar_arrive_noinc(&full[s]);
+          // the zero stores (generic proxy) become visible to the tensor core
+          // (async proxy) before the arrival releases the stage
+          ptx::fence_proxy_async_smem();
+          ptx::mbar_arrive(&full[s]);
         } else {
           ptx::cp_async_mbar_arrive(&full[s]);  // pending count raised until the copies land
           ptx::named_bar_sync(3, 128);          // every thread's raise precedes the arrival
@@ -580,7 +613,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
           for (int ks = 0; ks < nsteps; ++ks) {
             // A: K-major, a K step is 32 bytes along the row; B: N-major, a K
             // step is 16 k-rows, atoms kr k-rows apart
-            const uint64_t adesc = ptx::make_smem_desc(sa + ks * 32, 16, 8 * lay.wa, ptx::umma_layout_code(lay.wa));
+            const uint64_t adesc =
+                lay.slab ? ptx::make_smem_desc(sa + ks * 4096, 16, 256, ptx::umma_layout_code(32))
+                         : ptx::make_smem_desc(sa + ks * 32, 16, 8 * lay.wa, ptx::umma_layout_code(lay.wa));
             const uint64_t bdesc = ptx::make_smem_desc(sb + ks * 16 * lay.wb, lay.kr * lay.wb, 8 * lay.wb,
                                                        ptx::umma_layout_code(lay.wb));
             ptx::umma_f16_ss(d_tmem, adesc, bdesc, idesc, (kc | ks) != 0);
@@ -1033,19 +1068,35 @@ kami_status_t tc16_spmm_bsr_launch(int m, int n, int k, long long batch, bool bf
   p.batch = batch;
   p.G = packing(m, n);
   p.bsr = 1;
-  if (n % 64 == 0) {  // dense B by TMA (the producer then copies only A's nonzero blocks)
+  {
+    // dense B by TMA: G entries x 64 k-rows x n per stage, N-major atoms of
+    // Wn = 64, 32 or 16 columns (128-, 64-, 32-byte swizzle), zero-filled
+    // past k and past the batch
     PFN_encodeTiled enc = get_encode_tiled();
     if (!enc) return KAMI_ERROR_CUDA;
-    cuuint64_t dims[4] = {64, (cuuint64_t)k, (cuuint64_t)(n / 64), (cuuint64_t)batch};
-    cuuint64_t strides[3] = {(cuuint64_t)n * 2, 128, (cuuint64_t)k * n * 2};
-    cuuint32_t box[4] = {64, 64, (cuuint32_t)(n / 64), (cuuint32_t)p.G};
+    const CUtensorMapDataType dt = bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+    const int wn = n % 64 == 0 ? 64 : n % 32 == 0 ? 32 : 16;
+    const CUtensorMapSwizzle sw =
+        wn == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : wn == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+    cuuint64_t dims[4] = {(cuuint64_t)wn, (cuuint64_t)k, (cuuint64_t)(n / wn), (cuuint64_t)batch};
+    cuuint64_t strides[3] = {(cuuint64_t)n * 2, (cuuint64_t)wn * 2, (cuuint64_t)k * n * 2};
+    cuuint32_t box[4] = {(cuuint32_t)wn, 64, (cuuint32_t)(n / wn), (cuuint32_t)p.G};
     cuuint32_t es[4] = {1, 1, 1, 1};
-    if (enc(&p.tmB, bf16 ? CU_TENSOR_MAP_DATA_TYPE_BFLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 4,
-            const_cast<void*>(B), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+    if (enc(&p.tmB, dt, 4, const_cast<void*>(B), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
     p.b_tma = 1;
-    p.b_tx = (uint32_t)(8192 * (n / 64) * p.G);
+    p.b_wb = 2 * wn;
+    p.b_tx = (uint32_t)(128 * n * p.G);
+    // A's blocks: (16 columns, 16 rows, batch max_nnzb blocks), one block per box
+    const long long nb = batch * (long long)max_nnzb;
+    cuuint64_t adims[3] = {16, 16, (cuuint64_t)(nb > 0 ? nb : 1)};
+    cuuint64_t astr[2] = {32, 512};
+    cuuint32_t abox[3] = {16, 16, 1};
+    if (enc(&p.tmA, dt, 3, const_cast<void*>(nb > 0 ? vals : B), adims, astr, abox, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_32B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
   }
   p.max_nnzb = max_nnzb;
   p.rowptr = row_ptr;
