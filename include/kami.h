@@ -280,6 +280,10 @@ const char* kami_status_string(kami_status_t status);
 /* Name of the last kernel this thread launched ("" if none). */
 const char* kami_last_kernel(void);
 
+/* Diagnostic: the CUDA runtime's message for the last launch error a call
+ * reported as KAMI_ERROR_CUDA on this thread ("no error" if none). */
+const char* kami_last_cuda_error(void);
+
 int kami_version(void); /* (MAJOR << 16) | MINOR */
 
 /* Diagnostic: the FP64 DMMA roofline denominator measured on this device.

@@ -34,7 +34,7 @@ EXPORTS = [
     "kami_gemm_strided_batched_host", "kami_release_workspace", "kami_plan", "kami_paper_cost",
     "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level", "kami_gemm_vbatched",
     "kami_spmm_bsr_strided_batched", "kami_gemm_strided_batched_axpby", "kami_probe_dmma_peak",
-    "kami_set_grid_cap", "kami_plan_candidates", "kami_spmm_zmorton_strided_batched",
+    "kami_set_grid_cap", "kami_plan_candidates", "kami_spmm_zmorton_strided_batched", "kami_last_cuda_error",
 ]
 
 
@@ -106,6 +106,8 @@ def lib() -> ctypes.CDLL:
     L.kami_status_string.argtypes = [ctypes.c_int]
     L.kami_last_kernel.restype = ctypes.c_char_p
     L.kami_last_kernel.argtypes = []
+    L.kami_last_cuda_error.restype = ctypes.c_char_p
+    L.kami_last_cuda_error.argtypes = []
     L.kami_version.restype = ctypes.c_int
     _lib = L
     return L
@@ -113,6 +115,8 @@ def lib() -> ctypes.CDLL:
 
 def _check(status: int, what: str):
     if status != 0:
+        if status == 4:  # KAMI_ERROR_CUDA: append the runtime's message
+            what = f"{what} ({lib().kami_last_cuda_error().decode()})"
         raise KamiError(status, what)
 
 

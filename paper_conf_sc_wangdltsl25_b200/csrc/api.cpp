@@ -21,6 +21,11 @@ namespace kami {
 
 static thread_local const char* g_last_kernel = "";
 void set_last_kernel(const char* name) { g_last_kernel = name; }
+static thread_local int g_last_cuda = 0;
+int launch_status(int e) {
+  if (e != 0) g_last_cuda = e;
+  return e == 0 ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+}
 static std::atomic<int> g_grid_cap{0};
 int grid_cap() { return g_grid_cap.load(std::memory_order_relaxed); }
 
@@ -350,6 +355,7 @@ const char* kami_status_string(kami_status_t s) {
 }
 
 const char* kami_last_kernel(void) { return g_last_kernel; }
+const char* kami_last_cuda_error(void) { return cudaGetErrorString((cudaError_t)g_last_cuda); }
 
 int kami_version(void) { return (KAMI_VERSION_MAJOR << 16) | KAMI_VERSION_MINOR; }
 

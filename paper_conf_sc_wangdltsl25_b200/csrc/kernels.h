@@ -17,6 +17,8 @@ typedef CUresult (*PFN_encodeTiled)(CUtensorMap*, CUtensorMapDataType, cuuint32_
                                     CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 PFN_encodeTiled get_encode_tiled();
 void set_last_kernel(const char* name);
+// records e for kami_last_cuda_error(); returns KAMI_SUCCESS iff e == cudaSuccess
+int launch_status(int cuda_error);
 // kami_set_grid_cap (tests): every persistent launcher clamps its grid to this (0 = no cap)
 int grid_cap();
 inline long long apply_grid_cap(long long grid) {

@@ -98,11 +98,13 @@ struct alignas(64) VbParams {
   int early;  // release the accumulator before the copy-out (KAMI_VB_EARLY, A/B experiments)
   // Variable-size batches, class-sorted: a pre-pass buckets the
   // entries by (m, n, k) and packs each bucket's entries G(m, n) to a tile like
-  // a uniform batch.  utab[u] = {first position, ng | mt << 8, class, G}; A, B,
-  // C are then the pointer arrays in bucket order (position -> entry's
-  // pointers, written by the pre-pass); *nunits = live unit count.
+  // a uniform batch.  Unit u's record is rec[16 u .. 16 u + 15]: slot g < 8 =
+  // {A_g, B_g} (entry pointers), slot 8 + g = {C_g, hdr, 0} with hdr = ng |
+  // mt << 4 | G << 8 | class << 12 in every slot.  Every role reads a unit
+  // with ONE load per thread (no table -> pointer chain), a unit ahead;
+  // *nunits = live unit count.
   int sorted;
-  const int4* utab;
+  const int4* rec;
   const int* nunits;  // prefetch the next unit's maps (KAMI_VB_PREFETCH=0 disables, A/B experiments)
 };
 
@@ -185,16 +187,25 @@ __host__ __device__ __forceinline__ int vb_pack(int m, int n) {
   const int g = g1 < g2 ? g1 : g2;
   return g < 1 ? 1 : (g > 8 ? 8 : g);
 }
-// sorted mode: unit u from the pre-pass table
-__device__ __forceinline__ void unit_fill_sorted(const VbParams& p, long long u, Unit& U) {
-  const int4 t = __ldg(p.utab + u);
-  U.e0 = t.x;
-  U.ng = t.y & 0xFF;
-  U.mt = t.y >> 8;
-  U.m = ((t.z >> 10) + 1) << 3;
-  U.n = (((t.z >> 5) & 31) + 1) << 3;
-  U.k = ((t.z & 31) + 1) << 3;
-  U.G = t.w;
+// sorted mode: slot q of unit u's record.  Loaded a unit (or two) before it
+// is decoded (unit_decode): decoding right after the load would stall the
+// role for a global-memory round trip per unit (ncu).
+__device__ __forceinline__ int4 rec_slot(const VbParams& p, long long u, int q) {
+  return __ldg(p.rec + u * 16 + q);
+}
+__device__ __forceinline__ int vb_hdr(int ng, int mt, int G, int c) { return ng | (mt << 4) | (G << 8) | (c << 12); }
+__device__ __forceinline__ void unit_decode(const int hdr, Unit& U) {
+  U.e0 = 0;  // (sorted mode: pointers come from the record)
+  U.ng = hdr & 15;
+  U.mt = (hdr >> 4) & 15;
+  U.G = (hdr >> 8) & 15;
+  const int c = hdr >> 12;
+  U.m = ((c >> 10) + 1) << 3;
+  U.n = (((c >> 5) & 31) + 1) << 3;
+  U.k = ((c & 31) + 1) << 3;
+}
+__device__ __forceinline__ const uint16_t* rec_ptr(int lo, int hi) {
+  return reinterpret_cast<const uint16_t*>((unsigned long long)(unsigned)lo | ((unsigned long long)(unsigned)hi << 32));
 }
 // entry index of slot g of a unit (sorted mode: its position in bucket order)
 __device__ __forceinline__ long long unit_entry(const VbParams&, const Unit& U, int g) { return U.e0 + g; }
@@ -218,7 +229,10 @@ __device__ __forceinline__ void trace(int ev, uint32_t i) {
 }
 
 template <bool kBF16>
-__global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __grid_constant__ VbParams p) {
+// 13 warps: the SM sub-partition holding four of them has 16 K registers, so
+// 128 per thread is the ceiling (a 150-register build fails to launch)
+__global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
+    (const __grid_constant__ VbParams p) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   // 1024-byte aligned base; pointer arithmetic on the __shared__ array keeps
   // the address space, so table reads compile to LDS rather than generic loads
@@ -242,7 +256,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       // Otherwise one regular arrival by producer thread 0 per stage (after
       // the TMA issue, or after every copy thread raised the pending count
       // with its cp.async arrival and a named barrier).
-      ptx::mbar_init(&full[s], p.bsr ? 128 + (p.b_tma ? 1 : 0) : 1);
+      ptx::mbar_init(&full[s], p.bsr ? 128 + (p.b_tma ? 1 : 0) : 4);
       ptx::mbar_init(&empty[s], 1);
     }
     for (int a = 0; a < p.acc_bufs; ++a) {
@@ -278,7 +292,6 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     // pointers itself (one broadcast address per warp), so no shared table or
     // table barrier is needed.
     const bool one = p.G == 1 && !p.bsr && !p.sorted;
-    long long uf = blockIdx.x;  // sorted mode: the next unit to fetch
     // SpMM: the next unit's block structure is fetched ahead too, without the
     // row_ptr -> col_blk dependency: every col_blk slot of the unit's entries
     // (<= 2 per thread: G mb kb <= 256) and every row_ptr value (<= 17)
@@ -288,18 +301,24 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       const uint16_t *pa, *pb;
       int cb[2], rp;
     };
-    auto fetch = [&](PSlot& S) {
-      if (p.sorted) {
-        unit_fill_sorted(p, uf, S.U);
-        uf += gridDim.x;
-      } else {
-        unit_fill(p, ui.grp, ui.mt, S.U);
-      }
+    // sorted mode: R = this lane's record slot (lane & 15) of the unit,
+    // loaded one fetch earlier: lanes g < ng of every producer warp hold
+    // entry g's A and B pointers, lane 8's slot the header
+    auto fetch = [&](PSlot& S, const int4 R) {
       S.pa = S.pb = nullptr;
       S.cb[0] = S.cb[1] = -1;
       S.rp = 0;
-      if (one || tid < S.U.ng) {
-        const long long e = one ? S.U.e0 : unit_entry(p, S.U, tid);
+      if (p.sorted) {
+        unit_decode(__shfl_sync(0xffffffffu, R.z, 8), S.U);
+        if ((tid & 31) < S.U.ng) {
+          S.pa = rec_ptr(R.x, R.y);
+          S.pb = rec_ptr(R.z, R.w);
+        }
+        return;
+      }
+      unit_fill(p, ui.grp, ui.mt, S.U);
+      if (one || (tid & 31) < S.U.ng) {
+        const long long e = one ? S.U.e0 : unit_entry(p, S.U, tid & 31);
         S.pa = p.bsr ? nullptr
                : p.strided ? p.As + e * (long long)p.m * p.k
                            : reinterpret_cast<const uint16_t*>(p.A[e]);
@@ -323,47 +342,42 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
       const int m = U.m, n = U.n, k = U.k, G = U.G;
       const int kchunks = (k + 63) / 64;
       const int rows = G > 1 ? U.ng * m : min(128, m - U.mt * 128);  // live tile rows
-      // ---- all-TMA unit (A and B through views): warp 0 alone; lane g holds
-      // entry g's pointers, lane 0 issues every box and makes the stage's one
-      // arrival.  The other warps only follow the ring.
+      // ---- all-TMA unit (A and B through views): lane g of every producer
+      // warp holds entry g's pointers; warp w issues the boxes of entries
+      // g = w, w + 4, ... (the TMA issue of a packed unit is ~50 instructions
+      // per entry, one warp's serial issue was the bound for small entries)
+      // and makes one of the stage's four arrivals with its own byte count.
       const VbLayout lay = vb_layout(p, n, k);
       if (!p.bsr && lay.va && lay.vb && !(p.dbg & 2)) {
-        if (tid < 32) {
-          const int rows_e = G > 1 ? m : rows;
-          const uint32_t a_e = (uint32_t)rows_e * lay.wa, b_e = lay.kr * (uint32_t)n * 2u;
-          const uint32_t tx = (uint32_t)U.ng * (a_e + b_e);
-          const CUtensorMap* ma = p.vmap + vidx(k) * 16 + (rows_e >> 3) - 1;
-          const CUtensorMap* mb = p.vmap + 96 + vidx(n) * 6 + vidx(k);
-          const int arow = G > 1 ? 0 : U.mt * 128;
-          int alo = 0, ahi = 0, blo = 0, bhi = 0;
-          if (one || tid < U.ng) {
-            view_coords(pa, alo, ahi);
-            view_coords(pb, blo, bhi);
-          }
-          for (int kc = 0; kc < kchunks; ++kc, rs.next(p.stages), ++it) {
-            const uint32_t s = rs.s;
-            ptx::mbar_wait(&empty[s], rs.ph ^ 1);
-            if (p.dbg & 4) trace(0, it);
-            uint8_t* st = smem + s * p.stage_bytes;
-            if (tid == 0) ptx::mbar_arrive_expect_tx(&full[s], tx);
+        const int w = tid >> 5, ln = tid & 31;
+        const int rows_e = G > 1 ? m : rows;
+        const uint32_t a_e = (uint32_t)rows_e * lay.wa, b_e = lay.kr * (uint32_t)n * 2u;
+        const int mine = U.ng > w ? (U.ng - w + 3) >> 2 : 0;  // entries this warp issues
+        const uint32_t tx = (uint32_t)mine * (a_e + b_e);
+        const CUtensorMap* ma = p.vmap + vidx(k) * 16 + (rows_e >> 3) - 1;
+        const CUtensorMap* mb = p.vmap + 96 + vidx(n) * 6 + vidx(k);
+        const int arow = G > 1 ? 0 : U.mt * 128;
+        int alo = 0, ahi = 0, blo = 0, bhi = 0;
+        if (one || ln < U.ng) {
+          view_coords(pa, alo, ahi);
+          view_coords(pb, blo, bhi);
+        }
+        for (int kc = 0; kc < kchunks; ++kc, rs.next(p.stages), ++it) {
+          const uint32_t s = rs.s;
+          ptx::mbar_wait(&empty[s], rs.ph ^ 1);
+          if (p.dbg & 4) trace(0, it);
+          uint8_t* st = smem + s * p.stage_bytes;
+          if (ln == 0) ptx::mbar_arrive_expect_tx(&full[s], tx);
 #pragma unroll 1
-            for (int g = 0; g < U.ng; ++g) {
-              const int xa = __shfl_sync(0xffffffffu, alo, g), ya = __shfl_sync(0xffffffffu, ahi, g);
-              const int xb = __shfl_sync(0xffffffffu, blo, g), yb = __shfl_sync(0xffffffffu, bhi, g);
-              if (tid == 0) {
-                ptx::tma_load_4d(st + g * a_e, ma, &full[s], kc * 64, arow, xa, ya);
-                ptx::tma_load_5d(st + kAReg + g * b_e, mb, &full[s], 0, kc * 64, 0, xb, yb);
-              }
+          for (int g = w; g < U.ng; g += 4) {
+            const int xa = __shfl_sync(0xffffffffu, alo, g), ya = __shfl_sync(0xffffffffu, ahi, g);
+            const int xb = __shfl_sync(0xffffffffu, blo, g), yb = __shfl_sync(0xffffffffu, bhi, g);
+            if (ln == 0) {
+              ptx::tma_load_4d(st + g * a_e, ma, &full[s], kc * 64, arow, xa, ya);
+              ptx::tma_load_5d(st + kAReg + g * b_e, mb, &full[s], 0, kc * 64, 0, xb, yb);
             }
-            if (p.dbg & 4) trace(1, it);
           }
-        } else {
-          // the other warps only advance their ring position; the next copy
-          // unit starts with a warpgroup barrier (below), so they never wait
-          // on a slot more than one lap away from warp 0 (mbarrier waits test
-          // the phase parity only: a lap ahead or behind would alias)
-          for (int kc = 0; kc < kchunks; ++kc) rs.next(p.stages);
-          it += kchunks;
+          if (p.dbg & 4) trace(1, it);
         }
         return;
       }
@@ -535,7 +549,7 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
         } else {
           ptx::cp_async_mbar_arrive(&full[s]);  // pending count raised until the copies land
           ptx::named_bar_sync(3, 128);          // every thread's raise precedes the arrival
-          if (tid == 0) ptx::mbar_arrive(&full[s]);
+          if (tid == 0) ptx::mbar_arrive_cnt(&full[s], 4);  // the four producer warps' share
         }
         if (p.dbg & 4) trace(1, it);
       }
@@ -554,24 +568,54 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     };
     const long long g1 = gridDim.x, g2 = 2 * g1;
     long long u = blockIdx.x;
-    PSlot S0, S1;
-    if (u < units) fetch(S0);
-    if (u + g1 < units) fetch(S1);
-    while (u < units) {
-      {
-        const PSlot c = S0;
-        if (u + g2 < units) fetch(S0);
-        if (p.vprefetch && p.vmap && u + g1 < units) prefetch_maps(S1);
-        body(c);
+    if (p.sorted) {
+      // class-sorted units: the slots are the raw record slots (4 registers
+      // each, loaded two units ahead), decoded right before the unit's body
+      // (PSlot state two units deep spilled, and a spilled load result is a
+      // stall on that load)
+      int4 R0 = make_int4(0, 0, 0, 0), R1 = R0;
+      if (u < units) R0 = rec_slot(p, u, tid & 15);
+      if (u + g1 < units) R1 = rec_slot(p, u + g1, tid & 15);
+      while (u < units) {
+        {
+          const int4 c = R0;
+          if (u + g2 < units) R0 = rec_slot(p, u + g2, tid & 15);
+          PSlot S;
+          fetch(S, c);
+          body(S);
+        }
+        if ((u += g1) >= units) break;
+        {
+          const int4 c = R1;
+          if (u + g2 < units) R1 = rec_slot(p, u + g2, tid & 15);
+          PSlot S;
+          fetch(S, c);
+          body(S);
+        }
+        u += g1;
       }
-      if ((u += g1) >= units) break;
-      {
-        const PSlot c = S1;
-        if (u + g2 < units) fetch(S1);
-        if (p.vprefetch && p.vmap && u + g1 < units) prefetch_maps(S0);
-        body(c);
+    } else {
+      // slots S0 / S1 = units u and u + g1 (pointers in flight or landed)
+      const int4 z = make_int4(0, 0, 0, 0);
+      PSlot S0, S1;
+      if (u < units) fetch(S0, z);
+      if (u + g1 < units) fetch(S1, z);
+      while (u < units) {
+        {
+          const PSlot c = S0;
+          if (u + g2 < units) fetch(S0, z);
+          if (p.vprefetch && p.vmap && u + g1 < units) prefetch_maps(S1);
+          body(c);
+        }
+        if ((u += g1) >= units) break;
+        {
+          const PSlot c = S1;
+          if (u + g2 < units) fetch(S1, z);
+          if (p.vprefetch && p.vmap && u + g1 < units) prefetch_maps(S0);
+          body(c);
+        }
+        u += g1;
       }
-      u += g1;
     }
     ptx::cp_async_wait<0>();  // nothing may be in flight when the CTA exits
   } else if (warp == 4) {
@@ -580,15 +624,18 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     uint32_t it = 0, acc_it = 0;  // trace indices
     UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
     Unit Un;
-    auto fill = [&](long long v) {
-      if (p.sorted) unit_fill_sorted(p, v, Un);
-      else unit_fill(p, ui.grp, ui.mt, Un);
-    };
-    if ((long long)blockIdx.x < units) fill(blockIdx.x);
+    // sorted mode: hn = the next unit's header, decoded one unit later
+    int hn = 0;
+    if (!p.sorted && (long long)blockIdx.x < units) unit_fill(p, ui.grp, ui.mt, Un);
+    if (p.sorted && (long long)blockIdx.x < units) hn = __ldg(&p.rec[(long long)blockIdx.x * 16 + 8].z);
     for (long long u = blockIdx.x; u < units; u += gridDim.x) {
+      if (p.sorted) unit_decode(hn, Un);
       const Unit U = Un;
       ui.next();
-      if (u + gridDim.x < units) fill(u + gridDim.x);
+      if (u + gridDim.x < units) {
+        if (p.sorted) hn = __ldg(&p.rec[(u + gridDim.x) * 16 + 8].z);
+        else unit_fill(p, ui.grp, ui.mt, Un);
+      }
       if (U.mt * 128 >= U.m) continue;
       const uint32_t a = ra.s;
       ptx::mbar_wait(&tempty[a], ra.ph ^ 1);
@@ -641,17 +688,32 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel(const __gri
     UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
     Unit Un;
     uint16_t* pc_n = nullptr;
-    auto fetch = [&](long long v) {
-      if (p.sorted) unit_fill_sorted(p, v, Un);
-      else unit_fill(p, ui.grp, ui.mt, Un);
-      if (L < Un.ng) pc_n = entry_C(p, unit_entry(p, Un, L), Un.m, Un.n);
+    // sorted mode: Rn = this thread's record slot 8 + (L & 7) of the next
+    // unit ({C pointer, header}), decoded one unit later
+    int4 Rn = make_int4(0, 0, 0, 0);
+    auto fetch = [&]() {
+      if (p.sorted) {
+        // the header from lane 0's slot 8 (slots 8 + g, g >= ng, are never written)
+        unit_decode(__shfl_sync(0xffffffffu, Rn.z, 0), Un);
+        if (L < Un.ng) pc_n = const_cast<uint16_t*>(rec_ptr(Rn.x, Rn.y));
+      } else {
+        unit_fill(p, ui.grp, ui.mt, Un);
+        if (L < Un.ng) pc_n = entry_C(p, unit_entry(p, Un, L), Un.m, Un.n);
+      }
     };
-    if ((long long)blockIdx.x < units) fetch(blockIdx.x);
+    if ((long long)blockIdx.x < units) {
+      if (p.sorted) Rn = rec_slot(p, blockIdx.x, 8 + (L & 7));
+      fetch();
+      if (p.sorted && (long long)blockIdx.x + gridDim.x < units) Rn = rec_slot(p, blockIdx.x + gridDim.x, 8 + (L & 7));
+    }
     for (long long u = blockIdx.x; u < units; u += gridDim.x) {
       const Unit U = Un;
       uint16_t* const pc = pc_n;
       ui.next();
-      if (u + gridDim.x < units) fetch(u + gridDim.x);
+      if (u + gridDim.x < units) {
+        fetch();
+        if (p.sorted && u + 2ll * gridDim.x < units) Rn = rec_slot(p, u + 2ll * gridDim.x, 8 + (L & 7));
+      }
       if (U.mt * 128 >= U.m) continue;
       const uint32_t a = ra.s;
       const uint32_t aph = ra.ph;
@@ -937,12 +999,11 @@ __global__ void __launch_bounds__(1024) vb_class_scan(const int* hist, int* eoff
   }
 }
 
-// scatter: entry -> its bucket position; the first entry of every tile writes
-// the tile's units (one per m-tile)
+// scatter: entry -> its bucket position; each entry writes its pointers into
+// the record slots of its unit(s) (one per m-tile)
 __global__ void vb_class_scatter(long long batch, const int* dm, const int* dn, const int* dk, const int* hist,
-                                 const int* eoff, const int* uoff, int* cursor, const void* const* A,
-                                 const void* const* B, void* const* C, const void** sA, const void** sB, void** sC,
-                                 int4* utab) {
+                                 const int* uoff, int* cursor, const void* const* A, const void* const* B,
+                                 void* const* C, int4* rec) {
   for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < batch;
        e += (long long)gridDim.x * blockDim.x) {
     const int m = __ldg(dm + e), n = __ldg(dn + e), k = __ldg(dk + e);
@@ -956,15 +1017,13 @@ __global__ void vb_class_scatter(long long batch, const int* dm, const int* dn, 
     base = __shfl_sync(peers, base, leader);
     if (!ok) continue;
     const int pos = base + __popc(peers & ((1u << lane) - 1u));
-    const int first = eoff[c] + pos;
-    sA[first] = A[e];
-    sB[first] = B[e];
-    sC[first] = C[e];
-    const int G = vb_pack(m, n);
-    if (pos % G == 0) {
-      const int cnt = hist[c], ng = cnt - pos < G ? cnt - pos : G, mt_n = (m + 127) >> 7;
-      for (int mt = 0; mt < mt_n; ++mt)
-        utab[uoff[c] + (pos / G) * mt_n + mt] = make_int4(first, ng | (mt << 8), c, G);
+    const int G = vb_pack(m, n), cnt = hist[c], tile = pos / G, g = pos - tile * G;
+    const int ng = cnt - tile * G < G ? cnt - tile * G : G, mt_n = (m + 127) >> 7;
+    const unsigned long long a = (unsigned long long)A[e], b = (unsigned long long)B[e], cc = (unsigned long long)C[e];
+    for (int mt = 0; mt < mt_n; ++mt) {
+      int4* r = rec + (long long)(uoff[c] + tile * mt_n + mt) * 16;
+      r[g] = make_int4((int)(a & 0xffffffffu), (int)(a >> 32), (int)(b & 0xffffffffu), (int)(b >> 32));
+      r[8 + g] = make_int4((int)(cc & 0xffffffffu), (int)(cc >> 32), vb_hdr(ng, mt, G, c), 0);
     }
   }
 }
@@ -1027,19 +1086,19 @@ kami_status_t vb_launch(VbParams& p, bool bf16, int n_max, int max_m, cudaStream
   fn<<<(unsigned)grid, kVbThreads, smem, stream>>>(p);
   if (p.strided) {
     set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16,strided>" : "kami_tc16_vb_kernel<f16,strided>");
-    return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+    return (kami_status_t)launch_status((int)cudaGetLastError());
   }
   if (p.zorder) {
     set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16,spmm_zmorton>" : "kami_tc16_vb_kernel<f16,spmm_zmorton>");
-    return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+    return (kami_status_t)launch_status((int)cudaGetLastError());
   }
   if (p.sorted) {
     set_last_kernel(bf16 ? "kami_tc16_vb_kernel<bf16,sorted>" : "kami_tc16_vb_kernel<f16,sorted>");
-    return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+    return (kami_status_t)launch_status((int)cudaGetLastError());
   }
   set_last_kernel(p.bsr ? (bf16 ? "kami_tc16_vb_kernel<bf16,spmm_bsr>" : "kami_tc16_vb_kernel<f16,spmm_bsr>")
                         : (bf16 ? "kami_tc16_vb_kernel<bf16>" : "kami_tc16_vb_kernel<f16>"));
-  return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+  return (kami_status_t)launch_status((int)cudaGetLastError());
 }
 
 int packing(int m, int n) {  // entries per 128-lane tile (same rule as tc16.cu)
@@ -1146,8 +1205,8 @@ kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, co
   const bool sort = dm && batch < (1ll << 30) && (env ? atoi(env) != 0 : batch >= 256);
   if (!sort) return vb_launch(p, bf16, dm ? max_n : n, dm ? max_m : m, stream);
   const long long mt_max = (max_m + 127) / 128;
-  const size_t bytes =
-      sizeof(int) * (4 * (size_t)kClasses + 4) + sizeof(int4) * (size_t)(batch * mt_max) + 3 * sizeof(void*) * (size_t)batch;
+  // records: 256 bytes per unit, at most batch * mt_max units
+  const size_t bytes = sizeof(int) * (4 * (size_t)kClasses + 4) + 256 * (size_t)(batch * mt_max);
   void* ws = nullptr;
   cudaMemPool_t pool = vb_pool();
   if (!pool || cudaMallocFromPoolAsync(&ws, bytes, pool, stream) != cudaSuccess) return KAMI_ERROR_CUDA;
@@ -1156,10 +1215,7 @@ kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, co
   int* eoff = cursor + kClasses;
   int* uoff = eoff + kClasses;
   int* nunits = uoff + kClasses;
-  int4* utab = reinterpret_cast<int4*>(nunits + 4);  // 16-byte aligned (4 kClasses + 4 ints)
-  const void** sA = reinterpret_cast<const void**>(utab + batch * mt_max);
-  const void** sB = sA + batch;
-  void** sC = const_cast<void**>(sB + batch);
+  int4* rec = reinterpret_cast<int4*>(nunits + 4);  // 16-byte aligned (4 kClasses + 4 ints)
   kami_status_t st = KAMI_SUCCESS;
   if (cudaMemsetAsync(hist, 0, sizeof(int) * 2 * kClasses, stream) != cudaSuccess) st = KAMI_ERROR_CUDA;
   if (cudaFuncSetAttribute(vb_class_scan, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1169,17 +1225,13 @@ kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, co
     const int blocks = (int)((batch + 255) / 256 < 1184 ? (batch + 255) / 256 : 1184);
     vb_class_hist<<<blocks, 256, 0, stream>>>(batch, dm, dn, dk, hist);
     vb_class_scan<<<1, 1024, kClasses * sizeof(int), stream>>>(hist, eoff, uoff, nunits);
-    vb_class_scatter<<<blocks, 256, 0, stream>>>(batch, dm, dn, dk, hist, eoff, uoff, cursor, A, B, C, sA, sB, sC,
-                                                 utab);
+    vb_class_scatter<<<blocks, 256, 0, stream>>>(batch, dm, dn, dk, hist, uoff, cursor, A, B, C, rec);
     if (cudaGetLastError() != cudaSuccess) st = KAMI_ERROR_CUDA;
   }
   if (st == KAMI_SUCCESS) {
     p.sorted = 1;
     p.G = 8;  // buffer sizing: the widest packed tile (G n <= min(8 max_n, 256))
-    p.utab = utab;
-    p.A = sA;
-    p.B = sB;
-    p.C = sC;
+    p.rec = rec;
     p.nunits = nunits;
     st = vb_launch(p, bf16, max_n, max_m, stream);
   }
