@@ -202,10 +202,22 @@ kami_status_t kami_spmm_bsr_strided_batched(int m, int n, int k, int64_t batch, 
  * of 32): the 2D schedule across a CTA pair, CTA r taking block rows
  * [8r, 8r+8) = the Morton codes [128r, 128r+128), one contiguous range of the
  * sorted codes; otherwise the 1D kernel, which decodes each block's position
- * from its code. */
+ * from its code.  (This entry point is the _ex form with KAMI_ALGO_AUTO.) */
 kami_status_t kami_spmm_zmorton_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
                                                 const int* nnzb, const int* zcode, const void* vals, int max_nnzb,
                                                 const void* B, void* C, kami_stream_t stream);
+
+/* Same with an explicit schedule: KAMI_ALGO_1D runs the 1D kernel (every
+ * CTA decodes its tile's block positions from the codes); KAMI_ALGO_2D /
+ * KAMI_ALGO_2D_PAIR the 2D schedule across a CTA pair (m > 128, n a multiple
+ * of 32; NOT_SUPPORTED otherwise), each CTA taking the contiguous Morton
+ * range of its block rows (Sec. 4.6).  KAMI_ALGO_AUTO = the faster
+ * on B200, the 1D kernel (256^3 at 50 % blocks 0.75 vs 0.48
+ * of the roofline).  Other algos: NOT_SUPPORTED. */
+kami_status_t kami_spmm_zmorton_strided_batched_ex(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                                   const int* nnzb, const int* zcode, const void* vals,
+                                                   int max_nnzb, const void* B, void* C, kami_algo_t algo,
+                                                   kami_stream_t stream);
 
 /* Block-level (on-chip-resident) mode -- the paper's block-level experiment
  * (Sec. 5.1, Sec. 5.2, Fig. 8/9): every entry is owned by one

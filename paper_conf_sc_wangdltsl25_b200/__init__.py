@@ -35,6 +35,7 @@ EXPORTS = [
     "kami_status_string", "kami_last_kernel", "kami_version", "kami_gemm_block_level", "kami_gemm_vbatched",
     "kami_spmm_bsr_strided_batched", "kami_gemm_strided_batched_axpby", "kami_probe_dmma_peak",
     "kami_set_grid_cap", "kami_plan_candidates", "kami_spmm_zmorton_strided_batched", "kami_last_cuda_error",
+    "kami_spmm_zmorton_strided_batched_ex",
 ]
 
 
@@ -84,6 +85,8 @@ def lib() -> ctypes.CDLL:
     L.kami_spmm_bsr_strided_batched.argtypes = [i, i, i, i64, i, vp, vp, vp, i, vp, vp, st]
     L.kami_spmm_zmorton_strided_batched.argtypes = [i, i, i, i64, i, vp, vp, vp, i, vp, vp, st]
     L.kami_spmm_zmorton_strided_batched.restype = ctypes.c_int
+    L.kami_spmm_zmorton_strided_batched_ex.argtypes = [i, i, i, i64, i, vp, vp, vp, i, vp, vp, i, st]
+    L.kami_spmm_zmorton_strided_batched_ex.restype = ctypes.c_int
     L.kami_gemm_strided_batched_axpby.argtypes = [i, i, i, i64, i, i, ctypes.c_double, vp, vp, ctypes.c_double, vp,
                                                   st]
     L.kami_release_workspace.argtypes = []
@@ -219,14 +222,16 @@ def spmm_bsr_strided_batched(m, n, k, batch, dtype, row_ptr, col_blk, vals, B, C
     return C
 
 
-def spmm_zmorton_strided_batched(m, n, k, batch, dtype, nnzb, zcode, vals, B, C, stream=None):
+def spmm_zmorton_strided_batched(m, n, k, batch, dtype, nnzb, zcode, vals, B, C, stream=None, algo="auto"):
     """Block-sparse A in Z-Morton block storage (Sec. 4.6, Fig. 7(b))
     times dense B.  nnzb [batch] and zcode [batch, max_nnzb] int32, vals
-    [batch, max_nnzb, 16, 16], B/C packed row-major -- all device tensors."""
+    [batch, max_nnzb, 16, 16], B/C packed row-major -- all device tensors.
+    algo: "auto" / "1d" (Morton-decoding 1D kernel) or "2d" / "2d_pair" (CTA pair)."""
     max_nnzb = zcode.shape[-1]
-    _check(lib().kami_spmm_zmorton_strided_batched(m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _ptr(nnzb),
-                                                   _ptr(zcode), _ptr(vals), max_nnzb, _ptr(B), _ptr(C),
-                                                   _stream(stream)), "kami_spmm_zmorton_strided_batched")
+    _check(lib().kami_spmm_zmorton_strided_batched_ex(m, n, k, batch, _enum(DTYPE, dtype, "dtype"), _ptr(nnzb),
+                                                      _ptr(zcode), _ptr(vals), max_nnzb, _ptr(B), _ptr(C),
+                                                      _enum(ALGO, algo, "algo"), _stream(stream)),
+           "kami_spmm_zmorton_strided_batched_ex")
     return C
 
 

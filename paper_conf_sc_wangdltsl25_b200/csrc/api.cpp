@@ -268,25 +268,37 @@ kami_status_t kami_spmm_bsr_strided_batched(int m, int n, int k, int64_t batch, 
                               reinterpret_cast<cudaStream_t>(stream));
 }
 
-kami_status_t kami_spmm_zmorton_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
-                                                const int* nnzb, const int* zcode, const void* vals, int max_nnzb,
-                                                const void* B, void* C, kami_stream_t stream) {
+kami_status_t kami_spmm_zmorton_strided_batched_ex(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                                   const int* nnzb, const int* zcode, const void* vals,
+                                                   int max_nnzb, const void* B, void* C, kami_algo_t algo,
+                                                   kami_stream_t stream) {
   kami_status_t st = check_common(m, n, k, batch, dtype, KAMI_ROW_MAJOR, KAMI_ALGO_AUTO);
   if (st != KAMI_SUCCESS) return st;
   if (!is16(dtype) || k % 16 || m % 16) return KAMI_ERROR_NOT_SUPPORTED;
   if (max_nnzb < 0 || max_nnzb > (m / 16) * (k / 16)) return KAMI_ERROR_INVALID_VALUE;
+  const bool two_d = algo == KAMI_ALGO_2D || algo == KAMI_ALGO_2D_PAIR;
+  if (!(algo == KAMI_ALGO_AUTO || algo == KAMI_ALGO_1D || two_d)) return KAMI_ERROR_NOT_SUPPORTED;
+  if (two_d && !tc16_pair_supported(m, n, k)) return KAMI_ERROR_NOT_SUPPORTED;
   if (batch == 0) return KAMI_SUCCESS;
   if (!nnzb || !zcode || !vals || !B || !C || max_nnzb == 0) return KAMI_ERROR_INVALID_VALUE;
   if (!aligned16(vals) || !aligned16(B) || !aligned16(C)) return KAMI_ERROR_MISALIGNED;
   if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
-  // m > 128: the 2D schedule across a CTA pair, each CTA finding its block
-  // rows as one contiguous Morton range (tc16_pair.cu); else the 1D kernel,
-  // which decodes each block's position from its code (tc16_vb.cu)
-  if (tc16_pair_supported(m, n, k))
+  // 2D: the schedule across a CTA pair, each CTA finding its block rows as
+  // one contiguous Morton range (tc16_pair.cu).  AUTO / 1D: the 1D kernel,
+  // which decodes each block's position from its code (tc16_vb.cu) -- on
+  // B200 the faster of the two since its A blocks arrive by TMA
+  if (two_d)
     return tc16_pair_launch(m, n, k, batch, dtype == KAMI_DTYPE_BF16, nullptr, B, C,
                             reinterpret_cast<cudaStream_t>(stream), nnzb, zcode, vals, max_nnzb);
   return tc16_spmm_bsr_launch(m, n, k, batch, dtype == KAMI_DTYPE_BF16, nnzb, zcode, vals, max_nnzb, B, C,
                               reinterpret_cast<cudaStream_t>(stream), /*zorder=*/true);
+}
+
+kami_status_t kami_spmm_zmorton_strided_batched(int m, int n, int k, int64_t batch, kami_dtype_t dtype,
+                                                const int* nnzb, const int* zcode, const void* vals, int max_nnzb,
+                                                const void* B, void* C, kami_stream_t stream) {
+  return kami_spmm_zmorton_strided_batched_ex(m, n, k, batch, dtype, nnzb, zcode, vals, max_nnzb, B, C,
+                                              KAMI_ALGO_AUTO, stream);
 }
 
 kami_status_t kami_gemm_block_level(int m, int n, int k, int64_t batch, kami_dtype_t dtype, kami_layout_t layout,

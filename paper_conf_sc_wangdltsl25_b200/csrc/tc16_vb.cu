@@ -424,8 +424,12 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
             continue;
           }
           if (j >= rpg[mbk]) continue;  // unused tail slot
+          // block row of slot j: the last br with rp[br] <= j (binary search
+          // over the <= 17 row pointers: 5 dependent shared loads, not <= 16)
           br = 0;
-          while (rpg[br + 1] <= j) ++br;
+#pragma unroll
+          for (int step = 8; step > 0; step >>= 1)
+            if (br + step <= mbk - 1 && rpg[br + step] <= j) br += step;
           if (br < br0 || br >= br1) continue;
           blk_tab[(g * mbk + br - br0) * 16 + col] = (int)((U.e0 + g) * p.max_nnzb + j);
         }

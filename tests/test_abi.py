@@ -76,6 +76,23 @@ def test_null_misaligned_and_empty():
     assert L.kami_gemm_strided_batched_host(64, 64, 64, 2, 0, 0, None, None, None) == INVALID
 
 
+def test_spmm_zmorton_ex_host_checks():
+    """Schedule selection of the Z-Morton SpMM entry point, decided before any
+    launch: unknown schedules and the 2D pair on m <= 128 are NOT_SUPPORTED,
+    an empty batch is a no-op, null arrays are INVALID."""
+    L = kami.lib()
+    f = L.kami_spmm_zmorton_strided_batched_ex
+    for algo in (3, 4, 5, 6, 7):  # 3D, non-CA, TMA-1D, TMEM variants: no sparse form
+        assert f(256, 64, 64, 4, 0, FAKE, FAKE, FAKE, 16, FAKE, FAKE, algo, None) == UNSUP
+    assert f(128, 64, 64, 4, 0, FAKE, FAKE, FAKE, 16, FAKE, FAKE, 8, None) == UNSUP  # pair needs m > 128
+    assert f(128, 64, 64, 4, 0, FAKE, FAKE, FAKE, 16, FAKE, FAKE, 2, None) == UNSUP
+    for algo in (0, 1, 2, 8):
+        assert f(256, 64, 64, 0, 0, None, None, None, 16, None, None, algo, None) == 0
+        assert f(256, 64, 64, 4, 0, None, FAKE, FAKE, 16, FAKE, FAKE, algo, None) == INVALID
+    assert f(256, 64, 64, 4, 2, FAKE, FAKE, FAKE, 16, FAKE, FAKE, 0, None) == UNSUP  # FP64: no sparse path
+    assert f(256, 64, 64, 4, 0, FAKE, FAKE, FAKE, 65, FAKE, FAKE, 0, None) == INVALID  # max_nnzb > (m/16)(k/16)
+
+
 def test_plan_host_logic():
     p = kami.plan(64, 64, 64, "f16")
     assert p["kernel"] == "tcgen05" and p["algo"] == "1d" and p["p"] == 4 and p["stages"] >= 2

@@ -28,6 +28,7 @@ ap.add_argument("--reps", type=int, default=10)
 ap.add_argument("--density", type=float, default=0.5)
 ap.add_argument("--orders", default="16,32,64,128,192,256", help="vb mode: the order set")
 ap.add_argument("--nmax", type=int, default=256, help="vb mode: max_n passed to the call")
+ap.add_argument("--algo", default="auto", help="zmorton mode: auto / 1d / 2d")
 ap.add_argument("--noperm", action="store_true", help="ptr mode: pointers in entry order (no scatter)")
 a = ap.parse_args()
 hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
@@ -67,7 +68,7 @@ elif a.mode == "zmorton":
     zv[ent_s, rank] = v[ent_s, old_s]
     nz = nnz.int()
     C = torch.empty(a.batch * m * n, dtype=B.dtype, device="cuda")
-    run = lambda: kami.spmm_zmorton_strided_batched(m, n, k, a.batch, a.dtype, nz, zc, zv, B, C)  # noqa: E731
+    run = lambda: kami.spmm_zmorton_strided_batched(m, n, k, a.batch, a.dtype, nz, zc, zv, B, C, algo=a.algo)  # noqa: E731
     nnzb = float(nnz.sum())
     flops = 2.0 * nnzb * 256 * n
     byts = nnzb * (512 + 4) + a.batch * (4 + (k * n + m * n) * 2)
