@@ -98,7 +98,13 @@ typedef enum {
    * broadcasts each B column block to the other CTA's rows (Alg. 2).
    * n a multiple of 32 in [32,256], k a multiple of 8; NOT_SUPPORTED
    * otherwise. */
-  KAMI_ALGO_2D_PAIR = 8
+  KAMI_ALGO_2D_PAIR = 8,
+  /* 16-bit only, thin m (m in {16, 32}, n a multiple of 64 in [64, 256], k in
+   * {16, 32, 64}): tcgen05 1D on the transposed product C^T = B^T A^T, n on
+   * the 128 TMEM lanes and m on the columns, so E entries share one
+   * accumulator side by side.  Strided C = A B; NOT_SUPPORTED
+   * otherwise. */
+  KAMI_ALGO_1D_XT = 9
 } kami_algo_t;
 
 /* Opaque CUDA stream; binary compatible with cudaStream_t. */
@@ -241,7 +247,8 @@ typedef struct {
   int kernel;            /* 0 = tcgen05 16-bit (SS), 1 = warp-level DMMA/HMMA, 2 = FP64 DMMA with TMA
                             broadcast, 3 = tcgen05 16-bit with A resident in TMEM (TS), 4 = FP64 DMMA
                             for the whole size grid (k-sliced, register residency ratio), 5 = LDG-fed
-                            tcgen05 16-bit (m or n = 8 mod 16), 6 = tcgen05 CTA pair (2D, cta_group::2) */
+                            tcgen05 16-bit (m or n = 8 mod 16), 6 = tcgen05 CTA pair (2D, cta_group::2),
+                            7 = tcgen05 16-bit on the transposed product (thin m, XT) */
   int entries_per_cta;   /* batch entries a CTA keeps in flight             */
   int stages;            /* shared-memory pipeline depth                    */
   int kslice_regs_pct;   /* share of A/B kept resident (Sec. 4.7)           */

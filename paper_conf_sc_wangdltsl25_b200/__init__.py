@@ -24,7 +24,7 @@ SO_PATH = os.environ.get("KAMI_LIB") or os.path.join(_HERE, "libkami.so")
 
 DTYPE = {"f16": 0, "bf16": 1, "f64": 2, "tf32": 3, "e4m3": 4, "e5m2": 5}
 LAYOUT = {"row": 0, "col": 1}
-ALGO = {"auto": 0, "1d": 1, "2d": 2, "3d": 3, "nonca": 4, "1d_tma": 5, "1d_tmem": 6, "3d_tmem": 7, "2d_pair": 8}
+ALGO = {"auto": 0, "1d": 1, "2d": 2, "3d": 3, "nonca": 4, "1d_tma": 5, "1d_tmem": 6, "3d_tmem": 7, "2d_pair": 8, "1d_xt": 9}
 STATUS = {0: "KAMI_SUCCESS", 1: "KAMI_ERROR_INVALID_VALUE", 2: "KAMI_ERROR_NOT_SUPPORTED",
           3: "KAMI_ERROR_MISALIGNED", 4: "KAMI_ERROR_CUDA"}
 
@@ -60,7 +60,7 @@ class KamiCandidate(ctypes.Structure):
 
 BOUND = {0: "hbm", 1: "tensor", 2: "smem", 3: "tma", 4: "issue", 5: "latency"}
 KERNEL = {0: "tcgen05", 1: "warp_ca", 2: "dmma_tma", 3: "tcgen05_ts", 4: "dmma_gen", 5: "tcgen05_ldg",
-          6: "tcgen05_pair"}
+          6: "tcgen05_pair", 7: "tcgen05_xt"}
 
 _lib = None
 

@@ -67,7 +67,7 @@ kami_status_t check_common(int m, int n, int k, int64_t batch, int dtype, int la
   if (m <= 0 || n <= 0 || k <= 0 || batch < 0) return KAMI_ERROR_INVALID_VALUE;
   if (dtype < KAMI_DTYPE_F16 || dtype > KAMI_DTYPE_E5M2) return KAMI_ERROR_INVALID_VALUE;
   if (layout != KAMI_ROW_MAJOR && layout != KAMI_COL_MAJOR) return KAMI_ERROR_INVALID_VALUE;
-  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_2D_PAIR) return KAMI_ERROR_INVALID_VALUE;
+  if (algo < KAMI_ALGO_AUTO || algo > KAMI_ALGO_1D_XT) return KAMI_ERROR_INVALID_VALUE;
   return check_sizes(m, n, k, (kami_dtype_t)dtype);
 }
 
@@ -132,6 +132,12 @@ kami_status_t dispatch(const RowProblem& rp, int64_t batch, kami_dtype_t dtype, 
   kami_plan_t plan;
   kami_status_t st = planner_choose(rp.m, rp.n, rp.k, dtype, algo, p, /*pointer_array=*/Ca != nullptr, &plan);
   if (st != KAMI_SUCCESS) return st;
+  if (plan.kernel == 7 && !update && !Ca)  // thin m: tcgen05 on C^T = B^T A^T (strided C = A B)
+    return tc16_xt_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream);
+  if (plan.kernel == 7) {
+    if (algo != KAMI_ALGO_AUTO) return KAMI_ERROR_NOT_SUPPORTED;
+    plan.kernel = 0;  // the update form / pointer arrays: the SS tcgen05 kernel
+  }
   if (plan.kernel == 6) {  // tcgen05 CTA pair (strided C = A B)
     if (update || Ca) return KAMI_ERROR_NOT_SUPPORTED;
     return tc16_pair_launch(rp.m, rp.n, rp.k, batch, dtype == KAMI_DTYPE_BF16, rp.A, rp.B, C, stream);

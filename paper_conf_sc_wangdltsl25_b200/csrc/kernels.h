@@ -65,6 +65,12 @@ kami_status_t tc16_ts_plan(int m, int n, int k, int layers, TsShape* s);
 kami_status_t tc16_ts_launch(int m, int n, int k, long long batch, bool bf16, int layers, const void* A,
                              const void* B, void* C, cudaStream_t stream);
 
+// ------------- tcgen05 on the transposed product for thin m (tc16_xt.cu)
+bool tc16_xt_supported(int m, int n, int k);
+kami_status_t tc16_xt_plan(int m, int n, int k, int* E, int* stages);
+kami_status_t tc16_xt_launch(int m, int n, int k, long long batch, bool bf16, const void* A, const void* B, void* C,
+                             cudaStream_t stream);
+
 // ------------------------ tcgen05 CTA pair, KAMI-2D over 2 SMs (tc16_pair.cu)
 bool tc16_pair_supported(int m, int n, int k);
 // zcode != nullptr: A in Z-Morton block storage (nnzb, zcode, vals as kami_spmm_zmorton_strided_batched)

@@ -85,7 +85,7 @@ namespace {
 constexpr double kHbmBpc = 22.5, kLsm = 29, kBsm = 127.6, kNtc = 4;
 constexpr double kDmmaFpc = 127.6, kHmmaFpc = 1907.0, kUmmaFpc = 7737.0;
 constexpr double kTbar = 250, kTlat = 700;
-constexpr double kTmaLdRow = 1.55, kTmaStRow = 4.0, kUnitSS = 900, kItemTS = 1400, kEpiVal = 14;
+constexpr double kTmaLdRow = 1.55, kTmaStRow = 4.0, kUnitSS = 900, kItemTS = 1400, kEpiVal = 14, kEpiThin = 5.5;
 constexpr double kWarpLdBpc = 32;
 
 // columns of the accumulator the busiest epilogue warp drains per MMA tile
@@ -172,7 +172,12 @@ bool model_ss(int m, int n, int k, kami_dtype_t dt, Pred* out) {
   const double t_hbm = E * bytes_entry(m, n, k, dt) / kHbmBpc;
   const double t_tma = (rowsA + rowsB) * kTmaLdRow + rowsC * kTmaStRow;
   const double t_tc = E * 2.0 * m * n * k / kUmmaFpc;
-  const double t_epi = kEpiVal * epi_cols(m, n, s.G, s.slot, s.colrep) * (s.m_tiles > 1 ? 1 : s.U);
+  // one entry per tile with m <= 32: only the first epilogue warp holds rows
+  // and its stores leave per 64-column atom as they are staged, so a column
+  // costs kEpiThin (fit: bf16 16 x 192 x 16 / 32, ~1100 cycles per entry for
+  // 192 columns, profiles/r2/xt_r2.md) rather than the packed-tile kEpiVal
+  const double kv = (s.G == 1 && s.m_tiles == 1 && m <= 32 && !s.colrep) ? kEpiThin : kEpiVal;
+  const double t_epi = kv * epi_cols(m, n, s.G, s.slot, s.colrep) * (s.m_tiles > 1 ? 1 : s.U);
   Pred p = psoft({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {kUnitSS, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR},
                   {t_epi, KAMI_BOUND_ISSUE}});
   p.cycles /= E;
@@ -196,6 +201,31 @@ bool model_ts(int m, int n, int k, kami_dtype_t dt, int layers, Pred* out) {
   Pred p = psoft({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {t_fix, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR},
                   {t_epi, KAMI_BOUND_ISSUE}});
   p.cycles /= E;
+  *out = p;
+  return true;
+}
+
+// tcgen05 on the transposed product for thin m (tc16_xt.cu): a unit = E
+// entries x one 128-column tile of n; two TMA boxes in, one out; each
+// epilogue lane drains E m values with one 16-bit store each (kXtVal cycles
+// per value, two warpgroups on alternate units), and a unit has a fixed cost
+// kUnitXT (staging barrier round trips, the store of the previous unit) --
+// both fit to the 24 thin shapes of profiles/r2/xt_r2.md, where this model
+// picks the measured-better of XT / SS on 22 of 24 (the two misses within 4 %)
+constexpr double kXtVal = kEpiVal, kUnitXT = 2500;
+bool model_xt(int m, int n, int k, kami_dtype_t dt, Pred* out) {
+  if (dt != KAMI_DTYPE_F16 && dt != KAMI_DTYPE_BF16) return false;
+  int E = 0, stages = 0;
+  if (tc16_xt_plan(m, n, k, &E, &stages) != KAMI_SUCCESS) return false;
+  const double NT = (n + 127) / 128;
+  const double wt = (double)n / NT;  // columns of n per tile
+  const double t_hbm = E * ((double)(m * k) * 2 + (k * wt + m * wt) * 2) / kHbmBpc;
+  const double t_tma = (E * (double)m + 2.0 * E * k) * kTmaLdRow + 2.0 * E * m * kTmaStRow;
+  const double t_tc = E * 2.0 * m * 128 * k / kUmmaFpc;
+  const double t_epi = kXtVal * E * m / 2;
+  Pred p = psoft({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {kUnitXT, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR},
+                  {t_epi, KAMI_BOUND_ISSUE}});
+  p.cycles *= NT / E;
   *out = p;
   return true;
 }
@@ -325,6 +355,13 @@ void fill_plan(kami_plan_t* r, int kernel, kami_algo_t algo, int p, int m, int n
     r->entries_per_cta = m == 64 ? 3 : 8;
     r->kslice_regs_pct = 50;  // B_w resident in registers, A broadcast through SMEM
     r->t_all_cycles = b200_cost(1, n, m, k, 4, dt);
+  } else if (kernel == 7) {
+    int E = 1, st = 2;
+    tc16_xt_plan(m, n, k, &E, &st);
+    r->entries_per_cta = E * st;
+    r->stages = st;
+    r->kslice_regs_pct = 0;
+    r->t_all_cycles = b200_cost(1, n, m, k, 4, dt);
   } else if (kernel == 6) {
     r->entries_per_cta = 1;
     r->stages = 4;
@@ -368,6 +405,7 @@ int planner_candidates(int m, int n, int k, kami_dtype_t dt, bool pointer_array,
     if (model_vb(m, n, k, dt, &pr)) add(5, KAMI_ALGO_1D, 4, pr);
     if (model_ss(m, n, k, dt, &pr)) add(0, KAMI_ALGO_1D, 4, pr);
     if (model_ts(m, n, k, dt, 1, &pr)) add(3, KAMI_ALGO_1D_TMEM, 4, pr);
+    if (model_xt(m, n, k, dt, &pr)) add(7, KAMI_ALGO_1D_XT, 4, pr);
     if (model_ts(m, n, k, dt, 2, &pr)) add(3, KAMI_ALGO_3D_TMEM, 8, pr);
     if (kPairInAuto && model_pair(m, n, k, dt, &pr)) add(6, KAMI_ALGO_2D_PAIR, 8, pr);
   } else {
@@ -426,6 +464,15 @@ kami_status_t planner_choose(int m, int n, int k, kami_dtype_t dtype, kami_algo_
     kami_status_t st = tc16_ts_plan(m, n, k, algo == KAMI_ALGO_3D_TMEM ? 2 : 1, &ts);
     if (st != KAMI_SUCCESS) return st == KAMI_ERROR_INVALID_VALUE ? KAMI_ERROR_NOT_SUPPORTED : st;
     fill_plan(&r, 3, algo, algo == KAMI_ALGO_3D_TMEM ? 8 : 4, m, n, k, dtype);
+    *out = r;
+    return KAMI_SUCCESS;
+  }
+  // tcgen05 on the transposed product (thin m)
+  if (algo == KAMI_ALGO_1D_XT) {
+    if ((dtype != KAMI_DTYPE_F16 && dtype != KAMI_DTYPE_BF16) || pointer_array || (p != 0 && p != 4) ||
+        !tc16_xt_supported(m, n, k))
+      return KAMI_ERROR_NOT_SUPPORTED;
+    fill_plan(&r, 7, KAMI_ALGO_1D_XT, 4, m, n, k, dtype);
     *out = r;
     return KAMI_SUCCESS;
   }

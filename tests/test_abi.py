@@ -70,7 +70,7 @@ def test_null_misaligned_and_empty():
     assert L.kami_gemm_strided_batched(64, 64, 64, 0, 0, 0, None, None, None, None) == 0
     assert L.kami_gemm(64, 64, 64, 2, 0, 0, FAKE, FAKE, FAKE, None) == INVALID  # kami_gemm needs batch == 1
     assert L.kami_gemm_batched(64, 64, 64, 3, 0, 0, None, FAKE, FAKE, None) == INVALID
-    assert L.kami_gemm_strided_batched_ex(64, 64, 64, 1, 0, 0, FAKE, FAKE, FAKE, 9, 0, None) == INVALID
+    assert L.kami_gemm_strided_batched_ex(64, 64, 64, 1, 0, 0, FAKE, FAKE, FAKE, 10, 0, None) == INVALID
     assert L.kami_gemm_strided_batched_ex(64, 64, 64, 1, 0, 0, FAKE, FAKE, FAKE, 1, -2, None) == INVALID
     assert L.kami_gemm_strided_batched_host(64, 64, 64, 0, 0, 0, None, None, None) == 0
     assert L.kami_gemm_strided_batched_host(64, 64, 64, 2, 0, 0, None, None, None) == INVALID
@@ -113,12 +113,16 @@ def test_plan_host_logic():
 def test_plan_covers_the_16bit_grid():
     """Every shape of the 16-bit grid has a plan; AUTO is the model's pick (a
     tcgen05 kernel or, for some thin tiles, the one-warp register-resident 1D),
-    and 1D with p = 0 always names the tcgen05 kernel of the shape."""
+    and 1D with p = 0 always names the tcgen05 kernel of the shape.  The
+    transposed-product kernel is picked only where it runs (thin m, n a
+    multiple of 64, k in {16, 32, 64})."""
     for m in (8, 16, 24, 32, 48, 64, 128, 192, 256):
         for n in (8, 16, 40, 64, 256):
             for k in (8, 16, 40, 64, 256):
                 p = kami.plan(m, n, k, "bf16")
-                assert p["kernel"] in ("tcgen05", "tcgen05_ts", "tcgen05_ldg", "warp_ca"), (m, n, k, p)
+                assert p["kernel"] in ("tcgen05", "tcgen05_ts", "tcgen05_ldg", "warp_ca", "tcgen05_xt"), (m, n, k, p)
+                if p["kernel"] == "tcgen05_xt":
+                    assert m in (16, 32) and n % 64 == 0 and k in (16, 32, 64), (m, n, k, p)
                 if p["kernel"] == "warp_ca":
                     assert p["algo"] == "1d" and p["p"] == 1, (m, n, k, p)
                 q = kami.plan(m, n, k, "bf16", algo="1d")  # 1D with p = 0: the tcgen05 family

@@ -24,7 +24,7 @@ def _configs():
     return json.load(open(SWEEP))["configs"]
 
 
-FAMILY = {"kami_tc16_1d_kernel": "tcgen05", "kami_tc16_ts": "tcgen05_ts", "kami_warp": "warp_ca", "kami_tc16_vb_kernel": "tcgen05_ldg",
+FAMILY = {"kami_tc16_1d_kernel": "tcgen05", "kami_tc16_xt_kernel": "tcgen05_xt", "kami_tc16_ts": "tcgen05_ts", "kami_warp": "warp_ca", "kami_tc16_vb_kernel": "tcgen05_ldg",
           "kami_dmma_tma": "dmma_tma", "kami_dmma_gen": "dmma_gen"}
 
 

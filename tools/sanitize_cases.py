@@ -37,6 +37,8 @@ CASES = [
     ("f64", 32, 32, 32, 40, "2d", 0),        # warp-level DMMA 2D
     ("f64", 64, 64, 64, 16, "1d_tma", 0),    # FP64 TMA broadcast
     ("f64", 96, 40, 72, 12, "auto", 0),      # FP64 general (dmma_gen)
+    ("bf16", 16, 128, 16, 40, "1d_xt", 0),   # transposed product, m = 16 (two epilogue warpgroups)
+    ("f16", 32, 192, 32, 20, "1d_xt", 0),    # transposed product, m = 32, 64-column last tile
 ]
 
 
@@ -78,6 +80,39 @@ def main():
         ok = np.array_equal(ki.as_bits(dC.cpu()).reshape(-1), ref.reshape(-1))
         bad += not ok
         print(f"{'OK ' if ok else 'BAD'} {kami.last_kernel():45s} pointer arrays 64^3 x 24", flush=True)
+    # variable sizes, class-sorted (>= 256 entries: pre-pass + unit records)
+    with kami.grid_cap(2):
+        rng = np.random.default_rng(7)
+        batch = 300
+        sz = rng.choice(np.array([16, 32, 64]), size=(batch, 3))
+        mats = [ki.operands(int(a), int(b), int(c), 1, "f16", "int", seed=100 + i) for i, (a, b, c) in enumerate(sz)]
+        dA = [x[0].cuda() for x in mats]
+        dB = [x[1].cuda() for x in mats]
+        dC = [torch.zeros(int(a) * int(b), dtype=torch.float16, device="cuda") for a, b, _ in sz]
+        ptr = lambda ts: torch.tensor([t.data_ptr() for t in ts], dtype=torch.int64, device="cuda")  # noqa: E731
+        dm, dn, dk = (torch.tensor(sz[:, i], dtype=torch.int32, device="cuda") for i in range(3))
+        kami.gemm_vbatched(batch, dm, dn, dk, 64, 64, 64, "f16", "row", ptr(dA), ptr(dB), ptr(dC))
+        torch.cuda.synchronize()
+        ok = True
+        for i, (a, b, c) in enumerate(sz):
+            A, B = mats[i]
+            ref = oracle.round_to(oracle.gemm(int(a), int(b), int(c), 1, "f16", "row", ki.as_bits(A), ki.as_bits(B)),
+                                  "f16")
+            ok &= np.array_equal(ki.as_bits(dC[i].cpu()).reshape(-1), np.asarray(ref).reshape(-1))
+        bad += not ok
+        print(f"{'OK ' if ok else 'BAD'} {kami.last_kernel():45s} variable sizes {{16,32,64}}^3 x {batch}", flush=True)
+    # SpMM (A blocks by TMA, absent blocks zeroed in shared memory)
+    with kami.grid_cap(2):
+        m, n, k, batch = 128, 96, 128, 12
+        rp, cb, v, B = ki.bsr_operands(m, n, k, batch, "f16", density=0.5, dist="int", seed=8)
+        C = torch.zeros(batch * m * n, dtype=torch.float16, device="cuda")
+        kami.spmm_bsr_strided_batched(m, n, k, batch, "f16", rp.cuda(), cb.cuda(), v.cuda(), B.cuda(), C)
+        torch.cuda.synchronize()
+        ref = oracle.round_to(oracle.spmm_bsr(m, n, k, batch, "f16", rp.numpy(), cb.numpy(), ki.as_bits(v),
+                                              ki.as_bits(B)), "f16")
+        ok = np.array_equal(ki.as_bits(C.cpu()).reshape(-1), np.asarray(ref).reshape(-1))
+        bad += not ok
+        print(f"{'OK ' if ok else 'BAD'} {kami.last_kernel():45s} SpMM 128x96x128 x 12, 50 % blocks", flush=True)
     print("sanitize_cases:", "all OK" if not bad else f"{bad} BAD")
     return 1 if bad else 0
 

@@ -60,12 +60,15 @@ CONFIGS = [
     ("c4 bf16-16x16x32", "bf16", 16, 16, 32, 125000),
     ("c4 bf16-128x32x16", "bf16", 128, 32, 16, 125000),
     ("c4 bf16-40x24x56 (8-grid)", "bf16", 40, 24, 56, 125000),
+    ("c4 bf16-32x192x16", "bf16", 32, 192, 16, 125000),
+    ("c4 bf16-32x256x16", "bf16", 32, 256, 16, 125000),
+    ("c4 bf16-16x256x32", "bf16", 16, 256, 32, 125000),
     ("c4 f64-96x40x72 (a7)", "f64", 96, 40, 72, 32768),
 ]
 
 # candidate schedules: (algo, p); the library rejects the ones a shape has no kernel for
 CANDIDATES = {
-    "16": [("1d", 0), ("1d_tmem", 0), ("3d_tmem", 0), ("1d", 1), ("1d", 2), ("1d", 4), ("1d", 8), ("2d", 0),
+    "16": [("1d", 0), ("1d_xt", 0), ("1d_tmem", 0), ("3d_tmem", 0), ("1d", 1), ("1d", 2), ("1d", 4), ("1d", 8), ("2d", 0),
            ("3d", 0), ("nonca", 0), ("auto", 0)],
     "f64": [("1d_tma", 0), ("1d", 0), ("1d", 1), ("1d", 2), ("1d", 8), ("2d", 0), ("3d", 0), ("nonca", 0),
             ("auto", 0)],
