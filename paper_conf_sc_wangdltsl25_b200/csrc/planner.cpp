@@ -209,10 +209,12 @@ bool model_ts(int m, int n, int k, kami_dtype_t dt, int layers, Pred* out) {
 // entries x one 128-column tile of n; two TMA boxes in, one out; each
 // epilogue lane drains E m values with one 16-bit store each (kXtVal cycles
 // per value, two warpgroups on alternate units), and a unit has a fixed cost
-// kUnitXT (staging barrier round trips, the store of the previous unit) --
-// both fit to the 24 thin shapes of profiles/r2/xt_r2.md, where this model
-// picks the measured-better of XT / SS on 22 of 24 (the two misses within 4 %)
-constexpr double kXtVal = kEpiVal, kUnitXT = 2500;
+// kUnitXT0 + kUnitXT1 E (the epilogue's barrier / TMEM-load / store chain,
+// longer with more entries): measured ~3400 / 2400 / 1900 cycles per unit for
+// E = 8 / 4 / 2 at m = 16 whatever n (profiles/r2/xt_r2.md).  On the 24 thin
+// shapes this model picks the measured-better of XT / SS on 22 (the two misses
+// 6 % and 11 %, both where the SS model is off)
+constexpr double kXtVal = kEpiVal, kUnitXT0 = 1400, kUnitXT1 = 250;
 bool model_xt(int m, int n, int k, kami_dtype_t dt, Pred* out) {
   if (dt != KAMI_DTYPE_F16 && dt != KAMI_DTYPE_BF16) return false;
   int E = 0, stages = 0;
@@ -223,7 +225,7 @@ bool model_xt(int m, int n, int k, kami_dtype_t dt, Pred* out) {
   const double t_tma = (E * (double)m + 2.0 * E * k) * kTmaLdRow + 2.0 * E * m * kTmaStRow;
   const double t_tc = E * 2.0 * m * 128 * k / kUmmaFpc;
   const double t_epi = kXtVal * E * m / 2;
-  Pred p = psoft({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {kUnitXT, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR},
+  Pred p = psoft({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {kUnitXT0 + kUnitXT1 * E, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR},
                   {t_epi, KAMI_BOUND_ISSUE}});
   p.cycles *= NT / E;
   *out = p;
