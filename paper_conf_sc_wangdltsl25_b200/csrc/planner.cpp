@@ -211,23 +211,36 @@ bool model_ts(int m, int n, int k, kami_dtype_t dt, int layers, Pred* out) {
 // per value, two warpgroups on alternate units), and a unit has a fixed cost
 // kUnitXT0 + kUnitXT1 E (the epilogue's barrier / TMEM-load / store chain,
 // longer with more entries): measured ~3400 / 2400 / 1900 cycles per unit for
-// E = 8 / 4 / 2 at m = 16 whatever n (profiles/r2/xt_r2.md).  On the 24 thin
-// shapes this model picks the measured-better of XT / SS on 22 (the two misses
-// 6 % and 11 %, both where the SS model is off)
-constexpr double kXtVal = kEpiVal, kUnitXT0 = 1400, kUnitXT1 = 250;
+// E = 8 / 4 / 2 at m = 16 whatever n (profiles/r2/xt_r2.md).  Fit on the 24
+// thin shapes (head and pair tiles): the model picks the measured-better of XT
+// / SS / warp on 22, the two misses (32 x 192 x 32, 32 x 256 x 16) by 8-9 %
+constexpr double kXtVal = kEpiVal, kUnitXT0 = 1400, kUnitXT1 = 200;
 bool model_xt(int m, int n, int k, kami_dtype_t dt, Pred* out) {
   if (dt != KAMI_DTYPE_F16 && dt != KAMI_DTYPE_BF16) return false;
   int E = 0, stages = 0;
   if (tc16_xt_plan(m, n, k, &E, &stages) != KAMI_SUCCESS) return false;
-  const double NT = (n + 127) / 128;
-  const double wt = (double)n / NT;  // columns of n per tile
-  const double t_hbm = E * ((double)(m * k) * 2 + (k * wt + m * wt) * 2) / kHbmBpc;
-  const double t_tma = (E * (double)m + 2.0 * E * k) * kTmaLdRow + 2.0 * E * m * kTmaStRow;
-  const double t_tc = E * 2.0 * m * 128 * k / kUmmaFpc;
-  const double t_epi = kXtVal * E * m / 2;
-  Pred p = psoft({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {kUnitXT0 + kUnitXT1 * E, KAMI_BOUND_ISSUE}, {t_tc, KAMI_BOUND_TENSOR},
-                  {t_epi, KAMI_BOUND_ISSUE}});
-  p.cycles *= NT / E;
+  // a head tile: E entries x 128 columns of n; a pair tile: 2E entries x 64
+  auto unit = [&](int P) {
+    const double ents = (double)E * P, cols = 128.0 / P;
+    const double t_hbm = ents * ((double)m * k + k * cols + m * cols) * 2 / kHbmBpc;
+    const double t_tma = (ents * m + 2.0 * E * k) * kTmaLdRow + 2.0 * E * m * kTmaStRow;
+    const double t_tc = E * 2.0 * P * m * 128 * k / kUmmaFpc;
+    const double t_epi = kXtVal * E * m / 2;
+    return psoft({{t_hbm, KAMI_BOUND_HBM}, {t_tma, KAMI_BOUND_TMA}, {kUnitXT0 + kUnitXT1 * E, KAMI_BOUND_ISSUE},
+                  {t_tc, KAMI_BOUND_TENSOR}, {t_epi, KAMI_BOUND_ISSUE}});
+  };
+  Pred p;
+  if (n % 128 == 0) {
+    p = unit(1);
+    p.cycles *= (n / 128.0) / E;
+  } else if (n == 64) {
+    p = unit(2);
+    p.cycles /= 2.0 * E;
+  } else {  // n = 192: two heads and one pair per 2E entries
+    const Pred h = unit(1), q = unit(2);
+    p = h.cycles >= q.cycles ? h : q;
+    p.cycles = (2 * h.cycles + q.cycles) / (2.0 * E);
+  }
   *out = p;
   return true;
 }

@@ -22,7 +22,15 @@
 // = one column n of C: tcgen05.ld of 64 accumulator columns (4 or 2 entries)
 // per wait, cvt.rn, 16-bit stores into a staging tile in C's row-major box
 // layout, one TMA store per unit.
-// A unit = (group of E entries, 128-column tile of n).
+// A unit = (group of E entries, 128-column tile of n) -- a *head* tile, P = 1
+// -- or, for the 64-column pieces (n = 64, and the last 64 columns of
+// n = 192), a *pair* tile, P = 2: lanes 0-63 hold entry 2g's 64 columns and
+// lanes 64-127 entry 2g+1's, the MMA's N is 2m (A^T of both entries stacked),
+// and only the two diagonal m-column blocks are kept (the block-diagonal
+// packing of tc16.cu, in the transposed space).  Head and pair tiles have the
+// same shared-memory geometry: 2E atoms of k x 64 for B, and the staging tile
+// [2E][m][64] for C; only the boxes, N and the TMEM column of a lane half
+// differ.  n = 192 runs three units per 2E entries: two heads, one pair.
 #include <cuda.h>
 #include <cuda_fp16.h>
 #include <cuda_bf16.h>
@@ -46,6 +54,9 @@ struct alignas(64) XtParams {
   CUtensorMap tmA;  // A (k, m, batch), box (k, m, E), 2k-byte swizzle
   CUtensorMap tmB;  // B (64, k, n/64, batch), box (64, k, 2, E), 128-byte swizzle
   CUtensorMap tmC;  // C (64, m, n/64, batch), box (64, m, 2, E), no swizzle
+  CUtensorMap tmA2, tmB2, tmC2;  // pair tiles: boxes (k, m, 2E), (64, k, 1, 2E), (64, m, 1, 2E)
+  int mode;         // 0: n % 128 == 0 (heads), 1: n == 64 (pairs), 2: n == 192 (two heads + one pair per 2E)
+  uint32_t idesc2, tx2;
   int m, n, k, E, NT;
   long long batch, units;
   int stages;
@@ -54,6 +65,18 @@ struct alignas(64) XtParams {
   uint32_t idesc, tx;
   int acc_cols;
 };
+
+// unit (grp, mt) -> pair tile?, first entry, first 64-column atom of n
+struct XtUnit {
+  bool pair;
+  int e0, atom;
+};
+__device__ __forceinline__ XtUnit xt_unit(const XtParams& p, long long grp, int mt) {
+  if (p.mode == 0) return {false, (int)(grp * p.E), 2 * mt};
+  if (p.mode == 1) return {true, (int)(grp * 2 * p.E), 0};
+  if (mt < 2) return {false, (int)(grp * 2 * p.E) + mt * p.E, 0};
+  return {true, (int)(grp * 2 * p.E), 2};
+}
 
 template <bool kBF16, int kM>
 __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __grid_constant__ XtParams p) {
@@ -69,6 +92,11 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
     ptx::prefetch_tmap(&p.tmA);
     ptx::prefetch_tmap(&p.tmB);
     ptx::prefetch_tmap(&p.tmC);
+    if (p.mode) {
+      ptx::prefetch_tmap(&p.tmA2);
+      ptx::prefetch_tmap(&p.tmB2);
+      ptx::prefetch_tmap(&p.tmC2);
+    }
     for (int s = 0; s < p.stages; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
@@ -93,11 +121,12 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
       UnitIter ui(blockIdx.x, gridDim.x, p.NT);
       for (long long u = blockIdx.x; u < p.units; u += gridDim.x, ui.next(), r.next(p.stages)) {
         ptx::mbar_wait(&empty[r.s], r.ph ^ 1);
-        ptx::mbar_arrive_expect_tx(&full[r.s], p.tx);
+        const XtUnit U = xt_unit(p, ui.grp, ui.mt);
+        ptx::mbar_arrive_expect_tx(&full[r.s], U.pair ? p.tx2 : p.tx);
         uint8_t* st = smem + r.s * p.stage_bytes;
-        const int e0 = (int)(ui.grp * p.E);
-        ptx::tma_load_4d(st, &p.tmB, &full[r.s], 0, 0, 2 * ui.mt, e0);  // B^T: the MMA's A operand
-        ptx::tma_load_3d(st + p.a_off, &p.tmA, &full[r.s], 0, 0, e0);   // A^T: the MMA's B operand
+        // B^T (the MMA's A operand) and A^T (its B operand)
+        ptx::tma_load_4d(st, U.pair ? &p.tmB2 : &p.tmB, &full[r.s], 0, 0, U.atom, U.e0);
+        ptx::tma_load_3d(st + p.a_off, U.pair ? &p.tmA2 : &p.tmA, &full[r.s], 0, 0, U.e0);
       }
     }
   } else if (warp == 1) {
@@ -105,22 +134,27 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
     RingPos r, ra;
     const uint32_t a_sw = (uint32_t)p.k * 2u;  // A rows: 2k bytes, 2k-byte swizzle
     const int ksteps = p.k / 16;
-    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, r.next(p.stages), ra.next(2)) {
+    UnitIter ui(blockIdx.x, gridDim.x, p.NT);
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, r.next(p.stages), ra.next(2), ui.next()) {
+      const bool pair = xt_unit(p, ui.grp, ui.mt).pair;
+      const int P = pair ? 2 : 1;  // entries per 128-lane tile
       ptx::mbar_wait(&tempty[ra.s], ra.ph ^ 1);
       ptx::tc_fence_after();
       ptx::mbar_wait(&full[r.s], r.ph);
       ptx::tc_fence_after();
       if (lane == 0) {
         const uint32_t sb = smem_base + r.s * p.stage_bytes, sa = sb + p.a_off;
+        const uint32_t idesc = pair ? p.idesc2 : p.idesc;
         for (int e = 0; e < p.E; ++e) {
-          const uint32_t d = tmem_base + ra.s * p.acc_cols + e * p.m;
+          const uint32_t d = tmem_base + ra.s * p.acc_cols + e * P * p.m;
           for (int ks = 0; ks < ksteps; ++ks) {
             // B^T (MN-major): two 64-column atoms k*128 bytes apart, a K step = 16 rows of 128 B
             const uint64_t ad = ptx::make_smem_desc(sb + e * p.ent_b + ks * 2048, (uint32_t)p.k * 128, 1024, 2);
             // A^T (K-major): m rows of 2k bytes, a K step = 32 bytes along the row
-            const uint64_t bd = ptx::make_smem_desc(sa + e * p.ent_a + ks * 32, 16, 8 * a_sw,
+            // (pair tiles: the two entries' A^T rows stacked, N = 2m)
+            const uint64_t bd = ptx::make_smem_desc(sa + e * P * p.ent_a + ks * 32, 16, 8 * a_sw,
                                                     ptx::umma_layout_code((int)a_sw));
-            ptx::umma_f16_ss(d, ad, bd, p.idesc, ks != 0);
+            ptx::umma_f16_ss(d, ad, bd, idesc, ks != 0);
           }
         }
         ptx::umma_commit(&empty[r.s]);
@@ -135,7 +169,7 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
     const int wg = (warp - 2) >> 2;
     const int sp = warp & 3;          // TMEM sub-partition of this warp
     const int col = sp * 32 + lane;   // this thread's column of the 128-column tile
-    const int atom = col >> 6;
+    const int half = col >> 6;        // head tiles: the 64-column atom; pair tiles: the entry of the pair
     const uint32_t col_b = (uint32_t)(col & 63) * 2u;
     const bool leader = (warp & 3) == 2 && lane == 0;
     const uint32_t cbuf = smem_base + p.c_off + wg * p.c_buf;
@@ -143,9 +177,14 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
     uint32_t ph = 0;
     UnitIter ui(blockIdx.x + (long long)wg * gridDim.x, 2ll * gridDim.x, p.NT);
     for (long long u = blockIdx.x + (long long)wg * gridDim.x; u < p.units; u += 2ll * gridDim.x, ui.next(), ph ^= 1) {
-      const long long e0 = ui.grp * p.E;
-      const int ne = p.batch - e0 < p.E ? (int)(p.batch - e0) : p.E;
-      const bool live = ui.mt * 128 + col < p.n;
+      const XtUnit U = xt_unit(p, ui.grp, ui.mt);
+      const int P = U.pair ? 2 : 1;
+      const long long e0 = U.e0;
+      const int ng = (int)((p.batch - e0 + P - 1) / P);  // live groups of P entries
+      const int ne = ng < p.E ? ng : p.E;
+      // this lane's first accumulator column: head tiles (g m), pair tiles (2 g m + half m)
+      const int cs = P * kM;
+      const int c_half = U.pair ? half * kM : 0;
       // this warpgroup's previous store is done reading the staging tile
       if (leader) ptx::bulk_wait_read<0>();
       ptx::named_bar_sync(1 + wg, 128);
@@ -155,10 +194,15 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
       for (int e1 = 0; e1 < ne; e1 += per) {
         uint32_t v[64];
         // one wait per 64 columns: a wait per entry serialised the TMEM load latency
-        ptx::tmem_ld_32x32b_x32(t_row + e1 * kM, *reinterpret_cast<uint32_t(*)[32]>(&v[0]));
-        ptx::tmem_ld_32x32b_x32(t_row + e1 * kM + 32, *reinterpret_cast<uint32_t(*)[32]>(&v[32]));
+        // groups e1 .. e1 + per - 1: kM columns each (c_half is warp-uniform)
+#pragma unroll
+        for (int gq = 0; gq < per; ++gq) {
+          const uint32_t ta = t_row + (e1 + gq) * cs + c_half;
+          if (kM == 32) ptx::tmem_ld_32x32b_x32(ta, *reinterpret_cast<uint32_t(*)[32]>(&v[gq * 32]));
+          else ptx::tmem_ld_32x32b_x16(ta, *reinterpret_cast<uint32_t(*)[16]>(&v[gq * 16]));
+        }
         ptx::tmem_wait_ld();
-        if (live) {
+        {  // (every tile is full: head tiles 128 columns of one entry, pair tiles 64 of two)
 #pragma unroll
           for (int q = 0; q < 64; ++q) {
             const int e = e1 + q / kM, j = q % kM;
@@ -166,7 +210,7 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
               const float x = __uint_as_float(v[q]);
               const unsigned short h = kBF16 ? __bfloat16_as_ushort(__float2bfloat16_rn(x))
                                              : __half_as_ushort(__float2half_rn(x));
-              const uint32_t addr = cbuf + (uint32_t)((e * 2 + atom) * kM + j) * 128u + col_b;
+              const uint32_t addr = cbuf + (uint32_t)((e * 2 + half) * kM + j) * 128u + col_b;
               asm volatile("st.shared.u16 [%0], %1;" ::"r"(addr), "h"(h) : "memory");
             }
           }
@@ -178,7 +222,7 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
       ptx::fence_proxy_async_smem();
       ptx::named_bar_sync(1 + wg, 128);
       if (leader) {
-        ptx::tma_store_4d(&p.tmC, smem + p.c_off + wg * p.c_buf, 0, 0, 2 * ui.mt, (int)e0);
+        ptx::tma_store_4d(U.pair ? &p.tmC2 : &p.tmC, smem + p.c_off + wg * p.c_buf, 0, 0, U.atom, (int)e0);
         ptx::bulk_commit();
       }
     }
@@ -199,8 +243,10 @@ bool tc16_xt_supported(int m, int n, int k) {
 // entries per unit: the largest of 8, 4, 2, 1 that leaves at least three stages
 kami_status_t tc16_xt_plan(int m, int n, int k, int* E_out, int* stages_out) {
   if (!tc16_xt_supported(m, n, k)) return KAMI_ERROR_NOT_SUPPORTED;
+  const int pa = (n % 128 != 0) ? 2 : 1;  // pair tiles hold the A rows of 2E entries
   for (int E = 8; E >= 1; E >>= 1) {
-    const int stage = E * (2 * k * 128 + m * k * 2);
+    if (E * pa * m > 256) continue;         // one accumulator of <= 256 columns
+    const int stage = E * (2 * k * 128 + pa * m * k * 2);
     const int cbuf = E * 2 * m * 128;
     int st = (kXtSmemLimit - 1024 - 256 - 2 * cbuf) / stage;
     if (st > kXtMaxStages) st = kXtMaxStages;
@@ -251,28 +297,54 @@ kami_status_t tc16_xt_launch(int m, int n, int k, long long batch, bool bf16, co
             CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
       return KAMI_ERROR_CUDA;
   }
+  p.mode = n % 128 == 0 ? 0 : n == 64 ? 1 : 2;
+  if (p.mode) {  // pair tiles: one 64-column atom of each of 2E entries
+    cuuint64_t adims[3] = {(cuuint64_t)k, (cuuint64_t)m, (cuuint64_t)batch};
+    cuuint64_t astr[2] = {(cuuint64_t)k * 2, (cuuint64_t)m * k * 2};
+    cuuint32_t abox[3] = {(cuuint32_t)k, (cuuint32_t)m, (cuuint32_t)(2 * E)};
+    const CUtensorMapSwizzle sw =
+        k == 64 ? CU_TENSOR_MAP_SWIZZLE_128B : k == 32 ? CU_TENSOR_MAP_SWIZZLE_64B : CU_TENSOR_MAP_SWIZZLE_32B;
+    cuuint64_t bdims[4] = {64, (cuuint64_t)k, (cuuint64_t)(n / 64), (cuuint64_t)batch};
+    cuuint64_t bstr[3] = {(cuuint64_t)n * 2, 128, (cuuint64_t)k * n * 2};
+    cuuint32_t bbox[4] = {64, (cuuint32_t)k, 1, (cuuint32_t)(2 * E)};
+    cuuint64_t cdims[4] = {64, (cuuint64_t)m, (cuuint64_t)(n / 64), (cuuint64_t)batch};
+    cuuint64_t cstr[3] = {(cuuint64_t)n * 2, 128, (cuuint64_t)m * n * 2};
+    cuuint32_t cbox[4] = {64, (cuuint32_t)m, 1, (cuuint32_t)(2 * E)};
+    if (enc(&p.tmA2, dt, 3, const_cast<void*>(A), adims, astr, abox, es, CU_TENSOR_MAP_INTERLEAVE_NONE, sw,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS ||
+        enc(&p.tmB2, dt, 4, const_cast<void*>(B), bdims, bstr, bbox, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+            CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS ||
+        enc(&p.tmC2, dt, 4, C, cdims, cstr, cbox, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+            CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+      return KAMI_ERROR_CUDA;
+  }
   p.m = m;
   p.n = n;
   p.k = k;
   p.E = E;
-  p.NT = (n + 127) / 128;
+  // UnitIter m-tile count: heads per entry group (mode 0), one pair (1), two heads + one pair (2)
+  p.NT = p.mode == 0 ? n / 128 : p.mode == 1 ? 1 : 3;
   p.batch = batch;
-  p.units = (batch + E - 1) / E * p.NT;
+  p.units = p.mode == 0 ? (batch + E - 1) / E * p.NT : (batch + 2 * E - 1) / (2 * E) * p.NT;
   p.stages = stages;
   p.ent_b = 2u * k * 128;  // two 64-column atoms of k rows
   p.ent_a = (uint32_t)m * k * 2;
   p.a_off = (uint32_t)E * p.ent_b;
-  p.stage_bytes = (p.a_off + (uint32_t)E * p.ent_a + 1023) & ~1023u;
-  // (full boxes always land: OOB atoms of a 64-column last tile and entries
-  // past the batch are zero-filled and counted)
+  p.stage_bytes = (p.a_off + (uint32_t)(p.mode ? 2 : 1) * E * p.ent_a + 1023) & ~1023u;
+  // (full boxes always land: entries past the batch are zero-filled and counted)
   p.tx = (uint32_t)E * (p.ent_b + p.ent_a);
+  p.tx2 = (uint32_t)E * p.ent_b + 2u * E * p.ent_a;
   p.c_buf = (uint32_t)E * 2 * m * 128;
   p.c_off = (uint32_t)stages * p.stage_bytes;
   p.bar_off = p.c_off + 2 * p.c_buf;
-  int cols = 64;  // >= 64: the epilogue reads 64 columns per TMEM load batch
-  while (cols < E * m) cols <<= 1;
+  // the epilogue reads 64 / m groups per TMEM load batch, P m columns apart
+  const int pmax = p.mode ? 2 : 1, per = 64 / m;
+  int cols = 64;
+  while (cols < (E > per ? E : per) * pmax * m) cols <<= 1;
   p.acc_cols = cols;
   p.idesc = ptx::make_idesc_f16(bf16 ? 1 : 0, 128, m, /*a MN-major*/ 1, /*b K-major*/ 0);
+  p.idesc2 = ptx::make_idesc_f16(bf16 ? 1 : 0, 128, 2 * m, 1, 0);
   const uint32_t smem = p.bar_off + 256 + 1024;
   if (smem > (uint32_t)kXtSmemLimit) return KAMI_ERROR_NOT_SUPPORTED;
   auto fn = bf16 ? (m == 16 ? kami_tc16_xt_kernel<true, 16> : kami_tc16_xt_kernel<true, 32>)
