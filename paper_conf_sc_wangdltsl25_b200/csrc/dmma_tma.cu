@@ -78,8 +78,12 @@ __device__ __forceinline__ void load_a_entry(void* dst, const DmmaTmaParams& prm
 // columns 2a, 2a + 1; t = 2, 3: 2a + 8, 2a + 9) gives the four rows of a
 // half-warp eight distinct units.  Any permutation of k applied to A and B
 // alike leaves the product unchanged.
+// Used for k = 64 only (FK = 16 k-steps): at 32^3 the permuted B_w loads
+// measured slower (14.8 vs 17.0-17.4 TF/s, profiles/r2/fp64_kperm_r2.txt)
+// than the half-warp conflicts they remove.
+template <bool kP>
 __device__ __forceinline__ int kperm(int kk, int t) {
-  return ((kk >> 2) << 4) + ((kk & 3) << 1) + (t & 1) + ((t >> 1) << 3);
+  return kP ? ((kk >> 2) << 4) + ((kk & 3) << 1) + (t & 1) + ((t >> 1) << 3) : kk * 4 + t;
 }
 
 // B_w fragments of k-steps [K0, K1) of one entry (k = kperm(kk, t), n = g of each 8x8 block).
@@ -90,7 +94,7 @@ __device__ __forceinline__ void load_b_steps(double (&b)[FK][FN], const double* 
   for (int kk = K0; kk < K1; ++kk)
 #pragma unroll
     for (int j = 0; j < FN; ++j)
-      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(b[kk][j]) : "l"(Bg + kperm(kk, t) * N + j * 8 + g));
+      asm volatile("ld.global.nc.f64 %0, [%1];" : "=d"(b[kk][j]) : "l"(Bg + kperm<(FK >= 16)>(kk, t) * N + j * 8 + g));
 }
 
 // One k-step range of the entry: A fragments from the swizzled broadcast tile
@@ -100,7 +104,7 @@ __device__ __forceinline__ void mma_steps(double (&c)[FM][FN][2], const double (
                                           int g) {
 #pragma unroll
   for (int kk = K0; kk < K1; ++kk) {
-    const int col = kperm(kk, t);
+    const int col = kperm<(FK >= 16)>(kk, t);
     const uint32_t chunk_off = (uint32_t)(col >> 4) * (M * 128) + ((col & 1) << 3);
     const uint32_t unit = (uint32_t)((col & 15) >> 1);
 #pragma unroll
@@ -187,7 +191,7 @@ __global__ void __launch_bounds__(P * 32 * TEAMS, 1) kami_dmma_tma_1d_kernel(con
 #pragma unroll
       for (int kk = 0; kk < Cfg::FK; ++kk)
 #pragma unroll
-        for (int j = 0; j < Cfg::FN; ++j) b[kk][j] = __ldg(Bg + kperm(kk, t) * N + j * 8 + g);
+        for (int j = 0; j < Cfg::FN; ++j) b[kk][j] = __ldg(Bg + kperm<(Cfg::FK >= 16)>(kk, t) * N + j * 8 + g);
     }
     double c[Cfg::FM][Cfg::FN][2];
 #pragma unroll
