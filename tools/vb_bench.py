@@ -29,6 +29,7 @@ ap.add_argument("--density", type=float, default=0.5)
 ap.add_argument("--orders", default="16,32,64,128,192,256", help="vb mode: the order set")
 ap.add_argument("--nmax", type=int, default=256, help="vb mode: max_n passed to the call")
 ap.add_argument("--algo", default="auto", help="zmorton mode: auto / 1d / 2d")
+ap.add_argument("--sortalloc", action="store_true", help="vb mode: entries allocated in (m, n, k) class order")
 ap.add_argument("--noperm", action="store_true", help="ptr mode: pointers in entry order (no scatter)")
 a = ap.parse_args()
 hbm = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"] if os.path.exists(
@@ -88,6 +89,8 @@ else:
     rng = np.random.default_rng(0)
     orders = np.array([int(x) for x in a.orders.split(",")])
     sz = rng.choice(orders, size=(a.batch, 3))
+    if a.sortalloc:  # memory order = the kernel's class-sorted unit order (address locality experiment)
+        sz = sz[np.lexsort((sz[:, 2], sz[:, 1], sz[:, 0]))]
     mm, nn, kk = sz[:, 0], sz[:, 1], sz[:, 2]
     es = 2
     offA = np.concatenate([[0], np.cumsum(mm * kk)])
