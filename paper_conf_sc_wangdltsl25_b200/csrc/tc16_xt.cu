@@ -63,7 +63,7 @@ struct alignas(64) XtParams {
   uint32_t stage_bytes, a_off, ent_b, ent_a;
   uint32_t c_off, c_buf, bar_off;
   uint32_t idesc, tx;
-  int acc_cols;
+  int acc_cols, acc_bufs;  // accumulators of acc_cols TMEM columns (2 or 4)
 };
 
 // unit (grp, mt) -> pair tile?, first entry, first 64-column atom of n
@@ -85,8 +85,8 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + p.bar_off);
   uint64_t* empty = full + kXtMaxStages;
   uint64_t* tfull = empty + kXtMaxStages;
-  uint64_t* tempty = tfull + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+  uint64_t* tempty = tfull + 4;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 4);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     ptx::prefetch_tmap(&p.tmA);
@@ -101,13 +101,13 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
     }
-    for (int a = 0; a < 2; ++a) {
+    for (int a = 0; a < p.acc_bufs; ++a) {
       ptx::mbar_init(&tfull[a], 1);
-      ptx::mbar_init(&tempty[a], 4);  // the four warps of epilogue warpgroup a
+      ptx::mbar_init(&tempty[a], 4);  // the four warps of the epilogue warpgroup draining it
     }
     ptx::fence_mbar_init();
   }
-  if (warp == 1) ptx::tmem_alloc(tmem_slot, 2 * p.acc_cols);
+  if (warp == 1) ptx::tmem_alloc(tmem_slot, p.acc_bufs * p.acc_cols);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
@@ -135,7 +135,7 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
     const uint32_t a_sw = (uint32_t)p.k * 2u;  // A rows: 2k bytes, 2k-byte swizzle
     const int ksteps = p.k / 16;
     UnitIter ui(blockIdx.x, gridDim.x, p.NT);
-    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, r.next(p.stages), ra.next(2), ui.next()) {
+    for (long long u = blockIdx.x; u < p.units; u += gridDim.x, r.next(p.stages), ra.next(p.acc_bufs), ui.next()) {
       const bool pair = xt_unit(p, ui.grp, ui.mt).pair;
       const int P = pair ? 2 : 1;  // entries per 128-lane tile
       ptx::mbar_wait(&tempty[ra.s], ra.ph ^ 1);
@@ -164,8 +164,8 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
     }
   } else {
     // ------------------------------------------------------------ epilogue
-    // warpgroup wg takes the CTA's units i = wg, wg + 2, ... and always
-    // accumulator wg (the MMA alternates accumulators unit by unit)
+    // warpgroup wg takes the CTA's units i = wg, wg + 2, ...; unit i lives in
+    // accumulator i mod acc_bufs (the MMA's ring), phase (i / acc_bufs) & 1
     const int wg = (warp - 2) >> 2;
     const int sp = warp & 3;          // TMEM sub-partition of this warp
     const int col = sp * 32 + lane;   // this thread's column of the 128-column tile
@@ -174,9 +174,10 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
     const bool leader = (warp & 3) == 2 && lane == 0;
     const uint32_t cbuf = smem_base + p.c_off + wg * p.c_buf;
     constexpr int per = 64 / kM;      // entries per TMEM load batch (64 columns)
-    uint32_t ph = 0;
+    uint32_t li = wg;  // the CTA-local unit index i
     UnitIter ui(blockIdx.x + (long long)wg * gridDim.x, 2ll * gridDim.x, p.NT);
-    for (long long u = blockIdx.x + (long long)wg * gridDim.x; u < p.units; u += 2ll * gridDim.x, ui.next(), ph ^= 1) {
+    for (long long u = blockIdx.x + (long long)wg * gridDim.x; u < p.units; u += 2ll * gridDim.x, ui.next(), li += 2) {
+      const uint32_t acc = li % (uint32_t)p.acc_bufs, ph = (li / (uint32_t)p.acc_bufs) & 1u;
       const XtUnit U = xt_unit(p, ui.grp, ui.mt);
       const int P = U.pair ? 2 : 1;
       const long long e0 = U.e0;
@@ -188,9 +189,9 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
       // this warpgroup's previous store is done reading the staging tile
       if (leader) ptx::bulk_wait_read<0>();
       ptx::named_bar_sync(1 + wg, 128);
-      ptx::mbar_wait(&tfull[wg], ph);
+      ptx::mbar_wait(&tfull[acc], ph);
       ptx::tc_fence_after();
-      const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + wg * p.acc_cols;
+      const uint32_t t_row = tmem_base + (uint32_t(sp * 32) << 16) + acc * p.acc_cols;
       for (int e1 = 0; e1 < ne; e1 += per) {
         uint32_t v[64];
         // one wait per 64 columns: a wait per entry serialised the TMEM load latency
@@ -202,6 +203,13 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
           else ptx::tmem_ld_32x32b_x16(ta, *reinterpret_cast<uint32_t(*)[16]>(&v[gq * 16]));
         }
         ptx::tmem_wait_ld();
+        if (e1 + per >= ne) {
+          // every column of the unit is in registers: release the accumulator
+          // before the conversions and stores of the last batch
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
+        }
         {  // (every tile is full: head tiles 128 columns of one entry, pair tiles 64 of two)
 #pragma unroll
           for (int q = 0; q < 64; ++q) {
@@ -216,9 +224,6 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
           }
         }
       }
-      ptx::tc_fence_before();  // accumulator wg may be overwritten by the MMA of this warpgroup's next unit
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&tempty[wg]);
       ptx::fence_proxy_async_smem();
       ptx::named_bar_sync(1 + wg, 128);
       if (leader) {
@@ -231,7 +236,7 @@ __global__ void __launch_bounds__(kXtThreads, 1) kami_tc16_xt_kernel(const __gri
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
-  if (warp == 1) ptx::tmem_dealloc(tmem_base, 2 * p.acc_cols);
+  if (warp == 1) ptx::tmem_dealloc(tmem_base, p.acc_bufs * p.acc_cols);
 }
 
 }  // namespace
@@ -343,6 +348,7 @@ kami_status_t tc16_xt_launch(int m, int n, int k, long long batch, bool bf16, co
   int cols = 64;
   while (cols < (E > per ? E : per) * pmax * m) cols <<= 1;
   p.acc_cols = cols;
+  p.acc_bufs = 512 / cols >= 4 ? 4 : 2;
   p.idesc = ptx::make_idesc_f16(bf16 ? 1 : 0, 128, m, /*a MN-major*/ 1, /*b K-major*/ 0);
   p.idesc2 = ptx::make_idesc_f16(bf16 ? 1 : 0, 128, 2 * m, 1, 0);
   const uint32_t smem = p.bar_off + 256 + 1024;
