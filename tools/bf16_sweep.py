@@ -3,7 +3,8 @@
     python tools/bf16_sweep.py [--orders 16,32,64,128,192,256] [--squares-only]
                                [--global-batch 1000000] [--gpus-share 8] [--out profiles/r1/bf16_sweep.json]
 
-Reading (R16/SURVEY 8(d)): uniform size per point, 10^6 entries per
+Timing: the reps launches are captured in one CUDA graph and replayed
+between two CUDA events (as bench.py).  Reading (R16/SURVEY 8(d)): uniform size per point, 10^6 entries per
 point globally, sharded over 8 B200 -> 125 000 entries per GPU; one GPU runs
 its shard (chunked when the shard does not fit the memory budget).  Each point
 reports TFLOP/s and the fraction of its HBM roofline (measured copy
@@ -54,16 +55,30 @@ def main():
         for _ in range(2):
             kami.gemm_strided_batched(m, n, k, chunk, "bf16", "row", A, B, C)
         torch.cuda.synchronize()
+        # the reps x (shard / chunk) launches are captured in one CUDA graph and
+        # replayed between two events, as bench.py times its steps: eager
+        # launches put the host's per-call work (planning, tensor-map encode)
+        # between kernels of a few tens of microseconds (r1/r2 sweeps before
+        # this change: 16^3 0.69 eager vs 0.83 in a graph)
+        n_launch = 0
+
+        def body():
+            nonlocal n_launch
+            for _ in range(a.reps):
+                done = 0
+                while done < shard:  # the shard is streamed through the resident chunk
+                    nb = min(chunk, shard - done)
+                    kami.gemm_strided_batched(m, n, k, nb, "bf16", "row", A, B, C)
+                    done += nb
+                    n_launch += 1
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):  # (the binding launches on torch's current = capture stream)
+            body()
+        g.replay()
+        torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        n_launch = 0
-        for _ in range(a.reps):
-            done = 0
-            while done < shard:  # the shard is streamed through the resident chunk
-                nb = min(chunk, shard - done)
-                kami.gemm_strided_batched(m, n, k, nb, "bf16", "row", A, B, C)
-                done += nb
-                n_launch += 1
+        g.replay()
         e1.record()
         torch.cuda.synchronize()
         t = e0.elapsed_time(e1) * 1e-3 / a.reps
