@@ -247,7 +247,12 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
   const uint16_t** a_tab = reinterpret_cast<const uint16_t**>(blk_tab + 128);
   const uint16_t** b_tab = a_tab + 8;
   uint16_t** c_tab = reinterpret_cast<uint16_t**>(const_cast<uint16_t**>(b_tab + 8));  // [2 warpgroups][8]
-  int* rp_tab = reinterpret_cast<int*>(c_tab + 16);  // SpMM: the unit's row_ptr values [G][mb + 1] (<= 32)
+  int* rp_tab = reinterpret_cast<int*>(c_tab + 16);  // (unused since the SpMM row pointers live in lanes)
+  // SpMM: the block table is double-buffered by unit parity (blk_tab, blk_tab2)
+  // and tagged with the unit, so it needs neither a reset nor a barrier before
+  // it is rebuilt: a buffer was last read two units ago, before every producer
+  // thread passed the previous unit's publish barrier
+  int* blk_tab2 = rp_tab + 32;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < p.stages; ++s) {
@@ -266,6 +271,9 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
     ptx::fence_mbar_init();
   }
   if (warp == 4) ptx::tmem_alloc(tmem_slot, p.acc_cols * p.acc_bufs);
+  // SpMM block tables: tag 0 (never written) -- shared memory keeps an earlier
+  // launch's tags otherwise
+  for (int i = threadIdx.x; i < 128; i += blockDim.x) blk_tab[i] = blk_tab2[i] = 0;
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
@@ -280,7 +288,8 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
     // several stages stream concurrently without register staging.
     const int tid = threadIdx.x;  // 0..127
     RingPos rs;
-    uint32_t it = 0;  // stages issued (trace index)
+    uint32_t it = 0;     // stages issued (trace index)
+    uint32_t nunit = 0;  // units issued (SpMM table buffer / tag)
     UnitIter ui(blockIdx.x, gridDim.x, p.mtiles);
     // The sizes and entry pointers of a unit are fetched TWO units ahead into
     // alternating register slots: their global-load latency (the pointer and
@@ -330,7 +339,8 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
           const int idx = tid + 128 * q;
           S.cb[q] = idx < S.U.ng * p.max_nnzb ? __ldg(p.colblk + S.U.e0 * (long long)p.max_nnzb + idx) : -1;
         }
-        if (tid < S.U.ng * rpn) S.rp = __ldg(p.rowptr + S.U.e0 * (long long)rpn + tid);
+        // every warp holds the unit's <= 32 row pointers in its lanes (shuffled below)
+        if ((tid & 31) < S.U.ng * rpn) S.rp = __ldg(p.rowptr + S.U.e0 * (long long)rpn + (tid & 31));
       }
       ui.next();
     };
@@ -384,18 +394,18 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
       if (one && !p.bsr && p.vmap) {
         ptx::named_bar_sync(3, 128);  // warp 0 has issued every earlier TMA unit (see above)
       }
-      if (!one) {
+      if (!one && !p.bsr) {
         ptx::named_bar_sync(3, 128);  // previous unit's items issued: tables reusable
         if (tid < U.ng) {
           a_tab[tid] = pa;
           b_tab[tid] = pb;
         }
-        if (p.bsr) {
-          blk_tab[tid] = -1;
-          if (tid < U.ng * rpn) rp_tab[tid] = rpv;
-        }
         ptx::named_bar_sync(3, 128);
       }
+      // SpMM table entry: tag << 11 | g << 8 | j (tag = unit + 1 mod 2^21; 0 = never written)
+      const uint32_t btag = ((nunit & 0x1FFFFFu) + 1u) << 11;
+      int* const bt = (nunit & 1u) ? blk_tab2 : blk_tab;
+      ++nunit;
       if (p.bsr) {
         // block lookup table of this tile: tile block row -> global block slot.
         // Slot idx = g max_nnzb + j of entry g lies in block row br with
@@ -405,12 +415,13 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
         for (int q = 0; q < 2; ++q) {
           const int idx = tid + 128 * q;
           const int col = q ? cb1 : cb0;
-          if (col < 0) continue;
           const int g = idx / p.max_nnzb, j = idx - g * p.max_nnzb;
-          const int* rpg = rp_tab + g * rpn;
+          // row pointers of entry g from the lanes (every lane shuffles, valid or not)
+          const int gl = (col >= 0 && g < U.ng) ? g * rpn : 0;
           int br;
           if (p.zorder) {  // (row, column) from the Morton code: odd bits row, even bits column
-            if (j >= rpg[0]) continue;  // past the entry's nnzb
+            const int cnt = __shfl_sync(0xffffffffu, rpv, gl);
+            if (col < 0 || j >= cnt) continue;  // past the entry's nnzb
             const uint32_t z = (uint32_t)col;
             uint32_t r = 0, c = 0;
 #pragma unroll
@@ -420,18 +431,22 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
             }
             br = (int)r;
             if (br < br0 || br >= br1) continue;
-            blk_tab[(g * mbk + br - br0) * 16 + (int)c] = (int)((U.e0 + g) * p.max_nnzb + j);
+            bt[(g * mbk + br - br0) * 16 + (int)c] = (int)(btag | ((uint32_t)g << 8) | (uint32_t)j);  // g < 8, j < 256
             continue;
           }
-          if (j >= rpg[mbk]) continue;  // unused tail slot
+          const int last = __shfl_sync(0xffffffffu, rpv, gl + mbk);
           // block row of slot j: the last br with rp[br] <= j (binary search
-          // over the <= 17 row pointers: 5 dependent shared loads, not <= 16)
+          // over the <= 17 row pointers, shuffled from the lanes)
           br = 0;
 #pragma unroll
-          for (int step = 8; step > 0; step >>= 1)
-            if (br + step <= mbk - 1 && rpg[br + step] <= j) br += step;
+          for (int step = 8; step > 0; step >>= 1) {
+            const int cand = br + step;
+            const int v = __shfl_sync(0xffffffffu, rpv, gl + min(cand, mbk - 1));
+            if (cand <= mbk - 1 && v <= j) br = cand;
+          }
+          if (col < 0 || j >= last) continue;  // unused tail slot
           if (br < br0 || br >= br1) continue;
-          blk_tab[(g * mbk + br - br0) * 16 + col] = (int)((U.e0 + g) * p.max_nnzb + j);
+          bt[(g * mbk + br - br0) * 16 + col] = (int)(btag | ((uint32_t)g << 8) | (uint32_t)j);
         }
         ptx::named_bar_sync(3, 128);
       }
@@ -475,9 +490,10 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
           const int nib = rows >> 4, nks = kpad_c >> 4;
           const int slot = tid >> 2, part = tid & 3, ib = slot >> 2, ks = slot & 3;
           if (ib < nib && ks < nks) {
-            const int idx = blk_tab[ib * 16 + kc * 4 + ks];
+            const int v = bt[ib * 16 + kc * 4 + ks];
             const uint32_t off = s * p.stage_bytes + (uint32_t)ks * 4096u + (uint32_t)ib * 512u;
-            if (idx >= 0) {
+            if (((uint32_t)v & 0xFFFFF800u) == btag) {  // present in this unit's table
+              const int idx = (int)((U.e0 + ((v >> 8) & 0x7)) * p.max_nnzb + (v & 0xFF));
               if (part == 0) {
                 ptx::mbar_expect_tx(&full[s], 512u);
                 ptx::tma_load_3d(smem + off, &p.tmA, &full[s], 0, 0, idx);
