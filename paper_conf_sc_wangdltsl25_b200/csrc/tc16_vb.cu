@@ -807,6 +807,37 @@ __global__ void __launch_bounds__(kVbThreads, 1) kami_tc16_vb_kernel
         const int cpr = hw / 8;
         const int cpr_shift = (cpr & (cpr - 1)) == 0 ? __ffs(cpr) - 1 : -1;
         const uint32_t inv_m = (65536u + m - 1) / m;  // r / m == (r inv_m) >> 16 for r < 256
+        if (cpr_shift >= 0 && !(p.dbg & 1)) {
+          // power-of-two chunks per row (hw = 8 .. 128): this thread's chunk
+          // column is fixed and its rows step by 128 / cpr, so shared and
+          // global addresses advance by constants -- ~4 instructions per 16
+          // bytes instead of ~12 (the general loop below bound the
+          // write-heavy classes, ncu r2)
+          const int c = L & (cpr - 1), rstep = 128 >> cpr_shift;
+          int r = L >> cpr_shift;
+          uint32_t sa = cst + (uint32_t)r * kCRow + (uint32_t)c * 16u;
+          const uint32_t sstep = (uint32_t)rstep * kCRow;
+          if (G == 1) {
+            uint16_t* ga = c_tab[wg * 8] + (long long)(U.mt * 128 + r) * n + h0 + c * 8;
+            const long long gstep = (long long)rstep * n;
+#pragma unroll 4
+            for (; r < rows; r += rstep, sa += sstep, ga += gstep) {
+              uint32_t x0, x1, x2, x3;
+              ptx::ld_shared_v4(sa, x0, x1, x2, x3);
+              ptx::st_global_v4(ga, make_uint4(x0, x1, x2, x3));
+            }
+          } else {
+#pragma unroll 2
+            for (; r < rows; r += rstep, sa += sstep) {
+              const int ge = (int)(((uint32_t)r * inv_m) >> 16), er = r - ge * m;
+              uint32_t x0, x1, x2, x3;
+              ptx::ld_shared_v4(sa, x0, x1, x2, x3);
+              ptx::st_global_v4(c_tab[wg * 8 + ge] + (long long)er * n + h0 + c * 8, make_uint4(x0, x1, x2, x3));
+            }
+          }
+          ptx::named_bar_sync(1 + wg, 128);  // staging buffer reusable
+          continue;
+        }
         for (int i = L; i < rows * cpr; i += 128) {
           const int r = cpr_shift >= 0 ? i >> cpr_shift : i / cpr, c = i - r * cpr;
           const int ge = G > 1 ? (int)(((uint32_t)r * inv_m) >> 16) : 0;

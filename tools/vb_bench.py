@@ -28,6 +28,9 @@ ap.add_argument("--reps", type=int, default=10)
 ap.add_argument("--density", type=float, default=0.5)
 ap.add_argument("--orders", default="16,32,64,128,192,256", help="vb mode: the order set")
 ap.add_argument("--nmax", type=int, default=256, help="vb mode: max_n passed to the call")
+ap.add_argument("--morders", default="", help="vb mode: m's own order set (default --orders)")
+ap.add_argument("--norders", default="", help="vb mode: n's own order set")
+ap.add_argument("--korders", default="", help="vb mode: k's own order set")
 ap.add_argument("--algo", default="auto", help="zmorton mode: auto / 1d / 2d")
 ap.add_argument("--sortalloc", action="store_true", help="vb mode: entries allocated in (m, n, k) class order")
 ap.add_argument("--noperm", action="store_true", help="ptr mode: pointers in entry order (no scatter)")
@@ -89,6 +92,9 @@ else:
     rng = np.random.default_rng(0)
     orders = np.array([int(x) for x in a.orders.split(",")])
     sz = rng.choice(orders, size=(a.batch, 3))
+    for i, o in enumerate((a.morders, a.norders, a.korders)):
+        if o:
+            sz[:, i] = rng.choice(np.array([int(x) for x in o.split(",")]), size=a.batch)
     if a.sortalloc:  # memory order = the kernel's class-sorted unit order (address locality experiment)
         sz = sz[np.lexsort((sz[:, 2], sz[:, 1], sz[:, 0]))]
     mm, nn, kk = sz[:, 0], sz[:, 1], sz[:, 2]
