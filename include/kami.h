@@ -138,9 +138,12 @@ kami_status_t kami_gemm_batched(int m, int n, int k, int64_t batch, kami_dtype_t
  * 16-byte aligned, packed matrices in `layout`).  max_m/max_n/max_k are host
  * upper bounds used for planning and validated against the size grid; every
  * entry must itself be on the grid (16-bit: m, n multiples of 16 <= 256, k a
- * multiple of 8 <= 256) -- entries off the grid are undefined behaviour (the
- * sizes live on the device and are not read by the host).  16-bit types only
- * (FP64 returns KAMI_ERROR_NOT_SUPPORTED). */
+ * multiple of 8 <= 256; FP64: m, n, k multiples of 8 <= 256) and within the
+ * max bounds -- entries off the grid are undefined behaviour for 16-bit and
+ * skipped (C untouched) for FP64 (the sizes live on the device and are not
+ * read by the host).  FP16 / BF16 run the class-sorted tcgen05 kernel, FP64
+ * the k-sliced DMMA kernel with per-entry sizes; TF32 / FP8 return
+ * KAMI_ERROR_NOT_SUPPORTED. */
 kami_status_t kami_gemm_vbatched(int64_t batch, const int* m_array, const int* n_array, const int* k_array,
                                  int max_m, int max_n, int max_k, kami_dtype_t dtype, kami_layout_t layout,
                                  const void* const* A_array, const void* const* B_array, void* const* C_array,

@@ -247,13 +247,17 @@ kami_status_t kami_gemm_vbatched(int64_t batch, const int* m_array, const int* n
                                  kami_stream_t stream) {
   kami_status_t st = check_common(max_m, max_n, max_k, batch, dtype, layout, KAMI_ALGO_AUTO);
   if (st != KAMI_SUCCESS) return st;
-  if (!is16(dtype)) return KAMI_ERROR_NOT_SUPPORTED;
+  if (!is16(dtype) && dtype != KAMI_DTYPE_F64) return KAMI_ERROR_NOT_SUPPORTED;
   if (batch == 0) return KAMI_SUCCESS;
   if (!m_array || !n_array || !k_array || !A_array || !B_array || !C_array) return KAMI_ERROR_INVALID_VALUE;
   if (!aligned16(A_array) || !aligned16(B_array) || !aligned16(C_array)) return KAMI_ERROR_MISALIGNED;
   if (batch > (int64_t)INT32_MAX) return KAMI_ERROR_NOT_SUPPORTED;
   // column-major: C^T = B^T A^T per entry -> swap m<->n and A<->B
   const bool col = layout == KAMI_COL_MAJOR;
+  if (dtype == KAMI_DTYPE_F64)  // the k-sliced DMMA kernel with per-entry sizes
+    return dmma_gen_vb_launch(batch, col ? n_array : m_array, col ? m_array : n_array, k_array, col ? max_n : max_m,
+                              col ? max_m : max_n, max_k, col ? B_array : A_array, col ? A_array : B_array, C_array,
+                              reinterpret_cast<cudaStream_t>(stream));
   return tc16_vb_launch(batch, dtype == KAMI_DTYPE_BF16, 0, 0, 0, col ? n_array : m_array, col ? m_array : n_array,
                         k_array, col ? max_n : max_m, col ? max_m : max_n, col ? B_array : A_array,
                         col ? A_array : B_array, C_array, reinterpret_cast<cudaStream_t>(stream));

@@ -71,7 +71,47 @@ struct DmmaGenParams {
   const double* const* Aa;
   const double* const* Ba;
   double* const* Ca;
+  // variable sizes (kami_gemm_vbatched; pointer arrays): per-entry m, n, k in
+  // device arrays, units enumerated as (entry, 64-column block < max n); a
+  // unit past its entry's n, or an entry off the FP64 grid, is skipped
+  const int* dm;
+  const int* dn;
+  const int* dk;
 };
+
+// an entry's sizes and the quantities the kernel derives from them
+struct GenDims {
+  int m, n, k, ks, rs, mblocks, ce_shift;
+  uint32_t swz_bits;
+};
+__device__ __forceinline__ GenDims gen_dims(const DmmaGenParams& p, long long e) {
+  GenDims d;
+  if (p.dm) {
+    d.m = __ldg(p.dm + e);
+    d.n = __ldg(p.dn + e);
+    d.k = __ldg(p.dk + e);
+    d.ks = d.k / 4;
+    d.rs = d.ks < p.rs ? d.ks : p.rs;  // the plan's resident count is for the largest k
+    d.ce_shift = (d.k % 16 == 0) ? 4 : 3;
+  } else {
+    d.m = p.m;
+    d.n = p.n;
+    d.k = p.k;
+    d.ks = p.ks;
+    d.rs = p.rs;
+    d.ce_shift = p.ce_shift;
+  }
+  d.mblocks = (d.m + kGTM - 1) / kGTM;
+  d.swz_bits = d.ce_shift == 4 ? 3u : 2u;
+  return d;
+}
+// a unit with work: its 64-column block inside the entry's n, the entry on the grid
+__device__ __forceinline__ bool gen_live(const DmmaGenParams& p, const GenDims& d, int nb) {
+  if (!p.dm) return true;
+  const bool grid = d.m >= 8 && d.n >= 8 && d.k >= 8 && d.m <= 256 && d.n <= 256 && d.k <= 256 &&
+                    d.m % 8 == 0 && d.n % 8 == 0 && d.k % 8 == 0 && d.k <= p.k && d.n <= p.n && d.m <= p.m;
+  return grid && nb * kGNB < d.n;
+}
 
 template <int RK, bool kPtr>
 __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
@@ -101,21 +141,21 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   const uint32_t park = ptx::smem_u32(tbase + p.nbuf * p.a_block_bytes + w * p.park_bytes);
   // the team's block sequence: units u = first, first + nteams, ...; m-blocks 0.. of each
   const int tid = w * 32 + lane;  // 0..127 within the team
-  auto issue = [&](long long u, int mb, int s) {
+  auto issue = [&](long long u, int mb, int s, const GenDims& d) {
     const long long e = u / p.nblocks;
     if constexpr (kPtr) {  // every thread of the team: 16-byte chunks of the 32 x k block
       const double* Ae = p.Aa[e];
       const uint32_t dst0 = ptx::smem_u32(tbase + s * p.a_block_bytes);
-      const int cpr = p.k >> 1;  // 16-byte chunks per row
-      const uint32_t rowb = 8u << p.ce_shift;
+      const int cpr = d.k >> 1;  // 16-byte chunks per row
+      const uint32_t rowb = 8u << d.ce_shift;
       for (int i = tid; i < kGTM * cpr; i += kGP * 32) {
         const int r = i / cpr, c = i - r * cpr;  // row, chunk (two doubles)
         const int col = 2 * c;
         const int row = mb * kGTM + r;
-        const uint32_t off = (uint32_t)(col >> p.ce_shift) * (kGTM * rowb) +
-                             ptx::swz((uint32_t)r * rowb + (uint32_t)(col & ((1 << p.ce_shift) - 1)) * 8, p.swz_bits);
-        const bool ok = row < p.m;
-        ptx::cp_async_16(dst0 + off, ok ? Ae + (long long)row * p.k + col : Ae, ok ? 16u : 0u);
+        const uint32_t off = (uint32_t)(col >> d.ce_shift) * (kGTM * rowb) +
+                             ptx::swz((uint32_t)r * rowb + (uint32_t)(col & ((1 << d.ce_shift) - 1)) * 8, d.swz_bits);
+        const bool ok = row < d.m;
+        ptx::cp_async_16(dst0 + off, ok ? Ae + (long long)row * d.k + col : Ae, ok ? 16u : 0u);
       }
       ptx::cp_async_mbar_arrive_noinc(&full[s]);
     } else {
@@ -123,16 +163,31 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
       ptx::tma_load_4d(tbase + s * p.a_block_bytes, &p.tmA, &full[s], 0, mb * kGTM, 0, (int)e);
     }
   };
-  // prologue: the first nbuf blocks
+  // the producer's cursor (pu, pmb) walks the live units' A blocks nbuf ahead
+  // of the consumer; pd = the sizes of pu's entry
   long long pu = first;
   int pmb = 0;
+  GenDims pd{};
+  auto skip_dead = [&]() {
+    for (; pu < p.units; pu += nteams) {
+      const long long e = pu / p.nblocks;
+      pd = gen_dims(p, e);
+      if (gen_live(p, pd, (int)(pu - e * p.nblocks))) break;
+    }
+  };
+  auto advance = [&]() {
+    if (++pmb == pd.mblocks) {
+      pmb = 0;
+      pu += nteams;
+      skip_dead();
+    }
+  };
+  // prologue: the first nbuf blocks
+  skip_dead();
   if (issuer || kPtr) {
     for (int s = 0; s < p.nbuf && pu < p.units; ++s) {
-      issue(pu, pmb, s);
-      if (++pmb == p.mblocks) {
-        pmb = 0;
-        pu += nteams;
-      }
+      issue(pu, pmb, s, pd);
+      advance();
     }
   }
   double b[RK][kGFN];
@@ -140,32 +195,35 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   for (long long u = first; u < p.units; u += nteams) {
     const long long e = u / p.nblocks;
     const int nb = (int)(u - e * p.nblocks);
-    if (issuer && p.nblocks == 1 && u + nteams < p.units) {  // the next unit's B into L2 while this one computes
+    const GenDims d = gen_dims(p, e);
+    if (!gen_live(p, d, nb)) continue;  // (the producer cursor skips it too)
+    if (issuer && !p.dm && p.nblocks == 1 && u + nteams < p.units) {  // the next unit's B into L2 while this one computes
       const long long en = (u + nteams) / p.nblocks;
       ptx::prefetch_l2_bulk(kPtr ? p.Ba[en] : p.B + en * (long long)p.k * p.n, (uint32_t)(p.k * p.n * 8));
     }
     const int col0 = nb * kGNB + w * (kGFN * 8);
     const double* Bg = kPtr ? p.Ba[e] : p.B + e * (long long)p.k * p.n;
+    const int n_e = d.n, ks_e = d.ks, rs_e = d.rs, ce_e = d.ce_shift;
     // GMem2Reg: the resident k-steps of B_w; the parked ones go to this warp's slab
 #pragma unroll
     for (int kk = 0; kk < RK; ++kk)
 #pragma unroll
       for (int j = 0; j < kGFN; ++j) {
         const int col = col0 + j * 8 + g;
-        b[kk][j] = (kk < p.rs && col0 + j * 8 < p.n) ? __ldg(Bg + kcol(kk, t, p.ce_shift) * (long long)p.n + col)
+        b[kk][j] = (kk < rs_e && col0 + j * 8 < n_e) ? __ldg(Bg + kcol(kk, t, ce_e) * (long long)n_e + col)
                                                       : 0.0;
       }
-    for (int kk = p.rs; kk < p.ks; ++kk)
+    for (int kk = rs_e; kk < ks_e; ++kk)
 #pragma unroll
       for (int j = 0; j < kGFN; ++j) {
         const int col = col0 + j * 8 + g;
-        const double v = col0 + j * 8 < p.n ? __ldg(Bg + kcol(kk, t, p.ce_shift) * (long long)p.n + col) : 0.0;
-        asm volatile("st.shared.f64 [%0], %1;" ::"r"(park + (uint32_t)(((kk - p.rs) * kGFN + j) * 32 + lane) * 8),
+        const double v = col0 + j * 8 < n_e ? __ldg(Bg + kcol(kk, t, ce_e) * (long long)n_e + col) : 0.0;
+        asm volatile("st.shared.f64 [%0], %1;" ::"r"(park + (uint32_t)(((kk - rs_e) * kGFN + j) * 32 + lane) * 8),
                      "d"(v)
                      : "memory");
       }
     __syncwarp();
-    for (int mb = 0; mb < p.mblocks; ++mb, ab.next(p.nbuf)) {
+    for (int mb = 0; mb < d.mblocks; ++mb, ab.next(p.nbuf)) {
       const uint32_t s = ab.s;
       double c[kGFM][kGFN][2];
 #pragma unroll
@@ -174,18 +232,18 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
         for (int j = 0; j < kGFN; ++j) c[i][j][0] = c[i][j][1] = 0.0;
       ptx::mbar_wait(&full[s], ab.ph);
       const uint32_t a_s = ptx::smem_u32(tbase + s * p.a_block_bytes);
-      const uint32_t rowb = 8u << p.ce_shift;  // bytes of one swizzled row of a chunk
+      const uint32_t rowb = 8u << ce_e;  // bytes of one swizzled row of a chunk
       auto step = [&](int kk, const double (&bb)[kGFN]) {
-        const int col = kcol(kk, t, p.ce_shift);
-        const uint32_t chunk_off = (uint32_t)(col >> p.ce_shift) * (kGTM * rowb);
-        const uint32_t in_row = (uint32_t)(col & ((1 << p.ce_shift) - 1)) * 8;
+        const int col = kcol(kk, t, ce_e);
+        const uint32_t chunk_off = (uint32_t)(col >> ce_e) * (kGTM * rowb);
+        const uint32_t in_row = (uint32_t)(col & ((1 << ce_e) - 1)) * 8;
 #pragma unroll
         for (int i = 0; i < kGFM; ++i) {
           const int row = i * 8 + g;
           double a;
           asm volatile("ld.shared.f64 %0, [%1];"
                        : "=d"(a)
-                       : "r"(a_s + chunk_off + ptx::swz(row * rowb + in_row, p.swz_bits)));
+                       : "r"(a_s + chunk_off + ptx::swz(row * rowb + in_row, d.swz_bits)));
 #pragma unroll
           for (int j = 0; j < kGFN; ++j)
             asm volatile("mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0,%1}, {%2}, {%3}, {%0,%1};"
@@ -196,16 +254,16 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
       // resident k-steps: B fragments from registers
 #pragma unroll
       for (int kk = 0; kk < RK; ++kk)
-        if (kk < p.rs) step(kk, b[kk]);
+        if (kk < rs_e) step(kk, b[kk]);
       // parked k-steps: B fragments from the warp's slab (one LDS.64 per fragment)
 #pragma unroll 4
-      for (int kk = p.rs; kk < p.ks; ++kk) {
+      for (int kk = rs_e; kk < ks_e; ++kk) {
         double bb[kGFN];
 #pragma unroll
         for (int j = 0; j < kGFN; ++j)
           asm volatile("ld.shared.f64 %0, [%1];"
                        : "=d"(bb[j])
-                       : "r"(park + (uint32_t)(((kk - p.rs) * kGFN + j) * 32 + lane) * 8));
+                       : "r"(park + (uint32_t)(((kk - rs_e) * kGFN + j) * 32 + lane) * 8));
         step(kk, bb);
       }
       // Reg2GMem: C_w block; lane holds (row g, cols 2t, 2t+1) of each 8x8 fragment
@@ -215,16 +273,13 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
         const int row = mb * kGTM + i * 8 + g;
 #pragma unroll
         for (int j = 0; j < kGFN; ++j)
-          if (row < p.m && col0 + j * 8 < p.n)
-            ptx::st_global_v2_f64(Cg + (long long)row * p.n + col0 + j * 8 + 2 * t, c[i][j][0], c[i][j][1]);
+          if (row < d.m && col0 + j * 8 < n_e)
+            ptx::st_global_v2_f64(Cg + (long long)row * n_e + col0 + j * 8 + 2 * t, c[i][j][0], c[i][j][1]);
       }
       ptx::named_bar_sync(bar, kGP * 32);  // every warp finished reading buffer s
       if ((issuer || kPtr) && pu < p.units) {  // refill it with the block nbuf ahead
-        issue(pu, pmb, s);
-        if (++pmb == p.mblocks) {
-          pmb = 0;
-          pu += nteams;
-        }
+        issue(pu, pmb, s, pd);
+        advance();
       }
     }
   }
@@ -336,6 +391,53 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
   fn<<<(unsigned)grid, kGP * 32 * (gp.rk == kRK ? 2 : 4), smem, stream>>>(p);
   set_last_kernel(ptr ? "kami_dmma_gen_1d<ptr>" : "kami_dmma_gen_1d");
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
+}
+
+// Variable sizes (kami_gemm_vbatched, FP64; "supports various
+// matrix orders in a batch"): the pointer-array kernel with per-entry m, n, k
+// read on the device, planned for the largest (max_m, max_n, max_k).
+kami_status_t dmma_gen_vb_launch(long long batch, const int* dm, const int* dn, const int* dk, int max_m, int max_n,
+                                 int max_k, const void* const* Aa, const void* const* Ba, void* const* Ca,
+                                 cudaStream_t stream) {
+  if (!dmma_gen_supported(max_m, max_n, max_k)) return KAMI_ERROR_NOT_SUPPORTED;
+  if (!dm || !dn || !dk || !Aa || !Ba || !Ca) return KAMI_ERROR_INVALID_VALUE;
+  DmmaGenParams p;
+  memset(&p, 0, sizeof(p));
+  p.Aa = reinterpret_cast<const double* const*>(Aa);
+  p.Ba = reinterpret_cast<const double* const*>(Ba);
+  p.Ca = reinterpret_cast<double* const*>(Ca);
+  p.dm = dm;
+  p.dn = dn;
+  p.dk = dk;
+  p.batch = batch;
+  p.m = max_m;
+  p.n = max_n;
+  p.k = max_k;
+  p.ks = max_k / 4;
+  const GenPlan gp = gen_plan(max_m, max_n, max_k);
+  if (gp.smem > (uint32_t)kGenSmem) return KAMI_ERROR_NOT_SUPPORTED;
+  p.rs = gp.rs;
+  p.nblocks = (max_n + kGNB - 1) / kGNB;
+  p.mblocks = (max_m + kGTM - 1) / kGTM;
+  p.ce_shift = gp.ce_shift;
+  p.swz_bits = gp.ce_shift == 4 ? 3 : 2;
+  p.units = batch * p.nblocks;
+  p.a_block_bytes = gp.a_block_bytes;
+  p.park_bytes = gp.park_bytes;
+  p.teams = gp.teams;
+  p.nbuf = gp.nbuf;
+  auto fn = gp.rk == kRK ? kami_dmma_gen_kernel<kRK, true> : kami_dmma_gen_kernel<kRKSmall, true>;
+  if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)gp.smem) != cudaSuccess)
+    return KAMI_ERROR_CUDA;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const long long need = (p.units + p.teams - 1) / p.teams;
+  long long grid = sms < need ? sms : need;
+  grid = apply_grid_cap(grid);
+  fn<<<(unsigned)grid, kGP * 32 * (gp.rk == kRK ? 2 : 4), gp.smem, stream>>>(p);
+  set_last_kernel("kami_dmma_gen_1d<vbatched>");
+  return (kami_status_t)launch_status((int)cudaGetLastError());
 }
 
 }  // namespace kami

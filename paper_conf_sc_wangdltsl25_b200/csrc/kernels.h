@@ -107,6 +107,11 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
                               cudaStream_t stream, const void* const* Aa = nullptr, const void* const* Ba = nullptr,
                               void* const* Ca = nullptr);
 
+// FP64 variable sizes: the pointer-array dmma_gen kernel with per-entry sizes (device arrays)
+kami_status_t dmma_gen_vb_launch(long long batch, const int* dm, const int* dn, const int* dk, int max_m, int max_n,
+                                 int max_k, const void* const* Aa, const void* const* Ba, void* const* Ca,
+                                 cudaStream_t stream);
+
 // ------------------------- 16-bit pointer-array / variable-size (tc16_vb.cu)
 // dm/dn/dk: device arrays of per-entry sizes, or nullptr for uniform m, n, k.
 kami_status_t tc16_vb_launch(long long batch, bool bf16, int m, int n, int k, const int* dm, const int* dn,

@@ -160,7 +160,7 @@ def test_vbatched_rejects():
     with pytest.raises(kami.KamiError):
         kami.gemm_vbatched(4, 16, 16, 16, 300, 16, 16, "f16", "row", 16, 16, 16)  # max_m off the grid
     with pytest.raises(kami.KamiError):
-        kami.gemm_vbatched(4, 16, 16, 16, 64, 64, 64, "f64", "row", 16, 16, 16)  # fp64 not supported
+        kami.gemm_vbatched(4, 16, 16, 16, 64, 64, 64, "tf32", "row", 16, 16, 16)  # tf32: no variable-size path
 
 
 @pytest.mark.gpu
@@ -279,3 +279,38 @@ def test_vbatched_sorted_many_classes(dtype, monkeypatch):
             if not oracle.normalised_error(got.reshape(1, m, n), Cref, S) <= _tol(dtype, k):
                 bad.append((name, e, m, n, k))
     assert not bad and not diff, (bad[:20], [(e,) + sizes[e] for e in diff[:20]], len(diff))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("layout", ["row", "col"])
+@pytest.mark.parametrize("cap", [0, 3])
+def test_vbatched_f64_mixed_orders(layout, cap):
+    """FP64 variable sizes on the k-sliced DMMA kernel with
+    per-entry sizes: every entry against the oracle (FP64 bound), entries of
+    the whole FP64 grid (non-square, k not a multiple of 16, n past one
+    64-column block, m past one 32-row block), with and without a grid cap
+    (steady state: every team walks many units and skips dead ones)."""
+    rng = np.random.default_rng(21)
+    orders = [8, 16, 24, 40, 64, 72, 128, 136, 200, 256]
+    batch = 37
+    sizes = [(int(rng.choice(orders)), int(rng.choice(orders)), int(rng.choice(orders))) for _ in range(batch)]
+    sizes[0] = (256, 256, 256)
+    sizes[1] = (8, 8, 8)
+    bufs = []
+    for e, (m, n, k) in enumerate(sizes):
+        A, B = ki.operands(m, n, k, 1, "f64", "unif", seed=23, entry0=e)
+        bufs.append((A, B, A.cuda(), B.cuda(), torch.full((m * n,), float("nan"), dtype=torch.float64, device="cuda")))
+    dm = torch.tensor([s[0] for s in sizes], dtype=torch.int32, device="cuda")
+    dn = torch.tensor([s[1] for s in sizes], dtype=torch.int32, device="cuda")
+    dk = torch.tensor([s[2] for s in sizes], dtype=torch.int32, device="cuda")
+    pa = torch.tensor([b[2].data_ptr() for b in bufs], dtype=torch.int64, device="cuda")
+    pb = torch.tensor([b[3].data_ptr() for b in bufs], dtype=torch.int64, device="cuda")
+    pc = torch.tensor([b[4].data_ptr() for b in bufs], dtype=torch.int64, device="cuda")
+    with kami.grid_cap(cap):
+        kami.gemm_vbatched(batch, dm, dn, dk, 256, 256, 256, "f64", layout, pa, pb, pc)
+    torch.cuda.synchronize()
+    assert kami.last_kernel().startswith("kami_dmma_gen"), kami.last_kernel()
+    for (m, n, k), (A, B, _, _, C) in zip(sizes, bufs):
+        Cref, S = oracle.gemm(m, n, k, 1, "f64", layout, ki.as_bits(A), ki.as_bits(B), with_scale=True)
+        got = oracle.decode(oracle.to_row_major(ki.as_bits(C.cpu()), 1, m, n, layout).reshape(-1), "f64")
+        assert oracle.normalised_error(got.reshape(1, m, n), Cref, S) <= k * 2.0 ** -52, (m, n, k)

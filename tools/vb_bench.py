@@ -98,11 +98,12 @@ else:
     if a.sortalloc:  # memory order = the kernel's class-sorted unit order (address locality experiment)
         sz = sz[np.lexsort((sz[:, 2], sz[:, 1], sz[:, 0]))]
     mm, nn, kk = sz[:, 0], sz[:, 1], sz[:, 2]
-    es = 2
+    es = 8 if a.dtype == "f64" else 2
     offA = np.concatenate([[0], np.cumsum(mm * kk)])
     offB = np.concatenate([[0], np.cumsum(kk * nn)])
     offC = np.concatenate([[0], np.cumsum(mm * nn)])
-    A = torch.empty(int(offA[-1]), dtype=torch.bfloat16 if a.dtype == "bf16" else torch.float16, device="cuda")
+    A = torch.empty(int(offA[-1]), dtype={"bf16": torch.bfloat16, "f64": torch.float64}.get(a.dtype, torch.float16),
+                    device="cuda")
     B = torch.empty(int(offB[-1]), dtype=A.dtype, device="cuda")
     A.uniform_(-1, 1)
     B.uniform_(-1, 1)
