@@ -77,6 +77,11 @@ struct DmmaGenParams {
   const int* dm;
   const int* dn;
   const int* dk;
+  // unit records written by a pre-pass (gen_vb_units): {entry, 64-column
+  // block, m | n << 16, k} of every live unit, *count of them -- no dead
+  // units to walk and one load per unit
+  const int4* recs;
+  const int* count;
 };
 
 // an entry's sizes and the quantities the kernel derives from them
@@ -84,15 +89,18 @@ struct GenDims {
   int m, n, k, ks, rs, mblocks, ce_shift;
   uint32_t swz_bits;
 };
+__device__ __forceinline__ void gen_derive(const DmmaGenParams& p, GenDims& d) {
+  d.ks = d.k / 4;
+  d.rs = d.ks < p.rs ? d.ks : p.rs;  // the plan's resident count is for the largest k
+  d.ce_shift = (d.k % 16 == 0) ? 4 : 3;
+}
 __device__ __forceinline__ GenDims gen_dims(const DmmaGenParams& p, long long e) {
   GenDims d;
   if (p.dm) {
     d.m = __ldg(p.dm + e);
     d.n = __ldg(p.dn + e);
     d.k = __ldg(p.dk + e);
-    d.ks = d.k / 4;
-    d.rs = d.ks < p.rs ? d.ks : p.rs;  // the plan's resident count is for the largest k
-    d.ce_shift = (d.k % 16 == 0) ? 4 : 3;
+    gen_derive(p, d);
   } else {
     d.m = p.m;
     d.n = p.n;
@@ -106,6 +114,35 @@ __device__ __forceinline__ GenDims gen_dims(const DmmaGenParams& p, long long e)
   return d;
 }
 // a unit with work: its 64-column block inside the entry's n, the entry on the grid
+__device__ __forceinline__ bool gen_live(const DmmaGenParams& p, const GenDims& d, int nb);
+// unit u -> entry, column block, sizes, live
+struct GenUnit {
+  long long e;
+  int nb;
+  GenDims d;
+  bool live;
+};
+__device__ __forceinline__ GenUnit gen_unit(const DmmaGenParams& p, long long u) {
+  GenUnit r;
+  if (p.recs) {
+    const int4 q = __ldg(p.recs + u);
+    r.e = q.x;
+    r.nb = q.y;
+    r.d.m = q.z & 0xFFFF;
+    r.d.n = q.z >> 16;
+    r.d.k = q.w;
+    gen_derive(p, r.d);
+    r.d.mblocks = (r.d.m + kGTM - 1) / kGTM;
+    r.d.swz_bits = r.d.ce_shift == 4 ? 3u : 2u;
+    r.live = true;
+  } else {
+    r.e = u / p.nblocks;
+    r.nb = (int)(u - r.e * p.nblocks);
+    r.d = gen_dims(p, r.e);
+    r.live = gen_live(p, r.d, r.nb);
+  }
+  return r;
+}
 __device__ __forceinline__ bool gen_live(const DmmaGenParams& p, const GenDims& d, int nb) {
   if (!p.dm) return true;
   const bool grid = d.m >= 8 && d.n >= 8 && d.k >= 8 && d.m <= 256 && d.n <= 256 && d.k <= 256 &&
@@ -134,6 +171,7 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   }
   __syncthreads();
   if (team >= p.teams) return;
+  const long long units = p.recs ? (long long)*p.count : p.units;
   const long long nteams = (long long)gridDim.x * p.teams;
   const long long first = (long long)blockIdx.x * p.teams + team;
   const bool issuer = (w == 0 && lane == 0);
@@ -141,8 +179,7 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   const uint32_t park = ptx::smem_u32(tbase + p.nbuf * p.a_block_bytes + w * p.park_bytes);
   // the team's block sequence: units u = first, first + nteams, ...; m-blocks 0.. of each
   const int tid = w * 32 + lane;  // 0..127 within the team
-  auto issue = [&](long long u, int mb, int s, const GenDims& d) {
-    const long long e = u / p.nblocks;
+  auto issue = [&](long long e, int mb, int s, const GenDims& d) {
     if constexpr (kPtr) {  // every thread of the team: 16-byte chunks of the 32 x k block
       const double* Ae = p.Aa[e];
       const uint32_t dst0 = ptx::smem_u32(tbase + s * p.a_block_bytes);
@@ -167,16 +204,15 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   // of the consumer; pd = the sizes of pu's entry
   long long pu = first;
   int pmb = 0;
-  GenDims pd{};
+  GenUnit pd{};
   auto skip_dead = [&]() {
-    for (; pu < p.units; pu += nteams) {
-      const long long e = pu / p.nblocks;
-      pd = gen_dims(p, e);
-      if (gen_live(p, pd, (int)(pu - e * p.nblocks))) break;
+    for (; pu < units; pu += nteams) {
+      pd = gen_unit(p, pu);
+      if (pd.live) break;
     }
   };
   auto advance = [&]() {
-    if (++pmb == pd.mblocks) {
+    if (++pmb == pd.d.mblocks) {
       pmb = 0;
       pu += nteams;
       skip_dead();
@@ -185,19 +221,20 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   // prologue: the first nbuf blocks
   skip_dead();
   if (issuer || kPtr) {
-    for (int s = 0; s < p.nbuf && pu < p.units; ++s) {
-      issue(pu, pmb, s, pd);
+    for (int s = 0; s < p.nbuf && pu < units; ++s) {
+      issue(pd.e, pmb, s, pd.d);
       advance();
     }
   }
   double b[RK][kGFN];
   RingPos ab;  // A buffer ring (slot, parity)
-  for (long long u = first; u < p.units; u += nteams) {
-    const long long e = u / p.nblocks;
-    const int nb = (int)(u - e * p.nblocks);
-    const GenDims d = gen_dims(p, e);
-    if (!gen_live(p, d, nb)) continue;  // (the producer cursor skips it too)
-    if (issuer && !p.dm && p.nblocks == 1 && u + nteams < p.units) {  // the next unit's B into L2 while this one computes
+  for (long long u = first; u < units; u += nteams) {
+    const GenUnit gu = gen_unit(p, u);
+    if (!gu.live) continue;  // (the producer cursor skips it too)
+    const long long e = gu.e;
+    const int nb = gu.nb;
+    const GenDims d = gu.d;
+    if (issuer && !p.dm && p.nblocks == 1 && u + nteams < units) {  // the next unit's B into L2 while this one computes
       const long long en = (u + nteams) / p.nblocks;
       ptx::prefetch_l2_bulk(kPtr ? p.Ba[en] : p.B + en * (long long)p.k * p.n, (uint32_t)(p.k * p.n * 8));
     }
@@ -277,8 +314,8 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
             ptx::st_global_v2_f64(Cg + (long long)row * n_e + col0 + j * 8 + 2 * t, c[i][j][0], c[i][j][1]);
       }
       ptx::named_bar_sync(bar, kGP * 32);  // every warp finished reading buffer s
-      if ((issuer || kPtr) && pu < p.units) {  // refill it with the block nbuf ahead
-        issue(pu, pmb, s, pd);
+      if ((issuer || kPtr) && pu < units) {  // refill it with the block nbuf ahead
+        issue(pd.e, pmb, s, pd.d);
         advance();
       }
     }
@@ -393,6 +430,30 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
 }
 
+// the live units of a variable-size batch as records (warp-aggregated append)
+__global__ void gen_vb_units(long long batch, const int* dm, const int* dn, const int* dk, int max_m, int max_n,
+                             int max_k, int4* recs, int* count) {
+  for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < batch;
+       e += (long long)gridDim.x * blockDim.x) {
+    const int m = __ldg(dm + e), n = __ldg(dn + e), k = __ldg(dk + e);
+    const bool ok = m >= 8 && n >= 8 && k >= 8 && m <= max_m && n <= max_n && k <= max_k && m % 8 == 0 &&
+                    n % 8 == 0 && k % 8 == 0;
+    const int nb = ok ? (n + kGNB - 1) / kGNB : 0;
+    const unsigned act = __activemask();
+    int incl = nb;  // inclusive warp scan of the unit counts
+    const int lane = threadIdx.x & 31;
+    for (int o = 1; o < 32; o <<= 1) {
+      const int v = __shfl_up_sync(act, incl, o);
+      if (lane >= o) incl += v;
+    }
+    const int last = 31 - __clz(act);
+    int base = 0;
+    if (lane == last) base = atomicAdd(count, incl);
+    base = __shfl_sync(act, base, last) + incl - nb;
+    for (int j = 0; j < nb; ++j) recs[base + j] = make_int4((int)e, j, m | (n << 16), k);
+  }
+}
+
 // Variable sizes (kami_gemm_vbatched, FP64; "supports various
 // matrix orders in a batch"): the pointer-array kernel with per-entry m, n, k
 // read on the device, planned for the largest (max_m, max_n, max_k).
@@ -426,6 +487,18 @@ kami_status_t dmma_gen_vb_launch(long long batch, const int* dm, const int* dn, 
   p.park_bytes = gp.park_bytes;
   p.teams = gp.teams;
   p.nbuf = gp.nbuf;
+  // unit records of the live units (stream-ordered workspace, freed after the kernel)
+  void* ws = nullptr;
+  if (cudaMallocAsync(&ws, 16 + sizeof(int4) * (size_t)p.units, stream) != cudaSuccess) return KAMI_ERROR_CUDA;
+  int* count = static_cast<int*>(ws);
+  int4* recs = reinterpret_cast<int4*>(static_cast<char*>(ws) + 16);
+  cudaMemsetAsync(count, 0, sizeof(int), stream);
+  {
+    const int blocks = (int)((batch + 255) / 256 < 1184 ? (batch + 255) / 256 : 1184);
+    gen_vb_units<<<blocks, 256, 0, stream>>>(batch, dm, dn, dk, max_m, max_n, max_k, recs, count);
+  }
+  p.recs = recs;
+  p.count = count;
   auto fn = gp.rk == kRK ? kami_dmma_gen_kernel<kRK, true> : kami_dmma_gen_kernel<kRKSmall, true>;
   if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)gp.smem) != cudaSuccess)
     return KAMI_ERROR_CUDA;
@@ -436,8 +509,10 @@ kami_status_t dmma_gen_vb_launch(long long batch, const int* dm, const int* dn, 
   long long grid = sms < need ? sms : need;
   grid = apply_grid_cap(grid);
   fn<<<(unsigned)grid, kGP * 32 * (gp.rk == kRK ? 2 : 4), gp.smem, stream>>>(p);
+  const cudaError_t le = cudaGetLastError();
+  cudaFreeAsync(ws, stream);  // stream-ordered: after the kernel
   set_last_kernel("kami_dmma_gen_1d<vbatched>");
-  return (kami_status_t)launch_status((int)cudaGetLastError());
+  return (kami_status_t)launch_status((int)le);
 }
 
 }  // namespace kami
