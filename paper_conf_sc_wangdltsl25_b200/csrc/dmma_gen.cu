@@ -430,87 +430,109 @@ kami_status_t dmma_gen_launch(int m, int n, int k, long long batch, const void* 
   return cudaGetLastError() == cudaSuccess ? KAMI_SUCCESS : KAMI_ERROR_CUDA;
 }
 
-// the live units of a variable-size batch as records (warp-aggregated append)
+// the live units of a variable-size batch as records, in three k buckets
+// (k <= 32, k <= 128, k > 128: each launched with its own plan), by a
+// warp-aggregated append per bucket
+constexpr int kVbBuckets = 3;
+__host__ __device__ __forceinline__ int gen_bucket(int k) { return k <= 32 ? 0 : k <= 128 ? 1 : 2; }
 __global__ void gen_vb_units(long long batch, const int* dm, const int* dn, const int* dk, int max_m, int max_n,
-                             int max_k, int4* recs, int* count) {
+                             int max_k, int4* recs, long long stride, int* count) {
   for (long long e = blockIdx.x * (long long)blockDim.x + threadIdx.x; e < batch;
        e += (long long)gridDim.x * blockDim.x) {
     const int m = __ldg(dm + e), n = __ldg(dn + e), k = __ldg(dk + e);
     const bool ok = m >= 8 && n >= 8 && k >= 8 && m <= max_m && n <= max_n && k <= max_k && m % 8 == 0 &&
                     n % 8 == 0 && k % 8 == 0;
     const int nb = ok ? (n + kGNB - 1) / kGNB : 0;
+    const int bk = gen_bucket(k);
     const unsigned act = __activemask();
-    int incl = nb;  // inclusive warp scan of the unit counts
-    const int lane = threadIdx.x & 31;
-    for (int o = 1; o < 32; o <<= 1) {
-      const int v = __shfl_up_sync(act, incl, o);
-      if (lane >= o) incl += v;
+    const int lane = threadIdx.x & 31, last = 31 - __clz(act);
+#pragma unroll
+    for (int b = 0; b < kVbBuckets; ++b) {
+      const int mine = bk == b ? nb : 0;
+      int incl = mine;  // inclusive warp scan of this bucket's unit counts
+      for (int o = 1; o < 32; o <<= 1) {
+        const int v = __shfl_up_sync(act, incl, o);
+        if (lane >= o) incl += v;
+      }
+      int base = 0;
+      if (lane == last && incl) base = atomicAdd(count + b, incl);
+      base = __shfl_sync(act, base, last) + incl - mine;
+      for (int j = 0; j < mine; ++j) recs[b * stride + base + j] = make_int4((int)e, j, m | (n << 16), k);
     }
-    const int last = 31 - __clz(act);
-    int base = 0;
-    if (lane == last) base = atomicAdd(count, incl);
-    base = __shfl_sync(act, base, last) + incl - nb;
-    for (int j = 0; j < nb; ++j) recs[base + j] = make_int4((int)e, j, m | (n << 16), k);
   }
 }
 
 // Variable sizes (kami_gemm_vbatched, FP64; "supports various
 // matrix orders in a batch"): the pointer-array kernel with per-entry m, n, k
-// read on the device, planned for the largest (max_m, max_n, max_k).
+// read on the device, one launch per k bucket planned for (max_m, max_n,
+// the bucket's largest k): the A buffers and parked slabs of a k <= 32 bucket
+// leave four teams per SM where a plan for k = 256 leaves one.
 kami_status_t dmma_gen_vb_launch(long long batch, const int* dm, const int* dn, const int* dk, int max_m, int max_n,
                                  int max_k, const void* const* Aa, const void* const* Ba, void* const* Ca,
                                  cudaStream_t stream) {
   if (!dmma_gen_supported(max_m, max_n, max_k)) return KAMI_ERROR_NOT_SUPPORTED;
   if (!dm || !dn || !dk || !Aa || !Ba || !Ca) return KAMI_ERROR_INVALID_VALUE;
-  DmmaGenParams p;
-  memset(&p, 0, sizeof(p));
-  p.Aa = reinterpret_cast<const double* const*>(Aa);
-  p.Ba = reinterpret_cast<const double* const*>(Ba);
-  p.Ca = reinterpret_cast<double* const*>(Ca);
-  p.dm = dm;
-  p.dn = dn;
-  p.dk = dk;
-  p.batch = batch;
-  p.m = max_m;
-  p.n = max_n;
-  p.k = max_k;
-  p.ks = max_k / 4;
-  const GenPlan gp = gen_plan(max_m, max_n, max_k);
-  if (gp.smem > (uint32_t)kGenSmem) return KAMI_ERROR_NOT_SUPPORTED;
-  p.rs = gp.rs;
-  p.nblocks = (max_n + kGNB - 1) / kGNB;
-  p.mblocks = (max_m + kGTM - 1) / kGTM;
-  p.ce_shift = gp.ce_shift;
-  p.swz_bits = gp.ce_shift == 4 ? 3 : 2;
-  p.units = batch * p.nblocks;
-  p.a_block_bytes = gp.a_block_bytes;
-  p.park_bytes = gp.park_bytes;
-  p.teams = gp.teams;
-  p.nbuf = gp.nbuf;
-  // unit records of the live units (stream-ordered workspace, freed after the kernel)
+  const int nbmax = (max_n + kGNB - 1) / kGNB;
+  const long long stride = batch * nbmax;
   void* ws = nullptr;
-  if (cudaMallocAsync(&ws, 16 + sizeof(int4) * (size_t)p.units, stream) != cudaSuccess) return KAMI_ERROR_CUDA;
+  if (cudaMallocAsync(&ws, 16 + sizeof(int4) * (size_t)stride * kVbBuckets, stream) != cudaSuccess)
+    return KAMI_ERROR_CUDA;
   int* count = static_cast<int*>(ws);
   int4* recs = reinterpret_cast<int4*>(static_cast<char*>(ws) + 16);
-  cudaMemsetAsync(count, 0, sizeof(int), stream);
+  cudaMemsetAsync(count, 0, sizeof(int) * kVbBuckets, stream);
   {
     const int blocks = (int)((batch + 255) / 256 < 1184 ? (batch + 255) / 256 : 1184);
-    gen_vb_units<<<blocks, 256, 0, stream>>>(batch, dm, dn, dk, max_m, max_n, max_k, recs, count);
+    gen_vb_units<<<blocks, 256, 0, stream>>>(batch, dm, dn, dk, max_m, max_n, max_k, recs, stride, count);
   }
-  p.recs = recs;
-  p.count = count;
-  auto fn = gp.rk == kRK ? kami_dmma_gen_kernel<kRK, true> : kami_dmma_gen_kernel<kRKSmall, true>;
-  if (cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)gp.smem) != cudaSuccess)
-    return KAMI_ERROR_CUDA;
+  cudaError_t le = cudaGetLastError();
   int dev = 0, sms = 148;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  const long long need = (p.units + p.teams - 1) / p.teams;
-  long long grid = sms < need ? sms : need;
-  grid = apply_grid_cap(grid);
-  fn<<<(unsigned)grid, kGP * 32 * (gp.rk == kRK ? 2 : 4), gp.smem, stream>>>(p);
-  const cudaError_t le = cudaGetLastError();
-  cudaFreeAsync(ws, stream);  // stream-ordered: after the kernel
+  const int kb_hi[kVbBuckets] = {32, 128, 256};
+  for (int b = 0; b < kVbBuckets && le == cudaSuccess; ++b) {
+    const int klo = b == 0 ? 8 : kb_hi[b - 1] + 8;
+    if (max_k < klo) break;  // no entry can fall in this bucket
+    const int kb = max_k < kb_hi[b] ? max_k : kb_hi[b];
+    DmmaGenParams p;
+    memset(&p, 0, sizeof(p));
+    p.Aa = reinterpret_cast<const double* const*>(Aa);
+    p.Ba = reinterpret_cast<const double* const*>(Ba);
+    p.Ca = reinterpret_cast<double* const*>(Ca);
+    p.dm = dm;
+    p.dn = dn;
+    p.dk = dk;
+    p.batch = batch;
+    p.m = max_m;
+    p.n = max_n;
+    p.k = kb;
+    p.ks = kb / 4;
+    const GenPlan gp = gen_plan(max_m, max_n, kb);
+    if (gp.smem > (uint32_t)kGenSmem) {
+      le = cudaErrorInvalidValue;
+      break;
+    }
+    p.rs = gp.rs;
+    p.nblocks = nbmax;
+    p.mblocks = (max_m + kGTM - 1) / kGTM;
+    p.ce_shift = gp.ce_shift;
+    p.swz_bits = gp.ce_shift == 4 ? 3 : 2;
+    p.units = stride;  // upper bound; the kernel reads the bucket's count
+    p.a_block_bytes = gp.a_block_bytes;
+    p.park_bytes = gp.park_bytes;
+    p.teams = gp.teams;
+    p.nbuf = gp.nbuf;
+    p.recs = recs + b * stride;
+    p.count = count + b;
+    auto fn = gp.rk == kRK ? kami_dmma_gen_kernel<kRK, true> : kami_dmma_gen_kernel<kRKSmall, true>;
+    if ((le = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)gp.smem)) != cudaSuccess)
+      break;
+    const long long need = (p.units + p.teams - 1) / p.teams;
+    long long grid = sms < need ? sms : need;
+    grid = apply_grid_cap(grid);
+    fn<<<(unsigned)grid, kGP * 32 * (gp.rk == kRK ? 2 : 4), gp.smem, stream>>>(p);
+    le = cudaGetLastError();
+  }
+  cudaFreeAsync(ws, stream);  // stream-ordered: after the kernels
   set_last_kernel("kami_dmma_gen_1d<vbatched>");
   return (kami_status_t)launch_status((int)le);
 }
