@@ -177,3 +177,26 @@ def test_product_and_oracle_share_no_code():
             txt = open(os.path.join(ROOT, "oracle", f)).read()
             assert not re.search(r"^\s*(import|from)\s+(paper_conf_sc_wangdltsl25_b200|kami_inputs)\b|"
                                  r"#include\s+\"[^\"]*(kami|csrc)", txt, re.M), f
+
+
+def test_xt_plan_host_rules():
+    """The transposed-product kernel (kernel 7, KAMI_ALGO_1D_XT): the shapes it
+    runs, its unit geometry, and the model picks measured on one B200
+    (profiles/r2/xt_r2.md): XT for thin m with k = 16 and n >= 128 / the pair
+    tiles of n = 64, the SS kernel where its single-entry tiles stream better."""
+    for m, n, k in [(16, 128, 16), (16, 192, 16), (16, 64, 16), (32, 256, 64)]:
+        p = kami.plan(m, n, k, "bf16", algo="1d_xt")
+        assert p["kernel"] == "tcgen05_xt" and p["algo"] == "1d_xt", (m, n, k, p)
+        assert p["stages"] >= 3 and p["entries_per_cta"] >= 3, p
+    for m, n, k in [(48, 128, 16), (16, 96, 16), (16, 128, 48), (16, 128, 128), (8, 128, 16)]:
+        with pytest.raises(kami.KamiError):
+            kami.plan(m, n, k, "bf16", algo="1d_xt")
+    with pytest.raises(kami.KamiError):
+        kami.plan(16, 128, 16, "f64", algo="1d_xt")
+    assert kami.plan(16, 128, 16, "bf16")["kernel"] == "tcgen05_xt"   # 0.88 vs 0.43 (SS)
+    assert kami.plan(16, 192, 16, "bf16")["kernel"] == "tcgen05_xt"   # 0.87 vs 0.52
+    assert kami.plan(16, 64, 16, "bf16")["kernel"] == "tcgen05_xt"    # 0.88 vs 0.65 (pair tiles)
+    assert kami.plan(16, 192, 64, "bf16")["kernel"] == "tcgen05"      # 1.00 vs 0.96
+    assert kami.plan(64, 64, 64, "f16")["kernel"] == "tcgen05"        # the headline stays on SS
+    # column-major C is the row problem n x m: thin n runs the XT kernel
+    assert kami.plan(128, 16, 16, "bf16", layout="col")["kernel"] == "tcgen05_xt"
