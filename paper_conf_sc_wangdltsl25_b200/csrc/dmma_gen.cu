@@ -122,10 +122,22 @@ struct GenUnit {
   GenDims d;
   bool live;
 };
+__device__ __forceinline__ GenUnit gen_unit_rec(const DmmaGenParams& p, const int4 q);
 __device__ __forceinline__ GenUnit gen_unit(const DmmaGenParams& p, long long u) {
   GenUnit r;
-  if (p.recs) {
-    const int4 q = __ldg(p.recs + u);
+  if (p.recs) return gen_unit_rec(p, __ldg(p.recs + u));
+  {
+    r.e = u / p.nblocks;
+    r.nb = (int)(u - r.e * p.nblocks);
+    r.d = gen_dims(p, r.e);
+    r.live = gen_live(p, r.d, r.nb);
+  }
+  return r;
+}
+// a unit record already in registers (loaded a unit earlier by the consumer)
+__device__ __forceinline__ GenUnit gen_unit_rec(const DmmaGenParams& p, const int4 q) {
+  GenUnit r;
+  {
     r.e = q.x;
     r.nb = q.y;
     r.d.m = q.z & 0xFFFF;
@@ -135,11 +147,6 @@ __device__ __forceinline__ GenUnit gen_unit(const DmmaGenParams& p, long long u)
     r.d.mblocks = (r.d.m + kGTM - 1) / kGTM;
     r.d.swz_bits = r.d.ce_shift == 4 ? 3u : 2u;
     r.live = true;
-  } else {
-    r.e = u / p.nblocks;
-    r.nb = (int)(u - r.e * p.nblocks);
-    r.d = gen_dims(p, r.e);
-    r.live = gen_live(p, r.d, r.nb);
   }
   return r;
 }
@@ -228,8 +235,14 @@ __global__ void __launch_bounds__(RK == kRK ? kGP * 32 * 2 : kGP * 32 * 4, 1)
   }
   double b[RK][kGFN];
   RingPos ab;  // A buffer ring (slot, parity)
+  // records: the next unit's record is loaded one unit ahead and decoded at
+  // its turn (decoding right after the load put a global round trip on every
+  // unit's critical path)
+  int4 qn = make_int4(0, 0, 0, 0);
+  if (p.recs && first < units) qn = __ldg(p.recs + first);
   for (long long u = first; u < units; u += nteams) {
-    const GenUnit gu = gen_unit(p, u);
+    const GenUnit gu = p.recs ? gen_unit_rec(p, qn) : gen_unit(p, u);
+    if (p.recs && u + nteams < units) qn = __ldg(p.recs + u + nteams);
     if (!gu.live) continue;  // (the producer cursor skips it too)
     const long long e = gu.e;
     const int nb = gu.nb;
